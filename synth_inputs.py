@@ -1,0 +1,110 @@
+"""Seeded synthetic input generators shared by the oracle tests, the GPU
+parity tests and bench.py.
+
+This module holds NONE of the method's arithmetic (no checksums, no
+thresholds, no factorizations): it only draws matrices and fault plans from
+seeded generators, following the input recipe of DESIGN.md §3:
+
+* general (LU, QR, bandwidth sweep): A_ij ~ U(-1, 1);
+* SPD (Cholesky): A = (M + M^T)/2 + n*I with M ~ U(-1, 1);
+* integer tiles (exact-sum pins): A_ij uniform integers in [-R, R];
+* bit-flip plans (paper §X.A): element positions and XOR masks.
+
+Host arrays are numpy, float64 unless a dtype is given; `*_device` variants
+draw on the GPU with a seeded torch generator so the multi-GiB bench inputs
+never touch the host.  Semantics are mathematical (A[i, j] = row i, column
+j); the binding is responsible for the column-major layout of the C ABI.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+
+def rng(seed: int) -> np.random.Generator:
+    return np.random.Generator(np.random.PCG64(seed))
+
+
+def general(m: int, n: int | None = None, seed: int = 0, dtype=np.float64) -> np.ndarray:
+    """U(-1,1) general matrix (SURVEY §8d 'general')."""
+    n = m if n is None else n
+    return rng(seed).uniform(-1.0, 1.0, size=(m, n)).astype(dtype)
+
+
+def spd(n: int, seed: int = 0, dtype=np.float64) -> np.ndarray:
+    """(M + M^T)/2 + n*I, M ~ U(-1,1): diagonally dominant SPD."""
+    M = rng(seed).uniform(-1.0, 1.0, size=(n, n))
+    S = (M + M.T) * 0.5
+    S[np.diag_indices(n)] += n
+    return S.astype(dtype)
+
+
+def integers(m: int, n: int | None = None, seed: int = 0, R: int = 64, dtype=np.float64) -> np.ndarray:
+    """Integer-valued matrix in [-R, R]; every checksum of it is an exactly
+    representable integer, so sums are bit-exact in any order."""
+    n = m if n is None else n
+    return rng(seed).integers(-R, R + 1, size=(m, n)).astype(dtype)
+
+
+def flip_bits(value: float, bits, dtype=np.float64) -> float:
+    """XOR the given bit positions of one IEEE value (the paper's XOR fault,
+    L540).  Pure bit manipulation, no arithmetic of the method."""
+    if dtype == np.float64:
+        u = np.array([value], dtype=np.float64).view(np.uint64)
+        mask = np.uint64(0)
+        for b in bits:
+            mask |= np.uint64(1) << np.uint64(b)
+        return float((u ^ mask).view(np.float64)[0])
+    u = np.array([value], dtype=np.float32).view(np.uint32)
+    mask = np.uint32(0)
+    for b in bits:
+        mask |= np.uint32(1) << np.uint32(b)
+    return float((u ^ mask).view(np.float32)[0])
+
+
+def mask_of(bits) -> int:
+    m = 0
+    for b in bits:
+        m |= 1 << int(b)
+    return m
+
+
+def random_positions(n_tiles_r: int, n_tiles_c: int, nb: int, seed: int, lower_only: bool = False):
+    """One random (local i, local j) per tile: the config-1 'one flip per
+    tile' plan (BASELINE configs[0], paper L275 single-fault assumption)."""
+    g = rng(seed)
+    out = []
+    for J in range(n_tiles_c):
+        for I in range(n_tiles_r):
+            if lower_only and I < J:
+                continue
+            out.append((I, J, int(g.integers(0, nb)), int(g.integers(0, nb))))
+    return out
+
+
+# ---------------------------------------------------------------- device --
+def general_device(m: int, n: int | None = None, seed: int = 0, dtype=None, device="cuda"):
+    """Column-major U(-1,1) matrix drawn on the GPU (bench-sized inputs)."""
+    import torch
+
+    n = m if n is None else n
+    dtype = dtype or torch.float64
+    g = torch.Generator(device=device)
+    g.manual_seed(seed)
+    # storage (n, m) row-major == (m, n) column-major
+    buf = torch.rand((n, m), generator=g, dtype=dtype, device=device)
+    buf.mul_(2.0).sub_(1.0)
+    return buf.t()
+
+
+def spd_device(n: int, seed: int = 0, dtype=None, device="cuda"):
+    """Column-major (M + M^T)/2 + n*I drawn on the GPU."""
+    import torch
+
+    dtype = dtype or torch.float64
+    M = general_device(n, n, seed, dtype, device)  # column-major view
+    S = M.t().contiguous()  # row-major copy of M^T
+    S.add_(M.t().t())  # += M  (M^T + M), elementwise in place
+    S.mul_(0.5)
+    S.diagonal().add_(float(n))
+    del M
+    return S.t()  # symmetric: column-major view of the same data
