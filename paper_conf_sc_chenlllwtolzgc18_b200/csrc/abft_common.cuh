@@ -1,0 +1,136 @@
+// Internal helpers of the sm_100a ABFT library (not part of the C ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdio.h>
+
+#include "abft.h"
+
+#define ABFT_CUDA_TRY(expr)                                                              \
+  do {                                                                                   \
+    cudaError_t _e = (expr);                                                             \
+    if (_e != cudaSuccess) {                                                             \
+      fprintf(stderr, "[abft] CUDA error %s at %s:%d: %s\n", cudaGetErrorName(_e),      \
+              __FILE__, __LINE__, cudaGetErrorString(_e));                               \
+      return ABFT_E_CUDA;                                                                \
+    }                                                                                    \
+  } while (0)
+
+namespace abft {
+
+// ---------------------------------------------------------------- tiles --
+// Enumerate the tiles of a range in column-major tile order (J outer, I
+// inner), skipping I < J when lower_only.  Device and host.
+__host__ __device__ inline int64_t tiles_count(const abft_tiles_t& t) {
+  int64_t c = 0;
+  for (int J = t.J0; J < t.J1; ++J) {
+    int lo = t.lower_only ? (t.I0 > J ? t.I0 : J) : t.I0;
+    if (t.I1 > lo) c += t.I1 - lo;
+  }
+  return c;
+}
+
+__host__ __device__ inline void tile_of(const abft_tiles_t& t, int64_t idx, int& I, int& J) {
+  for (J = t.J0; J < t.J1; ++J) {
+    int lo = t.lower_only ? (t.I0 > J ? t.I0 : J) : t.I0;
+    int64_t cnt = t.I1 > lo ? t.I1 - lo : 0;
+    if (idx < cnt) {
+      I = lo + (int)idx;
+      return;
+    }
+    idx -= cnt;
+  }
+  I = -1;
+}
+
+// ------------------------------------------------------------ precision --
+template <typename T> struct Prec;
+template <> struct Prec<double> {
+  static constexpr double u = 1.1102230246251565e-16;  // 2^-53
+};
+template <> struct Prec<float> {
+  static constexpr double u = 5.9604644775390625e-08;  // 2^-24
+};
+
+// tau_e = scale * 2 * gamma_nb * m  (DESIGN.md c-6; gamma_k = k u/(1-k u), L133)
+template <typename T>
+__host__ __device__ inline double tau_factor(int nb, double scale) {
+  double ku = nb * Prec<T>::u;
+  return scale * 2.0 * ku / (1.0 - ku);
+}
+
+// ------------------------------------------------------------- PTX bits --
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_fence_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      " .reg .pred p;\n"
+      "WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+// 1-D TMA bulk copy global -> shared, completion counted on `bar` (bytes).
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// --------------------------------------------------------------- math --
+// Explicit round-to-nearest ops so the compiler cannot re-contract: the
+// encode and verify instantiations then produce bit-identical sums.
+__device__ __forceinline__ double fadd(double a, double b) { return __dadd_rn(a, b); }
+__device__ __forceinline__ float fadd(float a, float b) { return __fadd_rn(a, b); }
+__device__ __forceinline__ double ffma(double a, double b, double c) { return __fma_rn(a, b, c); }
+__device__ __forceinline__ float ffma(float a, float b, float c) { return __fmaf_rn(a, b, c); }
+
+template <typename T>
+__device__ __forceinline__ T shfl_xor(T v, int m) {
+  return __shfl_xor_sync(0xffffffffu, v, m);
+}
+
+// Value of view element (i, j) of a diagonal tile (c-3) given the stored
+// element x = A[i][j] (for SYM the caller handles mirroring).
+template <typename T>
+__device__ __forceinline__ T view_mask(int view, int i, int j, T x) {
+  switch (view) {
+    case ABFT_LOWER: return i >= j ? x : T(0);
+    case ABFT_UNIT_LOWER: return i > j ? x : (i == j ? T(1) : T(0));
+    case ABFT_UPPER: return i <= j ? x : T(0);
+    default: return x;
+  }
+}
+
+}  // namespace abft
+
+// Runtime (abft_runtime.cu)
+namespace abft {
+struct Workspace {
+  void* ptr = nullptr;
+  size_t bytes = 0;
+};
+// Per-stream scratch of at least `bytes` (grown on demand, never shrunk).
+int workspace_get(cudaStream_t s, size_t bytes, void** out);
+// Per-stream zero-initialised counter area (self-resetting kernels use it).
+int counters_get(cudaStream_t s, size_t n_ints, int** out);
+}  // namespace abft

@@ -1,0 +1,292 @@
+"""GPU parity of the checksum hot path (§8 rows a1–a3) against the oracle,
+called through the C ABI (ctypes binding)."""
+import numpy as np
+import pytest
+import torch
+
+import synth_inputs as si
+from oracle import checksum as ck
+from tests.gpu_helpers import dev, gpu_state_to_oracle, host, normwise_err
+
+pytestmark = pytest.mark.gpu
+
+TOL = {"f64": 1e-12, "f32": 1e-5}
+TDT = {"f64": torch.float64, "f32": torch.float32}
+NDT = {"f64": np.float64, "f32": np.float32}
+
+
+def _encode(lib, A_np, nb, prec="f64", view=ck.GENERAL, lower_only=False, which=ck.BOTH, mags=True, ld=None):
+    A = dev(A_np, TDT[prec], ld=ld)
+    mat = lib.Mat.alloc(A, nb, mags=mags)
+    t = lib.tiles(0, mat.mt, 0, mat.nt, lower_only, view)
+    lib.abft_encode(mat, t, which)
+    torch.cuda.synchronize()
+    return mat, t
+
+
+def _oracle_state(A_np, nb, prec="f64", view=ck.GENERAL, lower_only=False, which=ck.BOTH, mags=True):
+    A64 = A_np.astype(NDT[prec]).astype(np.float64)
+    st = ck.State.alloc(A64, nb, prec=prec, mags=mags)
+    ck.encode(st, ck.Tiles(0, st.mt, 0, st.nt, lower_only, view), which)
+    return st
+
+
+def _compare_encode(mat, st, prec, lower_only=False, view=ck.GENERAL, exact=False):
+    g = gpu_state_to_oracle(mat, prec)
+    nb = st.nb
+    worst = 0.0
+    for I, J in ck.Tiles(0, st.mt, 0, st.nt, lower_only, view):
+        v = view if I == J else ck.GENERAL
+        X = ck.tile_view(st.A, I, J, nb, v)
+        cs, rs = slice(J * nb, (J + 1) * nb), slice(I * nb, (I + 1) * nb)
+        cg, cr = g.colchk[2 * I:2 * I + 2, cs], st.colchk[2 * I:2 * I + 2, cs]
+        rg, rr = g.rowchk[rs, 2 * J:2 * J + 2], st.rowchk[rs, 2 * J:2 * J + 2]
+        if exact:
+            assert np.array_equal(cg, cr) and np.array_equal(rg, rr), (I, J)
+            assert np.array_equal(g.colmag[I, cs], st.colmag[I, cs])
+        worst = max(worst, normwise_err(cg, cr, X, 0), normwise_err(rg, rr, X, 1))
+        mag_err = np.abs(g.colmag[I, cs] - st.colmag[I, cs]) / np.maximum(st.colmag[I, cs], 1e-300)
+        worst = max(worst, float(mag_err.max()))
+    assert worst <= TOL[prec], worst
+    return worst
+
+
+@pytest.mark.parametrize("prec", ["f64", "f32"])
+@pytest.mark.parametrize("nb", [32, 64, 128, 256, 512, 1024])
+def test_encode_integer_bit_exact(lib, prec, nb):
+    n = 2 * nb if nb >= 512 else 4 * nb
+    A = si.integers(n, seed=nb, R=8 if prec == "f32" else 1000)
+    mat, _ = _encode(lib, A, nb, prec)
+    st = _oracle_state(A, nb, prec)
+    _compare_encode(mat, st, prec, exact=True)
+
+
+@pytest.mark.parametrize("prec", ["f64", "f32"])
+@pytest.mark.parametrize("nb,m,n", [(32, 256, 256), (64, 192, 320), (128, 384, 256), (256, 512, 768),
+                                    (512, 1024, 1536), (1024, 2048, 1024)])
+def test_encode_random_normwise(lib, prec, nb, m, n):
+    A = si.general(m, n, seed=m + n)
+    mat, _ = _encode(lib, A, nb, prec)
+    st = _oracle_state(A, nb, prec)
+    _compare_encode(mat, st, prec)
+
+
+@pytest.mark.parametrize("view", [ck.SYM_LOWER, ck.LOWER, ck.UNIT_LOWER, ck.UPPER])
+@pytest.mark.parametrize("nb", [32, 256, 1024])
+def test_encode_diag_views(lib, view, nb):
+    n = 2 * nb
+    A = si.spd(n, seed=3) if view == ck.SYM_LOWER else si.general(n, seed=3)
+    lower = view == ck.SYM_LOWER
+    mat, _ = _encode(lib, A, nb, "f64", view=view, lower_only=lower)
+    st = _oracle_state(A, nb, "f64", view=view, lower_only=lower)
+    _compare_encode(mat, st, "f64", lower_only=lower, view=view)
+
+
+def test_encode_odd_leading_dimension(lib):
+    # lda*8 not a multiple of 16 -> the non-TMA staging path
+    A = si.general(256, seed=4)
+    mat, _ = _encode(lib, A, 64, "f64", ld=257)
+    assert mat.A.stride(1) == 257
+    st = _oracle_state(A, 64, "f64")
+    _compare_encode(mat, st, "f64")
+
+
+@pytest.mark.parametrize("prec", ["f64", "f32"])
+@pytest.mark.parametrize("nb,n", [(32, 256), (256, 1024), (512, 2048), (1024, 2048), (1024, 4096), (512, 8192)])
+def test_verify_after_encode_is_exactly_zero(lib, prec, nb, n):
+    """c-27 pin: one deterministic reduction order -> delta == 0 bit-exactly,
+    whatever slab split the launcher picks for the tile count."""
+    A = si.general(n, seed=nb)
+    mat, t = _encode(lib, A, nb, prec)
+    rep = lib.Report.alloc(mat, deltas=True)
+    lib.abft_verify(mat, t, ck.BOTH, lib.abft_tol_t(ck.TOL_MAGNITUDE, 1.0), rep)
+    # a sub-range (different grid / slab split) must also be exact
+    sub = lib.tiles(1, mat.mt, 0, 1)
+    lib.abft_verify(mat, sub, ck.BOTH, lib.abft_tol_t(ck.TOL_MAGNITUDE, 1.0), rep)
+    torch.cuda.synchronize()
+    assert torch.count_nonzero(rep.dcol) == 0 and torch.count_nonzero(rep.drow) == 0
+    assert torch.count_nonzero(rep.status) == 0 and torch.count_nonzero(rep.counts) == 0
+
+
+def test_verify_sym_lower_after_encode_is_zero(lib):
+    A = si.spd(1024, seed=5)
+    mat, t = _encode(lib, A, 256, "f64", view=ck.SYM_LOWER, lower_only=True)
+    rep = lib.Report.alloc(mat, deltas=True)
+    lib.abft_verify(mat, t, ck.BOTH, lib.abft_tol_t(ck.TOL_MAGNITUDE, 1.0), rep)
+    torch.cuda.synchronize()
+    assert torch.count_nonzero(rep.status) == 0 and torch.count_nonzero(rep.dcol) == 0
+
+
+def _fix_tuple_list(fixes):
+    return sorted((f[0], f[1], f[4], f[5]) for f in fixes)
+
+
+def _run_locate(lib, mat, t, which, view=ck.GENERAL, tol=None):
+    tol = tol or lib.abft_tol_t(ck.TOL_MAGNITUDE, 1.0)
+    rep = lib.Report.alloc(mat)
+    lib.abft_verify(mat, t, which, tol, rep)
+    status_v = host(rep.status.clone()).astype(int)
+    fixbuf = torch.zeros(4096 * lib.FIX_BYTES, dtype=torch.uint8, device="cuda")
+    nfix = torch.zeros(1, dtype=torch.int32, device="cuda")
+    lib.abft_locate_correct(mat, t, which, tol, rep, fixbuf, nfix)
+    torch.cuda.synchronize()
+    n = int(nfix.item())
+    return status_v, host(rep.status).astype(int), rep.counts.cpu().numpy(), lib.decode_fixes(fixbuf, n)
+
+
+def _oracle_locate(st, t_or, which):
+    status_v, counts_v = ck.verify(st, t_or, which)
+    status_f, fixes, counts_f = ck.locate_correct(st, t_or, which)
+    return status_v, counts_v, status_f, fixes, counts_f
+
+
+def _compare_locate(lib, A_np, nb, mutate, which=ck.BOTH, view=ck.GENERAL, lower_only=False):
+    """Apply the same corruption on both sides; flags, classes, positions must
+    agree exactly; corrected data within the fp64 tolerance."""
+    mat, t = _encode(lib, A_np, nb, "f64", view=view, lower_only=lower_only)
+    st = _oracle_state(A_np, nb, "f64", view=view, lower_only=lower_only)
+    mutate(st, mat)
+    torch.cuda.synchronize()
+    sv, sf, counts, fixes = _run_locate(lib, mat, t, which, view)
+    t_or = ck.Tiles(0, st.mt, 0, st.nt, lower_only, view)
+    osv, ocv, osf, ofixes, ocf = _oracle_locate(st, t_or, which)
+    for (I, J), s in osv.items():
+        assert sv[I, J] == s, ((I, J), sv[I, J], s)
+    assert list(counts[:4]) == ocv, (counts, ocv)
+    for (I, J), s in osf.items():
+        assert sf[I, J] == s, ((I, J), sf[I, J], s)
+    assert list(counts[4:]) == ocf, (counts[4:], ocf)
+    assert _fix_tuple_list(fixes) == sorted((f.gi, f.gj, f.cls, f.kind) for f in ofixes)
+    g = gpu_state_to_oracle(mat)
+    scale = np.abs(st.A).max()
+    assert np.abs(g.A - st.A).max() <= 1e-12 * scale
+    return fixes
+
+
+def _set(st, mat, i, j, value):
+    st.A[i, j] = value
+    mat.A[i, j] = value
+
+
+def test_locate_0d_every_tile_config1(lib):
+    """BASELINE configs[0] shape: fp64 SPD n=256 nb=32, one MUST-band flip in
+    every lower tile (paper L275: one fault per block between checks)."""
+    nb, n = 32, 256
+    A = si.spd(n, seed=0)
+    plan = si.random_positions(n // nb, n // nb, nb, seed=1, lower_only=True)
+    g = si.rng(2)
+
+    def mutate(st, mat):
+        for I, J, i, j in plan:
+            gi, gj = I * nb + i, J * nb + j
+            if I == J and i < j:
+                gi, gj = I * nb + j, J * nb + i  # stored lower element
+            bit = int(g.integers(40, 64))
+            _set(st, mat, gi, gj, si.flip_bits(A[gi, gj], [bit]))
+
+    fixes = _compare_locate(lib, A, nb, mutate, view=ck.SYM_LOWER, lower_only=True)
+    assert len([f for f in fixes if f[5] == ck.FIX_DATA]) == len(plan)
+
+
+@pytest.mark.parametrize("case", ["1d_row", "1d_col", "chk_e", "chk_w", "stale_r", "stale_c", "2d", "inf", "nan",
+                                  "huge"])
+def test_locate_classes_match_oracle(lib, case):
+    A = si.general(128, seed=30)
+    nb = 64
+
+    def mutate(st, mat):
+        if case == "1d_row":
+            for j in range(64, 72):
+                _set(st, mat, 70, j, A[70, j] + j)
+        elif case == "1d_col":
+            for i in range(0, 64, 5):
+                _set(st, mat, i, 100, A[i, 100] - 3.0)
+        elif case in ("chk_e", "chk_w"):
+            w = 0 if case == "chk_e" else 1
+            st.colchk[2 + w, 10] += 50.0
+            mat.colchk[2 + w, 10] += 50.0
+        elif case == "stale_r":
+            for r, de, dw in [(3, 2.0, 11.0), (9, 3.0, 7.0)]:
+                st.rowchk[r, 0] += de
+                st.rowchk[r, 1] += dw
+                mat.rowchk[r, 0] += de
+                mat.rowchk[r, 1] += dw
+        elif case == "stale_c":
+            for c, de, dw in [(65, 2.0, 3.3), (70, 1.0, 2.7)]:
+                st.colchk[0, c] += de
+                st.colchk[1, c] += dw
+                mat.colchk[0, c] += de
+                mat.colchk[1, c] += dw
+        elif case == "2d":
+            _set(st, mat, 3, 4, A[3, 4] + 5.0)
+            _set(st, mat, 9, 11, A[9, 11] + 7.0)
+        elif case == "inf":
+            _set(st, mat, 33, 40, np.inf)
+        elif case == "nan":
+            _set(st, mat, 33, 40, np.nan)
+        elif case == "huge":
+            _set(st, mat, 33, 40, 1e308)
+
+    _compare_locate(lib, A, nb, mutate)
+
+
+@pytest.mark.parametrize("which", [ck.COL, ck.ROW])
+def test_locate_single_side(lib, which):
+    A = si.general(128, seed=31)
+
+    def mutate(st, mat):
+        if which == ck.COL:
+            for j in range(0, 40, 3):
+                _set(st, mat, 20, j, A[20, j] * -2.0)
+        else:
+            for i in range(64, 128, 7):
+                _set(st, mat, i, 90, A[i, 90] + 4.0)
+
+    _compare_locate(lib, A, 64, mutate, which=which)
+
+
+def test_locate_sym_pair_and_cross(lib):
+    A = si.spd(128, seed=32)
+
+    def mutate(st, mat):
+        _set(st, mat, 20, 4, A[20, 4] + 9.0)  # mirrored pair in tile (0,0)
+        r = 64 + 9  # cross in tile (1,1)
+        for j in range(64, r):
+            _set(st, mat, r, j, A[r, j] + 1.5)
+        for i in range(r + 1, 128):
+            _set(st, mat, i, r, A[i, r] + 3.5)
+        _set(st, mat, r, r, A[r, r] + 5.0)
+
+    _compare_locate(lib, A, 64, mutate, view=ck.SYM_LOWER, lower_only=True)
+
+
+def test_inject_is_xor(lib):
+    A = dev(si.general(64, seed=1))
+    before = A[5, 7].item()
+    lib.abft_inject(A, 5, 7, 1 << 62)
+    torch.cuda.synchronize()
+    assert A[5, 7].item() == si.flip_bits(before, [62])
+
+
+@pytest.mark.parametrize("prec", ["f64", "f32"])
+def test_full_size_sampled_tiles(lib, prec):
+    """BASELINE config-4 sized matrix (n=16384, nb=512): sampled tiles vs the
+    oracle, plus the verify-after-encode invariant over the whole matrix."""
+    n, nb = 16384, 512
+    A = si.general_device(n, seed=7, dtype=TDT[prec])
+    mat = lib.Mat.alloc(A, nb)
+    t = lib.tiles(0, n // nb, 0, n // nb)
+    lib.abft_encode(mat, t)
+    rep = lib.Report.alloc(mat)
+    lib.abft_verify(mat, t, ck.BOTH, lib.abft_tol_t(ck.TOL_MAGNITUDE, 1.0), rep)
+    torch.cuda.synchronize()
+    assert torch.count_nonzero(rep.counts) == 0
+    g = si.rng(3)
+    for _ in range(6):
+        I, J = int(g.integers(0, n // nb)), int(g.integers(0, n // nb))
+        X = host(A[I * nb:(I + 1) * nb, J * nb:(J + 1) * nb])
+        c, r, mc, mr = ck.encode_tile(X)
+        cg = host(mat.colchk[2 * I:2 * I + 2, J * nb:(J + 1) * nb])
+        rg = host(mat.rowchk[I * nb:(I + 1) * nb, 2 * J:2 * J + 2])
+        assert normwise_err(cg, c, X, 0) <= TOL[prec]
+        assert normwise_err(rg, r, X, 1) <= TOL[prec]
