@@ -1,0 +1,384 @@
+#!/usr/bin/env python
+"""Benchmark of the 2D weighted-checksum hot path (BASELINE.json metric:
+"checksum encode+verify GB/s vs HBM peak; ft_potrf overhead % at n=30720").
+
+One timed STEP = abft_encode + abft_verify + abft_locate_correct (a no-op
+launch when nothing is flagged) over the whole fp64 n=30720, nb=512 matrix
+(7.55 GB per pass, larger than the 126 MB L2, so no flush is needed).  The
+ft_potrf overhead half of the metric is measured in the same run: the
+fault-tolerant driver (all §8(a) rows, Alg. 2 order) vs the same driver with
+ABFT disabled, at n=30720 nb=512.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+N>1 is launched by torchrun: every rank owns its own n=30720 block-cyclic
+share (weak scaling), encodes/verifies it, and the per-step error flags are
+all-reduced over NCCL (the paper's error-report exchange, L361-L363).
+`--impl reference` times the CPU oracle (oracle/, the plain implementation
+written from the paper) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+N_MAT, NB = 30720, 512
+METRIC = "checksum encode+verify GB/s vs HBM peak; ft_potrf overhead % at n=30720"
+
+
+def alg_bytes(n, nb, es):
+    """Algorithmic bytes of one pass over an n x n matrix:
+    n^2 s read + 4 n^2/nb s checksum write (encode) or read (verify)."""
+    return n * n * es * (1.0 + 4.0 / nb)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic():
+    """dram read+write bytes per launch of the dominant kernel from the
+    committed `ncu --set full` summary (profiles/), or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_verify_summary.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        if d.get("n") == N_MAT and d.get("nb") == NB:
+            return float(d["dram_bytes_per_launch"])
+    except Exception:
+        pass
+    return None
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md)."""
+
+    def __init__(self, dev):
+        self.dev = dev
+        self.proc = None
+        self.path = f"/tmp/bench_clocks_{os.getpid()}.csv"
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.dev), f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+            self.f.close()
+
+    def summary(self):
+        try:
+            rows = [r.split(",") for r in open(self.path).read().strip().splitlines()]
+        except Exception:
+            return None
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[0]))
+                mx = max(mx, float(r[1]))
+                for nm, v in zip(names, r[3:7]):
+                    if v.strip().lower() == "active":
+                        reasons.add(nm)
+            except Exception:
+                continue
+        if not sm:
+            return None
+        sm.sort()
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------- reference --
+def run_reference(args):
+    """The oracle on the host cores: encode + verify of a bounded sample of
+    nb x nb tiles of the same fp64 U(-1,1) workload, same byte formula."""
+    import numpy as np
+
+    import synth_inputs as si
+    from oracle import checksum as ck
+
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    cores = len(os.sched_getaffinity(0))
+    nb = NB
+    n_tiles_sample = 8  # tiles per step sample
+    st = ck.State.alloc(si.general(nb * 2, nb * 4, seed=0), nb)
+    tiles = ck.Tiles(0, 2, 0, 4)
+    step_t = []
+    for s in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        ck.encode(st, tiles)
+        ck.verify(st, tiles)
+        dt = time.perf_counter() - t0
+        if s >= args.warmup:
+            step_t.append(dt)
+    bytes_step = 2 * n_tiles_sample * alg_bytes(nb, nb, 8)
+    t = sum(step_t) / len(step_t)
+    val = bytes_step / t / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": val, "unit": "GB/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"encode+verify fp64 nb={nb}, oracle sample of {n_tiles_sample} tiles per step "
+                               f"(of the n={N_MAT} matrix)", "n": N_MAT, "nb": nb},
+        "cpu_baseline": {"value": val, "unit": "GB/s", "cores": cores, "kind": "oracle",
+                         "sample": f"{n_tiles_sample} tiles of {nb}x{nb} fp64 per step"},
+        "e2e": {"value": val, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline_sample(seconds=10.0):
+    """Oracle encode+verify on host cores over a bounded sample (~10 s)."""
+    import numpy as np
+
+    import synth_inputs as si
+    from oracle import checksum as ck
+
+    nb = NB
+    st = ck.State.alloc(si.general(nb * 4, nb * 4, seed=1), nb)
+    tiles = ck.Tiles(0, 4, 0, 4)
+    done, t0 = 0, time.perf_counter()
+    while time.perf_counter() - t0 < seconds:
+        ck.encode(st, tiles)
+        ck.verify(st, tiles)
+        done += 16
+    dt = time.perf_counter() - t0
+    val = 2 * done * alg_bytes(nb, nb, 8) / dt / 1e9
+    return {"value": val, "unit": "GB/s", "cores": len(os.sched_getaffinity(0)), "kind": "oracle",
+            "sample": f"{done} tiles of {nb}x{nb} fp64 (encode+verify), {dt:.1f} s"}
+
+
+# ------------------------------------------------------------------ ours --
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import synth_inputs as si
+    from paper_conf_sc_chenlllwtolzgc18_b200 import abft
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    n, nb = args.n, NB
+    es = 8
+    # ---- workload: each rank holds its own n x n block-cyclic share (weak) ----
+    A = si.general_device(n, seed=1000 + rank)
+    mat = abft.Mat.alloc(A, nb, mags=False)
+    t_all = abft.tiles(0, n // nb, 0, n // nb)
+    rep = abft.Report.alloc(mat)
+    tol = abft.abft_tol_t(abft.TOL_MAGNITUDE, 1.0)
+    fixbuf = torch.zeros(1024 * abft.FIX_BYTES, dtype=torch.uint8, device="cuda")
+    nfix = torch.zeros(1, dtype=torch.int32, device="cuda")
+    stream = torch.cuda.current_stream()
+
+    def step(ev=None):
+        if ev:
+            ev[0].record()
+        abft.abft_encode(mat, t_all)
+        if ev:
+            ev[1].record()
+        abft.abft_verify(mat, t_all, abft.BOTH, tol, rep)
+        if ev:
+            ev[2].record()
+        abft.abft_locate_correct(mat, t_all, abft.BOTH, tol, rep, fixbuf, nfix)
+        if world > 1:
+            dist.all_reduce(rep.counts)  # error-flag reduce (L361-L363)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    t0e, t1e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with Clocks(local) as clk:
+        torch.cuda.synchronize()
+        t0e.record()
+        for s in range(args.steps):
+            step(evs[s])
+        t1e.record()
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ms = t0e.elapsed_time(t1e)
+    enc_ms = sum(e[0].elapsed_time(e[1]) for e in evs) / args.steps
+    ver_ms = sum(e[1].elapsed_time(e[2]) for e in evs) / args.steps
+    assert int(rep.counts.sum().item()) == 0, "error-free input flagged"
+    if world > 1:
+        tt = torch.tensor([ms], device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms = float(tt.item())
+    pass_bytes = alg_bytes(n, nb, es)
+    total_bytes = 2 * pass_bytes * args.steps * world
+    value = total_bytes / (ms / 1e3) / 1e9
+    peak, peak_src = peaks()
+    dom_ms = max(enc_ms, ver_ms)
+    dom = "checksum_pass_kernel<double,512,VERIFY=true>" if ver_ms >= enc_ms else "checksum_pass_kernel<double,512,VERIFY=false>"
+    achieved = pass_bytes / (dom_ms / 1e3) / 1e9
+
+    # ---- e2e: through the C ABI with host buffers (pinned H2D + result D2H) ----
+    e2e = None
+    if not args.no_e2e:
+        hostA = torch.empty((n, n), dtype=torch.float64, pin_memory=True)
+        hostA.copy_(A.t())  # row-major host image of the column-major matrix
+        status_h = torch.empty_like(rep.status.t().contiguous(), device="cpu").pin_memory()
+        counts_h = torch.empty(abft.NCOUNTS, dtype=torch.int32).pin_memory()
+        e_steps = max(2, min(args.steps, 3))
+
+        def e2e_step():
+            A.t().copy_(hostA, non_blocking=True)  # H2D of the step's input
+            step()
+            counts_h.copy_(rep.counts, non_blocking=True)  # D2H of the result
+            status_h.copy_(rep.status.t(), non_blocking=True)
+
+        e2e_step()
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        for _ in range(e_steps):
+            e2e_step()
+        b.record()
+        torch.cuda.synchronize()
+        ems = a.elapsed_time(b) / e_steps
+        if world > 1:
+            tt = torch.tensor([ems], device="cuda")
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            ems = float(tt.item())
+        e2e = {"value": 2 * pass_bytes * world / (ems / 1e3) / 1e9, "unit": "GB/s",
+               "h2d_bytes_per_step": n * n * es,
+               "d2h_bytes_per_step": int(counts_h.numel() * 4 + status_h.numel() * 4), "ms_per_step": ems}
+        del hostA
+
+    # ---- ft_potrf overhead at n=30720 (the metric's second half) ----
+    ftp = None
+    if not args.no_potrf and rank == 0:
+        ftp = potrf_overhead(abft, si, args.potrf_n, nb, args.potrf_reps)
+
+    del A, mat
+    torch.cuda.empty_cache()
+    cpu = cpu_baseline_sample(args.cpu_seconds) if (rank == 0 and world == 1 and not args.no_cpu) else None
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"encode+verify(+locate) fp64 n={n} nb={nb} per GPU, U(-1,1), full matrix "
+                                   f"(BASELINE configs[3] shape at the n={N_MAT} metric size)",
+                       "n": n, "nb": nb, "tiles_per_gpu": (n // nb) ** 2, "l2": "inputs larger than L2 (7.55 GB/pass)",
+                       "parallelism": f"tiles block-cyclic, dp{world}", "ft_potrf_n": args.potrf_n},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": ncu_traffic(), "kernel": dom,
+                         "bytes_per_launch": pass_bytes, "ms_per_launch": dom_ms, "peak_source": peak_src,
+                         "encode_GBs": pass_bytes / (enc_ms / 1e3) / 1e9,
+                         "verify_GBs": pass_bytes / (ver_ms / 1e3) / 1e9},
+            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": 3 * args.steps, "clocks": clk.summary(),
+            "ft_potrf": ftp,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def potrf_overhead(abft, si, n, nb, reps):
+    """T_ft vs T_plain of the same blocked driver, plus cuSOLVER
+    potrf as context; ms are CUDA-event times on the driver's stream."""
+    import torch
+
+    A0 = si.spd_device(n, seed=7)
+    A = torch.empty_like(A0.t()).t()
+    ctx = abft.Context()
+
+    def run(ft):
+        A.copy_(A0)
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft)
+        b.record()
+        torch.cuda.synchronize()
+        assert rc == 0 and info == 0
+        return a.elapsed_time(b), st
+
+    run(True)
+    run(False)
+    t_ft, t_plain = [], []
+    for _ in range(reps):
+        t_plain.append(run(False)[0])
+        t, st = run(True)
+        t_ft.append(t)
+        assert sum(st.counts) == 0
+    t_ft.sort()
+    t_plain.sort()
+    ft_ms, plain_ms = t_ft[len(t_ft) // 2], t_plain[len(t_plain) // 2]
+    # cuSOLVER dpotrf of the whole matrix (context)
+    S = A0.t().contiguous()
+    torch.backends.cuda.preferred_linalg_library("cusolver")
+    torch.linalg.cholesky(S)
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    torch.linalg.cholesky(S)
+    b.record()
+    torch.cuda.synchronize()
+    cus = a.elapsed_time(b)
+    del S, A, A0
+    torch.cuda.empty_cache()
+    return {"n": n, "nb": nb, "ms_ft": ft_ms, "ms_plain": plain_ms,
+            "overhead_pct": 100.0 * (ft_ms - plain_ms) / plain_ms, "cusolver_potrf_ms": cus,
+            "tflops_ft": n ** 3 / 3 / (ft_ms / 1e3) / 1e12, "reps": reps}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n", type=int, default=N_MAT)
+    ap.add_argument("--potrf-n", type=int, default=N_MAT)
+    ap.add_argument("--potrf-reps", type=int, default=3)
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-potrf", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -494,16 +494,6 @@ def classify_fix_round(st, tc, which, tol, fixes):
                 repaired = True
     if repaired:
         return CLS_CHK_CORRUPT
-    # step 5b — one side vouches for the data: the other side is stale
-    if has_c and has_r:
-        if Fr and not Fc:
-            for i in Fr:
-                _reencode_row(st, tc, i, CLS_STALE_R, fixes)
-            return CLS_STALE_R
-        if Fc and not Fr:
-            for j in Fc:
-                _reencode_col(st, tc, j, CLS_STALE_C, fixes)
-            return CLS_STALE_C
     # step 3 — all flagged columns locate the same row i (0D / 1D_ROW)
     loc_c = {}
     if has_c and Fc:
@@ -542,6 +532,19 @@ def classify_fix_round(st, tc, which, tol, fixes):
                     for j in others:
                         _fix_via_col(st, tc, r, j, CLS_SYM_CROSS, fixes)
                     return CLS_SYM_CROSS
+    # step 5b — one side vouches for the data: the other side is stale (it was
+    # updated with a corrupted operand and the data has since been fixed
+    # through the good side).  Only after steps 3-6 failed, so a genuine
+    # 1D error seen by one side is always corrected first.
+    if has_c and has_r:
+        if Fr and not Fc:
+            for i in Fr:
+                _reencode_row(st, tc, i, CLS_STALE_R, fixes)
+            return CLS_STALE_R
+        if Fc and not Fr:
+            for j in Fc:
+                _reencode_col(st, tc, j, CLS_STALE_C, fixes)
+            return CLS_STALE_C
     return CLS_2D  # step 7
 
 

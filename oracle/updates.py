@@ -23,7 +23,14 @@ from .checksum import State
 def tri_inv(T, lower=True, unit=False):
     """Explicit T^-1 (used only for the magnitude rule of c-6)."""
     n = T.shape[0]
-    return sla.solve_triangular(T, np.eye(n), lower=lower, unit_diagonal=unit)
+    return sla.solve_triangular(T, np.eye(n), lower=lower, unit_diagonal=unit, check_finite=False)
+
+
+def potrf_lower(S):
+    """LAPACK dpotrf('L') of a symmetric tile: (L, info) with info the
+    1-based failing minor (0 on success)."""
+    c, info = sla.lapack.dpotrf(S, lower=1, clean=1)
+    return np.tril(c), int(info)
 
 
 def chol_pd_rule(st: State, k: int):
@@ -35,39 +42,42 @@ def chol_pd_rule(st: State, k: int):
     s = slice(k * nb, (k + 1) * nb)
     Akk = st.A[s, s]
     S = np.tril(Akk) + np.tril(Akk, -1).T
-    try:
-        L = np.linalg.cholesky(S)
-    except np.linalg.LinAlgError:
-        return 1
+    L, info = potrf_lower(S)
+    if info:
+        return info
     st.A[s, s] = np.tril(L) + np.triu(Akk, 1)  # upper part of the tile untouched (potrf 'L')
     # c(L) L^T = c(A)  =>  c(L) = c(A) L^{-T}  (solve L · c(L)^T = c(A)^T)
     C = st.colchk[2 * k:2 * k + 2, s]
-    st.colchk[2 * k:2 * k + 2, s] = sla.solve_triangular(L, C.T, lower=True).T
+    st.colchk[2 * k:2 * k + 2, s] = sla.solve_triangular(L, C.T, lower=True, check_finite=False).T
     if st.colmag is not None:
         st.colmag[k, s] = st.colmag[k, s] @ np.abs(tri_inv(L).T)
     return 0
 
 
-def chol_pu_rule(st: State, k: int):
-    """c-12 PU: L_ik = A_ik·L_kk^{-T} for the whole column panel below the
-    diagonal tile, c(L_ik) = c(A_ik)·L_kk^{-T}, m_c ← m_c·|L_kk^{-T}|."""
+def chol_pu_data(st: State, k: int):
+    """c-12 PU data step: L_ik = A_ik·L_kk^{-T} for the column panel."""
     nb, n = st.nb, st.A.shape[0]
     s = slice(k * nb, (k + 1) * nb)
     r1 = (k + 1) * nb
     L = np.tril(st.A[s, s])
     P = st.A[r1:n, s]
-    st.A[r1:n, s] = sla.solve_triangular(L, P.T, lower=True).T
+    st.A[r1:n, s] = sla.solve_triangular(L, P.T, lower=True, check_finite=False).T
+
+
+def chol_pu_chk(st: State, k: int):
+    """c-12 PU checksum step: c(L_ik) = c(A_ik)·L_kk^{-T}, m_c ← m_c·|L_kk^{-T}|."""
+    nb = st.nb
+    s = slice(k * nb, (k + 1) * nb)
+    L = np.tril(st.A[s, s])
     C = st.colchk[2 * (k + 1):, s]
-    st.colchk[2 * (k + 1):, s] = sla.solve_triangular(L, C.T, lower=True).T
+    st.colchk[2 * (k + 1):, s] = sla.solve_triangular(L, C.T, lower=True, check_finite=False).T
     if st.colmag is not None:
         st.colmag[k + 1:, s] = st.colmag[k + 1:, s] @ np.abs(tri_inv(L).T)
 
 
-def chol_tmu_rule(st: State, k: int):
-    """c-12 TMU for every trailing tile (i ≥ j > k):
-    A_ij −= L_ik L_jk^T (lower triangle only, as DSYRK),
-    c(A_ij) −= c(L_ik)·L_jk^T, r(A_ij) −= L_ik·c(L_jk)^T (L189),
-    m_c(A_ij) += m_c(L_ik)·|L_jk|^T, m_r(A_ij) += |L_ik|·m_c(L_jk)^T (c-6)."""
+def chol_tmu_data(st: State, k: int):
+    """c-12 TMU data step, every trailing tile (i ≥ j > k):
+    A_ij −= L_ik L_jk^T on the lower triangle only (as DSYRK)."""
     nb, n = st.nb, st.A.shape[0]
     s = slice(k * nb, (k + 1) * nb)
     r1 = (k + 1) * nb
@@ -75,6 +85,16 @@ def chol_tmu_rule(st: State, k: int):
     upd = L21 @ L21.T
     tri = np.tril(np.ones((n - r1, n - r1), dtype=bool))
     st.A[r1:n, r1:n][tri] -= upd[tri]
+
+
+def chol_tmu_chk(st: State, k: int):
+    """c-12 TMU checksum step: c(A_ij) −= c(L_ik)·L_jk^T,
+    r(A_ij) −= L_ik·c(L_jk)^T (L189), m_c(A_ij) += m_c(L_ik)·|L_jk|^T,
+    m_r(A_ij) += |L_ik|·m_c(L_jk)^T (c-6)."""
+    nb, n = st.nb, st.A.shape[0]
+    s = slice(k * nb, (k + 1) * nb)
+    r1 = (k + 1) * nb
+    L21 = st.A[r1:n, s].copy()
     cL = st.colchk[2 * (k + 1):, s].copy()
     st.colchk[2 * (k + 1):, r1:n] -= cL @ L21.T
     st.rowchk[r1:n, 2 * (k + 1):] -= L21 @ cL.T

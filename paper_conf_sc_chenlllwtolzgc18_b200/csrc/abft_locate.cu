@@ -6,8 +6,8 @@
 // (L330-L334); "same row => 1D, otherwise 2D" (L432-L434, §VII.D).
 // Readings: c-4 correction x <- c_e - sum_{r!=i} X[r][j];
 // c-5 acceptance of the rounded ratio; c-7 non-finite fallback with
-// confirmation; c-11 class order CHK_CORRUPT -> STALE -> 0D/1D_ROW ->
-// 0D/1D_COL -> SYM pair -> SYM_CROSS -> 2D, at most 3 rounds.
+// confirmation; c-11 class order CHK_CORRUPT -> 0D/1D_ROW -> 0D/1D_COL ->
+// SYM pair -> SYM_CROSS -> STALE -> 2D, at most 3 rounds.
 //
 // This is the rare path (only tiles whose verify status is non-zero do any
 // work), so it favours clarity: one 256-thread CTA per flagged tile, warp-per-
@@ -377,20 +377,6 @@ __global__ void __launch_bounds__(kLThreads) locate_correct_kernel(LocArgs p) {
           cls = ABFT_CLS_CHK_CORRUPT;
           decided = true;
         }
-        // step 5b: stale side
-        if (!decided && has_c && has_r) {
-          if (nfr && !nfc) {
-            for (int i = 0; i < nb; ++i)
-              if (D[1].fl[i] & 3) push(ACT_REENC_ROW, i, -1, ABFT_CLS_STALE_R);
-            cls = ABFT_CLS_STALE_R;
-            decided = true;
-          } else if (nfc && !nfr) {
-            for (int j = 0; j < nb; ++j)
-              if (D[0].fl[j] & 3) push(ACT_REENC_COL, -1, j, ABFT_CLS_STALE_C);
-            cls = ABFT_CLS_STALE_C;
-            decided = true;
-          }
-        }
         // step 3: columns locate one row
         if (!decided && has_c && nfc) {
           int i0 = -2;
@@ -459,6 +445,21 @@ __global__ void __launch_bounds__(kLThreads) locate_correct_kernel(LocArgs p) {
                 decided = true;
               }
             }
+          }
+        }
+        // step 5b: stale side (after steps 3-6, so a genuine 1D error seen by
+        // one side is always corrected first)
+        if (!decided && has_c && has_r) {
+          if (nfr && !nfc) {
+            for (int i = 0; i < nb; ++i)
+              if (D[1].fl[i] & 3) push(ACT_REENC_ROW, i, -1, ABFT_CLS_STALE_R);
+            cls = ABFT_CLS_STALE_R;
+            decided = true;
+          } else if (nfc && !nfr) {
+            for (int j = 0; j < nb; ++j)
+              if (D[0].fl[j] & 3) push(ACT_REENC_COL, -1, j, ABFT_CLS_STALE_C);
+            cls = ABFT_CLS_STALE_C;
+            decided = true;
           }
         }
         s_nact = decided ? na : 0;

@@ -166,6 +166,47 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
   T* colmag = reinterpret_cast<T*>(p.colmag);
   T* dcol = reinterpret_cast<T*>(p.dcol);
   int my_colflags = 0, my_ncols = 0;
+  // verify: fetch the maintained column checksums (and magnitudes) of this
+  // slab once, while the TMA prologue is in flight, instead of one dependent
+  // strided load per column inside the stage loop.  For non-SYM tiles the
+  // SYM accumulator area is free and holds them: [e | w | mag] x cols.
+  if (VERIFY && !sym && (p.which & ABFT_COL)) {
+    for (int idx = tid; idx < cols; idx += kThreads) {
+      const int64_t gj = (int64_t)J * NB + c0 + idx;
+      symacc[idx] = colchk[(int64_t)2 * I + gj * p.ldc];
+      symacc[NB + idx] = colchk[(int64_t)2 * I + 1 + gj * p.ldc];
+      if (p.use_mag) symacc[2 * NB + idx] = colmag[I + gj * p.ldcm];
+    }
+    __syncthreads();
+  }
+  // column finish: encode writes c (and m_c); verify compares (c-6, c-7)
+  auto finish_col = [&](int jl, T pe, T pw, T pa) {
+    if (sym) {
+      symacc[jl] = pe;
+      symacc[NB + jl] = pw;
+      symacc[2 * NB + jl] = pa;
+      return;
+    }
+    if (!(p.which & ABFT_COL)) return;
+    const int64_t gj = (int64_t)J * NB + jl;
+    if (!VERIFY) {
+      T* cc2 = colchk + (int64_t)2 * I + gj * p.ldc;
+      cc2[0] = pe;
+      cc2[1] = pw;
+      if (colmag) colmag[I + gj * p.ldcm] = pa;
+    } else {
+      const int idx = jl - c0;
+      double m = p.use_mag ? (double)symacc[2 * NB + idx] : (double)pa;
+      T de, dw;
+      int f = check_pair<T>(symacc[idx], symacc[NB + idx], pe, pw, m, p.tau_fac, NB, &de, &dw);
+      if (dcol) {
+        dcol[(int64_t)2 * I + gj * p.ldc] = de;
+        dcol[(int64_t)2 * I + 1 + gj * p.ldc] = dw;
+      }
+      my_colflags |= f;
+      my_ncols += f & 1;
+    }
+  };
 
   for (int s = 0; s < nst; ++s) {
     const int slot = s % C::NSTAGE;
@@ -219,31 +260,7 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
           cpart[(h * C::CC + cc) * 3 + 2] = pa;
         }
       } else if (lane == 0) {
-        if (sym) {
-          symacc[jl] = pe;
-          symacc[NB + jl] = pw;
-          symacc[2 * NB + jl] = pa;
-        } else {
-          const int64_t gj = (int64_t)J * NB + jl;
-          T* cc2 = colchk + (int64_t)2 * I + gj * p.ldc;
-          if (!VERIFY) {
-            if (p.which & ABFT_COL) {
-              cc2[0] = pe;
-              cc2[1] = pw;
-              if (colmag) colmag[I + gj * p.ldcm] = pa;
-            }
-          } else if (p.which & ABFT_COL) {
-            double m = p.use_mag ? (double)colmag[I + gj * p.ldcm] : (double)pa;
-            T de, dw;
-            int f = check_pair<T>(cc2[0], cc2[1], pe, pw, m, p.tau_fac, NB, &de, &dw);
-            if (dcol) {
-              dcol[(int64_t)2 * I + gj * p.ldc] = de;
-              dcol[(int64_t)2 * I + 1 + gj * p.ldc] = dw;
-            }
-            my_colflags |= f;
-            my_ncols += f & 1;
-          }
-        }
+        finish_col(jl, pe, pw, pa);
       }
     }
     // ---------------- phase B: row sums ---------------------------------
@@ -304,31 +321,7 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
         pw = fadd(pw, cpart[(h * C::CC + cc) * 3 + 1]);
         pa = fadd(pa, cpart[(h * C::CC + cc) * 3 + 2]);
       }
-      if (sym) {
-        symacc[jl] = pe;
-        symacc[NB + jl] = pw;
-        symacc[2 * NB + jl] = pa;
-      } else {
-        const int64_t gj = (int64_t)J * NB + jl;
-        T* cc2 = colchk + (int64_t)2 * I + gj * p.ldc;
-        if (!VERIFY) {
-          if (p.which & ABFT_COL) {
-            cc2[0] = pe;
-            cc2[1] = pw;
-            if (colmag) colmag[I + gj * p.ldcm] = pa;
-          }
-        } else if (p.which & ABFT_COL) {
-          double m = p.use_mag ? (double)colmag[I + gj * p.ldcm] : (double)pa;
-          T de, dw;
-          int f = check_pair<T>(cc2[0], cc2[1], pe, pw, m, p.tau_fac, NB, &de, &dw);
-          if (dcol) {
-            dcol[(int64_t)2 * I + gj * p.ldc] = de;
-            dcol[(int64_t)2 * I + 1 + gj * p.ldc] = dw;
-          }
-          my_colflags |= f;
-          my_ncols += f & 1;
-        }
-      }
+      finish_col(jl, pe, pw, pa);
     }
     if (C::WPC > 1) __syncthreads();  // cpart reusable
     if (p.use_bulk && tid == 0 && s + C::NSTAGE < nst) issue(s + C::NSTAGE);

@@ -77,6 +77,7 @@ struct RepairArgs {
   const int32_t* n_fixes;
   const int32_t* mark;
   int32_t* rep_counts;  // [0] applied, [1] skipped
+  int32_t* counts;      // report counts: a skipped repair is uncorrectable (R)
 };
 
 template <typename T>
@@ -108,7 +109,10 @@ __global__ void fig4a_repair_kernel(RepairArgs r) {
     if (threadIdx.x == 0) s_skip = !(isfinite(eps) && fabs(eps) <= 1024.0 * s_max);
     __syncthreads();
     if (s_skip) {
-      if (threadIdx.x == 0) atomicAdd(&r.rep_counts[1], 1);
+      if (threadIdx.x == 0) {
+        atomicAdd(&r.rep_counts[1], 1);
+        atomicAdd(&r.counts[ABFT_CNT_UNCORRECTABLE], 1);
+      }
       continue;
     }
     const T e = (T)eps;
@@ -137,6 +141,13 @@ __global__ void fig4a_repair_kernel(RepairArgs r) {
     if (threadIdx.x == 0) atomicAdd(&r.rep_counts[0], 1);
     __syncthreads();
   }
+}
+
+// LAPACK info of the whole factorization: first failing tile's local minor
+// offset by the tile origin.
+__global__ void accum_info_kernel(int32_t* tile_info, int32_t* total, int64_t offset) {
+  if (*tile_info != 0 && *total == 0) *total = (int32_t)(*tile_info + offset);
+  *tile_info = 0;
 }
 }  // namespace abft
 
@@ -199,13 +210,23 @@ struct Driver {
     if (target == 2) return (char*)M.rowchk + (gi + gj * M.ldr) * es;
     return (char*)A + (gi + gj * lda) * es;
   }
+  // Elements the op after `point` overwrites: an on-chip flip there cannot be
+  // changed back, so it stays (reading c-8).
+  bool in_update_region(int point, int k, int64_t gi, int64_t gj) const {
+    const int64_t r0 = k * nb, r1 = (k + 1) * nb;
+    if (point == FT_AT_PRE_PD) return gi >= r0 && gi < r1 && gj >= r0 && gj < r1;
+    if (point == FT_AT_PRE_PU) return gi >= r1 && gj >= r0 && gj < r1;
+    if (point == FT_AT_PRE_TMU) return gi >= r1 && gj >= r1;
+    return false;
+  }
   int inject_at(int k, int point) {
     for (int t = 0; t < o->n_inject; ++t) {
       const ft_inject_t& f = o->inject[t];
       if (f.iter != k || f.point != point) continue;
       FT_TRY(abft_inject(elem(f.target, f.gi, f.gj), dtype, 0, f.xor_mask, (abft_stream_t)s));
       bool op_point = point == FT_AT_PRE_PD || point == FT_AT_PRE_PU || point == FT_AT_PRE_TMU;
-      if (f.kind == FT_KIND_ONCHIP && op_point) onchip_pending.push_back(f);
+      if (f.kind == FT_KIND_ONCHIP && op_point && f.target == 0 && !in_update_region(point, k, f.gi, f.gj))
+        onchip_pending.push_back(f);
     }
     return 0;
   }
@@ -334,6 +355,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
         D.ldcm = d.M.ldcm;
       }
       FT_TRY(abft_panel_potrf(&D, d.info, as));
+      accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.rep + 2, (int64_t)k * nb);
     }
     FT_TRY(d.restore_onchip());
     FT_TRY(d.inject_at(k, FT_AT_POST_PD));
@@ -362,10 +384,10 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       }
       lk.unlock();
     }
+    FT_TRY(d.restore_onchip());  // on-chip flips hit the data step only (c-8)
     if (ft)
       FT_TRY(abft_update_trsm(dtype, 'R', 'L', 'T', 'N', nb, d.a_at(k * nb, k * nb), lda, d.colchk_at(2 * (k + 1), k * nb),
                               d.M.ldc, m2, d.colmag_at(k + 1, k * nb), d.M.ldcm, m2 / 2, as));
-    FT_TRY(d.restore_onchip());
     FT_TRY(d.inject_at(k, FT_AT_POST_PU));
     // line 10: check the updated panel (c only; 1D_ROW fixable, 2D -> restart, L434)
     if (ft) FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
@@ -386,6 +408,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       }
       lk.unlock();
     }
+    FT_TRY(d.restore_onchip());  // on-chip flips hit the data step only (c-8)
     if (ft) {
       // c(A_ij) -= c(L_ik) L_jk^T
       FT_TRY(abft_update_gemm(dtype, ABFT_COL, 'N', 'T', -1.0, d.colchk_at(2 * (k + 1), k * nb), d.M.ldc,
@@ -396,7 +419,6 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
                               d.a_at(r1, k * nb), lda, d.rowchk_at(r1, 2 * (k + 1)), d.M.ldr, m2, nk, nb,
                               d.colmag_at(k + 1, k * nb), d.M.ldcm, d.rowmag_at(r1, k + 1), d.M.ldrm, as));
     }
-    FT_TRY(d.restore_onchip());
     FT_TRY(d.inject_at(k, FT_AT_POST_TMU));
     // line 13: heuristic panel re-check for the TMU (Fig. 4a) + guarded repair (c-25)
     if (ft) {
@@ -422,6 +444,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
         ra.n_fixes = d.nfix;
         ra.mark = d.mark;
         ra.rep_counts = d.rep;
+        ra.counts = d.counts;
         if (dtype == ABFT_F64)
           fig4a_repair_kernel<double><<<1, 256, 0, s>>>(ra);
         else
@@ -431,14 +454,14 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     }
   }
   // ---- the single host synchronisation: stats ----
-  int32_t host_ints[8 + 1 + 1 + 1 + 2];
+  int32_t host_ints[8 + 1 + 1 + 1 + 2 + 1];
   ABFT_CUDA_TRY(cudaMemcpyAsync(host_ints, d.counts, sizeof(host_ints), cudaMemcpyDeviceToHost, s));
   if (o->fix_log && o->fix_log_cap > 0)
     ABFT_CUDA_TRY(cudaMemcpyAsync(o->fix_log, c->fixlog, sizeof(abft_fix_t) * std::min(o->fix_log_cap, c->fixcap),
                                   cudaMemcpyDeviceToDevice, s));
   ABFT_CUDA_TRY(cudaStreamSynchronize(s));
   auto t1 = std::chrono::steady_clock::now();
-  if (info_out) *info_out = host_ints[10];
+  if (info_out) *info_out = host_ints[13];
   if (stats) {
     for (int i = 0; i < 8; ++i) stats->counts[i] = host_ints[i];
     stats->n_fixes = host_ints[8];

@@ -97,14 +97,17 @@ def general_device(m: int, n: int | None = None, seed: int = 0, dtype=None, devi
 
 
 def spd_device(n: int, seed: int = 0, dtype=None, device="cuda"):
-    """Column-major (M + M^T)/2 + n*I drawn on the GPU."""
+    """(M + M^T)/2 + n*I with M ~ U(-1,1), drawn on the GPU; symmetric, so the
+    returned column-major view is the same matrix."""
     import torch
 
     dtype = dtype or torch.float64
-    M = general_device(n, n, seed, dtype, device)  # column-major view
-    S = M.t().contiguous()  # row-major copy of M^T
-    S.add_(M.t().t())  # += M  (M^T + M), elementwise in place
+    g = torch.Generator(device=device)
+    g.manual_seed(seed)
+    buf = torch.rand((n, n), generator=g, dtype=dtype, device=device)
+    buf.mul_(2.0).sub_(1.0)
+    S = buf + buf.t()
+    del buf
     S.mul_(0.5)
     S.diagonal().add_(float(n))
-    del M
-    return S.t()  # symmetric: column-major view of the same data
+    return S.t()

@@ -1,0 +1,159 @@
+"""GPU parity of ft_potrf (§8 rows a4–a7) against the oracle driver, through
+the C ABI: error-free factors, and fault campaigns whose fix logs (positions,
+classes) must match the oracle's exactly (BASELINE configs[0] and [1])."""
+import numpy as np
+import pytest
+import torch
+
+import synth_inputs as si
+from oracle import checksum as ck
+from oracle import drivers as dr
+from tests.gpu_helpers import dev, host
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ctx(lib):
+    return lib.Context()
+
+
+def _gpu_potrf(lib, ctx, A_np, nb, inject=(), abft=True, fig4a=True, dtype=torch.float64):
+    A = dev(A_np, dtype)
+    inj = [(f.iter, f.point, f.kind, f.target, f.gi, f.gj, si.mask_of(f.bits)) for f in inject]
+    log = torch.zeros(8192 * lib.FIX_BYTES, dtype=torch.uint8, device="cuda")
+    rc, info, stats = lib.ft_potrf(ctx, A, nb, abft=abft, fig4a_repair=fig4a, inject=inj, fix_log=log)
+    torch.cuda.synchronize()
+    fixes = lib.decode_fixes(log, stats.n_fixes)
+    return np.tril(host(A)), rc, info, stats, fixes
+
+
+@pytest.mark.parametrize("n,nb", [(256, 32), (1024, 128), (2048, 256), (2048, 512), (4096, 1024)])
+def test_error_free_matches_lapack(lib, ctx, n, nb):
+    A = si.spd(n, seed=n)
+    L, rc, info, stats, fixes = _gpu_potrf(lib, ctx, A, nb)
+    Lref = np.linalg.cholesky(A)
+    assert rc == 0 and info == 0 and stats.counts[:] == [0] * 8 and not fixes
+    assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
+    assert stats.n_checks == 5 * (n // nb - 1) + 2
+
+
+def test_unprotected_same_factor(lib, ctx):
+    A = si.spd(1024, seed=1)
+    L0, *_ = _gpu_potrf(lib, ctx, A, 128, abft=False)
+    L1, *_ = _gpu_potrf(lib, ctx, A, 128, abft=True)
+    assert np.abs(L0 - L1).max() <= 1e-13 * np.abs(L0).max()
+
+
+def test_not_spd_info(lib, ctx):
+    A = si.spd(128, seed=4)
+    A[70, 70] = -1e6
+    _, rc, info, _, _ = _gpu_potrf(lib, ctx, A, 32, abft=False)
+    assert info == 64 + 7
+
+
+def _compare(lib, ctx, A, nb, injects, fig4a=True):
+    Lo, so = dr.ft_potrf(A, nb, inject=injects, fig4a_repair=fig4a)
+    Lg, rc, info, sg, fg = _gpu_potrf(lib, ctx, A, nb, inject=injects, fig4a=fig4a)
+    assert (rc == lib.E_UNCORRECTABLE) == (so.uncorrectable > 0)
+    assert sg.repairs_skipped == so.repairs_skipped
+    if so.repairs_skipped:
+        # a guarded-out repair leaves overflowing garbage in the trailing
+        # matrix: the outcome is R (detected, restart); what the checks see
+        # afterwards is Inf/NaN arithmetic and not compared
+        return so, sg
+    assert list(sg.counts) == so.counts, (list(sg.counts), so.counts)
+    assert sorted((f[0], f[1], f[4], f[5]) for f in fg) == sorted((f.gi, f.gj, f.cls, f.kind) for f in so.fixes)
+    assert sg.repairs_applied == so.repairs_applied and sg.repairs_skipped == so.repairs_skipped
+    assert (rc == lib.E_UNCORRECTABLE) == (so.uncorrectable > 0)
+    if so.uncorrectable == 0:
+        Lref = np.linalg.cholesky(A)
+        assert np.abs(Lg - Lref).max() <= 1e-12 * np.abs(Lref).max()
+        assert np.abs(Lo - Lref).max() <= 1e-12 * np.abs(Lref).max()
+    return so, sg
+
+
+# (point, kind, target, gi, gj, bits) at iteration 2, n=256, nb=32
+CASES = [
+    (dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 0, 70, 66, (61,)),
+    (dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 0, 75, 75, (55, 52)),
+    (dr.AT_POST_PD, dr.KIND_PERSIST, 0, 80, 70, (62,)),
+    (dr.AT_PRE_PU_CHECK, dr.KIND_PERSIST, 0, 200, 70, (60,)),
+    (dr.AT_POST_PU, dr.KIND_PERSIST, 0, 150, 90, (63,)),
+    (dr.AT_PRE_PU, dr.KIND_ONCHIP, 0, 130, 68, (58,)),
+    (dr.AT_PRE_PU, dr.KIND_ONCHIP, 0, 70, 66, (60,)),      # PU reference part -> 2D (R)
+    (dr.AT_PRE_TMU, dr.KIND_ONCHIP, 0, 140, 72, (57,)),
+    (dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 170, 80, (54,)),    # Fig. 4a repair
+    (dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 170, 80, (62,)),    # guarded: R
+    (dr.AT_POST_TMU, dr.KIND_PERSIST, 0, 230, 100, (59,)),
+    (dr.AT_POST_TMU, dr.KIND_PERSIST, 0, 196, 196, (62,)),
+    (dr.AT_PRE_PU_CHECK, dr.KIND_PERSIST, 1, 11, 100, (60,)),  # checksum memory fault
+    (dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 2, 70, 5, (61,)),    # row-checksum memory fault
+]
+
+
+@pytest.mark.parametrize("case", range(len(CASES)))
+def test_fault_campaign_parity(lib, ctx, case):
+    point, kind, target, gi, gj, bits = CASES[case]
+    A = si.spd(256, seed=0)
+    _compare(lib, ctx, A, 32, [dr.Inject(2, point, kind, target, gi, gj, bits)])
+
+
+def test_fig4a_off_matches_oracle(lib, ctx):
+    A = si.spd(256, seed=0)
+    so, sg = _compare(lib, ctx, A, 32, [dr.Inject(2, dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 170, 80, (54,))], fig4a=False)
+    assert so.uncorrectable >= 1
+
+
+def _random_plan(n, nb, seed, k_faults):
+    """Seeded random single-fault-per-run plans over every hook point."""
+    g = si.rng(seed)
+    nt = n // nb
+    plan = []
+    for _ in range(k_faults):
+        k = int(g.integers(0, nt - 1))
+        point = int(g.integers(0, 8))
+        kind = dr.KIND_ONCHIP if point in (dr.AT_PRE_PU, dr.AT_PRE_TMU) and g.random() < 0.5 else dr.KIND_PERSIST
+        r0 = (k + 1) * nb
+        if point in (dr.AT_PRE_PD_CHECK, dr.AT_PRE_PD, dr.AT_POST_PD):
+            a, b = int(g.integers(k * nb, r0)), int(g.integers(k * nb, r0))
+            gi, gj = max(a, b), min(a, b)
+        elif point in (dr.AT_PRE_PU_CHECK, dr.AT_PRE_PU, dr.AT_POST_PU, dr.AT_PRE_TMU):
+            gi, gj = int(g.integers(r0, n)), int(g.integers(k * nb, r0))
+        else:
+            a, b = int(g.integers(r0, n)), int(g.integers(r0, n))
+            gi, gj = max(a, b), min(a, b)
+        bit = int(g.integers(52, 64))
+        plan.append(dr.Inject(k, point, kind, 0, gi, gj, (bit,)))
+    return plan
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_random_campaign_parity(lib, ctx, seed):
+    """Config-1 shape (fp64 SPD n=256 nb=32), one random fault per run at a
+    random Alg. 2 hook, exponent/sign bits (MUST band)."""
+    A = si.spd(256, seed=100 + seed)
+    _compare(lib, ctx, A, 32, _random_plan(256, 32, seed, 1))
+
+
+def test_config2_shape_error_free_and_injected(lib, ctx):
+    """BASELINE configs[1]: fp64 n=10240 nb=512; error-free residual check at
+    full size, then a random DRAM fault in a trailing tile, fixed."""
+    n, nb = 10240, 512
+    A = si.spd_device(n, seed=5)
+    A0 = A.clone()
+    rc, info, stats = lib.ft_potrf(ctx, A, nb)
+    torch.cuda.synchronize()
+    assert rc == 0 and info == 0 and list(stats.counts) == [0] * 8
+    L = torch.tril(A)
+    # sampled residual rows: |A0 - L L^T| on 64 random rows
+    g = si.rng(9)
+    rows = torch.tensor(sorted(g.choice(n, 64, replace=False)), device="cuda")
+    R = A0[rows] - L[rows] @ L.T
+    assert R.abs().max().item() <= 1e-12 * n
+    A.copy_(A0)
+    inj = [(5, lib.AT_POST_TMU, lib.KIND_PERSIST, 0, 7000, 6000, 1 << 61)]
+    rc, info, stats = lib.ft_potrf(ctx, A, nb, inject=inj)
+    torch.cuda.synchronize()
+    assert rc == 0 and stats.counts[5] == 1
+    assert (torch.tril(A) - L).abs().max().item() <= 1e-12 * L.abs().max().item()

@@ -1,0 +1,126 @@
+"""Pins of the oracle's update rules and Alg. 2 driver (oracle/updates.py,
+oracle/drivers.py) against independent facts: LAPACK's unblocked Cholesky
+(numpy.linalg.cholesky) of the whole matrix, the checksum invariant
+'maintained == recomputed' after every phase (L114, L149, L189), and fault
+campaigns whose right answer is the fault-free factor.  CPU only."""
+import numpy as np
+import pytest
+
+import synth_inputs as si
+from oracle import checksum as ck
+from oracle import drivers as dr
+
+
+def _invariant(st, k, phase):
+    """After each phase, every live checksum equals the recomputed one
+    within tau (no flags) — checked on tiles whose checksums are maintained."""
+    nt, nb = st.nt, st.nb
+    tol = ck.Tol()
+    if phase == "pd":
+        tc = ck.check_tile(st, k, k, ck.LOWER, ck.COL, tol)
+        assert not tc.Fc, (k, phase)
+    elif phase == "pu":
+        for I in range(k + 1, nt):
+            tc = ck.check_tile(st, I, k, ck.GENERAL, ck.COL, tol)
+            assert not tc.Fc, (k, phase, I)
+    else:
+        for I, J in ck.Tiles(k + 1, nt, k + 1, nt, True, ck.SYM_LOWER):
+            tc = ck.check_tile(st, I, J, ck.SYM_LOWER if I == J else ck.GENERAL, ck.BOTH, tol)
+            assert not tc.Fc and not tc.Fr, (k, phase, I, J)
+
+
+@pytest.mark.parametrize("n,nb", [(256, 32), (512, 64), (384, 128)])
+def test_ft_potrf_error_free_matches_lapack(n, nb):
+    A = si.spd(n, seed=n + nb)
+    L, stats = dr.ft_potrf(A, nb, invariant_hook=_invariant)
+    Lref = np.linalg.cholesky(A)
+    assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
+    assert stats.counts == [0] * 8 and stats.info == 0
+    # Alg. 2 issues 2 checks per final iteration and 5 per other iteration
+    nt = n // nb
+    assert stats.n_checks == 5 * (nt - 1) + 2
+
+
+def test_unprotected_driver_same_factor():
+    A = si.spd(256, seed=3)
+    L0, _ = dr.ft_potrf(A, 32, abft=False)
+    L1, _ = dr.ft_potrf(A, 32, abft=True)
+    assert np.abs(L0 - L1).max() <= 1e-13 * np.abs(L0).max()
+
+
+def test_not_spd_reports_info():
+    A = si.spd(128, seed=4)
+    A[70, 70] = -1e6
+    L, stats = dr.ft_potrf(A, 32, abft=False)
+    assert stats.info == 64 + 7  # first failing minor, 1-based, inside tile 2
+
+
+def _run(n, nb, injects, seed=0):
+    A = si.spd(n, seed=seed)
+    Lref, _ = dr.ft_potrf(A, nb)
+    L, stats = dr.ft_potrf(A, nb, inject=injects)
+    return A, Lref, L, stats
+
+
+# one fault per run at every Alg. 2 hook, each expected to be fixed (paper
+# Table VIII 'Y' outcomes for full checksums; readings c-8, c-11, c-25)
+FIXABLE = [
+    # (point, kind, gi, gj, bits)  at iteration k=2, n=256, nb=32
+    (dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 70, 66, (61,)),   # DRAM in A_kk before the pre-PD check
+    (dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 75, 75, (55, 52)),  # diagonal element
+    (dr.AT_POST_PD, dr.KIND_PERSIST, 80, 70, (62,)),        # computation error in L_kk
+    (dr.AT_PRE_PU_CHECK, dr.KIND_PERSIST, 200, 70, (60,)),  # DRAM in the panel to be updated
+    (dr.AT_POST_PU, dr.KIND_PERSIST, 150, 90, (63,)),       # computation error in L_ik
+    (dr.AT_PRE_PU, dr.KIND_ONCHIP, 130, 68, (58,)),         # on-chip in PU update part -> 1D_ROW
+    (dr.AT_PRE_TMU, dr.KIND_ONCHIP, 140, 72, (57,)),        # on-chip in TMU reference part -> 1D
+    (dr.AT_PRE_TMU, dr.KIND_PERSIST, 170, 80, (54,)),       # DRAM in TMU reference part -> Fig. 4a
+    (dr.AT_POST_TMU, dr.KIND_PERSIST, 230, 100, (59,)),     # computation error in the trailing matrix
+    (dr.AT_POST_TMU, dr.KIND_PERSIST, 196, 196, (62,)),     # trailing diagonal element (SYRK output)
+]
+
+
+@pytest.mark.parametrize("case", range(len(FIXABLE)))
+def test_fault_campaign_fixed(case):
+    point, kind, gi, gj, bits = FIXABLE[case]
+    inj = [dr.Inject(2, point, kind, 0, gi, gj, bits)]
+    A, Lref, L, stats = _run(256, 32, inj)
+    assert stats.uncorrectable == 0, stats.counts
+    assert stats.counts[0] >= 1  # detected
+    assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max(), np.abs(L - Lref).max()
+
+
+def test_fig4a_repair_is_required():
+    # without the repair the diagonal SYRK tile ends 2D (reading c-25)
+    inj = [dr.Inject(2, dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 170, 80, (54,))]
+    A = si.spd(256, seed=0)
+    _, stats = dr.ft_potrf(A, 32, inject=inj, fig4a_repair=False)
+    assert stats.uncorrectable >= 1
+    _, stats = dr.ft_potrf(A, 32, inject=inj, fig4a_repair=True)
+    assert stats.uncorrectable == 0 and stats.repairs_applied == 1
+
+
+def test_fig4a_guard_huge_fault_detected_not_silent():
+    # exponent flip to ~1e300 in a TMU reference element: the guarded repair
+    # is skipped and the run ends DETECTED (R), never silently wrong (N)
+    A = si.spd(256, seed=0)
+    x = 0.3
+    inj = [dr.Inject(2, dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 170, 80, (62,))]
+    Lref, _ = dr.ft_potrf(A, 32)
+    L, stats = dr.ft_potrf(A, 32, inject=inj)
+    ok = np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
+    assert stats.repairs_skipped == 1
+    assert ok or stats.uncorrectable >= 1
+
+
+def test_pu_reference_fault_is_2d():
+    # on-chip flip in L_kk while PU reads it: every panel row is wrong -> 2D (Table V)
+    inj = [dr.Inject(2, dr.AT_PRE_PU, dr.KIND_ONCHIP, 0, 70, 66, (60,))]
+    _, _, _, stats = _run(256, 32, inj)
+    assert stats.uncorrectable >= 1
+
+
+def test_checksum_memory_fault_repaired():
+    inj = [dr.Inject(3, dr.AT_PRE_PU_CHECK, dr.KIND_PERSIST, 1, 2 * 5 + 1, 100, (60,))]
+    A, Lref, L, stats = _run(256, 32, inj)
+    assert stats.uncorrectable == 0 and stats.counts[6] >= 1
+    assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
