@@ -226,10 +226,39 @@ ABFT_API int abft_update_gemm(int32_t dtype, int32_t which, char transX, char tr
 /* a4 — abft_panel_potrf (PD of Cholesky, Table II, c-12).  `diag` is ONE
  * nb x nb tile (m = n = nb) whose colchk holds c_sym(A_kk) (SYM_LOWER view)
  * and colmag its magnitudes.  Computes L_kk = chol(A_kk) in place (lower;
- * cuSOLVER on the device), then c(L_kk) = c_sym(A_kk) * L_kk^-T and
- * m_c(L_kk) = m_c * |L_kk^-T|.  LAPACK info (0, or k > 0 if the leading minor
- * k is not positive definite) goes to *info (device int32). */
-ABFT_API int abft_panel_potrf(const abft_mat_t *diag, int32_t *info, abft_stream_t stream);
+ * cuSOLVER on the device), L_kk^-1 (into Linv, device nb x nb with leading
+ * dimension ldw, when non-NULL — the driver reuses it for the PU), then
+ * c(L_kk) = c_sym(A_kk) * L_kk^-T and m_c(L_kk) = m_c * |L_kk^-T|.  colchk
+ * may be NULL (plain PD).  LAPACK info (0, or k > 0 if the leading minor k is
+ * not positive definite) goes to *info (device int32). */
+ABFT_API int abft_panel_potrf(const abft_mat_t *diag, void *Linv, int64_t ldw, int32_t *info,
+                              abft_stream_t stream);
+
+/* W = T^-1 for an nb x nb triangular T (uplo 'L'/'U', diag 'N'/'U'); the
+ * other triangle of W is written as zero.  Helper of the a5 rule (the
+ * magnitude propagation needs |T^-1| explicitly, c-6). */
+ABFT_API int abft_tri_inverse(int32_t dtype, char uplo, char diag, int64_t nb, const void *T, int64_t ldt,
+                              void *W, int64_t ldw, abft_stream_t stream);
+
+/* a5 with a precomputed inverse W = T^-1 (as abft_update_trsm, without the
+ * triangular solve): side 'R': chk (nvec x nb) <- chk * op(W),
+ * mag (nmag x nb) <- mag * |op(W)|; side 'L': chk (nb x nvec) <- op(W) * chk,
+ * mag (nb x nmag) <- |op(W)| * mag.  Skinny DGEMMs, results copied back. */
+ABFT_API int abft_update_trsm_inv(int32_t dtype, char side, char trans, int64_t nb, const void *W,
+                                  int64_t ldw, void *chk, int64_t ldchk, int64_t nvec, void *mag,
+                                  int64_t ldmag, int64_t nmag, abft_stream_t stream);
+
+/* a6 for the symmetric (Cholesky) TMU A22 -= L21 L21^T over ntk trailing tile
+ * rows/columns (L189, c-12): with P = c(L21) L21^T (one 2ntk x ntk*nb DGEMM),
+ *   c(A_IJ) -= P[2I.., cols of J]          for I >= J  (Cc: colchk block at
+ *              tile row k+1, column (k+1)nb; leading dimension ldc)
+ *   r(A_IJ) -= P[2J.., cols of I]^T        for I >= J  (Rr: rowchk block, ldr)
+ * and, when mL != NULL, with Q = m_c(L21) |L21|^T: Cm += Q (lower tiles),
+ * Rm += Q^T (c-6).  L21: ntk*nb x nb (ldl); cL: 2ntk x nb panel column
+ * checksums (ld ldc, the colchk leading dimension); mL: ntk x nb (ldcm). */
+ABFT_API int abft_update_syrk(int32_t dtype, int64_t nb, int64_t ntk, const void *L21, int64_t ldl,
+                              const void *cL, int64_t ldc, const void *mL, int64_t ldcm, void *Cc,
+                              void *Rr, int64_t ldr, void *Cm, void *Rm, int64_t ldrm, abft_stream_t stream);
 
 /* ----------------------------------------------------- drivers (a7) -- */
 typedef struct ft_ctx ft_ctx_t;
@@ -261,6 +290,8 @@ typedef struct {
   const ft_inject_t *inject;
   abft_fix_t *fix_log;   /* optional device log of every fix (capacity fix_log_cap) */
   int32_t fix_log_cap;
+  int32_t pu_gemm;       /* 1: PU as L21 = A21 * L_kk^-T (DGEMM with the PD's explicit inverse) in
+                            both the protected and the unprotected driver; 0: cuBLAS DTRSM */
 } ft_opts_t;
 
 /* Host-side statistics, filled after the driver's final synchronisation. */

@@ -138,3 +138,176 @@ def chol_fig4a_repair(st: State, k: int, gi: int, gj: int, before: float, after:
         if st.rowmag is not None:
             st.rowmag[p, J] += abs(E) * st.colmag[J, k * nb + ql]
     return "applied"
+
+
+# ------------------------------------------------------------------- LU ----
+def lu_swap_rule(st: State, p: int, q: int, cols, vals_p, vals_q, row_chk_cols=()):
+    """Reading c-14 of the silent swap rule: exchanging global rows p and q
+    (p' = p mod nb in tile P, q' in tile Q) changes the column checksums of
+    every column `cols` by the moved values (x_p, x_q the values before the
+    swap):  P != Q: c(P) += [1, p'+1]^T (x_q − x_p), c(Q) += [1, q'+1]^T (x_p − x_q);
+    P == Q: c_w += (p' − q')(x_q − x_p); magnitudes follow |x|.  Row
+    checksums (and row magnitudes) of the tile columns `row_chk_cols` move
+    with the rows."""
+    nb = st.nb
+    P, Q, pl, ql = p // nb, q // nb, p % nb, q % nb
+    d = np.asarray(vals_q, dtype=np.float64) - np.asarray(vals_p, dtype=np.float64)
+    da = np.abs(vals_q) - np.abs(vals_p)
+    if P != Q:
+        st.colchk[2 * P, cols] += d
+        st.colchk[2 * P + 1, cols] += (pl + 1) * d
+        st.colchk[2 * Q, cols] -= d
+        st.colchk[2 * Q + 1, cols] -= (ql + 1) * d
+        if st.colmag is not None:
+            st.colmag[P, cols] += da
+            st.colmag[Q, cols] -= da
+    else:
+        st.colchk[2 * P + 1, cols] += (pl - ql) * d
+    for J in row_chk_cols:
+        st.rowchk[[p, q], 2 * J:2 * J + 2] = st.rowchk[[q, p], 2 * J:2 * J + 2]
+        if st.rowmag is not None:
+            st.rowmag[[p, q], J] = st.rowmag[[q, p], J]
+
+
+def lu_panel_getrf(st: State, k: int):
+    """c-13 PD, factor step: LAPACK dgetrf of the column panel
+    P = A[k·nb:, k·nb:(k+1)·nb] (partial pivoting, idamax ties → first).
+    Does not touch the state.  Returns (lu_panel, ipiv 0-based global,
+    info, pre-PD panel copy)."""
+    nb, n = st.nb, st.A.shape[0]
+    r0, r1 = k * nb, (k + 1) * nb
+    P0 = st.A[r0:n, r0:r1].copy()
+    lu, piv, info = sla.lapack.dgetrf(P0.copy())
+    return lu, r0 + np.asarray(piv, dtype=np.int64), int(info), P0
+
+
+def lu_swap_rows(ipiv, k, nb):
+    """The rows a panel's pivot sequence moves (each swap p = k·nb + j <-> ipiv[j])."""
+    rows = []
+    for j, q in enumerate(ipiv):
+        p = k * nb + j
+        if p != int(q):
+            rows += [p, int(q)]
+    return sorted(set(rows))
+
+
+def lu_pd_apply(st: State, k: int, lu, ipiv, P0):
+    """c-13/c-14 PD, apply step: the row swaps on the left (factored L
+    panels, c only) and right (trailing, c and r) columns with the swap rule,
+    the panel's own column checksums swapped with the PRE-PD copy (L430),
+    then c(L_I) = c(P~_I)·U_kk^{-1} (L_kk in UNIT_LOWER view) and
+    r(U_kk) = L_kk^{-1}·r(P~_kk), magnitudes by |U_kk^{-1}|, |L_kk^{-1}| (c-6)."""
+    nb, n = st.nb, st.A.shape[0]
+    nt = n // nb
+    r0, r1 = k * nb, (k + 1) * nb
+    copy = P0.copy()
+    panel_cols = np.arange(r0, r1)
+    left_cols = np.arange(0, r0)
+    right_cols = np.arange(r1, n)
+    for j in range(nb):
+        p, q = r0 + j, int(ipiv[j])
+        if p == q:
+            continue
+        lu_swap_rule(st, p, q, panel_cols, copy[p - r0].copy(), copy[q - r0].copy(), row_chk_cols=range(k, nt))
+        copy[[p - r0, q - r0]] = copy[[q - r0, p - r0]]
+        if r0 > 0:
+            lu_swap_rule(st, p, q, left_cols, st.A[p, :r0].copy(), st.A[q, :r0].copy())
+        if r1 < n:
+            lu_swap_rule(st, p, q, right_cols, st.A[p, r1:].copy(), st.A[q, r1:].copy())
+        st.A[[p, q], :r0] = st.A[[q, p], :r0]
+        st.A[[p, q], r1:] = st.A[[q, p], r1:]
+    st.A[r0:n, r0:r1] = lu
+    U = np.triu(lu[:nb, :nb])
+    Lkk = np.tril(lu[:nb, :nb], -1) + np.eye(nb)
+    Uinv = tri_inv(U, lower=False)
+    Linv = tri_inv(Lkk, lower=True, unit=True)
+    cs = slice(r0, r1)
+    st.colchk[2 * k:, cs] = st.colchk[2 * k:, cs] @ Uinv
+    st.rowchk[r0:r1, 2 * k:2 * k + 2] = Linv @ st.rowchk[r0:r1, 2 * k:2 * k + 2]
+    if st.colmag is not None:
+        st.colmag[k:, cs] = st.colmag[k:, cs] @ np.abs(Uinv)
+        st.rowmag[r0:r1, k] = np.abs(Linv) @ st.rowmag[r0:r1, k]
+
+
+def lu_pd(st: State, k: int):
+    """Factor + apply (no pre-swap check): returns (ipiv_global, info)."""
+    lu, ipiv, info, P0 = lu_panel_getrf(st, k)
+    lu_pd_apply(st, k, lu, ipiv, P0)
+    return ipiv, info
+
+
+def lu_pu_data(st: State, k: int):
+    """c-13 PU data step: U_kJ = L_kk^{-1}·A_kJ for the row panel."""
+    nb, n = st.nb, st.A.shape[0]
+    r0, r1 = k * nb, (k + 1) * nb
+    Lkk = np.tril(st.A[r0:r1, r0:r1], -1) + np.eye(nb)
+    st.A[r0:r1, r1:n] = sla.solve_triangular(Lkk, st.A[r0:r1, r1:n], lower=True, unit_diagonal=True,
+                                             check_finite=False)
+
+
+def lu_pu_chk(st: State, k: int):
+    """c-13 PU checksum step: r(U_kJ) = L_kk^{-1}·r(A_kJ), m_r ← |L_kk^{-1}|·m_r."""
+    nb = st.nb
+    r0, r1 = k * nb, (k + 1) * nb
+    Lkk = np.tril(st.A[r0:r1, r0:r1], -1) + np.eye(nb)
+    st.rowchk[r0:r1, 2 * (k + 1):] = sla.solve_triangular(Lkk, st.rowchk[r0:r1, 2 * (k + 1):], lower=True,
+                                                          unit_diagonal=True, check_finite=False)
+    if st.rowmag is not None:
+        st.rowmag[r0:r1, k + 1:] = np.abs(tri_inv(Lkk, lower=True, unit=True)) @ st.rowmag[r0:r1, k + 1:]
+
+
+def lu_tmu_data(st: State, k: int):
+    """c-13 TMU data step: A_IJ −= L_Ik·U_kJ for every trailing tile."""
+    nb, n = st.nb, st.A.shape[0]
+    r0, r1 = k * nb, (k + 1) * nb
+    st.A[r1:n, r1:n] -= st.A[r1:n, r0:r1] @ st.A[r0:r1, r1:n]
+
+
+def lu_tmu_chk(st: State, k: int):
+    """c-13 TMU checksum step: c(A_IJ) −= c(L_Ik)·U_kJ, r(A_IJ) −= L_Ik·r(U_kJ);
+    m_c += m_c(L)·|U|, m_r += |L|·m_r(U) (c-6)."""
+    nb, n = st.nb, st.A.shape[0]
+    r0, r1 = k * nb, (k + 1) * nb
+    L21, U12 = st.A[r1:n, r0:r1], st.A[r0:r1, r1:n]
+    st.colchk[2 * (k + 1):, r1:n] -= st.colchk[2 * (k + 1):, r0:r1] @ U12
+    st.rowchk[r1:n, 2 * (k + 1):] -= L21 @ st.rowchk[r0:r1, 2 * (k + 1):]
+    if st.colmag is not None:
+        st.colmag[k + 1:, r1:n] += st.colmag[k + 1:, r0:r1] @ np.abs(U12)
+        st.rowmag[r1:n, k + 1:] += np.abs(L21) @ st.rowmag[r0:r1, k + 1:]
+
+
+def lu_fig4a_repair(st: State, k: int, gi: int, gj: int, before: float, after: float):
+    """Reading c-25 for LU: the post-TMU re-check corrected a panel element by
+    E = after − before; the TMU had consumed the bad value.
+    L21[p, q] (column panel): A[p, r1:] −= E·U[q, r1:], r(A_i,J)[p', :] −= E·r(U_J)[q, :]
+      (c(A) was built from the good c(L), so only data and r change); m_r += |E|·m_r(U).
+    U12[q, c] (row panel): A[r1:, c] −= L21[:, q]·E, c(A_I,j)[:, c'] −= c(L_I)[:, q]·E
+      (r(A) was built from the good r(U)); m_c += |E|·m_c(L).
+    Guard as in Cholesky (2^10 × max |panel line|, finite)."""
+    nb, n = st.nb, st.A.shape[0]
+    nt = n // nb
+    r0, r1 = k * nb, (k + 1) * nb
+    E = after - before
+    if r0 <= gj < r1 and gi >= r1:  # element of L21
+        p, q = gi, gj - r0
+        mx = float(np.max(np.abs(st.A[r1:n, gj])))
+        if not (np.isfinite(E) and abs(E) <= 1024.0 * mx):
+            return "skipped"
+        st.A[p, r1:n] -= E * st.A[r0 + q, r1:n]
+        for J in range(k + 1, nt):
+            st.rowchk[p, 2 * J:2 * J + 2] -= E * st.rowchk[r0 + q, 2 * J:2 * J + 2]
+            if st.rowmag is not None:
+                st.rowmag[p, J] += abs(E) * st.rowmag[r0 + q, J]
+        return "applied"
+    if r0 <= gi < r1 and gj >= r1:  # element of U12
+        q, c = gi - r0, gj
+        mx = float(np.max(np.abs(st.A[gi, r1:n])))
+        if not (np.isfinite(E) and abs(E) <= 1024.0 * mx):
+            return "skipped"
+        st.A[r1:n, c] -= st.A[r1:n, r0 + q] * E
+        for I in range(k + 1, nt):
+            st.colchk[2 * I:2 * I + 2, c] -= E * st.colchk[2 * I:2 * I + 2, r0 + q]
+            if st.colmag is not None:
+                st.colmag[I, c] += abs(E) * st.colmag[I, r0 + q]
+        return "applied"
+    return None

@@ -77,7 +77,7 @@ class ft_inject_t(C.Structure):
 class ft_opts_t(C.Structure):
     _fields_ = [("nb", C.c_int64), ("abft", C.c_int32), ("tol_kind", C.c_int32), ("tol_scale", C.c_double),
                 ("fig4a_repair", C.c_int32), ("n_inject", C.c_int32), ("inject", C.POINTER(ft_inject_t)),
-                ("fix_log", C.c_void_p), ("fix_log_cap", C.c_int32)]
+                ("fix_log", C.c_void_p), ("fix_log_cap", C.c_int32), ("pu_gemm", C.c_int32)]
 
 
 class ft_stats_t(C.Structure):
@@ -99,7 +99,10 @@ _sig = {
     "abft_update_trsm": [_i32, _ch, _ch, _ch, _ch, _i64, _vp, _i64, _vp, _i64, _i64, _vp, _i64, _i64, _vp],
     "abft_update_gemm": [_i32, _i32, _ch, _ch, _d, _vp, _i64, _vp, _i64, _vp, _i64, _i64, _i64, _i64,
                          _vp, _i64, _vp, _i64, _vp],
-    "abft_panel_potrf": [_P(abft_mat_t), _vp, _vp],
+    "abft_panel_potrf": [_P(abft_mat_t), _vp, _i64, _vp, _vp],
+    "abft_tri_inverse": [_i32, _ch, _ch, _i64, _vp, _i64, _vp, _i64, _vp],
+    "abft_update_trsm_inv": [_i32, _ch, _ch, _i64, _vp, _i64, _vp, _i64, _i64, _vp, _i64, _i64, _vp],
+    "abft_update_syrk": [_i32, _i64, _i64, _vp, _i64, _vp, _i64, _vp, _i64, _vp, _vp, _i64, _vp, _vp, _i64, _vp],
     "ft_ctx_create": [_P(_vp), _i32, _vp],
     "ft_ctx_destroy": [_vp],
     "ft_potrf": [_vp, _i32, _i64, _vp, _i64, _P(ft_opts_t), _P(ft_stats_t), _P(_i64)],
@@ -281,9 +284,30 @@ def abft_update_gemm(which, transX, transY, alpha, Xchk, Y, Cchk, M2, N, K, Xmag
         _ptr(Cchk), ld_of(Cchk), M2, N, K, _ptr(Xmag), ld_of(Xmag), _ptr(Cmag), ld_of(Cmag), _stream(stream)))
 
 
-def abft_panel_potrf(diag: Mat, info: torch.Tensor, stream=None):
+def abft_panel_potrf(diag: Mat, info: torch.Tensor, Linv: torch.Tensor = None, stream=None):
     m = diag.c()
-    return _check("abft_panel_potrf", _L.abft_panel_potrf(C.byref(m), _ptr(info), _stream(stream)))
+    return _check("abft_panel_potrf", _L.abft_panel_potrf(C.byref(m), _ptr(Linv), ld_of(Linv) if Linv is not None
+                                                          else 0, _ptr(info), _stream(stream)))
+
+
+def abft_tri_inverse(uplo, diag, T, W, stream=None):
+    nb = T.shape[0]
+    return _check("abft_tri_inverse", _L.abft_tri_inverse(_dt(T), uplo.encode(), diag.encode(), nb, _ptr(T), ld_of(T),
+                                                          _ptr(W), ld_of(W), _stream(stream)))
+
+
+def abft_update_trsm_inv(side, trans, W, chk, nvec, mag=None, nmag=0, stream=None):
+    return _check("abft_update_trsm_inv", _L.abft_update_trsm_inv(
+        _dt(W), side.encode(), trans.encode(), W.shape[0], _ptr(W), ld_of(W), _ptr(chk), ld_of(chk), nvec,
+        _ptr(mag), ld_of(mag), nmag, _stream(stream)))
+
+
+def abft_update_syrk(nb, ntk, L21, cL, Cc, Rr, mL=None, Cm=None, Rm=None, stream=None):
+    """Cholesky TMU checksum rule; Cc/Rr/Cm/Rm are the trailing blocks of
+    colchk/rowchk/colmag/rowmag (views sharing their arrays' ld)."""
+    return _check("abft_update_syrk", _L.abft_update_syrk(
+        _dt(L21), nb, ntk, _ptr(L21), ld_of(L21), _ptr(cL), ld_of(cL), _ptr(mL), ld_of(mL), _ptr(Cc), _ptr(Rr),
+        ld_of(Rr), _ptr(Cm), _ptr(Rm), ld_of(Rm), _stream(stream)))
 
 
 def decode_fixes(buf: torch.Tensor, n: int):
@@ -304,13 +328,13 @@ class Context:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h is not None and h.value:
+        if h is not None and h.value and _L is not None:
             _L.ft_ctx_destroy(h)
             self._h = None
 
 
 def ft_potrf(ctx: Context, A: torch.Tensor, nb: int, abft=True, tol_kind=TOL_MAGNITUDE, tol_scale=1.0,
-             fig4a_repair=True, inject=(), fix_log=None):
+             fig4a_repair=True, inject=(), fix_log=None, pu_gemm=True):
     """Fault-tolerant lower Cholesky in place on a column-major A.  Returns
     (rc, info, stats) with rc 0 or E_UNCORRECTABLE (other codes raise)."""
     n = A.shape[0]
@@ -318,7 +342,7 @@ def ft_potrf(ctx: Context, A: torch.Tensor, nb: int, abft=True, tol_kind=TOL_MAG
     for k, f in enumerate(inject):
         inj[k] = ft_inject_t(*f)
     opts = ft_opts_t(nb, int(abft), tol_kind, tol_scale, int(fig4a_repair), len(inject), inj,
-                     _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES)
+                     _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES, int(pu_gemm))
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_potrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), C.byref(opts), C.byref(stats), C.byref(info))

@@ -77,6 +77,7 @@ struct PassArgs {
   void* drow;
   int32_t* counts;
   void* part;       // [ntiles][GROUPS][NB][3] (slabbed tiles only)
+  void* symws;      // [ntiles][3][NB] SYM column sums of slabbed diagonal tiles
   int* ticket;      // [ntiles] self-resetting
   int* tflags;      // [ntiles] self-resetting
 };
@@ -119,8 +120,10 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
   tile_of(p.tiles, tile, I, J);
   const int view = (I == J) ? p.tiles.diag_view : ABFT_GENERAL;
   const bool sym = view == ABFT_SYM_LOWER;
-  if (sym && slab != 0) return;  // symmetric diagonal tiles are never split
-  const int nslab = sym ? 1 : p.nslab;
+  const int nslab = p.nslab;
+  // SYM column sums of a split tile go through the workspace (the finishing
+  // CTA adds them to the row sums); an unsplit tile keeps them in smem
+  T* symcol = (sym && nslab > 1) ? reinterpret_cast<T*>(p.symws) + (size_t)tile * NB * 3 : symacc;
   const int cols = NB / nslab;
   const int c0 = slab * cols;
   const int nst = cols / C::CC;
@@ -182,9 +185,9 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
   // column finish: encode writes c (and m_c); verify compares (c-6, c-7)
   auto finish_col = [&](int jl, T pe, T pw, T pa) {
     if (sym) {
-      symacc[jl] = pe;
-      symacc[NB + jl] = pw;
-      symacc[2 * NB + jl] = pa;
+      symcol[jl] = pe;
+      symcol[NB + jl] = pw;
+      symcol[2 * NB + jl] = pa;
       return;
     }
     if (!(p.which & ABFT_COL)) return;
@@ -378,9 +381,15 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
     if (r >= NB) continue;
     T re = tot[q].e, rw = tot[q].w, ra = tot[q].a;
     if (sym) {  // c_sym[r] = colsum_lower[r] + rowsum_strict[r]; r_sym = c_sym^T
-      re = fadd(symacc[r], re);
-      rw = fadd(symacc[NB + r], rw);
-      ra = fadd(symacc[2 * NB + r], ra);
+      if (nslab > 1) {
+        re = fadd(__ldcg(symcol + r), re);
+        rw = fadd(__ldcg(symcol + NB + r), rw);
+        ra = fadd(__ldcg(symcol + 2 * NB + r), ra);
+      } else {
+        re = fadd(symacc[r], re);
+        rw = fadd(symacc[NB + r], rw);
+        ra = fadd(symacc[2 * NB + r], ra);
+      }
     }
     const int64_t gi = (int64_t)I * NB + r;
     const int64_t gj = (int64_t)J * NB + r;
@@ -466,13 +475,14 @@ static int launch_nb(PassArgs& a, int64_t ntiles, cudaStream_t s) {
   a.nslab = nslab;
   if (nslab > 1) {
     void* ws = nullptr;
-    size_t bytes = (size_t)ntiles * C::GROUPS * NB * 3 * sizeof(T);
+    size_t bytes = (size_t)ntiles * (C::GROUPS + 1) * NB * 3 * sizeof(T);
     int rc = workspace_get(s, bytes, &ws);
     if (rc) return rc;
     int* ctr = nullptr;
     rc = counters_get(s, (size_t)2 * ntiles, &ctr);
     if (rc) return rc;
     a.part = ws;
+    a.symws = reinterpret_cast<T*>(ws) + (size_t)ntiles * C::GROUPS * NB * 3;
     a.ticket = ctr;
     a.tflags = ctr + ntiles;
   }

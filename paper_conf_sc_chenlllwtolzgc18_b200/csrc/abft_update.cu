@@ -13,6 +13,7 @@
 
 #include <mutex>
 #include <unordered_map>
+#include <vector>
 
 #include "abft_common.cuh"
 
@@ -170,63 +171,253 @@ static cublasStatus_t trsm(cublasHandle_t h, cublasSideMode_t sd, cublasFillMode
 
 static cublasOperation_t op_of(char t) { return (t == 'T' || t == 't') ? CUBLAS_OP_T : CUBLAS_OP_N; }
 
-// |op(T)^-1| (nb x nb, ld nb) into scratch slot 1.
+// W = T^-1 (explicit triangular inverse; the other triangle of W is zero, a
+// unit diagonal is materialised).  Recursive block inversion:
+// the 64x64 diagonal blocks are inverted in shared memory by one CTA each
+// (row-by-row substitution, threads over columns), then pairs of inverted
+// blocks are merged level by level with two strided-batched DGEMMs,
+//   lower: inv([A 0; B C]) = [A^-1 0; -C^-1 B A^-1  C^-1]
+//   upper: inv([A B; 0 C]) = [A^-1  -A^-1 B C^-1; 0 C^-1].
+constexpr int kInvBS = 64;
+
 template <typename T>
-int abs_tri_inverse(cublasHandle_t h, char side, char uplo, char trans, char diag, int nb, const T* Tm, int ldt,
-                    cudaStream_t s, T** out) {
-  void* w = nullptr;
-  int rc = scratch_get(s, 1, (size_t)nb * nb * sizeof(T), &w);
+__global__ void __launch_bounds__(256) tri_inv_base_kernel(const T* __restrict__ Tm, int ldt, T* __restrict__ W,
+                                                           int ldw, int bs, int upper, int unit) {
+  // X = L^-1 by column-oriented forward elimination on X = I:
+  //   for k: X[k,:] /= L[k,k];  X[i,:] -= L[i,k] X[k,:] (i > k)
+  // 256 threads: thread (j, g) owns column j and rows i = g, g+4, ...
+  extern __shared__ __align__(16) unsigned char inv_sm[];
+  T(*Ls)[kInvBS + 1] = reinterpret_cast<T(*)[kInvBS + 1]>(inv_sm);
+  T(*Xs)[kInvBS + 1] = Ls + kInvBS;
+  const int b0 = blockIdx.x * bs;
+  const int tid = threadIdx.x;
+  for (int idx = tid; idx < bs * bs; idx += blockDim.x) {
+    const int i = idx % bs, j = idx / bs;  // coalesced along i (column-major source)
+    T v;
+    if (upper)  // Ls = U^T (lower): Ls[j][i] = U[i][j] for i <= j
+      v = Tm[(b0 + i) + (int64_t)(b0 + j) * ldt];
+    else
+      v = Tm[(b0 + i) + (int64_t)(b0 + j) * ldt];
+    if (upper) {
+      T u = (i <= j) ? v : T(0);
+      if (unit && i == j) u = T(1);
+      Ls[j][i] = u;
+    } else {
+      T l = (i >= j) ? v : T(0);
+      if (unit && i == j) l = T(1);
+      Ls[i][j] = l;
+    }
+    Xs[i][j] = (i == j) ? T(1) : T(0);
+  }
+  __syncthreads();
+  const int j = tid % kInvBS, g = tid / kInvBS, ng = blockDim.x / kInvBS;
+  for (int k = 0; k < bs; ++k) {
+    if (j < bs && g == 0) Xs[k][j] = Xs[k][j] / Ls[k][k];
+    __syncthreads();
+    if (j < bs) {
+      const T xk = Xs[k][j];
+      for (int i = k + 1 + g; i < bs; i += ng) Xs[i][j] -= Ls[i][k] * xk;
+    }
+    __syncthreads();
+  }
+  for (int idx = tid; idx < bs * bs; idx += blockDim.x) {
+    const int i = idx % bs, jj = idx / bs;
+    if (upper)  // W = X^T
+      W[(b0 + i) + (int64_t)(b0 + jj) * ldw] = Xs[jj][i];
+    else
+      W[(b0 + i) + (int64_t)(b0 + jj) * ldw] = Xs[i][jj];
+  }
+}
+
+static cublasStatus_t gemm_sb(cublasHandle_t h, cublasOperation_t ta, cublasOperation_t tb, int m, int n, int k,
+                              const double* al, const double* A, int lda, long long sa, const double* B, int ldb,
+                              long long sb, const double* be, double* C, int ldc, long long sc, int batch) {
+  return cublasDgemmStridedBatched(h, ta, tb, m, n, k, al, A, lda, sa, B, ldb, sb, be, C, ldc, sc, batch);
+}
+static cublasStatus_t gemm_sb(cublasHandle_t h, cublasOperation_t ta, cublasOperation_t tb, int m, int n, int k,
+                              const float* al, const float* A, int lda, long long sa, const float* B, int ldb,
+                              long long sb, const float* be, float* C, int ldc, long long sc, int batch) {
+  return cublasSgemmStridedBatched(h, ta, tb, m, n, k, al, A, lda, sa, B, ldb, sb, be, C, ldc, sc, batch);
+}
+
+template <typename T>
+int tri_inverse_t(char uplo, char diag, int nb, const T* Tm, int ldt, T* W, int ldw, cudaStream_t s) {
+  const bool upper = uplo == 'U' || uplo == 'u', unit = diag == 'U' || diag == 'u';
+  const int bs = nb < kInvBS ? nb : kInvBS;
+  if (nb % bs) return ABFT_E_UNSUPPORTED;
+  ABFT_CUDA_TRY(cudaMemset2DAsync(W, (size_t)ldw * sizeof(T), 0, (size_t)nb * sizeof(T), nb, s));
+  const size_t smem = 2 * kInvBS * (kInvBS + 1) * sizeof(T);
+  static bool attr = false;
+  if (!attr) {
+    ABFT_CUDA_TRY(cudaFuncSetAttribute(tri_inv_base_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    attr = true;
+  }
+  tri_inv_base_kernel<T><<<nb / bs, 256, smem, s>>>(Tm, ldt, W, ldw, bs, upper, unit);
+  ABFT_CUDA_TRY(cudaGetLastError());
+  if (bs == nb) return 0;
+  void* tv = nullptr;
+  int rc = scratch_get(s, 9, (size_t)nb * nb / 2 * sizeof(T), &tv);
   if (rc) return rc;
-  T* W = reinterpret_cast<T*>(w);
-  identity_kernel<T><<<grid_for((int64_t)nb * nb), 256, 0, s>>>(W, nb);
-  ABFT_CUDA_TRY(cudaGetLastError());
-  const T one = T(1);
-  // W = I * op(T)^-1 (right) or op(T)^-1 * I (left) -- the same matrix
-  ABFT_CUBLAS_TRY(trsm(h, (side == 'L' || side == 'l') ? CUBLAS_SIDE_LEFT : CUBLAS_SIDE_RIGHT,
-                       (uplo == 'U' || uplo == 'u') ? CUBLAS_FILL_MODE_UPPER : CUBLAS_FILL_MODE_LOWER, op_of(trans),
-                       (diag == 'U' || diag == 'u') ? CUBLAS_DIAG_UNIT : CUBLAS_DIAG_NON_UNIT, nb, nb, &one, Tm, ldt,
-                       W, nb));
-  abs_inplace_kernel<T><<<grid_for((int64_t)nb * nb), 256, 0, s>>>(W, (int64_t)nb * nb);
-  ABFT_CUDA_TRY(cudaGetLastError());
-  *out = W;
+  T* tmp = reinterpret_cast<T*>(tv);
+  std::unique_lock<std::mutex> lk;
+  cublasHandle_t h = blas_handle(s, lk);
+  const T one = T(1), zero = T(0), mone = T(-1);
+  for (int sz = bs; sz < nb; sz *= 2) {
+    const int batch = nb / (2 * sz);
+    const long long sW = (long long)(2 * sz) * (1 + ldw), sT = (long long)(2 * sz) * (1 + ldt);
+    const long long sTmp = (long long)sz * sz;
+    const T* Ai = W;                                  // A^-1 at (0,0) of each pair
+    const T* Ci = W + sz + (int64_t)sz * ldw;         // C^-1 at (s,s)
+    if (!upper) {
+      const T* B = Tm + sz;                           // B at (s,0) of T
+      T* X = W + sz;                                  // result block (s,0) of W
+      ABFT_CUBLAS_TRY(gemm_sb(h, CUBLAS_OP_N, CUBLAS_OP_N, sz, sz, sz, &one, B, ldt, sT, Ai, ldw, sW, &zero, tmp, sz,
+                              sTmp, batch));
+      ABFT_CUBLAS_TRY(gemm_sb(h, CUBLAS_OP_N, CUBLAS_OP_N, sz, sz, sz, &mone, Ci, ldw, sW, tmp, sz, sTmp, &zero, X, ldw,
+                              sW, batch));
+    } else {
+      const T* B = Tm + (int64_t)sz * ldt;            // B at (0,s) of T
+      T* X = W + (int64_t)sz * ldw;                   // result block (0,s) of W
+      ABFT_CUBLAS_TRY(gemm_sb(h, CUBLAS_OP_N, CUBLAS_OP_N, sz, sz, sz, &one, Ai, ldw, sW, B, ldt, sT, &zero, tmp, sz,
+                              sTmp, batch));
+      ABFT_CUBLAS_TRY(gemm_sb(h, CUBLAS_OP_N, CUBLAS_OP_N, sz, sz, sz, &mone, tmp, sz, sTmp, Ci, ldw, sW, &zero, X, ldw,
+                              sW, batch));
+    }
+  }
+  return 0;
+}
+
+// out (rows x cols, ld ldo) <- tmp (ld rows): stream-ordered copy back
+template <typename T>
+static int copy_back(T* out, int64_t ldo, const T* tmp, int64_t rows, int64_t cols, cudaStream_t s) {
+  ABFT_CUDA_TRY(cudaMemcpy2DAsync(out, ldo * sizeof(T), tmp, rows * sizeof(T), rows * sizeof(T), cols,
+                                  cudaMemcpyDeviceToDevice, s));
+  return 0;
+}
+
+// a5 with a precomputed inverse W = T^-1:
+//   side R: chk (nvec x nb) <- chk * op(W);  mag (nmag x nb) <- mag * |op(W)|
+//   side L: chk (nb x nvec) <- op(W) * chk;  mag (nb x nmag) <- |op(W)| * mag
+template <typename T>
+int update_trsm_inv_t(char side, char trans, int64_t nb, const T* W, int64_t ldw, T* chk, int64_t ldchk, int64_t nvec,
+                      T* mag, int64_t ldmag, int64_t nmag, cudaStream_t s) {
+  const bool left = side == 'L' || side == 'l';
+  const cublasOperation_t oW = op_of(trans);
+  const T one = T(1), zero = T(0);
+  const int64_t nmax = nvec > nmag ? nvec : nmag;
+  if (nmax <= 0) return 0;
+  void* tv = nullptr;
+  int rc = scratch_get(s, 2, (size_t)nb * nmax * sizeof(T), &tv);
+  if (rc) return rc;
+  T* tmp = reinterpret_cast<T*>(tv);
+  std::unique_lock<std::mutex> lk;
+  cublasHandle_t h = blas_handle(s, lk);
+  if (nvec > 0) {
+    if (!left) {
+      ABFT_CUBLAS_TRY(gemm(h, CUBLAS_OP_N, oW, (int)nvec, (int)nb, (int)nb, &one, chk, (int)ldchk, W, (int)ldw, &zero,
+                           tmp, (int)nvec));
+      rc = copy_back<T>(chk, ldchk, tmp, nvec, nb, s);
+    } else {
+      ABFT_CUBLAS_TRY(gemm(h, oW, CUBLAS_OP_N, (int)nb, (int)nvec, (int)nb, &one, W, (int)ldw, chk, (int)ldchk, &zero,
+                           tmp, (int)nb));
+      rc = copy_back<T>(chk, ldchk, tmp, nb, nvec, s);
+    }
+    if (rc) return rc;
+  }
+  if (mag && nmag > 0) {
+    void* av = nullptr;
+    rc = scratch_get(s, 1, (size_t)nb * nb * sizeof(T), &av);
+    if (rc) return rc;
+    T* aW = reinterpret_cast<T*>(av);
+    rc = abs_copy<T>(aW, W, nb, nb, ldw, s);
+    if (rc) return rc;
+    if (!left) {
+      ABFT_CUBLAS_TRY(gemm(h, CUBLAS_OP_N, oW, (int)nmag, (int)nb, (int)nb, &one, mag, (int)ldmag, aW, (int)nb, &zero,
+                           tmp, (int)nmag));
+      rc = copy_back<T>(mag, ldmag, tmp, nmag, nb, s);
+    } else {
+      ABFT_CUBLAS_TRY(gemm(h, oW, CUBLAS_OP_N, (int)nb, (int)nmag, (int)nb, &one, aW, (int)nb, mag, (int)ldmag, &zero,
+                           tmp, (int)nb));
+      rc = copy_back<T>(mag, ldmag, tmp, nb, nmag, s);
+    }
+    if (rc) return rc;
+  }
   return 0;
 }
 
 template <typename T>
 int update_trsm_t(char side, char uplo, char trans, char diag, int64_t nb, const void* Tv, int64_t ldt, void* chkv,
                   int64_t ldchk, int64_t nvec, void* magv, int64_t ldmag, int64_t nmag, cudaStream_t s) {
-  std::unique_lock<std::mutex> lk;
-  cublasHandle_t h = blas_handle(s, lk);
-  const T* Tm = reinterpret_cast<const T*>(Tv);
-  T* chk = reinterpret_cast<T*>(chkv);
-  const bool left = side == 'L' || side == 'l';
-  const T one = T(1), zero = T(0);
-  if (nvec > 0) {
-    ABFT_CUBLAS_TRY(trsm(h, left ? CUBLAS_SIDE_LEFT : CUBLAS_SIDE_RIGHT,
-                         (uplo == 'U' || uplo == 'u') ? CUBLAS_FILL_MODE_UPPER : CUBLAS_FILL_MODE_LOWER,
-                         op_of(trans), (diag == 'U' || diag == 'u') ? CUBLAS_DIAG_UNIT : CUBLAS_DIAG_NON_UNIT,
-                         left ? (int)nb : (int)nvec, left ? (int)nvec : (int)nb, &one, Tm, (int)ldt, chk, (int)ldchk));
+  void* wv = nullptr;
+  int rc = scratch_get(s, 5, (size_t)nb * nb * sizeof(T), &wv);
+  if (rc) return rc;
+  T* W = reinterpret_cast<T*>(wv);
+  rc = tri_inverse_t<T>(uplo, diag, (int)nb, reinterpret_cast<const T*>(Tv), (int)ldt, W, (int)nb, s);
+  if (rc) return rc;
+  return update_trsm_inv_t<T>(side, trans, nb, W, nb, reinterpret_cast<T*>(chkv), ldchk, nvec,
+                              reinterpret_cast<T*>(magv), ldmag, nmag, s);
+}
+
+// Cholesky TMU checksum rule from ONE product (c-12, L189).  P = c(L21) L21^T
+// (M2 x nk) gives c(A_IJ) -= P[2I.., cols of J] for I >= J and, transposed,
+// r(A_IJ) -= P[2J.., cols of I]^T for I >= J.  Magnitudes from
+// Q = m_c(L21) |L21|^T likewise (c-6).
+template <typename T>
+__global__ void syrk_scatter_col_kernel(T* __restrict__ C, int64_t ldc, const T* __restrict__ P, int64_t M, int64_t nk,
+                                        int nb, int rows_per_tile, T sign) {
+  const int64_t total = M * nk;
+  for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+       idx += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t x = idx / M, y = idx - x * M;
+    if (y / rows_per_tile >= x / nb) C[y + x * ldc] += sign * P[idx];
   }
-  if (magv && nmag > 0) {
-    T* W = nullptr;
-    int rc = abs_tri_inverse<T>(h, side, uplo, trans, diag, (int)nb, Tm, (int)ldt, s, &W);
+}
+template <typename T>
+__global__ void syrk_scatter_row_kernel(T* __restrict__ R, int64_t ldr, const T* __restrict__ P, int64_t M, int64_t nk,
+                                        int nb, int rows_per_tile, T sign) {
+  const int64_t total = M * nk;
+  for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+       idx += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t y = idx / nk, x = idx - y * nk;
+    if (x / nb >= y / rows_per_tile) R[x + y * ldr] += sign * P[y + x * M];
+  }
+}
+
+template <typename T>
+int update_syrk_t(int64_t nb, int64_t ntk, const T* L21, int64_t ldl, const T* cL, int64_t ldc, const T* mL,
+                  int64_t ldcm, T* Cc, T* Rr, int64_t ldr, T* Cm, T* Rm, int64_t ldrm, cudaStream_t s) {
+  const int64_t nk = ntk * nb, M2 = 2 * ntk;
+  if (nk == 0) return 0;
+  void* pv = nullptr;
+  int rc = scratch_get(s, 7, (size_t)M2 * nk * sizeof(T), &pv);
+  if (rc) return rc;
+  T* P = reinterpret_cast<T*>(pv);
+  const T one = T(1), zero = T(0);
+  {
+    std::unique_lock<std::mutex> lk;
+    cublasHandle_t h = blas_handle(s, lk);
+    ABFT_CUBLAS_TRY(gemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)M2, (int)nk, (int)nb, &one, cL, (int)ldc, L21, (int)ldl,
+                         &zero, P, (int)M2));
+  }
+  syrk_scatter_col_kernel<T><<<grid_for(M2 * nk), 256, 0, s>>>(Cc, ldc, P, M2, nk, (int)nb, 2, T(-1));
+  syrk_scatter_row_kernel<T><<<grid_for(M2 * nk), 256, 0, s>>>(Rr, ldr, P, M2, nk, (int)nb, 2, T(-1));
+  ABFT_CUDA_TRY(cudaGetLastError());
+  if (mL && Cm && Rm) {
+    void* av = nullptr;
+    rc = scratch_get(s, 3, (size_t)nk * nb * sizeof(T), &av);
     if (rc) return rc;
-    T* mag = reinterpret_cast<T*>(magv);
-    void* tmpv = nullptr;
-    rc = scratch_get(s, 2, (size_t)nb * nmag * sizeof(T), &tmpv);
+    T* aL = reinterpret_cast<T*>(av);
+    rc = abs_copy<T>(aL, L21, nk, nb, ldl, s);
     if (rc) return rc;
-    T* tmp = reinterpret_cast<T*>(tmpv);
-    if (!left) {  // tmp (nmag x nb) = mag * |W|
-      ABFT_CUBLAS_TRY(gemm(h, CUBLAS_OP_N, CUBLAS_OP_N, (int)nmag, (int)nb, (int)nb, &one, mag, (int)ldmag, W,
-                           (int)nb, &zero, tmp, (int)nmag));
-      ABFT_CUDA_TRY(cudaMemcpy2DAsync(mag, ldmag * sizeof(T), tmp, nmag * sizeof(T), nmag * sizeof(T), nb,
-                                      cudaMemcpyDeviceToDevice, s));
-    } else {  // tmp (nb x nmag) = |W| * mag
-      ABFT_CUBLAS_TRY(gemm(h, CUBLAS_OP_N, CUBLAS_OP_N, (int)nb, (int)nmag, (int)nb, &one, W, (int)nb, mag,
-                           (int)ldmag, &zero, tmp, (int)nb));
-      ABFT_CUDA_TRY(cudaMemcpy2DAsync(mag, ldmag * sizeof(T), tmp, nb * sizeof(T), nb * sizeof(T), nmag,
-                                      cudaMemcpyDeviceToDevice, s));
+    {
+      std::unique_lock<std::mutex> lk;
+      cublasHandle_t h = blas_handle(s, lk);
+      ABFT_CUBLAS_TRY(gemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)ntk, (int)nk, (int)nb, &one, mL, (int)ldcm, aL, (int)nk,
+                           &zero, P, (int)ntk));
     }
+    syrk_scatter_col_kernel<T><<<grid_for(ntk * nk), 256, 0, s>>>(Cm, ldcm, P, ntk, nk, (int)nb, 1, T(1));
+    syrk_scatter_row_kernel<T><<<grid_for(ntk * nk), 256, 0, s>>>(Rm, ldrm, P, ntk, nk, (int)nb, 1, T(1));
+    ABFT_CUDA_TRY(cudaGetLastError());
   }
   return 0;
 }
@@ -318,4 +509,56 @@ extern "C" int abft_update_gemm(int32_t dtype, int32_t which, char transX, char 
                                            Xmag, ldxm, Cmag, ldcm, s)
              : abft::update_gemm_t<float>(which, transX, transY, alpha, Xchk, ldx, Y, ldy, Cchk, ldcc, M2, N, K,
                                           Xmag, ldxm, Cmag, ldcm, s);
+}
+
+extern "C" int abft_tri_inverse(int32_t dtype, char uplo, char diag, int64_t nb, const void* T, int64_t ldt, void* W,
+                                int64_t ldw, abft_stream_t stream) {
+  if (dtype != ABFT_F32 && dtype != ABFT_F64) return -1;
+  if (uplo != 'L' && uplo != 'U') return -2;
+  if (diag != 'N' && diag != 'U') return -3;
+  if (nb <= 0) return -4;
+  if (!T || ldt < nb) return -5;
+  if (!W || ldw < nb) return -7;
+  cudaStream_t s = (cudaStream_t)stream;
+  return dtype == ABFT_F64
+             ? abft::tri_inverse_t<double>(uplo, diag, (int)nb, (const double*)T, (int)ldt, (double*)W, (int)ldw, s)
+             : abft::tri_inverse_t<float>(uplo, diag, (int)nb, (const float*)T, (int)ldt, (float*)W, (int)ldw, s);
+}
+
+extern "C" int abft_update_trsm_inv(int32_t dtype, char side, char trans, int64_t nb, const void* W, int64_t ldw,
+                                    void* chk, int64_t ldchk, int64_t nvec, void* mag, int64_t ldmag, int64_t nmag,
+                                    abft_stream_t stream) {
+  if (dtype != ABFT_F32 && dtype != ABFT_F64) return -1;
+  if (side != 'L' && side != 'R') return -2;
+  if (trans != 'N' && trans != 'T') return -3;
+  if (nb <= 0) return -4;
+  if (!W || ldw < nb) return -5;
+  if (nvec < 0) return -9;
+  if (nvec > 0 && (!chk || ldchk < (side == 'R' ? nvec : nb))) return -7;
+  if (mag && nmag > 0 && ldmag < (side == 'R' ? nmag : nb)) return -11;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (dtype == ABFT_F64)
+    return abft::update_trsm_inv_t<double>(side, trans, nb, (const double*)W, ldw, (double*)chk, ldchk, nvec,
+                                           (double*)mag, ldmag, nmag, s);
+  return abft::update_trsm_inv_t<float>(side, trans, nb, (const float*)W, ldw, (float*)chk, ldchk, nvec, (float*)mag,
+                                        ldmag, nmag, s);
+}
+
+extern "C" int abft_update_syrk(int32_t dtype, int64_t nb, int64_t ntk, const void* L21, int64_t ldl, const void* cL,
+                                int64_t ldc, const void* mL, int64_t ldcm, void* Cc, void* Rr, int64_t ldr, void* Cm,
+                                void* Rm, int64_t ldrm, abft_stream_t stream) {
+  if (dtype != ABFT_F32 && dtype != ABFT_F64) return -1;
+  if (nb <= 0) return -2;
+  if (ntk < 0) return -3;
+  if (ntk == 0) return 0;
+  if (!L21 || ldl < ntk * nb) return -4;
+  if (!cL || !Cc || ldc < 2 * ntk) return -6;
+  if (!Rr || ldr < ntk * nb) return -11;
+  if (mL && (!Cm || !Rm || ldcm < ntk || ldrm < ntk * nb)) return -8;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (dtype == ABFT_F64)
+    return abft::update_syrk_t<double>(nb, ntk, (const double*)L21, ldl, (const double*)cL, ldc, (const double*)mL,
+                                       ldcm, (double*)Cc, (double*)Rr, ldr, (double*)Cm, (double*)Rm, ldrm, s);
+  return abft::update_syrk_t<float>(nb, ntk, (const float*)L21, ldl, (const float*)cL, ldc, (const float*)mL, ldcm,
+                                    (float*)Cc, (float*)Rr, ldr, (float*)Cm, (float*)Rm, ldrm, s);
 }

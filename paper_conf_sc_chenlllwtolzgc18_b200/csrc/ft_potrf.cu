@@ -51,17 +51,27 @@ static int potrf_tile(const abft_mat_t* d, int32_t* info, cudaStream_t s) {
 }
 }  // namespace abft
 
-extern "C" int abft_panel_potrf(const abft_mat_t* d, int32_t* info, abft_stream_t stream) {
+extern "C" int abft_panel_potrf(const abft_mat_t* d, void* Linv, int64_t ldw, int32_t* info, abft_stream_t stream) {
   if (!d || d->m != d->nb || d->n != d->nb || !d->A || d->lda < d->nb) return -1;
-  if (!info) return -2;
+  if (Linv && ldw < d->nb) return -3;
+  if (!info) return -4;
   if (d->dtype != ABFT_F32 && d->dtype != ABFT_F64) return -1;
   cudaStream_t s = (cudaStream_t)stream;
   int rc = d->dtype == ABFT_F64 ? abft::potrf_tile<double>(d, info, s) : abft::potrf_tile<float>(d, info, s);
   if (rc) return rc;
+  if (!d->colchk && !Linv) return 0;
+  // L_kk^-1 once (reused by the caller for the PU when Linv is given)
+  void* W = Linv;
+  int64_t ldW = ldw;
+  if (!W) {
+    FT_TRY(abft::scratch(s, 8, (size_t)d->nb * d->nb * (d->dtype == ABFT_F64 ? 8 : 4), &W));
+    ldW = d->nb;
+  }
+  FT_TRY(abft_tri_inverse(d->dtype, 'L', 'N', d->nb, d->A, d->lda, W, ldW, stream));
   if (!d->colchk) return 0;
   // c(L_kk) = c_sym(A_kk) L_kk^-T ; m_c(L_kk) = m_c |L_kk^-T|   (c-12, c-6)
-  return abft_update_trsm(d->dtype, 'R', 'L', 'T', 'N', d->nb, d->A, d->lda, d->colchk, d->ldc, 2, d->colmag,
-                          d->ldcm, d->colmag ? 1 : 0, stream);
+  return abft_update_trsm_inv(d->dtype, 'R', 'T', d->nb, W, ldW, d->colchk, d->ldc, 2, d->colmag, d->ldcm,
+                              d->colmag ? 1 : 0, stream);
 }
 
 // --------------------------------------------------------- Fig. 4a repair --
@@ -161,6 +171,10 @@ struct ft_ctx {
   size_t ints_n = 0;
   abft_fix_t* fixlog = nullptr;
   int fixcap = 0;
+  void* linv = nullptr;  // nb x nb inverse of the current L_kk
+  size_t linv_bytes = 0;
+  void* putmp = nullptr;  // n x nb panel scratch for the GEMM-based PU
+  size_t putmp_bytes = 0;
 };
 
 extern "C" int ft_ctx_create(ft_ctx_t** ctx, int32_t device, abft_stream_t stream) {
@@ -184,6 +198,8 @@ extern "C" int ft_ctx_destroy(ft_ctx_t* c) {
   if (c->state) cudaFree(c->state);
   if (c->ints) cudaFree(c->ints);
   if (c->fixlog) cudaFree(c->fixlog);
+  if (c->linv) cudaFree(c->linv);
+  if (c->putmp) cudaFree(c->putmp);
   delete c;
   return 0;
 }
@@ -229,6 +245,18 @@ struct Driver {
         onchip_pending.push_back(f);
     }
     return 0;
+  }
+  // Fault-injection runs only: does the plan touch L_kk between the PD (which
+  // produced the inverse the GEMM-based PU reads) and the PU?  Then the PU
+  // must see the flipped L_kk, as an in-place TRSM would (reading c-8).
+  bool lkk_touched_before_pu(int k) const {
+    for (int t = 0; t < o->n_inject; ++t) {
+      const ft_inject_t& f = o->inject[t];
+      if (f.iter != k || f.target != 0) continue;
+      if (f.point != FT_AT_PRE_PU_CHECK && f.point != FT_AT_PRE_PU) continue;
+      if (f.gi >= k * nb && f.gi < (k + 1) * nb && f.gj >= k * nb && f.gj < (k + 1) * nb) return true;
+    }
+    return false;
   }
   int restore_onchip() {  // after the op: undo on-chip flips (the stored value was never wrong)
     for (auto& f : onchip_pending) FT_TRY(abft_inject(elem(f.target, f.gi, f.gj), dtype, 0, f.xor_mask, (abft_stream_t)s));
@@ -292,6 +320,17 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (cudaMalloc(&c->ints, ints_need * sizeof(int32_t)) != cudaSuccess) return ABFT_E_NOMEM;
     c->ints_n = ints_need;
   }
+  auto grow = [](void*& p, size_t& have, size_t need) -> int {
+    if (have >= need) return 0;
+    if (p) cudaFree(p);
+    p = nullptr;
+    have = 0;
+    if (cudaMalloc(&p, need) != cudaSuccess) return ABFT_E_NOMEM;
+    have = need;
+    return 0;
+  };
+  FT_TRY(grow(c->linv, c->linv_bytes, (size_t)nb * nb * d.es));
+  if (o->pu_gemm) FT_TRY(grow(c->putmp, c->putmp_bytes, (size_t)n * nb * d.es));
   d.status = c->ints;
   d.counts = d.status + nt * nt;
   d.nfix = d.counts + 8;
@@ -354,7 +393,8 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
         D.colmag = d.colmag_at(k, k * nb);
         D.ldcm = d.M.ldcm;
       }
-      FT_TRY(abft_panel_potrf(&D, d.info, as));
+      const bool need_inv = ft || o->pu_gemm;
+      FT_TRY(abft_panel_potrf(&D, need_inv ? c->linv : nullptr, nb, d.info, as));
       accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.rep + 2, (int64_t)k * nb);
     }
     FT_TRY(d.restore_onchip());
@@ -367,9 +407,30 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft) FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH));
     // line 9: PU  L_ik = A_ik L_kk^-T  (+ c(L_ik) = c(A_ik) L_kk^-T, c-12)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PU));
+    const bool refresh_inv = o->pu_gemm && d.lkk_touched_before_pu(k);
+    if (refresh_inv) FT_TRY(abft_tri_inverse(dtype, 'L', 'N', nb, d.a_at(k * nb, k * nb), lda, c->linv, nb, as));
     {
       cublasHandle_t h = blas_handle(s, lk);
-      if (dtype == ABFT_F64) {
+      if (o->pu_gemm) {
+        // L21 = A21 L_kk^-T as a DGEMM with the explicit inverse (tensor cores),
+        // written to scratch and copied back
+        if (dtype == ABFT_F64) {
+          const double one = 1.0, zero = 0.0;
+          if (cublasDgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)nk, (int)nb, (int)nb, &one, (const double*)d.a_at(r1, k * nb),
+                          (int)lda, (const double*)c->linv, (int)nb, &zero, (double*)c->putmp, (int)nk) !=
+              CUBLAS_STATUS_SUCCESS)
+            return ABFT_E_CUBLAS;
+        } else {
+          const float one = 1.0f, zero = 0.0f;
+          if (cublasSgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)nk, (int)nb, (int)nb, &one, (const float*)d.a_at(r1, k * nb),
+                          (int)lda, (const float*)c->linv, (int)nb, &zero, (float*)c->putmp, (int)nk) !=
+              CUBLAS_STATUS_SUCCESS)
+            return ABFT_E_CUBLAS;
+        }
+        lk.unlock();
+        ABFT_CUDA_TRY(cudaMemcpy2DAsync(d.a_at(r1, k * nb), lda * d.es, c->putmp, nk * d.es, nk * d.es, nb,
+                                        cudaMemcpyDeviceToDevice, s));
+      } else if (dtype == ABFT_F64) {
         const double one = 1.0;
         if (cublasDtrsm(h, CUBLAS_SIDE_RIGHT, CUBLAS_FILL_MODE_LOWER, CUBLAS_OP_T, CUBLAS_DIAG_NON_UNIT, (int)nk,
                         (int)nb, &one, (const double*)d.a_at(k * nb, k * nb), (int)lda, (double*)d.a_at(r1, k * nb),
@@ -382,12 +443,13 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
                         (int)lda) != CUBLAS_STATUS_SUCCESS)
           return ABFT_E_CUBLAS;
       }
-      lk.unlock();
+      if (lk.owns_lock()) lk.unlock();
     }
     FT_TRY(d.restore_onchip());  // on-chip flips hit the data step only (c-8)
-    if (ft)
-      FT_TRY(abft_update_trsm(dtype, 'R', 'L', 'T', 'N', nb, d.a_at(k * nb, k * nb), lda, d.colchk_at(2 * (k + 1), k * nb),
-                              d.M.ldc, m2, d.colmag_at(k + 1, k * nb), d.M.ldcm, m2 / 2, as));
+    if (refresh_inv) FT_TRY(abft_tri_inverse(dtype, 'L', 'N', nb, d.a_at(k * nb, k * nb), lda, c->linv, nb, as));
+    if (ft)  // c(L_ik) = c(A_ik) L_kk^-T, m_c <- m_c |L_kk^-T| with the PD's inverse (c-12, c-6)
+      FT_TRY(abft_update_trsm_inv(dtype, 'R', 'T', nb, c->linv, nb, d.colchk_at(2 * (k + 1), k * nb), d.M.ldc, m2,
+                                  d.colmag_at(k + 1, k * nb), d.M.ldcm, m2 / 2, as));
     FT_TRY(d.inject_at(k, FT_AT_POST_PU));
     // line 10: check the updated panel (c only; 1D_ROW fixable, 2D -> restart, L434)
     if (ft) FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
@@ -410,14 +472,11 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     }
     FT_TRY(d.restore_onchip());  // on-chip flips hit the data step only (c-8)
     if (ft) {
-      // c(A_ij) -= c(L_ik) L_jk^T
-      FT_TRY(abft_update_gemm(dtype, ABFT_COL, 'N', 'T', -1.0, d.colchk_at(2 * (k + 1), k * nb), d.M.ldc,
-                              d.a_at(r1, k * nb), lda, d.colchk_at(2 * (k + 1), r1), d.M.ldc, m2, nk, nb,
-                              d.colmag_at(k + 1, k * nb), d.M.ldcm, d.colmag_at(k + 1, r1), d.M.ldcm, as));
-      // r(A_ij) -= L_ik c(L_jk)^T  (transposed column checksum of the panel, L189)
-      FT_TRY(abft_update_gemm(dtype, ABFT_ROW, 'T', 'N', -1.0, d.colchk_at(2 * (k + 1), k * nb), d.M.ldc,
-                              d.a_at(r1, k * nb), lda, d.rowchk_at(r1, 2 * (k + 1)), d.M.ldr, m2, nk, nb,
-                              d.colmag_at(k + 1, k * nb), d.M.ldcm, d.rowmag_at(r1, k + 1), d.M.ldrm, as));
+      // c(A_ij) -= c(L_ik) L_jk^T and r(A_ij) -= L_ik c(L_jk)^T from one product (c-12, L189)
+      FT_TRY(abft_update_syrk(dtype, nb, nt - k - 1, d.a_at(r1, k * nb), lda, d.colchk_at(2 * (k + 1), k * nb), d.M.ldc,
+                              d.colmag_at(k + 1, k * nb), d.M.ldcm, d.colchk_at(2 * (k + 1), r1),
+                              d.rowchk_at(r1, 2 * (k + 1)), d.M.ldr, d.colmag_at(k + 1, r1), d.rowmag_at(r1, k + 1),
+                              d.M.ldrm, as));
     }
     FT_TRY(d.inject_at(k, FT_AT_POST_TMU));
     // line 13: heuristic panel re-check for the TMU (Fig. 4a) + guarded repair (c-25)

@@ -124,3 +124,86 @@ def test_checksum_memory_fault_repaired():
     A, Lref, L, stats = _run(256, 32, inj)
     assert stats.uncorrectable == 0 and stats.counts[6] >= 1
     assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
+
+
+# ------------------------------------------------------------------- LU ----
+import scipy.linalg as sla  # noqa: E402
+
+
+def _lu_invariant(st, k, phase):
+    nt = st.nt
+    tol = ck.Tol()
+    if phase == "pd":
+        for I in range(k, nt):
+            tc = ck.check_tile(st, I, k, ck.UNIT_LOWER if I == k else ck.GENERAL, ck.COL, tol)
+            assert not tc.Fc, (k, phase, I)
+        tc = ck.check_tile(st, k, k, ck.UPPER, ck.ROW, tol)
+        assert not tc.Fr
+        # trailing and left-panel checksums after the pivot swaps (c-14)
+        for I, J in ck.Tiles(k + 1, nt, k + 1, nt):
+            tc = ck.check_tile(st, I, J, ck.GENERAL, ck.BOTH, tol)
+            assert not tc.Fc and not tc.Fr, (k, "swap", I, J)
+        for I, J in ck.Tiles(0, nt, 0, k):
+            if I >= J:
+                tc = ck.check_tile(st, I, J, ck.UNIT_LOWER if I == J else ck.GENERAL, ck.COL, tol)
+                assert not tc.Fc, (k, "swap-left", I, J)
+    elif phase == "pu":
+        for J in range(k + 1, nt):
+            tc = ck.check_tile(st, k, J, ck.GENERAL, ck.ROW, tol)
+            assert not tc.Fr, (k, phase, J)
+    else:
+        for I, J in ck.Tiles(k + 1, nt, k + 1, nt):
+            tc = ck.check_tile(st, I, J, ck.GENERAL, ck.BOTH, tol)
+            assert not tc.Fc and not tc.Fr, (k, phase, I, J)
+
+
+@pytest.mark.parametrize("n,nb", [(256, 32), (512, 64), (384, 128)])
+def test_ft_getrf_error_free_matches_lapack(n, nb):
+    A = si.general(n, seed=n + nb)
+    LU, piv, stats = dr.ft_getrf(A, nb, invariant_hook=_lu_invariant)
+    lu, p = sla.lu_factor(A)
+    assert np.array_equal(piv, p)
+    assert np.abs(LU - lu).max() <= 1e-12 * np.abs(lu).max()
+    assert stats.counts == [0] * 8
+
+
+LU_FIXABLE = [
+    (dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 100, 70, (61,)),   # DRAM in the column panel before PD
+    (dr.AT_POST_PD, dr.KIND_PERSIST, 150, 80, (62,)),        # computation error in L21
+    (dr.AT_POST_PD, dr.KIND_PERSIST, 66, 90, (58,)),         # computation error in U_kk
+    (dr.AT_PRE_PU_CHECK, dr.KIND_PERSIST, 70, 200, (60,)),   # DRAM in the row panel
+    (dr.AT_POST_PU, dr.KIND_PERSIST, 75, 180, (63,)),        # computation error in U12
+    (dr.AT_PRE_PU, dr.KIND_ONCHIP, 72, 130, (57,)),          # on-chip in PU update part -> 1D_COL
+    (dr.AT_PRE_TMU, dr.KIND_ONCHIP, 140, 72, (57,)),         # on-chip in L21 during TMU -> 1D_ROW
+    (dr.AT_PRE_TMU, dr.KIND_ONCHIP, 70, 140, (56,)),         # on-chip in U12 during TMU -> 1D_COL
+    (dr.AT_PRE_TMU, dr.KIND_PERSIST, 170, 80, (54,)),        # DRAM in L21 -> Fig. 4a
+    (dr.AT_PRE_TMU, dr.KIND_PERSIST, 80, 170, (55,)),        # DRAM in U12 -> Fig. 4a
+    (dr.AT_POST_TMU, dr.KIND_PERSIST, 230, 100, (59,)),      # trailing computation error
+]
+
+
+@pytest.mark.parametrize("case", range(len(LU_FIXABLE)))
+def test_lu_fault_campaign_fixed(case):
+    point, kind, gi, gj, bits = LU_FIXABLE[case]
+    A = si.general(256, seed=0)
+    lu, p = sla.lu_factor(A)
+    LU, piv, stats = dr.ft_getrf(A, 32, inject=[dr.Inject(2, point, kind, 0, gi, gj, bits)])
+    assert stats.uncorrectable == 0, stats.counts
+    assert stats.counts[0] >= 1
+    assert np.array_equal(piv, p)
+    assert np.abs(LU - lu).max() <= 1e-12 * np.abs(lu).max()
+
+
+def test_lu_trailing_fault_in_a_pivot_row_fixed_before_the_swap():
+    """A DRAM fault in a trailing row that the next panel's pivoting moves
+    (row 70 = k·nb + 6 at k=2 is swapped unless it is its own pivot): the
+    pre-swap row check (c-14b) must fix it before the swap deltas use it."""
+    A = si.general(256, seed=0)
+    lu, p = sla.lu_factor(A)
+    assert p[70] != 70
+    inj = [dr.Inject(1, dr.AT_POST_TMU, dr.KIND_PERSIST, 0, 70, 200, (60,))]
+    LU, piv, stats = dr.ft_getrf(A, 32, inject=inj)
+    assert stats.uncorrectable == 0 and stats.counts[5] >= 1
+    assert any(c[1] == "pre_swap_rows" for c in stats.checks)
+    assert np.array_equal(piv, p)
+    assert np.abs(LU - lu).max() <= 1e-12 * np.abs(lu).max()
