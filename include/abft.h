@@ -234,6 +234,25 @@ ABFT_API int abft_update_gemm(int32_t dtype, int32_t which, char transX, char tr
 ABFT_API int abft_panel_potrf(const abft_mat_t *diag, void *Linv, int64_t ldw, int32_t *info,
                               abft_stream_t stream);
 
+/* a4 — abft_panel_getrf (PD of LU with partial pivoting for iteration k of
+ * the square matrix `mat`; [13] via L135-L145, c-13, c-14).  In order:
+ * cuSOLVER dgetrf of the column panel A[k*nb:, k*nb:(k+1)*nb] (pivots to
+ * ipiv[0..nb), 1-based global, LAPACK convention); when mat carries
+ * checksums: the pre-swap row check (c-14b) of every trailing row the pivots
+ * move (row checksums of tile columns > k; flagged tiles are classified and
+ * corrected by abft_locate_correct with `tol`, `rep`, `fixes`); the row swaps
+ * of all columns outside the panel (LAPACK laswp) with the column-checksum
+ * deltas of c-14 (panel columns from the pre-PD copy, L430), row checksums
+ * and magnitudes moved with their rows; then L_kk^-1 -> Linv, U_kk^-1 -> Uinv
+ * (nb x nb, ld nb, device) and c(L_I) = c(P~_I) U_kk^-1 (I >= k),
+ * r(U_kk) = L_kk^-1 r(P~_kk), magnitudes by the absolute inverses (c-6).
+ * mat->colchk == NULL gives the plain PD (getrf + swaps + inverses).
+ * LAPACK info (U(i,i) == 0) goes to *info (device int32). */
+ABFT_API int abft_panel_getrf(const abft_mat_t *mat, int32_t k, int64_t *ipiv, const abft_tol_t *tol,
+                              const abft_report_t *rep, abft_fix_t *fixes, int32_t max_fixes,
+                              int32_t *n_fixes, void *Linv, void *Uinv, int32_t *info,
+                              abft_stream_t stream);
+
 /* W = T^-1 for an nb x nb triangular T (uplo 'L'/'U', diag 'N'/'U'); the
  * other triangle of W is written as zero.  Helper of the a5 rule (the
  * magnitude propagation needs |T^-1| explicitly, c-6). */
@@ -319,6 +338,19 @@ ABFT_API int ft_ctx_destroy(ft_ctx_t *ctx);
  * DESIGN.md §8).  *info (host) follows LAPACK potrf. */
 ABFT_API int ft_potrf(ft_ctx_t *ctx, int32_t dtype, int64_t n, void *dA, int64_t lda,
              const ft_opts_t *opts, ft_stats_t *stats, int64_t *info);
+
+/* ft_getrf — fault-tolerant LU with partial pivoting, PA = LU, of the square
+ * n x n matrix dA (device, lda >= n, n % nb == 0), right-looking blocked,
+ * full checksums on the trailing matrix ([13], L135-L145), Alg. 2 order per
+ * iteration k: check the column panel (c+r) -> abft_panel_getrf (pre-swap row
+ * check, swaps, c(L), r(U_kk)) -> check L (UNIT_LOWER, c) and U_kk (UPPER, r)
+ * -> check the row panel (c+r) -> PU U12 = L_kk^-1 A12 + r(U12) -> check U12
+ * (r) -> TMU DGEMM + c/r rules -> re-check both panels (Fig. 4a) with the
+ * guarded repair (c-25).  ipiv: device int64[n], 1-based global pivots.
+ * Returns ABFT_E_UNCORRECTABLE if a 2D error remained.  *info (host) follows
+ * LAPACK getrf. */
+ABFT_API int ft_getrf(ft_ctx_t *ctx, int32_t dtype, int64_t n, void *dA, int64_t lda, int64_t *ipiv,
+                      const ft_opts_t *opts, ft_stats_t *stats, int64_t *info);
 
 #ifdef __cplusplus
 }

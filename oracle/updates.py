@@ -311,3 +311,137 @@ def lu_fig4a_repair(st: State, k: int, gi: int, gj: int, before: float, after: f
                 st.colmag[I, c] += abs(E) * st.colmag[I, r0 + q]
         return "applied"
     return None
+
+
+# ------------------------------------------------------------------- QR ----
+def _panel_weights(nb, nt_rows):
+    """W (2·nt_rows × nt_rows·nb): rows 2I / 2I+1 hold v1 / v2 of tile row I
+    of the panel (tile-local, 1-based; L108)."""
+    W = np.zeros((2 * nt_rows, nt_rows * nb))
+    v1, v2 = np.ones(nb), np.arange(1, nb + 1, dtype=np.float64)
+    for I in range(nt_rows):
+        W[2 * I, I * nb:(I + 1) * nb] = v1
+        W[2 * I + 1, I * nb:(I + 1) * nb] = v2
+    return W
+
+
+def qr_pd_alg1(st: State, k: int):
+    """Algorithm 1 (L228–L235, reconstruction c-15) with LAPACK's dlarfg
+    conventions (v(1) = 1, tau, beta = −sign(x1)·||x||; tau = 0 when x(2:) = 0):
+    Householder QR of the column panel P = A[k·nb:, k·nb:(k+1)·nb] extended
+    by its column checksums ck (per tile [v1 v2]^T P, the 'checksum row') and
+    its row checksums rck (P [v1 v2], the 'checksum column').  For j = 0..nb−1:
+      x = P[j:, j];  c_x = ck[:, j] − W[:, :j] P[:j, j]   (checksum of x from
+                                       the trusted checksum minus finished rows)
+      beta, tau, v = dlarfg(x);  v_ck = (c_x − beta·W[:, j]) / (x1 − beta)
+      y = v^T P[j:, j+1:];  P[j:, j+1:] −= tau v y;  ck[:, j+1:] −= tau v_ck y
+      rck[j:] −= tau v (v^T rck[j:])
+      store beta, v(2:) in P[:, j] and v_ck in ck[:, j]  (= c(V) in UNIT_LOWER view)
+    Magnitudes (c-6): m_x = mck[:, j]; m_v = (m_x + |beta|·[row j in tile]) / |x1 − beta|;
+    mck[:, j+1:] += |tau| m_v |y|;  mr[j:] += |tau| |v| (|v|^T mr[j:]).
+    At the end rck = Q^T P [v1 v2] = [r(R); 0].  Returns tau (nb)."""
+    nb, n = st.nb, st.A.shape[0]
+    nt = n // nb
+    r0, r1 = k * nb, (k + 1) * nb
+    m = n - r0
+    P = st.A[r0:n, r0:r1].copy()
+    W = _panel_weights(nb, nt - k)
+    ck = st.colchk[2 * k:, r0:r1].copy()
+    rck = st.rowchk[r0:n, 2 * k:2 * k + 2].copy()
+    mags = st.colmag is not None
+    if mags:
+        mck = st.colmag[k:, r0:r1].copy()
+        mr = st.rowmag[r0:n, k].copy()
+    tau = np.zeros(nb)
+    for j in range(nb):
+        x = P[j:, j].copy()
+        c_x = ck[:, j] - W[:, :j] @ P[:j, j]
+        alpha = x[0]
+        xnorm = float(np.linalg.norm(x[1:]))
+        e_row = (W[:, j] != 0).astype(np.float64)[0::2]  # tiles holding row j
+        if xnorm == 0.0:
+            t, beta = 0.0, alpha
+            v = np.zeros_like(x)
+            v[0] = 1.0
+            v_ck = W[:, j].copy()
+            if mags:
+                m_v = e_row.copy()
+        else:
+            beta = -np.copysign(np.hypot(alpha, xnorm), alpha)
+            t = (beta - alpha) / beta
+            v = x / (alpha - beta)
+            v[0] = 1.0
+            v_ck = (c_x - beta * W[:, j]) / (alpha - beta)
+            if mags:
+                m_v = (mck[:, j] + abs(beta) * e_row) / abs(alpha - beta)
+        tau[j] = t
+        if j + 1 < nb:
+            y = v @ P[j:, j + 1:]
+            P[j:, j + 1:] -= t * np.outer(v, y)
+            ck[:, j + 1:] -= t * np.outer(v_ck, y)
+            if mags:
+                mck[:, j + 1:] += abs(t) * np.outer(m_v, np.abs(y))
+        yr = v @ rck[j:]
+        rck[j:] -= t * np.outer(v, yr)
+        if mags:
+            mr[j:] += abs(t) * np.abs(v) * float(np.abs(v) @ mr[j:])
+        P[j, j] = beta
+        P[j + 1:, j] = v[1:]
+        ck[:, j] = v_ck
+        if mags:
+            mck[:, j] = m_v
+    st.A[r0:n, r0:r1] = P
+    st.colchk[2 * k:, r0:r1] = ck
+    st.rowchk[r0:n, 2 * k:2 * k + 2] = rck
+    if mags:
+        st.colmag[k:, r0:r1] = mck
+        st.rowmag[r0:n, k] = mr
+    return tau
+
+
+def qr_V(st: State, k: int):
+    """V (unit lower trapezoidal) of panel k as stored by dgeqrf."""
+    nb, n = st.nb, st.A.shape[0]
+    r0, r1 = k * nb, (k + 1) * nb
+    V = np.tril(st.A[r0:n, r0:r1], -1)
+    V[:nb, :nb] += np.eye(nb)
+    return V
+
+
+def qr_T(V, tau):
+    """CTF (the paper's 'computing triangular factor', L238; LAPACK dlarft,
+    forward, columnwise): T[j,j] = tau_j, T[:j, j] = −tau_j T[:j,:j] V[:, :j]^T v_j."""
+    nb = V.shape[1]
+    T = np.zeros((nb, nb))
+    for j in range(nb):
+        T[j, j] = tau[j]
+        if j:
+            T[:j, j] = -tau[j] * (T[:j, :j] @ (V[:, :j].T @ V[:, j]))
+    return T
+
+
+def qr_tmu_data(st: State, k: int, V, T):
+    """QR TMU data step (Table III): A2 ← (I − V T V^T)^T A2 = A2 − V (T^T V^T A2)
+    for A2 = A[k·nb:, (k+1)·nb:] (its first nb rows become R12)."""
+    nb, n = st.nb, st.A.shape[0]
+    r0, r1 = k * nb, (k + 1) * nb
+    A2 = st.A[r0:n, r1:n]
+    Wm = T.T @ (V.T @ A2)
+    st.A[r0:n, r1:n] = A2 - V @ Wm
+    return Wm
+
+
+def qr_tmu_chk(st: State, k: int, V, T, Wm):
+    """QR TMU checksum step (Table III, red symbols; c-15): with W = T^T V^T A2,
+    c(A2) −= c(V)·W and r(A2) −= V·(T^T V^T r(A2)); magnitudes
+    m_c += m_c(V)|W|, m_r += |V| (|T|^T (|V|^T m_r)) (c-6)."""
+    nb, n = st.nb, st.A.shape[0]
+    r0, r1 = k * nb, (k + 1) * nb
+    cV = st.colchk[2 * k:, r0:r1]
+    st.colchk[2 * k:, r1:n] -= cV @ Wm
+    rA = st.rowchk[r0:n, 2 * (k + 1):]
+    st.rowchk[r0:n, 2 * (k + 1):] = rA - V @ (T.T @ (V.T @ rA))
+    if st.colmag is not None:
+        st.colmag[k:, r1:n] += st.colmag[k:, r0:r1] @ np.abs(Wm)
+        mr = st.rowmag[r0:n, k + 1:]
+        st.rowmag[r0:n, k + 1:] = mr + np.abs(V) @ (np.abs(T).T @ (np.abs(V).T @ mr))

@@ -103,6 +103,9 @@ _sig = {
     "abft_tri_inverse": [_i32, _ch, _ch, _i64, _vp, _i64, _vp, _i64, _vp],
     "abft_update_trsm_inv": [_i32, _ch, _ch, _i64, _vp, _i64, _vp, _i64, _i64, _vp, _i64, _i64, _vp],
     "abft_update_syrk": [_i32, _i64, _i64, _vp, _i64, _vp, _i64, _vp, _i64, _vp, _vp, _i64, _vp, _vp, _i64, _vp],
+    "abft_panel_getrf": [_P(abft_mat_t), _i32, _vp, _P(abft_tol_t), _P(abft_report_t), _vp, _i32, _vp, _vp, _vp,
+                         _vp, _vp],
+    "ft_getrf": [_vp, _i32, _i64, _vp, _i64, _vp, _P(ft_opts_t), _P(ft_stats_t), _P(_i64)],
     "ft_ctx_create": [_P(_vp), _i32, _vp],
     "ft_ctx_destroy": [_vp],
     "ft_potrf": [_vp, _i32, _i64, _vp, _i64, _P(ft_opts_t), _P(ft_stats_t), _P(_i64)],
@@ -331,6 +334,40 @@ class Context:
         if h is not None and h.value and _L is not None:
             _L.ft_ctx_destroy(h)
             self._h = None
+
+
+def _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm):
+    inj = (ft_inject_t * max(1, len(inject)))()
+    for k, f in enumerate(inject):
+        inj[k] = ft_inject_t(*f)
+    opts = ft_opts_t(nb, int(abft), tol_kind, tol_scale, int(fig4a_repair), len(inject), inj,
+                     _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES, int(pu_gemm))
+    return opts, inj
+
+
+def abft_panel_getrf(mat: Mat, k: int, ipiv: torch.Tensor, Linv: torch.Tensor, Uinv: torch.Tensor,
+                     info: torch.Tensor, tol: abft_tol_t = None, rep: Report = None, fixes: torch.Tensor = None,
+                     n_fixes: torch.Tensor = None, stream=None):
+    m = mat.c()
+    r = rep.c() if rep is not None else None
+    cap = 0 if fixes is None else fixes.numel() // FIX_BYTES
+    return _check("abft_panel_getrf", _L.abft_panel_getrf(
+        C.byref(m), k, _ptr(ipiv), C.byref(tol) if tol is not None else None, C.byref(r) if r is not None else None,
+        _ptr(fixes), cap, _ptr(n_fixes), _ptr(Linv), _ptr(Uinv), _ptr(info), _stream(stream)))
+
+
+def ft_getrf(ctx: Context, A: torch.Tensor, nb: int, ipiv: torch.Tensor, abft=True, tol_kind=TOL_MAGNITUDE,
+             tol_scale=1.0, fig4a_repair=True, inject=(), fix_log=None):
+    """Fault-tolerant LU with partial pivoting in place on a column-major A;
+    ipiv: int64 device tensor (n), receives 1-based global pivots."""
+    n = A.shape[0]
+    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, True)
+    stats = ft_stats_t()
+    info = C.c_int64()
+    rc = _L.ft_getrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), _ptr(ipiv), C.byref(opts), C.byref(stats),
+                     C.byref(info))
+    _check("ft_getrf", rc, ok=(0, E_UNCORRECTABLE))
+    return rc, info.value, stats
 
 
 def ft_potrf(ctx: Context, A: torch.Tensor, nb: int, abft=True, tol_kind=TOL_MAGNITUDE, tol_scale=1.0,

@@ -1,0 +1,226 @@
+// Shared plumbing of the fault-tolerant drivers (ft_potrf, ft_getrf):
+// context buffers, the checksum state of the matrix, Alg. 2 check helper,
+// fault-injection hooks (reading c-8) and the final statistics read-back.
+#pragma once
+#include <cublas_v2.h>
+#include <cusolverDn.h>
+
+#include <algorithm>
+#include <chrono>
+#include <mutex>
+#include <vector>
+
+#include "abft_common.cuh"
+
+namespace abft {
+cublasHandle_t blas_handle(cudaStream_t s, std::unique_lock<std::mutex>& lk);
+cusolverDnHandle_t solver_handle(cudaStream_t s, std::unique_lock<std::mutex>& lk);
+int scratch(cudaStream_t s, int slot, size_t bytes, void** out);
+}  // namespace abft
+
+#define FT_TRY(expr)     \
+  do {                   \
+    int _rc = (expr);    \
+    if (_rc) return _rc; \
+  } while (0)
+
+struct ft_ctx {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  void* state = nullptr;  // colchk | rowchk | colmag | rowmag
+  size_t state_bytes = 0;
+  int32_t* ints = nullptr;  // status | counts[8] | n_fixes | mark | info | rep[2] | info_total | spare
+  size_t ints_n = 0;
+  abft_fix_t* fixlog = nullptr;
+  int fixcap = 0;
+  void* linv = nullptr;  // nb x nb inverse of the current L_kk
+  size_t linv_bytes = 0;
+  void* uinv = nullptr;  // nb x nb inverse of the current U_kk (LU)
+  size_t uinv_bytes = 0;
+  void* putmp = nullptr;  // n x nb panel scratch (GEMM-based PU, LU panel copy)
+  size_t putmp_bytes = 0;
+  void* aux = nullptr;  // driver-specific device scratch (LU pivots / swap rows)
+  size_t aux_bytes = 0;
+};
+
+namespace abft {
+
+inline int grow_buffer(void*& p, size_t& have, size_t need) {
+  if (have >= need) return 0;
+  if (p) cudaFree(p);
+  p = nullptr;
+  have = 0;
+  if (cudaMalloc(&p, need) != cudaSuccess) return ABFT_E_NOMEM;
+  have = need;
+  return 0;
+}
+
+// LAPACK info of the whole factorization: first failing panel's local value
+// offset by the panel origin.
+static __global__ void accum_info_kernel(int32_t* tile_info, int32_t* total, int64_t offset) {
+  if (*tile_info != 0 && *total == 0) *total = (int32_t)(*tile_info + offset);
+  *tile_info = 0;
+}
+
+struct Driver {
+  ft_ctx* c = nullptr;
+  cudaStream_t s = nullptr;
+  int32_t dtype = ABFT_F64;
+  int64_t n = 0, nb = 0, nt = 0, lda = 0;
+  size_t es = 8;
+  void* A = nullptr;
+  const ft_opts_t* o = nullptr;
+  bool lu = false;
+  abft_mat_t M{};
+  abft_report_t R{};
+  abft_tol_t tol{};
+  int32_t *status = nullptr, *counts = nullptr, *nfix = nullptr, *mark = nullptr, *info = nullptr, *rep = nullptr,
+          *info_total = nullptr;
+  std::vector<ft_inject_t> onchip_pending;
+  int n_checks = 0;
+
+  int setup(ft_ctx* ctx, int32_t dt, int64_t n_, int64_t nb_, void* dA, int64_t lda_, const ft_opts_t* opts,
+            bool is_lu) {
+    c = ctx;
+    s = ctx->stream;
+    dtype = dt;
+    n = n_;
+    nb = nb_;
+    nt = n_ / nb_;
+    lda = lda_;
+    es = dt == ABFT_F64 ? 8 : 4;
+    A = dA;
+    o = opts;
+    lu = is_lu;
+    const bool ft = o->abft != 0;
+    size_t need = ft ? (size_t)(2 * nt * n + n * 2 * nt + nt * n + n * nt) * es : 0;
+    FT_TRY(grow_buffer(c->state, c->state_bytes, need));
+    size_t ints_need = (size_t)nt * nt + 8 + 8;
+    void* ip = c->ints;
+    FT_TRY(grow_buffer(ip, c->ints_n, ints_need * sizeof(int32_t)));
+    c->ints = reinterpret_cast<int32_t*>(ip);
+    FT_TRY(grow_buffer(c->linv, c->linv_bytes, (size_t)nb * nb * es));
+    if (lu) FT_TRY(grow_buffer(c->uinv, c->uinv_bytes, (size_t)nb * nb * es));
+    if (o->pu_gemm || lu) FT_TRY(grow_buffer(c->putmp, c->putmp_bytes, (size_t)n * nb * es));
+    status = c->ints;
+    counts = status + nt * nt;
+    nfix = counts + 8;
+    mark = nfix + 1;
+    info = mark + 1;
+    rep = info + 1;
+    info_total = rep + 2;
+    ABFT_CUDA_TRY(cudaMemsetAsync(c->ints, 0, ints_need * sizeof(int32_t), s));
+    char* st = (char*)c->state;
+    M.dtype = dtype;
+    M.m = n;
+    M.n = n;
+    M.nb = nb;
+    M.A = dA;
+    M.lda = lda;
+    if (ft) {
+      M.colchk = st;
+      M.ldc = 2 * nt;
+      st += 2 * nt * n * es;
+      M.rowchk = st;
+      M.ldr = n;
+      st += n * 2 * nt * es;
+      M.colmag = st;
+      M.ldcm = nt;
+      st += nt * n * es;
+      M.rowmag = st;
+      M.ldrm = n;
+    }
+    R.status = status;
+    R.ld_status = nt;
+    R.counts = counts;
+    tol.kind = o->tol_kind;
+    tol.scale = o->tol_scale > 0 ? o->tol_scale : 1.0;
+    return 0;
+  }
+
+  char* elem(int target, int64_t gi, int64_t gj) {
+    if (target == 1) return (char*)M.colchk + (gi + gj * M.ldc) * es;
+    if (target == 2) return (char*)M.rowchk + (gi + gj * M.ldr) * es;
+    return (char*)A + (gi + gj * lda) * es;
+  }
+  // Elements the op after `point` overwrites: an on-chip flip there cannot be
+  // changed back, so it stays (reading c-8).
+  bool in_update_region(int point, int k, int64_t gi, int64_t gj) const {
+    const int64_t r0 = k * nb, r1 = (k + 1) * nb;
+    if (!lu) {
+      if (point == FT_AT_PRE_PD) return gi >= r0 && gi < r1 && gj >= r0 && gj < r1;
+      if (point == FT_AT_PRE_PU) return gi >= r1 && gj >= r0 && gj < r1;
+    } else {
+      if (point == FT_AT_PRE_PD) return gi >= r0 && gj >= r0 && gj < r1;
+      if (point == FT_AT_PRE_PU) return gi >= r0 && gi < r1 && gj >= r1;
+    }
+    if (point == FT_AT_PRE_TMU) return gi >= r1 && gj >= r1;
+    return false;
+  }
+  int inject_at(int k, int point) {
+    for (int t = 0; t < o->n_inject; ++t) {
+      const ft_inject_t& f = o->inject[t];
+      if (f.iter != k || f.point != point) continue;
+      FT_TRY(abft_inject(elem(f.target, f.gi, f.gj), dtype, 0, f.xor_mask, (abft_stream_t)s));
+      bool op_point = point == FT_AT_PRE_PD || point == FT_AT_PRE_PU || point == FT_AT_PRE_TMU;
+      if (f.kind == FT_KIND_ONCHIP && op_point && f.target == 0 && !in_update_region(point, k, f.gi, f.gj))
+        onchip_pending.push_back(f);
+    }
+    return 0;
+  }
+  // Fault-injection runs only: does the plan touch the diagonal tile between
+  // the PD (which produced the inverse the GEMM-based PU reads) and the PU?
+  // Then the PU must see the flipped tile, as an in-place TRSM would (c-8).
+  bool diag_touched_before_pu(int k) const {
+    for (int t = 0; t < o->n_inject; ++t) {
+      const ft_inject_t& f = o->inject[t];
+      if (f.iter != k || f.target != 0) continue;
+      if (f.point != FT_AT_PRE_PU_CHECK && f.point != FT_AT_PRE_PU) continue;
+      if (f.gi >= k * nb && f.gi < (k + 1) * nb && f.gj >= k * nb && f.gj < (k + 1) * nb) return true;
+    }
+    return false;
+  }
+  int restore_onchip() {  // after the op's data step: undo on-chip flips (the stored value was never wrong)
+    for (auto& f : onchip_pending)
+      FT_TRY(abft_inject(elem(f.target, f.gi, f.gj), dtype, 0, f.xor_mask, (abft_stream_t)s));
+    onchip_pending.clear();
+    return 0;
+  }
+  int check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only = false) {
+    abft_tiles_t t{I0, I1, J0, J1, lower_only ? 1 : 0, view};
+    FT_TRY(abft_verify(&M, &t, which, &tol, &R, (abft_stream_t)s));
+    FT_TRY(abft_locate_correct(&M, &t, which, &tol, &R, c->fixlog, c->fixcap, nfix, (abft_stream_t)s));
+    ++n_checks;
+    return 0;
+  }
+  void* colchk_at(int64_t r, int64_t col) { return (char*)M.colchk + (r + col * M.ldc) * es; }
+  void* colmag_at(int64_t r, int64_t col) { return (char*)M.colmag + (r + col * M.ldcm) * es; }
+  void* rowchk_at(int64_t r, int64_t col) { return (char*)M.rowchk + (r + col * M.ldr) * es; }
+  void* rowmag_at(int64_t r, int64_t col) { return (char*)M.rowmag + (r + col * M.ldrm) * es; }
+  void* a_at(int64_t r, int64_t col) { return (char*)A + (r + col * lda) * es; }
+
+  // The single host synchronisation: counters, info and the fix log.
+  int finish(std::chrono::steady_clock::time_point t0, ft_stats_t* stats, int64_t* info_out) {
+    int32_t h[8 + 8];
+    ABFT_CUDA_TRY(cudaMemcpyAsync(h, counts, sizeof(h), cudaMemcpyDeviceToHost, s));
+    if (o->fix_log && o->fix_log_cap > 0)
+      ABFT_CUDA_TRY(cudaMemcpyAsync(o->fix_log, c->fixlog, sizeof(abft_fix_t) * std::min(o->fix_log_cap, c->fixcap),
+                                    cudaMemcpyDeviceToDevice, s));
+    ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+    auto t1 = std::chrono::steady_clock::now();
+    // layout after counts: nfix(8) mark(9) info(10) rep(11,12) info_total(13)
+    if (info_out) *info_out = h[13];
+    if (stats) {
+      for (int i = 0; i < 8; ++i) stats->counts[i] = h[i];
+      stats->n_fixes = h[8];
+      stats->repairs_applied = h[11];
+      stats->repairs_skipped = h[12];
+      stats->uncorrectable = h[ABFT_CNT_UNCORRECTABLE];
+      stats->n_checks = n_checks;
+      stats->ms_total = std::chrono::duration<double, std::milli>(t1 - t0).count();
+    }
+    return h[ABFT_CNT_UNCORRECTABLE] ? ABFT_E_UNCORRECTABLE : 0;
+  }
+};
+
+}  // namespace abft

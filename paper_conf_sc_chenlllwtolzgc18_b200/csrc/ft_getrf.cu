@@ -1,0 +1,484 @@
+// ft_getrf.cu — LU with partial pivoting: PD checksum rules with pivot swaps
+// (a4), left TRSM rule (a5), LU TMU rule (a6) and the fault-tolerant driver in
+// Alg. 2 order (a7).
+//
+// Paper: full-checksum LU of [13] (L135-L145, §III.C): full checksums on the
+// trailing matrix, c on the column panel, r on the row panel; Alg. 2
+// (L364-L379); heuristic TMU check Fig. 4a (L359).  Readings: c-13 (LU rules),
+// c-14 (pivot swap deltas from the pre-PD panel copy, L430), c-14b (pre-swap
+// row check of every trailing row a swap moves), c-25 (Fig. 4a repair).
+#include "ft_driver.cuh"
+
+namespace abft {
+
+// 1-based local pivots of the panel (cuSOLVER) -> 1-based global (LAPACK).
+__global__ void lu_pivots_kernel(const int32_t* piv_local, int64_t* ipiv_global, int nb, int64_t r0) {
+  for (int j = threadIdx.x; j < nb; j += blockDim.x) ipiv_global[j] = r0 + piv_local[j];
+}
+
+// Distinct rows moved by the panel's swaps (c-14b), compacted into rows[],
+// count in *nrows.  One CTA of 1024 threads.
+__global__ void lu_swap_rows_kernel(const int32_t* piv_local, int nb, int64_t r0, int64_t* rows, int32_t* nrows) {
+  __shared__ int64_t cand[2048];
+  __shared__ int cnt;
+  if (threadIdx.x == 0) cnt = 0;
+  for (int s = threadIdx.x; s < 2 * nb; s += blockDim.x) {
+    const int j = s < nb ? s : s - nb;
+    const int64_t p = r0 + j, q = r0 + piv_local[j] - 1;
+    cand[s] = (p == q) ? -1 : (s < nb ? p : q);
+  }
+  __syncthreads();
+  for (int s = threadIdx.x; s < 2 * nb; s += blockDim.x) {
+    const int64_t r = cand[s];
+    if (r < 0) continue;
+    bool first = true;
+    for (int t = 0; t < s && first; ++t)
+      if (cand[t] == r) first = false;
+    if (first) rows[atomicAdd(&cnt, 1)] = r;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) *nrows = cnt;
+}
+
+// Pre-swap row check: row r of every trailing tile (I = r/nb, J > k) against
+// its row checksums; a flagged tile gets ST_ROW so locate_correct treats it.
+template <typename T>
+__global__ void lu_row_check_kernel(const T* A, int64_t lda, const T* rowchk, int64_t ldr, const T* rowmag,
+                                    int64_t ldrm, int use_mag, double tau_fac, int nb, int k, int nt,
+                                    const int64_t* rows, const int32_t* nrows, int32_t* status, int64_t ld_status,
+                                    int32_t* counts) {
+  const int lane = threadIdx.x & 31;
+  const int64_t item = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
+  const int ncols = nt - k - 1;
+  if (ncols <= 0) return;
+  const int64_t ri = item / ncols;
+  const int J = k + 1 + (int)(item % ncols);
+  if (ri >= *nrows) return;
+  const int64_t r = rows[ri];
+  T e = T(0), w = T(0), a = T(0);
+  for (int c = lane; c < nb; c += 32) {
+    T x = A[r + ((int64_t)J * nb + c) * lda];
+    e = fadd(e, x);
+    w = ffma(T(c + 1), x, w);
+    a = fadd(a, fabs(x));
+  }
+  for (int m = 16; m >= 1; m >>= 1) {
+    e = fadd(e, shfl_xor(e, m));
+    w = fadd(w, shfl_xor(w, m));
+    a = fadd(a, shfl_xor(a, m));
+  }
+  if (lane) return;
+  const T de = rowchk[r + (int64_t)(2 * J) * ldr] - e;
+  const T dw = rowchk[r + (int64_t)(2 * J + 1) * ldr] - w;
+  const double m = use_mag ? (double)rowmag[r + (int64_t)J * ldrm] : (double)a;
+  const double t = tau_fac * m;
+  const bool bad = !isfinite((double)de) || !isfinite((double)dw) || fabs((double)de) > t ||
+                   fabs((double)dw) > (double)nb * t;
+  if (!bad) return;
+  atomicAdd(&counts[ABFT_CNT_ROWS_FLAGGED], 1);
+  const int old = atomicOr(&status[r / nb + (int64_t)J * ld_status], ABFT_ST_ROW);
+  if (!(old & (ABFT_ST_COL | ABFT_ST_ROW))) atomicAdd(&counts[ABFT_CNT_TILES_FLAGGED], 1);
+}
+
+// Row swaps of every column outside the panel (LAPACK laswp) with the c-14
+// column-checksum deltas; panel columns update only their checksums, from the
+// pre-PD copy (swapped progressively).  One thread per matrix column.
+template <typename T>
+__global__ void lu_swap_cols_kernel(T* A, int64_t lda, int64_t n, int nb, int k, const int32_t* piv_local, T* pcopy,
+                                    int64_t ldp, T* colchk, int64_t ldc, T* colmag, int64_t ldcm) {
+  const int64_t r0 = (int64_t)k * nb, r1 = r0 + nb;
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x) {
+    const bool panel = c >= r0 && c < r1;
+    if (panel && !colchk) continue;  // getrf already swapped the panel; no checksums to move
+    T* col = panel ? pcopy + (c - r0) * ldp - r0 : A + c * lda;  // indexable by global row
+    for (int j = 0; j < nb; ++j) {
+      const int64_t p = r0 + j, q = r0 + piv_local[j] - 1;
+      if (p == q) continue;
+      const T xp = col[p], xq = col[q];
+      if (colchk) {
+        const int64_t P = p / nb, Q = q / nb, pl = p % nb, ql = q % nb;
+        const T d = xq - xp;
+        if (P != Q) {
+          colchk[2 * P + c * ldc] += d;
+          colchk[2 * P + 1 + c * ldc] += T(pl + 1) * d;
+          colchk[2 * Q + c * ldc] -= d;
+          colchk[2 * Q + 1 + c * ldc] -= T(ql + 1) * d;
+          if (colmag) {
+            const T da = fabs(xq) - fabs(xp);
+            colmag[P + c * ldcm] += da;
+            colmag[Q + c * ldcm] -= da;
+          }
+        } else {
+          colchk[2 * P + 1 + c * ldc] += T(pl - ql) * d;
+        }
+      }
+      col[p] = xq;
+      col[q] = xp;
+    }
+  }
+}
+
+// Row checksums (and row magnitudes) move with their rows (tile columns >= k).
+template <typename T>
+__global__ void lu_swap_rowchk_kernel(T* rowchk, int64_t ldr, T* rowmag, int64_t ldrm, int nb, int k, int nt,
+                                      const int32_t* piv_local) {
+  const int64_t r0 = (int64_t)k * nb;
+  for (int J = k + blockIdx.x * blockDim.x + threadIdx.x; J < nt; J += gridDim.x * blockDim.x) {
+    for (int j = 0; j < nb; ++j) {
+      const int64_t p = r0 + j, q = r0 + piv_local[j] - 1;
+      if (p == q) continue;
+      for (int t = 0; t < 2; ++t) {
+        T* e = rowchk + (int64_t)(2 * J + t) * ldr;
+        const T tmp = e[p];
+        e[p] = e[q];
+        e[q] = tmp;
+      }
+      if (rowmag) {
+        T* m = rowmag + (int64_t)J * ldrm;
+        const T tmp = m[p];
+        m[p] = m[q];
+        m[q] = tmp;
+      }
+    }
+  }
+}
+
+// Fig. 4a repair for LU (c-25): a correction E of L21[p, q] or U12[q, c] found
+// by the post-TMU panel re-check is pushed into the trailing matrix the TMU
+// built from the bad value.  Single CTA, fixes in log order.
+struct LuRepairArgs {
+  void* A;
+  int64_t lda, n, nb;
+  int k;
+  void *colchk, *rowchk, *colmag, *rowmag;
+  int64_t ldc, ldr, ldcm, ldrm;
+  const abft_fix_t* fixes;
+  int cap;
+  const int32_t* n_fixes;
+  const int32_t* mark;
+  int32_t* rep_counts;
+  int32_t* counts;
+};
+
+template <typename T>
+__global__ void lu_fig4a_repair_kernel(LuRepairArgs r) {
+  const int n0 = *r.mark, n1 = min(*r.n_fixes, r.cap);
+  T* A = reinterpret_cast<T*>(r.A);
+  T* colchk = reinterpret_cast<T*>(r.colchk);
+  T* rowchk = reinterpret_cast<T*>(r.rowchk);
+  T* colmag = reinterpret_cast<T*>(r.colmag);
+  T* rowmag = reinterpret_cast<T*>(r.rowmag);
+  const int64_t nb = r.nb, nt = r.n / nb, k = r.k, r0 = k * nb, r1 = r0 + nb;
+  __shared__ double s_max;
+  __shared__ int s_skip;
+  for (int f = n0; f < n1; ++f) {
+    const abft_fix_t fx = r.fixes[f];
+    if (fx.kind != ABFT_FIX_DATA) continue;
+    const bool inL = fx.gj >= r0 && fx.gj < r1 && fx.gi >= r1;
+    const bool inU = fx.gi >= r0 && fx.gi < r1 && fx.gj >= r1;
+    if (!inL && !inU) continue;
+    const double eps = fx.after - fx.before;
+    double mx = 0.0;
+    if (inL)
+      for (int64_t a = r1 + threadIdx.x; a < r.n; a += blockDim.x) mx = fmax(mx, fabs((double)A[a + fx.gj * r.lda]));
+    else
+      for (int64_t c = r1 + threadIdx.x; c < r.n; c += blockDim.x) mx = fmax(mx, fabs((double)A[fx.gi + c * r.lda]));
+    for (int m = 16; m >= 1; m >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, m));
+    if (threadIdx.x == 0) s_max = 0.0;
+    __syncthreads();
+    if ((threadIdx.x & 31) == 0) atomicMax((unsigned long long*)&s_max, __double_as_longlong(mx));
+    __syncthreads();
+    if (threadIdx.x == 0) s_skip = !(isfinite(eps) && fabs(eps) <= 1024.0 * s_max);
+    __syncthreads();
+    if (s_skip) {
+      if (threadIdx.x == 0) {
+        atomicAdd(&r.rep_counts[1], 1);
+        atomicAdd(&r.counts[ABFT_CNT_UNCORRECTABLE], 1);
+      }
+      __syncthreads();
+      continue;
+    }
+    const T e = (T)eps, ae = fabs(e);
+    if (inL) {  // row p of the trailing matrix: A[p, c] -= E U[q, c]; r(A_iJ)[p] -= E r(U_J)[q]
+      const int64_t p = fx.gi, q = fx.gj - r0;
+      for (int64_t c = r1 + threadIdx.x; c < r.n; c += blockDim.x) A[p + c * r.lda] -= e * A[r0 + q + c * r.lda];
+      for (int64_t J = k + 1 + threadIdx.x; J < nt; J += blockDim.x) {
+        rowchk[p + 2 * J * r.ldr] -= e * rowchk[r0 + q + 2 * J * r.ldr];
+        rowchk[p + (2 * J + 1) * r.ldr] -= e * rowchk[r0 + q + (2 * J + 1) * r.ldr];
+        if (rowmag) rowmag[p + J * r.ldrm] += ae * rowmag[r0 + q + J * r.ldrm];
+      }
+    } else {  // column c: A[a, c] -= L[a, q] E; c(A_Ij)[:, c] -= E c(L_I)[:, q]
+      const int64_t q = fx.gi - r0, c = fx.gj;
+      for (int64_t a = r1 + threadIdx.x; a < r.n; a += blockDim.x) A[a + c * r.lda] -= A[a + (r0 + q) * r.lda] * e;
+      for (int64_t I = k + 1 + threadIdx.x; I < nt; I += blockDim.x) {
+        colchk[2 * I + c * r.ldc] -= e * colchk[2 * I + (r0 + q) * r.ldc];
+        colchk[2 * I + 1 + c * r.ldc] -= e * colchk[2 * I + 1 + (r0 + q) * r.ldc];
+        if (colmag) colmag[I + c * r.ldcm] += ae * colmag[I + (r0 + q) * r.ldcm];
+      }
+    }
+    if (threadIdx.x == 0) atomicAdd(&r.rep_counts[0], 1);
+    __syncthreads();
+  }
+}
+
+static unsigned blocks_for(int64_t work, int per) {
+  int64_t g = (work + per - 1) / per;
+  return (unsigned)(g < 1 ? 1 : (g > 148 * 32 ? 148 * 32 : g));
+}
+
+}  // namespace abft
+
+// ------------------------------------------------------------ panel getrf --
+extern "C" int abft_panel_getrf(const abft_mat_t* mat, int32_t k, int64_t* ipiv, const abft_tol_t* tol,
+                                const abft_report_t* rep, abft_fix_t* fixes, int32_t max_fixes, int32_t* n_fixes,
+                                void* Linv, void* Uinv, int32_t* info, abft_stream_t stream) {
+  using namespace abft;
+  if (!mat || mat->m != mat->n || mat->nb < 32 || mat->nb > 1024 || (mat->nb & (mat->nb - 1)) ||
+      mat->n % mat->nb || !mat->A || mat->lda < mat->m)
+    return -1;
+  const int64_t nb = mat->nb, n = mat->n, nt = n / nb;
+  if (k < 0 || k >= nt) return -2;
+  if (!ipiv) return -3;
+  const bool ft = mat->colchk != nullptr;
+  if (ft && (!mat->rowchk || !tol || !rep || !rep->status || !rep->counts || !n_fixes)) return -4;
+  if (!Linv) return -9;
+  if (!Uinv) return -10;
+  if (!info) return -11;
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t es = mat->dtype == ABFT_F64 ? 8 : 4;
+  const int64_t r0 = k * nb, mk = n - r0;
+  char* A = (char*)mat->A;
+  char* panel = A + (r0 + r0 * mat->lda) * es;
+  // scratch: pre-PD panel copy | local pivots | swap rows | nrows | getrf work
+  int lwork = 0;
+  {
+    std::unique_lock<std::mutex> lk;
+    cusolverDnHandle_t h = solver_handle(s, lk);
+    cusolverStatus_t st = mat->dtype == ABFT_F64
+                              ? cusolverDnDgetrf_bufferSize(h, (int)mk, (int)nb, (double*)panel, (int)mat->lda, &lwork)
+                              : cusolverDnSgetrf_bufferSize(h, (int)mk, (int)nb, (float*)panel, (int)mat->lda, &lwork);
+    if (st != CUSOLVER_STATUS_SUCCESS) return ABFT_E_CUSOLVER;
+  }
+  const size_t copy_bytes = ft ? (size_t)mk * nb * es : 0;
+  const size_t off_piv = (copy_bytes + 255) / 256 * 256;
+  const size_t off_rows = off_piv + ((size_t)nb * 4 + 255) / 256 * 256;
+  const size_t off_nrows = off_rows + (size_t)2 * nb * 8;
+  const size_t off_work = (off_nrows + 4 + 255) / 256 * 256;
+  void* scr = nullptr;
+  FT_TRY(scratch(s, 10, off_work + (size_t)(lwork + 1) * es, &scr));
+  char* base = (char*)scr;
+  int32_t* piv_local = (int32_t*)(base + off_piv);
+  int64_t* rows = (int64_t*)(base + off_rows);
+  int32_t* nrows = (int32_t*)(base + off_nrows);
+  if (ft)
+    ABFT_CUDA_TRY(cudaMemcpy2DAsync(base, mk * es, panel, mat->lda * es, mk * es, nb, cudaMemcpyDeviceToDevice, s));
+  {
+    std::unique_lock<std::mutex> lk;
+    cusolverDnHandle_t h = solver_handle(s, lk);
+    cusolverStatus_t st =
+        mat->dtype == ABFT_F64
+            ? cusolverDnDgetrf(h, (int)mk, (int)nb, (double*)panel, (int)mat->lda, (double*)(base + off_work),
+                               piv_local, info)
+            : cusolverDnSgetrf(h, (int)mk, (int)nb, (float*)panel, (int)mat->lda, (float*)(base + off_work),
+                               piv_local, info);
+    if (st != CUSOLVER_STATUS_SUCCESS) return ABFT_E_CUSOLVER;
+  }
+  lu_pivots_kernel<<<1, 256, 0, s>>>(piv_local, ipiv, (int)nb, r0);
+  // c-14b: verify every trailing row a swap will move, fix before swapping
+  if (ft && k < nt - 1) {
+    lu_swap_rows_kernel<<<1, 1024, 0, s>>>(piv_local, (int)nb, r0, rows, nrows);
+    const int ncols = (int)(nt - k - 1);
+    const int64_t items = 2 * nb * ncols;
+    const bool use_mag = tol->kind == ABFT_TOL_MAGNITUDE && mat->rowmag;
+    const double tf = mat->dtype == ABFT_F64 ? tau_factor<double>((int)nb, tol->scale)
+                                             : tau_factor<float>((int)nb, tol->scale);
+    if (mat->dtype == ABFT_F64)
+      lu_row_check_kernel<double><<<(unsigned)((items + 7) / 8), 256, 0, s>>>(
+          (const double*)A, mat->lda, (const double*)mat->rowchk, mat->ldr, (const double*)mat->rowmag, mat->ldrm,
+          use_mag, tf, (int)nb, k, (int)nt, rows, nrows, rep->status, rep->ld_status, rep->counts);
+    else
+      lu_row_check_kernel<float><<<(unsigned)((items + 7) / 8), 256, 0, s>>>(
+          (const float*)A, mat->lda, (const float*)mat->rowchk, mat->ldr, (const float*)mat->rowmag, mat->ldrm,
+          use_mag, tf, (int)nb, k, (int)nt, rows, nrows, rep->status, rep->ld_status, rep->counts);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    abft_tiles_t tr{(int)k, (int)nt, (int)k + 1, (int)nt, 0, ABFT_GENERAL};
+    FT_TRY(abft_locate_correct(mat, &tr, ABFT_BOTH, tol, rep, fixes, max_fixes, n_fixes, stream));
+  }
+  // swaps: data outside the panel + c deltas (panel: from the pre-PD copy)
+  if (mat->dtype == ABFT_F64)
+    lu_swap_cols_kernel<double><<<blocks_for(n, 128), 128, 0, s>>>(
+        (double*)A, mat->lda, n, (int)nb, k, piv_local, (double*)base, mk, (double*)mat->colchk, mat->ldc,
+        (double*)mat->colmag, mat->ldcm);
+  else
+    lu_swap_cols_kernel<float><<<blocks_for(n, 128), 128, 0, s>>>((float*)A, mat->lda, n, (int)nb, k, piv_local,
+                                                                  (float*)base, mk, (float*)mat->colchk, mat->ldc,
+                                                                  (float*)mat->colmag, mat->ldcm);
+  ABFT_CUDA_TRY(cudaGetLastError());
+  if (ft) {
+    if (mat->dtype == ABFT_F64)
+      lu_swap_rowchk_kernel<double><<<1, 128, 0, s>>>((double*)mat->rowchk, mat->ldr, (double*)mat->rowmag,
+                                                       mat->ldrm, (int)nb, k, (int)nt, piv_local);
+    else
+      lu_swap_rowchk_kernel<float><<<1, 128, 0, s>>>((float*)mat->rowchk, mat->ldr, (float*)mat->rowmag, mat->ldrm,
+                                                      (int)nb, k, (int)nt, piv_local);
+    ABFT_CUDA_TRY(cudaGetLastError());
+  }
+  // inverses of the diagonal factors (reused by the PU) and the c-13 PD rules
+  FT_TRY(abft_tri_inverse(mat->dtype, 'L', 'U', nb, panel, mat->lda, Linv, nb, stream));
+  FT_TRY(abft_tri_inverse(mat->dtype, 'U', 'N', nb, panel, mat->lda, Uinv, nb, stream));
+  if (!ft) return 0;
+  // c(L_I) = c(P~_I) U_kk^-1 for I >= k ; m_c <- m_c |U_kk^-1|
+  FT_TRY(abft_update_trsm_inv(mat->dtype, 'R', 'N', nb, Uinv, nb, (char*)mat->colchk + (2 * k + r0 * mat->ldc) * es,
+                              mat->ldc, 2 * (nt - k),
+                              mat->colmag ? (char*)mat->colmag + (k + r0 * mat->ldcm) * es : nullptr, mat->ldcm,
+                              nt - k, stream));
+  // r(U_kk) = L_kk^-1 r(P~_kk) ; m_r <- |L_kk^-1| m_r
+  FT_TRY(abft_update_trsm_inv(mat->dtype, 'L', 'N', nb, Linv, nb, (char*)mat->rowchk + (r0 + 2 * k * mat->ldr) * es,
+                              mat->ldr, 2, mat->rowmag ? (char*)mat->rowmag + (r0 + k * mat->ldrm) * es : nullptr,
+                              mat->ldrm, 1, stream));
+  return 0;
+}
+
+// ----------------------------------------------------------------- driver --
+extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t lda, int64_t* ipiv,
+                        const ft_opts_t* o, ft_stats_t* stats, int64_t* info_out) {
+  using namespace abft;
+  if (!c) return -1;
+  if (dtype != ABFT_F32 && dtype != ABFT_F64) return -2;
+  if (!o) return -7;
+  const int64_t nb = o->nb;
+  if (n < 0 || nb < 32 || nb > 1024 || (nb & (nb - 1)) || n % nb) return -3;
+  if (!dA) return -4;
+  if (lda < std::max<int64_t>(1, n)) return -5;
+  if (!ipiv) return -6;
+  if (o->n_inject < 0 || (o->n_inject > 0 && !o->inject)) return -7;
+  ABFT_CUDA_TRY(cudaSetDevice(c->device));
+  Driver d;
+  FT_TRY(d.setup(c, dtype, n, nb, dA, lda, o, /*lu=*/true));
+  const int64_t nt = d.nt;
+  const bool ft = o->abft != 0;
+  cudaStream_t s = d.s;
+  const abft_stream_t as = (abft_stream_t)s;
+  std::unique_lock<std::mutex> lk;
+  auto t0 = std::chrono::steady_clock::now();
+  if (ft) {
+    abft_tiles_t all{0, (int)nt, 0, (int)nt, 0, ABFT_GENERAL};
+    FT_TRY(abft_encode(&d.M, &all, ABFT_BOTH, as));
+  }
+  for (int k = 0; k < nt; ++k) {
+    const int64_t r0 = k * nb, r1 = r0 + nb, nk = n - r1;
+    const int m2 = (int)(2 * (nt - k - 1));
+    // Alg. 2 lines 3-4: check the column panel to be decomposed (c + r)
+    FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
+    if (ft) FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH));
+    // line 5: PD with pivoting, swap rule, c(L), r(U_kk)
+    FT_TRY(d.inject_at(k, FT_AT_PRE_PD));
+    FT_TRY(abft_panel_getrf(&d.M, k, ipiv + r0, ft ? &d.tol : nullptr, ft ? &d.R : nullptr, c->fixlog, c->fixcap,
+                            d.nfix, c->linv, c->uinv, d.info, as));
+    if (ft && k < nt - 1) ++d.n_checks;  // the pre-swap row check (c-14b)
+    accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.info_total, r0);
+    FT_TRY(d.restore_onchip());
+    FT_TRY(d.inject_at(k, FT_AT_POST_PD));
+    // line 7: check the decomposed panel: L (UNIT_LOWER on the diagonal, c) and U_kk (r)
+    if (ft) {
+      FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_UNIT_LOWER, ABFT_COL));
+      FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_UPPER, ABFT_ROW));
+    }
+    if (k == nt - 1) break;
+    // line 8: check the row panel to be updated (c + r)
+    FT_TRY(d.inject_at(k, FT_AT_PRE_PU_CHECK));
+    if (ft) FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_BOTH));
+    // line 9: PU  U12 = L_kk^-1 A12 (DGEMM with the PD's inverse) + r rule
+    FT_TRY(d.inject_at(k, FT_AT_PRE_PU));
+    const bool refresh = d.diag_touched_before_pu(k);
+    if (refresh) FT_TRY(abft_tri_inverse(dtype, 'L', 'U', nb, d.a_at(r0, r0), lda, c->linv, nb, as));
+    {
+      cublasHandle_t h = blas_handle(s, lk);
+      cublasStatus_t st;
+      if (dtype == ABFT_F64) {
+        const double one = 1.0, zero = 0.0;
+        st = cublasDgemm(h, CUBLAS_OP_N, CUBLAS_OP_N, (int)nb, (int)nk, (int)nb, &one, (const double*)c->linv,
+                         (int)nb, (const double*)d.a_at(r0, r1), (int)lda, &zero, (double*)c->putmp, (int)nb);
+      } else {
+        const float one = 1.0f, zero = 0.0f;
+        st = cublasSgemm(h, CUBLAS_OP_N, CUBLAS_OP_N, (int)nb, (int)nk, (int)nb, &one, (const float*)c->linv, (int)nb,
+                         (const float*)d.a_at(r0, r1), (int)lda, &zero, (float*)c->putmp, (int)nb);
+      }
+      lk.unlock();
+      if (st != CUBLAS_STATUS_SUCCESS) return ABFT_E_CUBLAS;
+      ABFT_CUDA_TRY(cudaMemcpy2DAsync(d.a_at(r0, r1), lda * d.es, c->putmp, nb * d.es, nb * d.es, nk,
+                                      cudaMemcpyDeviceToDevice, s));
+    }
+    FT_TRY(d.restore_onchip());
+    if (refresh) FT_TRY(abft_tri_inverse(dtype, 'L', 'U', nb, d.a_at(r0, r0), lda, c->linv, nb, as));
+    if (ft)  // r(U_kJ) = L_kk^-1 r(A_kJ), m_r <- |L_kk^-1| m_r  (c-13)
+      FT_TRY(abft_update_trsm_inv(dtype, 'L', 'N', nb, c->linv, nb, d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, m2,
+                                  d.rowmag_at(r0, k + 1), d.M.ldrm, m2 / 2, as));
+    FT_TRY(d.inject_at(k, FT_AT_POST_PU));
+    // line 10: check the updated row panel (r)
+    if (ft) FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW));
+    // line 12: TMU  A22 -= L21 U12 (DGEMM on tensor cores) + c-13 rules
+    FT_TRY(d.inject_at(k, FT_AT_PRE_TMU));
+    {
+      cublasHandle_t h = blas_handle(s, lk);
+      cublasStatus_t st;
+      if (dtype == ABFT_F64) {
+        const double m1 = -1.0, one = 1.0;
+        st = cublasDgemm(h, CUBLAS_OP_N, CUBLAS_OP_N, (int)nk, (int)nk, (int)nb, &m1, (const double*)d.a_at(r1, r0),
+                         (int)lda, (const double*)d.a_at(r0, r1), (int)lda, &one, (double*)d.a_at(r1, r1), (int)lda);
+      } else {
+        const float m1 = -1.0f, one = 1.0f;
+        st = cublasSgemm(h, CUBLAS_OP_N, CUBLAS_OP_N, (int)nk, (int)nk, (int)nb, &m1, (const float*)d.a_at(r1, r0),
+                         (int)lda, (const float*)d.a_at(r0, r1), (int)lda, &one, (float*)d.a_at(r1, r1), (int)lda);
+      }
+      lk.unlock();
+      if (st != CUBLAS_STATUS_SUCCESS) return ABFT_E_CUBLAS;
+    }
+    FT_TRY(d.restore_onchip());
+    if (ft) {
+      // c(A_IJ) -= c(L_Ik) U_kJ
+      FT_TRY(abft_update_gemm(dtype, ABFT_COL, 'N', 'N', -1.0, d.colchk_at(2 * (k + 1), r0), d.M.ldc, d.a_at(r0, r1),
+                              lda, d.colchk_at(2 * (k + 1), r1), d.M.ldc, m2, nk, nb, d.colmag_at(k + 1, r0),
+                              d.M.ldcm, d.colmag_at(k + 1, r1), d.M.ldcm, as));
+      // r(A_IJ) -= L_Ik r(U_kJ)
+      FT_TRY(abft_update_gemm(dtype, ABFT_ROW, 'N', 'N', -1.0, d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, d.a_at(r1, r0),
+                              lda, d.rowchk_at(r1, 2 * (k + 1)), d.M.ldr, m2, nk, nb, d.rowmag_at(r0, k + 1),
+                              d.M.ldrm, d.rowmag_at(r1, k + 1), d.M.ldrm, as));
+    }
+    FT_TRY(d.inject_at(k, FT_AT_POST_TMU));
+    // line 13: heuristic re-check of both panels (Fig. 4a) + guarded repair
+    if (ft) {
+      ABFT_CUDA_TRY(cudaMemcpyAsync(d.mark, d.nfix, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
+      FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
+      FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW));
+      if (o->fig4a_repair) {
+        LuRepairArgs ra{};
+        ra.A = dA;
+        ra.lda = lda;
+        ra.n = n;
+        ra.nb = nb;
+        ra.k = k;
+        ra.colchk = d.M.colchk;
+        ra.rowchk = d.M.rowchk;
+        ra.colmag = d.M.colmag;
+        ra.rowmag = d.M.rowmag;
+        ra.ldc = d.M.ldc;
+        ra.ldr = d.M.ldr;
+        ra.ldcm = d.M.ldcm;
+        ra.ldrm = d.M.ldrm;
+        ra.fixes = c->fixlog;
+        ra.cap = c->fixcap;
+        ra.n_fixes = d.nfix;
+        ra.mark = d.mark;
+        ra.rep_counts = d.rep;
+        ra.counts = d.counts;
+        if (dtype == ABFT_F64)
+          lu_fig4a_repair_kernel<double><<<1, 256, 0, s>>>(ra);
+        else
+          lu_fig4a_repair_kernel<float><<<1, 256, 0, s>>>(ra);
+        ABFT_CUDA_TRY(cudaGetLastError());
+      }
+    }
+  }
+  return d.finish(t0, stats, info_out);
+}

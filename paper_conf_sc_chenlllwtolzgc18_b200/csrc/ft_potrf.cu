@@ -6,26 +6,7 @@
 // PD on the CPU in MAGMA (L61) — here the PD runs on the device (cuSOLVER),
 // DESIGN.md §7 explains why.  Readings: c-12 (Cholesky rules), c-24 (views
 // before/after PD), c-25 (guarded Fig. 4a trailing repair), c-8 (fault hooks).
-#include <cublas_v2.h>
-#include <cusolverDn.h>
-
-#include <chrono>
-#include <mutex>
-#include <vector>
-
-#include "abft_common.cuh"
-
-namespace abft {
-cublasHandle_t blas_handle(cudaStream_t s, std::unique_lock<std::mutex>& lk);
-cusolverDnHandle_t solver_handle(cudaStream_t s, std::unique_lock<std::mutex>& lk);
-int scratch(cudaStream_t s, int slot, size_t bytes, void** out);
-}  // namespace abft
-
-#define FT_TRY(expr)          \
-  do {                        \
-    int _rc = (expr);         \
-    if (_rc) return _rc;      \
-  } while (0)
+#include "ft_driver.cuh"
 
 // ------------------------------------------------------------ panel potrf --
 namespace abft {
@@ -153,30 +134,9 @@ __global__ void fig4a_repair_kernel(RepairArgs r) {
   }
 }
 
-// LAPACK info of the whole factorization: first failing tile's local minor
-// offset by the tile origin.
-__global__ void accum_info_kernel(int32_t* tile_info, int32_t* total, int64_t offset) {
-  if (*tile_info != 0 && *total == 0) *total = (int32_t)(*tile_info + offset);
-  *tile_info = 0;
-}
 }  // namespace abft
 
 // ----------------------------------------------------------------- driver --
-struct ft_ctx {
-  int device = 0;
-  cudaStream_t stream = nullptr;
-  void* state = nullptr;  // colchk | rowchk | colmag | rowmag
-  size_t state_bytes = 0;
-  int32_t* ints = nullptr;  // status | counts[8] | n_fixes | mark | info | rep[2]
-  size_t ints_n = 0;
-  abft_fix_t* fixlog = nullptr;
-  int fixcap = 0;
-  void* linv = nullptr;  // nb x nb inverse of the current L_kk
-  size_t linv_bytes = 0;
-  void* putmp = nullptr;  // n x nb panel scratch for the GEMM-based PU
-  size_t putmp_bytes = 0;
-};
-
 extern "C" int ft_ctx_create(ft_ctx_t** ctx, int32_t device, abft_stream_t stream) {
   if (!ctx) return -1;
   ABFT_CUDA_TRY(cudaSetDevice(device));
@@ -199,85 +159,12 @@ extern "C" int ft_ctx_destroy(ft_ctx_t* c) {
   if (c->ints) cudaFree(c->ints);
   if (c->fixlog) cudaFree(c->fixlog);
   if (c->linv) cudaFree(c->linv);
+  if (c->uinv) cudaFree(c->uinv);
   if (c->putmp) cudaFree(c->putmp);
+  if (c->aux) cudaFree(c->aux);
   delete c;
   return 0;
 }
-
-namespace {
-
-struct Driver {
-  ft_ctx* c;
-  cudaStream_t s;
-  int32_t dtype;
-  int64_t n, nb, nt, lda;
-  size_t es;
-  void* A;
-  const ft_opts_t* o;
-  abft_mat_t M{};
-  abft_report_t R{};
-  abft_tol_t tol{};
-  int32_t *status, *counts, *nfix, *mark, *info, *rep;
-  std::vector<ft_inject_t> onchip_pending;
-  int n_checks = 0;
-
-  char* elem(int target, int64_t gi, int64_t gj) {
-    if (target == 1) return (char*)M.colchk + (gi + gj * M.ldc) * es;
-    if (target == 2) return (char*)M.rowchk + (gi + gj * M.ldr) * es;
-    return (char*)A + (gi + gj * lda) * es;
-  }
-  // Elements the op after `point` overwrites: an on-chip flip there cannot be
-  // changed back, so it stays (reading c-8).
-  bool in_update_region(int point, int k, int64_t gi, int64_t gj) const {
-    const int64_t r0 = k * nb, r1 = (k + 1) * nb;
-    if (point == FT_AT_PRE_PD) return gi >= r0 && gi < r1 && gj >= r0 && gj < r1;
-    if (point == FT_AT_PRE_PU) return gi >= r1 && gj >= r0 && gj < r1;
-    if (point == FT_AT_PRE_TMU) return gi >= r1 && gj >= r1;
-    return false;
-  }
-  int inject_at(int k, int point) {
-    for (int t = 0; t < o->n_inject; ++t) {
-      const ft_inject_t& f = o->inject[t];
-      if (f.iter != k || f.point != point) continue;
-      FT_TRY(abft_inject(elem(f.target, f.gi, f.gj), dtype, 0, f.xor_mask, (abft_stream_t)s));
-      bool op_point = point == FT_AT_PRE_PD || point == FT_AT_PRE_PU || point == FT_AT_PRE_TMU;
-      if (f.kind == FT_KIND_ONCHIP && op_point && f.target == 0 && !in_update_region(point, k, f.gi, f.gj))
-        onchip_pending.push_back(f);
-    }
-    return 0;
-  }
-  // Fault-injection runs only: does the plan touch L_kk between the PD (which
-  // produced the inverse the GEMM-based PU reads) and the PU?  Then the PU
-  // must see the flipped L_kk, as an in-place TRSM would (reading c-8).
-  bool lkk_touched_before_pu(int k) const {
-    for (int t = 0; t < o->n_inject; ++t) {
-      const ft_inject_t& f = o->inject[t];
-      if (f.iter != k || f.target != 0) continue;
-      if (f.point != FT_AT_PRE_PU_CHECK && f.point != FT_AT_PRE_PU) continue;
-      if (f.gi >= k * nb && f.gi < (k + 1) * nb && f.gj >= k * nb && f.gj < (k + 1) * nb) return true;
-    }
-    return false;
-  }
-  int restore_onchip() {  // after the op: undo on-chip flips (the stored value was never wrong)
-    for (auto& f : onchip_pending) FT_TRY(abft_inject(elem(f.target, f.gi, f.gj), dtype, 0, f.xor_mask, (abft_stream_t)s));
-    onchip_pending.clear();
-    return 0;
-  }
-  int check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only = false) {
-    abft_tiles_t t{I0, I1, J0, J1, lower_only ? 1 : 0, view};
-    FT_TRY(abft_verify(&M, &t, which, &tol, &R, (abft_stream_t)s));
-    FT_TRY(abft_locate_correct(&M, &t, which, &tol, &R, c->fixlog, c->fixcap, nfix, (abft_stream_t)s));
-    ++n_checks;
-    return 0;
-  }
-  void* colchk_at(int64_t r, int64_t col) { return (char*)M.colchk + (r + col * M.ldc) * es; }
-  void* colmag_at(int64_t r, int64_t col) { return (char*)M.colmag + (r + col * M.ldcm) * es; }
-  void* rowchk_at(int64_t r, int64_t col) { return (char*)M.rowchk + (r + col * M.ldr) * es; }
-  void* rowmag_at(int64_t r, int64_t col) { return (char*)M.rowmag + (r + col * M.ldrm) * es; }
-  void* a_at(int64_t r, int64_t col) { return (char*)A + (r + col * lda) * es; }
-};
-
-}  // namespace
 
 extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t lda, const ft_opts_t* o,
                         ft_stats_t* stats, int64_t* info_out) {
@@ -292,78 +179,10 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
   if (o->n_inject < 0 || (o->n_inject > 0 && !o->inject)) return -6;
   ABFT_CUDA_TRY(cudaSetDevice(c->device));
   Driver d;
-  d.c = c;
-  d.s = c->stream;
-  d.dtype = dtype;
-  d.n = n;
-  d.nb = nb;
-  d.nt = n / nb;
-  d.lda = lda;
-  d.es = dtype == ABFT_F64 ? 8 : 4;
-  d.A = dA;
-  d.o = o;
+  FT_TRY(d.setup(c, dtype, n, nb, dA, lda, o, /*lu=*/false));
   const int64_t nt = d.nt;
   const bool ft = o->abft != 0;
   cudaStream_t s = d.s;
-  // ---- state buffers (grown, never shrunk) ----
-  size_t need = ft ? (size_t)(2 * nt * n + n * 2 * nt + nt * n + n * nt) * d.es : 0;
-  if (c->state_bytes < need) {
-    if (c->state) cudaFree(c->state);
-    c->state = nullptr;
-    c->state_bytes = 0;
-    if (cudaMalloc(&c->state, need) != cudaSuccess) return ABFT_E_NOMEM;
-    c->state_bytes = need;
-  }
-  size_t ints_need = (size_t)nt * nt + 8 + 1 + 1 + 1 + 2 + 4;
-  if (c->ints_n < ints_need) {
-    if (c->ints) cudaFree(c->ints);
-    if (cudaMalloc(&c->ints, ints_need * sizeof(int32_t)) != cudaSuccess) return ABFT_E_NOMEM;
-    c->ints_n = ints_need;
-  }
-  auto grow = [](void*& p, size_t& have, size_t need) -> int {
-    if (have >= need) return 0;
-    if (p) cudaFree(p);
-    p = nullptr;
-    have = 0;
-    if (cudaMalloc(&p, need) != cudaSuccess) return ABFT_E_NOMEM;
-    have = need;
-    return 0;
-  };
-  FT_TRY(grow(c->linv, c->linv_bytes, (size_t)nb * nb * d.es));
-  if (o->pu_gemm) FT_TRY(grow(c->putmp, c->putmp_bytes, (size_t)n * nb * d.es));
-  d.status = c->ints;
-  d.counts = d.status + nt * nt;
-  d.nfix = d.counts + 8;
-  d.mark = d.nfix + 1;
-  d.info = d.mark + 1;
-  d.rep = d.info + 1;
-  ABFT_CUDA_TRY(cudaMemsetAsync(c->ints, 0, ints_need * sizeof(int32_t), s));
-  char* st = (char*)c->state;
-  d.M.dtype = dtype;
-  d.M.m = n;
-  d.M.n = n;
-  d.M.nb = nb;
-  d.M.A = dA;
-  d.M.lda = lda;
-  if (ft) {
-    d.M.colchk = st;
-    d.M.ldc = 2 * nt;
-    st += 2 * nt * n * d.es;
-    d.M.rowchk = st;
-    d.M.ldr = n;
-    st += n * 2 * nt * d.es;
-    d.M.colmag = st;
-    d.M.ldcm = nt;
-    st += nt * n * d.es;
-    d.M.rowmag = st;
-    d.M.ldrm = n;
-  }
-  d.R.status = d.status;
-  d.R.ld_status = nt;
-  d.R.counts = d.counts;
-  d.tol.kind = o->tol_kind;
-  d.tol.scale = o->tol_scale > 0 ? o->tol_scale : 1.0;
-
   std::unique_lock<std::mutex> lk;
   auto t0 = std::chrono::steady_clock::now();
   const abft_stream_t as = (abft_stream_t)s;
@@ -395,7 +214,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       }
       const bool need_inv = ft || o->pu_gemm;
       FT_TRY(abft_panel_potrf(&D, need_inv ? c->linv : nullptr, nb, d.info, as));
-      accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.rep + 2, (int64_t)k * nb);
+      accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.info_total, (int64_t)k * nb);
     }
     FT_TRY(d.restore_onchip());
     FT_TRY(d.inject_at(k, FT_AT_POST_PD));
@@ -407,7 +226,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft) FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH));
     // line 9: PU  L_ik = A_ik L_kk^-T  (+ c(L_ik) = c(A_ik) L_kk^-T, c-12)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PU));
-    const bool refresh_inv = o->pu_gemm && d.lkk_touched_before_pu(k);
+    const bool refresh_inv = o->pu_gemm && d.diag_touched_before_pu(k);
     if (refresh_inv) FT_TRY(abft_tri_inverse(dtype, 'L', 'N', nb, d.a_at(k * nb, k * nb), lda, c->linv, nb, as));
     {
       cublasHandle_t h = blas_handle(s, lk);
@@ -512,23 +331,5 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       }
     }
   }
-  // ---- the single host synchronisation: stats ----
-  int32_t host_ints[8 + 1 + 1 + 1 + 2 + 1];
-  ABFT_CUDA_TRY(cudaMemcpyAsync(host_ints, d.counts, sizeof(host_ints), cudaMemcpyDeviceToHost, s));
-  if (o->fix_log && o->fix_log_cap > 0)
-    ABFT_CUDA_TRY(cudaMemcpyAsync(o->fix_log, c->fixlog, sizeof(abft_fix_t) * std::min(o->fix_log_cap, c->fixcap),
-                                  cudaMemcpyDeviceToDevice, s));
-  ABFT_CUDA_TRY(cudaStreamSynchronize(s));
-  auto t1 = std::chrono::steady_clock::now();
-  if (info_out) *info_out = host_ints[13];
-  if (stats) {
-    for (int i = 0; i < 8; ++i) stats->counts[i] = host_ints[i];
-    stats->n_fixes = host_ints[8];
-    stats->repairs_applied = host_ints[11];
-    stats->repairs_skipped = host_ints[12];
-    stats->uncorrectable = host_ints[ABFT_CNT_UNCORRECTABLE];
-    stats->n_checks = d.n_checks;
-    stats->ms_total = std::chrono::duration<double, std::milli>(t1 - t0).count();
-  }
-  return host_ints[ABFT_CNT_UNCORRECTABLE] ? ABFT_E_UNCORRECTABLE : 0;
+  return d.finish(t0, stats, info_out);
 }

@@ -207,3 +207,72 @@ def test_lu_trailing_fault_in_a_pivot_row_fixed_before_the_swap():
     assert any(c[1] == "pre_swap_rows" for c in stats.checks)
     assert np.array_equal(piv, p)
     assert np.abs(LU - lu).max() <= 1e-12 * np.abs(lu).max()
+
+
+# ------------------------------------------------------------------- QR ----
+def _qr_invariant(st, k, phase):
+    nt = st.nt
+    tol = ck.Tol()
+    if phase == "pd":
+        for I in range(k, nt):
+            tc = ck.check_tile(st, I, k, ck.UNIT_LOWER if I == k else ck.GENERAL, ck.COL, tol)
+            assert not tc.Fc, (k, phase, I)
+        tc = ck.check_tile(st, k, k, ck.UPPER, ck.ROW, tol)
+        assert not tc.Fr
+        # below the diagonal tile, Q^T P [v1 v2] = 0 (Alg. 1 end state)
+        n, nb = st.A.shape[0], st.nb
+        below = st.rowchk[(k + 1) * nb:n, 2 * k:2 * k + 2]
+        assert np.abs(below).max(initial=0) <= 1e-10 * max(1.0, np.abs(st.rowchk[k * nb:(k + 1) * nb, 2 * k]).max())
+    else:
+        for J in range(k + 1, nt):
+            tc = ck.check_tile(st, k, J, ck.GENERAL, ck.ROW, tol)
+            assert not tc.Fr, (k, "R12", J)
+        for I, J in ck.Tiles(k + 1, nt, k + 1, nt):
+            tc = ck.check_tile(st, I, J, ck.GENERAL, ck.BOTH, tol)
+            assert not tc.Fc and not tc.Fr, (k, phase, I, J)
+
+
+@pytest.mark.parametrize("n,nb", [(256, 32), (512, 64), (384, 128)])
+def test_ft_geqrf_error_free_matches_lapack(n, nb):
+    A = si.general(n, seed=n + nb + 1)
+    H, tau, stats = dr.ft_geqrf(A, nb, invariant_hook=_qr_invariant)
+    h, t = np.linalg.qr(A, mode="raw")  # LAPACK dgeqrf output (h transposed)
+    h = h.T
+    assert np.abs(H - h).max() <= 1e-12 * np.abs(h).max()
+    assert np.abs(tau - t).max() <= 1e-12
+    assert stats.counts == [0] * 8
+
+
+def test_qr_last_column_convention():
+    # dlarfg with x(2:) = 0 gives tau = 0 and R_nn = x_n (no sign flip, c-15)
+    A = si.general(64, seed=3)
+    H, tau, _ = dr.ft_geqrf(A, 32)
+    h, t = np.linalg.qr(A, mode="raw")
+    assert tau[-1] == 0.0 and t[-1] == 0.0 and H[-1, -1] == pytest.approx(h.T[-1, -1], rel=1e-12)
+
+
+QR_FIXABLE = [
+    (dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 100, 70, (61,)),   # DRAM in the column panel
+    (dr.AT_POST_PD, dr.KIND_PERSIST, 150, 80, (62,)),        # computation error in V
+    (dr.AT_POST_PD, dr.KIND_PERSIST, 66, 90, (58,)),         # computation error in R_kk
+    (dr.AT_POST_TMU, dr.KIND_PERSIST, 230, 100, (59,)),      # trailing computation error
+    (dr.AT_POST_TMU, dr.KIND_PERSIST, 70, 200, (60,)),       # R12 computation error
+]
+
+
+@pytest.mark.parametrize("case", range(len(QR_FIXABLE)))
+def test_qr_fault_campaign_fixed(case):
+    point, kind, gi, gj, bits = QR_FIXABLE[case]
+    A = si.general(256, seed=0)
+    h, t = np.linalg.qr(A, mode="raw")
+    H, tau, stats = dr.ft_geqrf(A, 32, inject=[dr.Inject(2, point, kind, 0, gi, gj, bits)])
+    assert stats.uncorrectable == 0, stats.counts
+    assert stats.counts[0] >= 1
+    assert np.abs(H - h.T).max() <= 1e-12 * np.abs(h).max()
+
+
+def test_qr_tmu_reference_fault_detected():
+    # DRAM fault in V consumed by the TMU: detected by the re-check, reported R
+    A = si.general(256, seed=0)
+    _, _, stats = dr.ft_geqrf(A, 32, inject=[dr.Inject(2, dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 170, 80, (54,))])
+    assert stats.uncorrectable >= 1 and stats.repairs_skipped == 1
