@@ -184,6 +184,7 @@ def run_ours(args):
 
     import synth_inputs as si
     from paper_conf_sc_chenlllwtolzgc18_b200 import abft
+    from paper_conf_sc_chenlllwtolzgc18_b200 import dist as D
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -214,7 +215,7 @@ def run_ours(args):
             ev[2].record()
         abft.abft_locate_correct(mat, t_all, abft.BOTH, tol, rep, fixbuf, nfix)
         if world > 1:
-            dist.all_reduce(rep.counts)  # error-flag reduce (L361-L363)
+            D.reduce_counts(rep.counts)  # error-report exchange (L361-L363)
 
     for _ in range(args.warmup):
         step()
@@ -282,9 +283,11 @@ def run_ours(args):
         del hostA
 
     # ---- ft_potrf overhead at n=30720 (the metric's second half) ----
-    ftp = None
+    ftp = lq = None
     if not args.no_potrf and rank == 0:
         ftp = potrf_overhead(abft, si, args.potrf_n, nb, args.potrf_reps)
+    if not args.no_lu_qr and rank == 0:
+        lq = lu_qr_overhead(abft, si, args.lu_qr_n, nb, args.lu_qr_reps)
 
     del A, mat
     torch.cuda.empty_cache()
@@ -304,7 +307,7 @@ def run_ours(args):
                          "encode_GBs": pass_bytes / (enc_ms / 1e3) / 1e9,
                          "verify_GBs": pass_bytes / (ver_ms / 1e3) / 1e9},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": 3 * args.steps, "clocks": clk.summary(),
-            "ft_potrf": ftp,
+            "ft_potrf": ftp, "ft_getrf_geqrf": lq,
         }
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -360,6 +363,53 @@ def potrf_overhead(abft, si, n, nb, reps):
             "tflops_ft": n ** 3 / 3 / (ft_ms / 1e3) / 1e12, "reps": reps}
 
 
+def lu_qr_overhead(abft, si, n, nb, reps):
+    """BASELINE configs[2]: ft_getrf / ft_geqrf at n=20480 nb=512, ABFT on vs
+    the same driver with ABFT off; cuSOLVER getrf / geqrf as context."""
+    import torch
+
+    A0 = si.general_device(n, seed=21)
+    A = torch.empty_like(A0.t()).t()
+    ctx = abft.Context()
+    ipiv = torch.zeros(n, dtype=torch.int64, device="cuda")
+    tau = torch.zeros(n, dtype=torch.float64, device="cuda")
+    out = {"n": n, "nb": nb, "reps": reps}
+
+    def run(fn, ft):
+        A.copy_(A0)
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        rc, info, st = fn(ft)
+        b.record()
+        torch.cuda.synchronize()
+        assert rc == 0 and sum(st.counts) == 0, (rc, list(st.counts))
+        return a.elapsed_time(b)
+
+    for name, fn, flops in [("getrf", lambda ft: abft.ft_getrf(ctx, A, nb, ipiv, abft=ft), 2 * n ** 3 / 3),
+                            ("geqrf", lambda ft: abft.ft_geqrf(ctx, A, nb, tau, abft=ft), 4 * n ** 3 / 3)]:
+        run(fn, True)
+        run(fn, False)
+        tf = sorted(run(fn, True) for _ in range(reps))[reps // 2]
+        tp = sorted(run(fn, False) for _ in range(reps))[reps // 2]
+        out[name] = {"ms_ft": tf, "ms_plain": tp, "overhead_pct": 100.0 * (tf - tp) / tp,
+                     "tflops_ft": flops / (tf / 1e3) / 1e12}
+    torch.backends.cuda.preferred_linalg_library("cusolver")
+    G = A0.t().contiguous()
+    for name, fn in [("getrf", lambda: torch.linalg.lu_factor(G)), ("geqrf", lambda: torch.geqrf(G))]:
+        fn()
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        fn()
+        b.record()
+        torch.cuda.synchronize()
+        out[name]["cusolver_ms"] = a.elapsed_time(b)
+    del G, A, A0
+    torch.cuda.empty_cache()
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -373,6 +423,9 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-potrf", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--lu-qr-n", type=int, default=20480)
+    ap.add_argument("--lu-qr-reps", type=int, default=1)
+    ap.add_argument("--no-lu-qr", action="store_true")
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args)

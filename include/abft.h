@@ -116,8 +116,12 @@ typedef struct {
 } abft_tiles_t;
 
 typedef struct {
-  int32_t kind;  /* ABFT_TOL_* */
-  double scale;  /* multiplies tau (default 1) */
+  int32_t kind;    /* ABFT_TOL_* */
+  double scale;    /* multiplies tau (default 1) */
+  int32_t refresh; /* abft_verify: rebase every UNFLAGGED checksum entry of a checked tile on the
+                      recomputed value and reset its magnitude to e^T|X| (c-6); flagged entries are
+                      left for abft_locate_correct.  Keeps the magnitude bound from compounding
+                      |T^-1| factors across iterations (LU/QR). */
 } abft_tol_t;
 
 /* Verification output.  status: device int32, (m/nb) x (n/nb) column-major,
@@ -253,6 +257,18 @@ ABFT_API int abft_panel_getrf(const abft_mat_t *mat, int32_t k, int64_t *ipiv, c
                               int32_t *n_fixes, void *Linv, void *Uinv, int32_t *info,
                               abft_stream_t stream);
 
+/* a4 — abft_panel_geqrf (PD of Householder QR for iteration k; Table III,
+ * Alg. 1, c-15).  cuSOLVER dgeqrf of the column panel (LAPACK
+ * storage: R on and above the diagonal, v(2:) below, tau[0..nb)), the unit
+ * lower trapezoidal V into V (device, (n-k*nb) x nb, ld n-k*nb), the
+ * triangular factor T of the compact WY form (CTF, L238; not protected, c-16)
+ * into T (nb x nb, ld nb); when mat carries checksums (panel_copy: device
+ * (n-k*nb) x nb scratch for the pre-PD panel): c(V) per panel tile by the
+ * Alg. 1 recurrences replayed on the checksum rows, r(R) = rows of Q^T r(P),
+ * magnitudes by c-6.  *info (device int32) from dgeqrf. */
+ABFT_API int abft_panel_geqrf(const abft_mat_t *mat, int32_t k, void *tau, void *V, void *T,
+                              void *panel_copy, int32_t *info, abft_stream_t stream);
+
 /* W = T^-1 for an nb x nb triangular T (uplo 'L'/'U', diag 'N'/'U'); the
  * other triangle of W is written as zero.  Helper of the a5 rule (the
  * magnitude propagation needs |T^-1| explicitly, c-6). */
@@ -311,6 +327,7 @@ typedef struct {
   int32_t fix_log_cap;
   int32_t pu_gemm;       /* 1: PU as L21 = A21 * L_kk^-T (DGEMM with the PD's explicit inverse) in
                             both the protected and the unprotected driver; 0: cuBLAS DTRSM */
+  int32_t refresh;       /* abft_tol_t.refresh for every check of the run (default 1) */
 } ft_opts_t;
 
 /* Host-side statistics, filled after the driver's final synchronisation. */
@@ -350,6 +367,17 @@ ABFT_API int ft_potrf(ft_ctx_t *ctx, int32_t dtype, int64_t n, void *dA, int64_t
  * Returns ABFT_E_UNCORRECTABLE if a 2D error remained.  *info (host) follows
  * LAPACK getrf. */
 ABFT_API int ft_getrf(ft_ctx_t *ctx, int32_t dtype, int64_t n, void *dA, int64_t lda, int64_t *ipiv,
+                      const ft_opts_t *opts, ft_stats_t *stats, int64_t *info);
+
+/* ft_geqrf — fault-tolerant Householder QR A = QR of the square n x n dA
+ * (device, lda >= n, n % nb == 0) with full checksums (Table III): per
+ * iteration k — check the column panel (c+r) -> abft_panel_geqrf -> check V
+ * (UNIT_LOWER, c) and R_kk (UPPER, r) -> TMU A2 <- Q^T A2 (three DGEMMs) with
+ * c(A2) -= c(V) W, r(A2) -= V T^T V^T r(A2) -> re-check V (a V correction
+ * after the TMU consumed it is outcome R) and R12 (r).  Output as LAPACK
+ * dgeqrf (R and V in dA, tau: device array of n).  Returns
+ * ABFT_E_UNCORRECTABLE if a 2D / consumed error remained. */
+ABFT_API int ft_geqrf(ft_ctx_t *ctx, int32_t dtype, int64_t n, void *dA, int64_t lda, void *tau,
                       const ft_opts_t *opts, ft_stats_t *stats, int64_t *info);
 
 #ifdef __cplusplus

@@ -123,6 +123,7 @@ class Tol:
 
     kind: int = TOL_MAGNITUDE
     scale: float = 1.0
+    refresh: bool = False  # rebase clean entries on the recomputed checksums (c-6)
 
 
 @dataclass
@@ -297,12 +298,36 @@ def verify(st: State, tiles: Tiles, which=BOTH, tol: Tol = Tol()):
         tc = check_tile(st, I, J, tiles.view(I, J), which, tol)
         s = tc.status
         status[(I, J)] = s
+        if tol.refresh:
+            _refresh(st, tc, which)
         if s & (ST_COL | ST_ROW):
             counts[0] += 1
         counts[1] += len(tc.Fc)
         counts[2] += len(tc.Fr)
         counts[3] += 1 if tc.nonfinite else 0
     return status, counts
+
+
+def _refresh(st: State, tc: TileCheck, which):
+    """Reading c-6 'refresh': every UNFLAGGED checksum entry of a verified
+    tile is rebased on the recomputed value and its magnitude reset to the
+    fresh e^T|X| (flagged entries are left for locate/correct).  Without it the
+    magnitude bound compounds |T^-1| factors over the iterations of LU/QR and
+    the threshold grows until it hides O(1) errors."""
+    nb = st.nb
+    c, r, mc, mr = encode_tile(tc.X)
+    cs = slice(tc.J * nb, (tc.J + 1) * nb)
+    rs = slice(tc.I * nb, (tc.I + 1) * nb)
+    if which & COL:
+        ok = ~(tc.fce | tc.fcw)
+        st.colchk[2 * tc.I:2 * tc.I + 2, cs][:, ok] = c[:, ok]
+        if st.colmag is not None:
+            st.colmag[tc.I, cs][ok] = mc[ok]
+    if which & ROW:
+        ok = ~(tc.fre | tc.frw)
+        st.rowchk[rs, 2 * tc.J:2 * tc.J + 2][ok, :] = r[ok, :]
+        if st.rowmag is not None:
+            st.rowmag[rs, tc.J][ok] = mr[ok]
 
 
 # ----------------------------------------------------------------- locate --

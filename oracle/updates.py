@@ -338,7 +338,7 @@ def qr_pd_alg1(st: State, k: int):
       rck[j:] −= tau v (v^T rck[j:])
       store beta, v(2:) in P[:, j] and v_ck in ck[:, j]  (= c(V) in UNIT_LOWER view)
     Magnitudes (c-6): m_x = mck[:, j]; m_v = (m_x + |beta|·[row j in tile]) / |x1 − beta|;
-    mck[:, j+1:] += |tau| m_v |y|;  mr[j:] += |tau| |v| (|v|^T mr[j:]).
+    mck[:, j+1:] += |tau| m_v |y|;  after the loop m_r += |V| (|T|^T (|V|^T m_r)).
     At the end rck = Q^T P [v1 v2] = [r(R); 0].  Returns tau (nb)."""
     nb, n = st.nb, st.A.shape[0]
     nt = n // nb
@@ -383,8 +383,6 @@ def qr_pd_alg1(st: State, k: int):
                 mck[:, j + 1:] += abs(t) * np.outer(m_v, np.abs(y))
         yr = v @ rck[j:]
         rck[j:] -= t * np.outer(v, yr)
-        if mags:
-            mr[j:] += abs(t) * np.abs(v) * float(np.abs(v) @ mr[j:])
         P[j, j] = beta
         P[j + 1:, j] = v[1:]
         ck[:, j] = v_ck
@@ -395,7 +393,11 @@ def qr_pd_alg1(st: State, k: int):
     st.rowchk[r0:n, 2 * k:2 * k + 2] = rck
     if mags:
         st.colmag[k:, r0:r1] = mck
-        st.rowmag[r0:n, k] = mr
+        # rck = Q^T r(P), Q^T = I − V T^T V^T: m_r += |V| (|T|^T (|V|^T m_r)) (c-6)
+        V = np.tril(P, -1)
+        V[:nb, :nb] += np.eye(nb)
+        T = qr_T(V, tau)
+        st.rowmag[r0:n, k] = mr + np.abs(V) @ (np.abs(T).T @ (np.abs(V).T @ mr))
     return tau
 
 

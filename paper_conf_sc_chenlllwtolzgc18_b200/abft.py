@@ -53,7 +53,7 @@ class abft_tiles_t(C.Structure):
 
 
 class abft_tol_t(C.Structure):
-    _fields_ = [("kind", C.c_int32), ("scale", C.c_double)]
+    _fields_ = [("kind", C.c_int32), ("scale", C.c_double), ("refresh", C.c_int32)]
 
 
 class abft_report_t(C.Structure):
@@ -77,7 +77,8 @@ class ft_inject_t(C.Structure):
 class ft_opts_t(C.Structure):
     _fields_ = [("nb", C.c_int64), ("abft", C.c_int32), ("tol_kind", C.c_int32), ("tol_scale", C.c_double),
                 ("fig4a_repair", C.c_int32), ("n_inject", C.c_int32), ("inject", C.POINTER(ft_inject_t)),
-                ("fix_log", C.c_void_p), ("fix_log_cap", C.c_int32), ("pu_gemm", C.c_int32)]
+                ("fix_log", C.c_void_p), ("fix_log_cap", C.c_int32), ("pu_gemm", C.c_int32),
+                ("refresh", C.c_int32)]
 
 
 class ft_stats_t(C.Structure):
@@ -106,6 +107,8 @@ _sig = {
     "abft_panel_getrf": [_P(abft_mat_t), _i32, _vp, _P(abft_tol_t), _P(abft_report_t), _vp, _i32, _vp, _vp, _vp,
                          _vp, _vp],
     "ft_getrf": [_vp, _i32, _i64, _vp, _i64, _vp, _P(ft_opts_t), _P(ft_stats_t), _P(_i64)],
+    "abft_panel_geqrf": [_P(abft_mat_t), _i32, _vp, _vp, _vp, _vp, _vp, _vp],
+    "ft_geqrf": [_vp, _i32, _i64, _vp, _i64, _vp, _P(ft_opts_t), _P(ft_stats_t), _P(_i64)],
     "ft_ctx_create": [_P(_vp), _i32, _vp],
     "ft_ctx_destroy": [_vp],
     "ft_potrf": [_vp, _i32, _i64, _vp, _i64, _P(ft_opts_t), _P(ft_stats_t), _P(_i64)],
@@ -336,12 +339,13 @@ class Context:
             self._h = None
 
 
-def _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm):
+def _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh=True):
     inj = (ft_inject_t * max(1, len(inject)))()
     for k, f in enumerate(inject):
         inj[k] = ft_inject_t(*f)
     opts = ft_opts_t(nb, int(abft), tol_kind, tol_scale, int(fig4a_repair), len(inject), inj,
-                     _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES, int(pu_gemm))
+                     _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES, int(pu_gemm),
+                     int(refresh))
     return opts, inj
 
 
@@ -370,16 +374,33 @@ def ft_getrf(ctx: Context, A: torch.Tensor, nb: int, ipiv: torch.Tensor, abft=Tr
     return rc, info.value, stats
 
 
+def abft_panel_geqrf(mat: Mat, k: int, tau: torch.Tensor, V: torch.Tensor, T: torch.Tensor,
+                     panel_copy: torch.Tensor, info: torch.Tensor, stream=None):
+    m = mat.c()
+    return _check("abft_panel_geqrf", _L.abft_panel_geqrf(C.byref(m), k, _ptr(tau), _ptr(V), _ptr(T),
+                                                          _ptr(panel_copy), _ptr(info), _stream(stream)))
+
+
+def ft_geqrf(ctx: Context, A: torch.Tensor, nb: int, tau: torch.Tensor, abft=True, tol_kind=TOL_MAGNITUDE,
+             tol_scale=1.0, inject=(), fix_log=None):
+    """Fault-tolerant Householder QR in place on a column-major A (LAPACK
+    dgeqrf storage); tau: device tensor (n) of A's dtype."""
+    n = A.shape[0]
+    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, True, inject, fix_log, True)
+    stats = ft_stats_t()
+    info = C.c_int64()
+    rc = _L.ft_geqrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), _ptr(tau), C.byref(opts), C.byref(stats),
+                     C.byref(info))
+    _check("ft_geqrf", rc, ok=(0, E_UNCORRECTABLE))
+    return rc, info.value, stats
+
+
 def ft_potrf(ctx: Context, A: torch.Tensor, nb: int, abft=True, tol_kind=TOL_MAGNITUDE, tol_scale=1.0,
-             fig4a_repair=True, inject=(), fix_log=None, pu_gemm=True):
+             fig4a_repair=True, inject=(), fix_log=None, pu_gemm=True, refresh=True):
     """Fault-tolerant lower Cholesky in place on a column-major A.  Returns
     (rc, info, stats) with rc 0 or E_UNCORRECTABLE (other codes raise)."""
     n = A.shape[0]
-    inj = (ft_inject_t * max(1, len(inject)))()
-    for k, f in enumerate(inject):
-        inj[k] = ft_inject_t(*f)
-    opts = ft_opts_t(nb, int(abft), tol_kind, tol_scale, int(fig4a_repair), len(inject), inj,
-                     _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES, int(pu_gemm))
+    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_potrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), C.byref(opts), C.byref(stats), C.byref(info))

@@ -70,6 +70,7 @@ struct PassArgs {
   int nslab;
   int use_bulk;
   int use_mag;      // verify: thresholds from maintained magnitude arrays
+  int refresh;      // verify: rebase unflagged entries on the recomputed checksums (c-6)
   double tau_fac;   // scale * 2 * gamma_nb
   int32_t* status;
   int64_t ld_status;
@@ -208,6 +209,12 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
       }
       my_colflags |= f;
       my_ncols += f & 1;
+      if (p.refresh && !(f & 1)) {
+        T* cc2 = colchk + (int64_t)2 * I + gj * p.ldc;
+        cc2[0] = pe;
+        cc2[1] = pw;
+        if (colmag) colmag[I + gj * p.ldcm] = pa;
+      }
     }
   };
 
@@ -416,6 +423,11 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
         }
         my_rowflags |= f;
         my_nrows += f & 1;
+        if (p.refresh && !(f & 1)) {
+          rowchk[gi + (int64_t)(2 * J) * p.ldr] = re;
+          rowchk[gi + (int64_t)(2 * J + 1) * p.ldr] = rw;
+          if (rowmag) rowmag[gi + (int64_t)J * p.ldrm] = ra;
+        }
       }
       if (sym && (p.which & ABFT_COL)) {
         double m = p.use_mag ? (double)colmag[I + gj * p.ldcm] : (double)ra;
@@ -428,6 +440,11 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
         }
         my_colflags |= f;
         my_symcols += f & 1;
+        if (p.refresh && !(f & 1)) {
+          colchk[(int64_t)2 * I + gj * p.ldc] = re;
+          colchk[(int64_t)2 * I + 1 + gj * p.ldc] = rw;
+          if (colmag) colmag[I + gj * p.ldcm] = ra;
+        }
       }
     }
   }
@@ -552,6 +569,7 @@ static int run_pass(const abft_mat_t* m, const abft_tiles_t* t, int which, const
                 (!(which & ABFT_ROW) || m->rowmag);
     a.tau_fac = m->dtype == ABFT_F64 ? tau_factor<double>((int)m->nb, tol->scale)
                                      : tau_factor<float>((int)m->nb, tol->scale);
+    a.refresh = tol->refresh;
     a.status = rep->status;
     a.ld_status = rep->ld_status;
     a.dcol = rep->dcol;

@@ -71,6 +71,7 @@ struct Driver {
   void* A = nullptr;
   const ft_opts_t* o = nullptr;
   bool lu = false;
+  bool qr = false;
   abft_mat_t M{};
   abft_report_t R{};
   abft_tol_t tol{};
@@ -135,6 +136,7 @@ struct Driver {
     R.counts = counts;
     tol.kind = o->tol_kind;
     tol.scale = o->tol_scale > 0 ? o->tol_scale : 1.0;
+    tol.refresh = o->refresh;
     return 0;
   }
 
@@ -154,7 +156,7 @@ struct Driver {
       if (point == FT_AT_PRE_PD) return gi >= r0 && gj >= r0 && gj < r1;
       if (point == FT_AT_PRE_PU) return gi >= r0 && gi < r1 && gj >= r1;
     }
-    if (point == FT_AT_PRE_TMU) return gi >= r1 && gj >= r1;
+    if (point == FT_AT_PRE_TMU) return gi >= (qr ? r0 : r1) && gj >= r1;
     return false;
   }
   int inject_at(int k, int point) {

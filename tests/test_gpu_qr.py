@@ -1,0 +1,112 @@
+"""GPU parity of ft_geqrf (QR rows of §8 a4–a7: Alg. 1 panel checksums, QR
+TMU rules, Alg. 2 order) against the oracle driver and LAPACK dgeqrf."""
+import numpy as np
+import pytest
+import torch
+
+import synth_inputs as si
+from oracle import drivers as dr
+from tests.gpu_helpers import dev, host
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ctx(lib):
+    return lib.Context()
+
+
+def _gpu_geqrf(lib, ctx, A_np, nb, inject=(), abft=True):
+    A = dev(A_np)
+    n = A.shape[0]
+    tau = torch.zeros(n, dtype=torch.float64, device="cuda")
+    inj = [(f.iter, f.point, f.kind, f.target, f.gi, f.gj, si.mask_of(f.bits)) for f in inject]
+    log = torch.zeros(8192 * lib.FIX_BYTES, dtype=torch.uint8, device="cuda")
+    rc, info, stats = lib.ft_geqrf(ctx, A, nb, tau, abft=abft, inject=inj, fix_log=log)
+    torch.cuda.synchronize()
+    return host(A), tau.cpu().numpy(), rc, info, stats, lib.decode_fixes(log, stats.n_fixes)
+
+
+@pytest.mark.parametrize("n,nb", [(256, 32), (1024, 128), (2048, 256), (2048, 512)])
+def test_error_free_matches_lapack(lib, ctx, n, nb):
+    A = si.general(n, seed=n + 5)
+    H, tau, rc, info, stats, fixes = _gpu_geqrf(lib, ctx, A, nb)
+    h, t = np.linalg.qr(A, mode="raw")
+    h = h.T
+    assert rc == 0 and info == 0 and list(stats.counts) == [0] * 8 and not fixes
+    assert np.abs(H - h).max() <= 1e-12 * np.abs(h).max() * max(1, n // 1024)
+    assert np.abs(tau - t).max() <= 1e-12 * max(1, n // 1024)
+
+
+def test_unprotected_same_factor(lib, ctx):
+    A = si.general(1024, seed=2)
+    a = _gpu_geqrf(lib, ctx, A, 128, abft=False)
+    b = _gpu_geqrf(lib, ctx, A, 128, abft=True)
+    assert np.abs(a[0] - b[0]).max() <= 1e-13 * np.abs(a[0]).max()
+
+
+def _compare(lib, ctx, A, nb, injects):
+    Ho, tauo, so = dr.ft_geqrf(A, nb, inject=injects)
+    Hg, taug, rc, info, sg, fg = _gpu_geqrf(lib, ctx, A, nb, inject=injects)
+    assert (rc == lib.E_UNCORRECTABLE) == (so.uncorrectable > 0)
+    assert sg.repairs_skipped == so.repairs_skipped
+    if so.uncorrectable:
+        return so, sg
+    assert list(sg.counts) == so.counts, (list(sg.counts), so.counts)
+    assert sorted((f[0], f[1], f[4], f[5]) for f in fg) == sorted((f.gi, f.gj, f.cls, f.kind) for f in so.fixes)
+    assert sg.n_checks == so.n_checks
+    h, t = np.linalg.qr(A, mode="raw")
+    assert np.abs(Hg - h.T).max() <= 1e-12 * np.abs(h).max()
+    return so, sg
+
+
+QR_CASES = [
+    (2, dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 0, 100, 70, (61,)),
+    (2, dr.AT_POST_PD, dr.KIND_PERSIST, 0, 150, 80, (62,)),
+    (2, dr.AT_POST_PD, dr.KIND_PERSIST, 0, 66, 90, (58,)),
+    (2, dr.AT_POST_TMU, dr.KIND_PERSIST, 0, 230, 100, (59,)),
+    (2, dr.AT_POST_TMU, dr.KIND_PERSIST, 0, 70, 200, (60,)),
+    (2, dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 170, 80, (54,)),     # consumed V fault -> R
+    (2, dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 1, 9, 75, (61,)),  # column-checksum memory fault
+    (2, dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 2, 100, 5, (61,)),  # row-checksum memory fault
+]
+
+
+@pytest.mark.parametrize("case", range(len(QR_CASES)))
+def test_qr_fault_campaign_parity(lib, ctx, case):
+    k, point, kind, target, gi, gj, bits = QR_CASES[case]
+    A = si.general(256, seed=0)
+    _compare(lib, ctx, A, 32, [dr.Inject(k, point, kind, target, gi, gj, bits)])
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_qr_random_campaign_parity(lib, ctx, seed):
+    g = si.rng(300 + seed)
+    nb, n = 32, 256
+    k = int(g.integers(0, n // nb - 1))
+    point = [dr.AT_PRE_PD_CHECK, dr.AT_POST_PD, dr.AT_POST_TMU][int(g.integers(0, 3))]
+    r0, r1 = k * nb, (k + 1) * nb
+    if point == dr.AT_POST_TMU:
+        gi, gj = int(g.integers(r0, n)), int(g.integers(r1, n))
+    else:
+        gi, gj = int(g.integers(r0, n)), int(g.integers(r0, r1))
+    A = si.general(n, seed=400 + seed)
+    _compare(lib, ctx, A, nb, [dr.Inject(k, point, dr.KIND_PERSIST, 0, gi, gj, (int(g.integers(52, 64)),))])
+
+
+def test_config3_shape_error_free(lib, ctx):
+    """BASELINE configs[2]: fp64 QR n=20480 nb=512 error free; sampled columns
+    of A − Q R (Q from the stored reflectors) — a property at any size."""
+    n, nb = 20480, 512
+    A0 = si.general_device(n, seed=13)
+    A = A0.clone()
+    tau = torch.zeros(n, dtype=torch.float64, device="cuda")
+    rc, info, stats = lib.ft_geqrf(ctx, A, nb, tau)
+    torch.cuda.synchronize()
+    assert rc == 0 and list(stats.counts) == [0] * 8
+    Q = torch.linalg.householder_product(A.contiguous(), tau)
+    g = si.rng(5)
+    cols = torch.tensor(sorted(g.choice(n, 16, replace=False)), device="cuda")
+    R = torch.triu(A)[:, cols]
+    res = (A0[:, cols] - Q @ R).abs().max().item()
+    assert res <= 1e-10 * A0.abs().max().item() * n ** 0.5
