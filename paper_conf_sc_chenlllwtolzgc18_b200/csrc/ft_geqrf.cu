@@ -65,16 +65,29 @@ __global__ void qr_fix_zero_tau_kernel(T* Tm, const T* tau, int nb) {
 
 // Alg. 1 checksum replay, one warp per checksum row rho of the panel's
 // colchk block (2 (nt-k) rows); tile row 0 of the block is the diagonal tile.
+// The row (and its magnitude row) lives in shared memory for the whole
+// recurrence; ZT = Z^T so step j reads row j of Z contiguously.
+constexpr int kReplayWarps = 4;
+
 template <typename T>
-__global__ void qr_replay_kernel(T* ck, int64_t ldc, T* mck, int64_t ldcm, int nrows, const T* panel, int64_t lda,
-                                 const T* tau, const T* Z, int nb) {
-  const int lane = threadIdx.x & 31;
-  const int rho = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
+__global__ void __launch_bounds__(32 * kReplayWarps) qr_replay_kernel(T* ck, int64_t ldc, T* mck, int64_t ldcm,
+                                                                      int nrows, const T* panel, int64_t lda,
+                                                                      const T* tau, const T* ZT, int nb) {
+  extern __shared__ __align__(16) unsigned char rp_sm[];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int rho = blockIdx.x * kReplayWarps + wid;
   if (rho >= nrows) return;
+  T* row = reinterpret_cast<T*>(rp_sm) + (size_t)wid * 2 * nb;
+  T* mrow = row + nb;
   const int I = rho / 2, wt = rho % 2;  // tile row (0 = diagonal tile), weight v1 / v2
   const bool emag = mck && wt == 0;
-  T* ckr = ck + rho;            // ck[rho, c] = ckr[c * ldc]
+  T* ckr = ck + rho;  // ck[rho, c] = ckr[c * ldc]
   T* mr = emag ? mck + I : nullptr;
+  for (int c = lane; c < nb; c += 32) {
+    row[c] = ckr[(int64_t)c * ldc];
+    mrow[c] = emag ? mr[(int64_t)c * ldcm] : T(0);
+  }
+  __syncwarp();
   for (int j = 0; j < nb; ++j) {
     // c_x = ck[rho, j] - W[rho, :j] R[:j, j]  (rows above j are in the diagonal tile)
     T acc = T(0);
@@ -89,22 +102,27 @@ __global__ void qr_replay_kernel(T* ck, int64_t ldc, T* mck, int64_t ldcm, int n
       vck = wj;
       if (emag) mv = I == 0 ? T(1) : T(0);
     } else {
-      const T cx = ckr[(int64_t)j * ldc] - acc;
+      const T cx = row[j] - acc;
       const T den = -t * beta;  // x1 - beta
       vck = (cx - beta * wj) / den;
-      if (emag) mv = (mr[(int64_t)j * ldcm] + fabs(beta) * (I == 0 ? T(1) : T(0))) / fabs(den);
+      if (emag) mv = (mrow[j] + fabs(beta) * (I == 0 ? T(1) : T(0))) / fabs(den);
+      const T* zr = ZT + (int64_t)j * nb;
       for (int c = j + 1 + lane; c < nb; c += 32) {
-        const T z = Z[j + (int64_t)c * nb];
-        ckr[(int64_t)c * ldc] -= vck * z;
-        if (emag) mr[(int64_t)c * ldcm] += mv * fabs(z);
+        const T z = zr[c];
+        row[c] -= vck * z;
+        if (emag) mrow[c] += mv * fabs(z);
       }
     }
     __syncwarp();
     if (lane == 0) {
-      ckr[(int64_t)j * ldc] = vck;
-      if (emag) mr[(int64_t)j * ldcm] = mv;
+      row[j] = vck;
+      mrow[j] = mv;
     }
     __syncwarp();
+  }
+  for (int c = lane; c < nb; c += 32) {
+    ckr[(int64_t)c * ldc] = row[c];
+    if (emag) mr[(int64_t)c * ldcm] = mrow[c];
   }
 }
 
@@ -215,22 +233,29 @@ static int panel_geqrf_t(const abft_mat_t* mat, int k, T* tau, T* Vbuf, T* Tout,
   qr_fix_zero_tau_kernel<T><<<(unsigned)nb, 128, 0, s>>>(Tout, tau, (int)nb);
   ABFT_CUDA_TRY(cudaGetLastError());
   if (!ft) return 0;
-  // Z = T^T (V^T P0): row j = tau_j v_j^T P^(j-1)
-  T* Z = S;  // reuse
+  // Z = T^T (V^T P0): row j = tau_j v_j^T P^(j-1); stored transposed,
+  // ZT = G^T T with G = V^T P0, so the replay reads row j of Z contiguously
+  T* ZT = S;  // reuse
   {
     std::unique_lock<std::mutex> lk;
     cublasHandle_t h = blas_handle(s, lk);
     if (gemmT<T>(h, CUBLAS_OP_T, CUBLAS_OP_N, (int)nb, (int)nb, (int)mk, T(1), Vbuf, (int)mk, P0, (int)mk, T(0), G,
                  (int)nb) ||
-        gemmT<T>(h, CUBLAS_OP_T, CUBLAS_OP_N, (int)nb, (int)nb, (int)nb, T(1), Tout, (int)nb, G, (int)nb, T(0), Z,
+        gemmT<T>(h, CUBLAS_OP_T, CUBLAS_OP_N, (int)nb, (int)nb, (int)nb, T(1), G, (int)nb, Tout, (int)nb, T(0), ZT,
                  (int)nb))
       return ABFT_E_CUBLAS;
   }
   const int nrows = (int)(2 * (nt - k));
   T* ck = reinterpret_cast<T*>(mat->colchk) + 2 * k + r0 * mat->ldc;
   T* mck = mat->colmag ? reinterpret_cast<T*>(mat->colmag) + k + r0 * mat->ldcm : nullptr;
-  qr_replay_kernel<T><<<(unsigned)((nrows + 7) / 8), 256, 0, s>>>(ck, mat->ldc, mck, mat->ldcm, nrows, panel,
-                                                                  mat->lda, tau, Z, (int)nb);
+  const size_t rsm = (size_t)kReplayWarps * 2 * nb * sizeof(T);
+  static bool rattr = false;
+  if (!rattr) {
+    ABFT_CUDA_TRY(cudaFuncSetAttribute(qr_replay_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024));
+    rattr = true;
+  }
+  qr_replay_kernel<T><<<(unsigned)((nrows + kReplayWarps - 1) / kReplayWarps), 32 * kReplayWarps, rsm, s>>>(
+      ck, mat->ldc, mck, mat->ldcm, nrows, panel, mat->lda, tau, ZT, (int)nb);
   ABFT_CUDA_TRY(cudaGetLastError());
   // r(R): r(P) <- Q^T r(P) for the panel's row checksums (m_k x 2)
   {

@@ -16,28 +16,80 @@ __global__ void lu_pivots_kernel(const int32_t* piv_local, int64_t* ipiv_global,
   for (int j = threadIdx.x; j < nb; j += blockDim.x) ipiv_global[j] = r0 + piv_local[j];
 }
 
-// Distinct rows moved by the panel's swaps (c-14b), compacted into rows[],
-// count in *nrows.  One CTA of 1024 threads.
-__global__ void lu_swap_rows_kernel(const int32_t* piv_local, int nb, int64_t r0, int64_t* rows, int32_t* nrows) {
-  __shared__ int64_t cand[2048];
+// The panel's pivot sequence as a permutation of the rows it moves: S (sorted
+// distinct moved rows), src[s] = slot in S of the row whose value ends at
+// S[s] after all nb swaps, tb[T - k] = first slot in tile row T (T = k..nt).
+// One CTA of 1024 threads: bitonic sort in shared memory, then the nb swaps
+// replayed on slot contents by one thread (binary search row -> slot).
+__global__ void __launch_bounds__(1024) lu_perm_kernel(const int32_t* piv_local, int nb, int64_t r0, int nt, int k,
+                                                       int64_t* S, int32_t* src, int32_t* tb, int32_t* nrows) {
+  __shared__ int64_t key[2048];
+  __shared__ int32_t content[2048];
   __shared__ int cnt;
-  if (threadIdx.x == 0) cnt = 0;
-  for (int s = threadIdx.x; s < 2 * nb; s += blockDim.x) {
+  const int tid = threadIdx.x;
+  for (int s = tid; s < 2048; s += blockDim.x) key[s] = INT64_MAX;
+  __syncthreads();
+  // candidates (p and q of every swap with p != q), duplicates kept for now
+  for (int s = tid; s < 2 * nb; s += blockDim.x) {
     const int j = s < nb ? s : s - nb;
     const int64_t p = r0 + j, q = r0 + piv_local[j] - 1;
-    cand[s] = (p == q) ? -1 : (s < nb ? p : q);
+    if (p != q) key[s] = s < nb ? p : q;
   }
   __syncthreads();
-  for (int s = threadIdx.x; s < 2 * nb; s += blockDim.x) {
-    const int64_t r = cand[s];
-    if (r < 0) continue;
-    bool first = true;
-    for (int t = 0; t < s && first; ++t)
-      if (cand[t] == r) first = false;
-    if (first) rows[atomicAdd(&cnt, 1)] = r;
+  for (int size = 2; size <= 2048; size <<= 1)  // bitonic sort ascending
+    for (int stride = size >> 1; stride > 0; stride >>= 1) {
+      for (int i = tid; i < 2048; i += blockDim.x) {
+        const int partner = i ^ stride;
+        if (partner > i) {
+          const bool up = (i & size) == 0;
+          const int64_t a = key[i], b = key[partner];
+          if ((a > b) == up) {
+            key[i] = b;
+            key[partner] = a;
+          }
+        }
+      }
+      __syncthreads();
+    }
+  if (tid == 0) {  // unique + permutation replay (serial, <= 2 nb entries)
+    int n = 0;
+    for (int i = 0; i < 2048 && key[i] != INT64_MAX; ++i)
+      if (n == 0 || key[i] != key[n - 1]) key[n++] = key[i];
+    cnt = n;
+    for (int i = 0; i < n; ++i) content[i] = i;
+    auto slot = [&](int64_t r) {
+      int lo = 0, hi = n - 1;
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (key[mid] < r) lo = mid + 1; else hi = mid;
+      }
+      return lo;
+    };
+    for (int j = 0; j < nb; ++j) {
+      const int64_t p = r0 + j, q = r0 + piv_local[j] - 1;
+      if (p == q) continue;
+      const int a = slot(p), b = slot(q);
+      const int t = content[a];
+      content[a] = content[b];
+      content[b] = t;
+    }
   }
   __syncthreads();
-  if (threadIdx.x == 0) *nrows = cnt;
+  const int n = cnt;
+  for (int s2 = tid; s2 < n; s2 += blockDim.x) {
+    S[s2] = key[s2];
+    src[s2] = content[s2];
+  }
+  for (int T = k + tid; T <= nt; T += blockDim.x) {  // first slot with row >= T*nb
+    const int64_t r = (int64_t)T * nb;
+    int lo = 0, hi = n;
+    while (lo < hi) {
+      const int mid = (lo + hi) >> 1;
+      if (key[mid] < r) lo = mid + 1; else hi = mid;
+    }
+    tb[T - k] = lo;
+  }
+  if (tid == 0) *nrows = n;
 }
 
 // Pre-swap row check: row r of every trailing tile (I = r/nb, J > k) against
@@ -80,66 +132,66 @@ __global__ void lu_row_check_kernel(const T* A, int64_t lda, const T* rowchk, in
   if (!(old & (ABFT_ST_COL | ABFT_ST_ROW))) atomicAdd(&counts[ABFT_CNT_TILES_FLAGGED], 1);
 }
 
-// Row swaps of every column outside the panel (LAPACK laswp) with the c-14
-// column-checksum deltas; panel columns update only their checksums, from the
-// pre-PD copy (swapped progressively).  One thread per matrix column.
+// Row interchanges of every column outside the panel (LAPACK laswp) with
+// the c-14 column-checksum deltas, applied as the net permutation of the moved
+// rows: one CTA per column gathers the moved values into shared memory, the
+// thread of each tile row sums its deltas in slot order (deterministic), then
+// the permuted values are written back.  Panel columns only update their
+// checksums, with values from the pre-PD copy (L430).  Equal to the sequential
+// swap rule in exact arithmetic.
 template <typename T>
-__global__ void lu_swap_cols_kernel(T* A, int64_t lda, int64_t n, int nb, int k, const int32_t* piv_local, T* pcopy,
-                                    int64_t ldp, T* colchk, int64_t ldc, T* colmag, int64_t ldcm) {
+__global__ void __launch_bounds__(256) lu_perm_cols_kernel(T* A, int64_t lda, int nb, int k, int nt, const int64_t* S,
+                                                           const int32_t* src, const int32_t* tb,
+                                                           const int32_t* nrows, const T* pcopy, int64_t ldp,
+                                                           T* colchk, int64_t ldc, T* colmag, int64_t ldcm) {
+  __shared__ T xs[2048];
+  const int64_t c = blockIdx.x;
   const int64_t r0 = (int64_t)k * nb, r1 = r0 + nb;
-  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x) {
-    const bool panel = c >= r0 && c < r1;
-    if (panel && !colchk) continue;  // getrf already swapped the panel; no checksums to move
-    T* col = panel ? pcopy + (c - r0) * ldp - r0 : A + c * lda;  // indexable by global row
-    for (int j = 0; j < nb; ++j) {
-      const int64_t p = r0 + j, q = r0 + piv_local[j] - 1;
-      if (p == q) continue;
-      const T xp = col[p], xq = col[q];
-      if (colchk) {
-        const int64_t P = p / nb, Q = q / nb, pl = p % nb, ql = q % nb;
-        const T d = xq - xp;
-        if (P != Q) {
-          colchk[2 * P + c * ldc] += d;
-          colchk[2 * P + 1 + c * ldc] += T(pl + 1) * d;
-          colchk[2 * Q + c * ldc] -= d;
-          colchk[2 * Q + 1 + c * ldc] -= T(ql + 1) * d;
-          if (colmag) {
-            const T da = fabs(xq) - fabs(xp);
-            colmag[P + c * ldcm] += da;
-            colmag[Q + c * ldcm] -= da;
-          }
-        } else {
-          colchk[2 * P + 1 + c * ldc] += T(pl - ql) * d;
-        }
+  const bool panel = c >= r0 && c < r1;
+  if (panel && !colchk) return;
+  const int n = *nrows;
+  const T* col = panel ? pcopy + (c - r0) * ldp - r0 : A + c * lda;
+  for (int s = threadIdx.x; s < n; s += blockDim.x) xs[s] = col[S[s]];
+  __syncthreads();
+  if (colchk) {
+    for (int T0 = threadIdx.x; T0 < nt - k; T0 += blockDim.x) {
+      const int b = tb[T0], e = tb[T0 + 1];
+      if (b == e) continue;
+      const int64_t base = (int64_t)(k + T0) * nb;
+      T de = T(0), dw = T(0), da = T(0);
+      for (int s = b; s < e; ++s) {
+        const T xn = xs[src[s]], xo = xs[s];
+        const T d = xn - xo;
+        de += d;
+        dw += T(S[s] - base + 1) * d;
+        da += fabs(xn) - fabs(xo);
       }
-      col[p] = xq;
-      col[q] = xp;
+      const int64_t P = k + T0;
+      colchk[2 * P + c * ldc] += de;
+      colchk[2 * P + 1 + c * ldc] += dw;
+      if (colmag) colmag[P + c * ldcm] += da;
     }
   }
+  if (panel) return;  // getrf already permuted the panel data
+  T* colw = A + c * lda;
+  for (int s = threadIdx.x; s < n; s += blockDim.x) colw[S[s]] = xs[src[s]];
 }
 
 // Row checksums (and row magnitudes) move with their rows (tile columns >= k).
 template <typename T>
-__global__ void lu_swap_rowchk_kernel(T* rowchk, int64_t ldr, T* rowmag, int64_t ldrm, int nb, int k, int nt,
-                                      const int32_t* piv_local) {
-  const int64_t r0 = (int64_t)k * nb;
-  for (int J = k + blockIdx.x * blockDim.x + threadIdx.x; J < nt; J += gridDim.x * blockDim.x) {
-    for (int j = 0; j < nb; ++j) {
-      const int64_t p = r0 + j, q = r0 + piv_local[j] - 1;
-      if (p == q) continue;
-      for (int t = 0; t < 2; ++t) {
-        T* e = rowchk + (int64_t)(2 * J + t) * ldr;
-        const T tmp = e[p];
-        e[p] = e[q];
-        e[q] = tmp;
-      }
-      if (rowmag) {
-        T* m = rowmag + (int64_t)J * ldrm;
-        const T tmp = m[p];
-        m[p] = m[q];
-        m[q] = tmp;
-      }
-    }
+__global__ void __launch_bounds__(256) lu_perm_rowchk_kernel(T* rowchk, int64_t ldr, T* rowmag, int64_t ldrm, int k,
+                                                             const int64_t* S, const int32_t* src,
+                                                             const int32_t* nrows) {
+  __shared__ T vs[2048];
+  const int J = k + blockIdx.x;
+  const int n = *nrows;
+  for (int a = 0; a < 3; ++a) {
+    T* arr = a < 2 ? rowchk + (int64_t)(2 * J + a) * ldr : (rowmag ? rowmag + (int64_t)J * ldrm : nullptr);
+    if (!arr) break;
+    for (int s = threadIdx.x; s < n; s += blockDim.x) vs[s] = arr[S[s]];
+    __syncthreads();
+    for (int s = threadIdx.x; s < n; s += blockDim.x) arr[S[s]] = vs[src[s]];
+    __syncthreads();
   }
 }
 
@@ -262,7 +314,9 @@ extern "C" int abft_panel_getrf(const abft_mat_t* mat, int32_t k, int64_t* ipiv,
   const size_t copy_bytes = ft ? (size_t)mk * nb * es : 0;
   const size_t off_piv = (copy_bytes + 255) / 256 * 256;
   const size_t off_rows = off_piv + ((size_t)nb * 4 + 255) / 256 * 256;
-  const size_t off_nrows = off_rows + (size_t)2 * nb * 8;
+  const size_t off_src = off_rows + (size_t)2 * nb * 8;
+  const size_t off_tb = off_src + (size_t)2 * nb * 4;
+  const size_t off_nrows = off_tb + ((size_t)nt + 2) * 4;
   const size_t off_work = (off_nrows + 4 + 255) / 256 * 256;
   void* scr = nullptr;
   FT_TRY(scratch(s, 10, off_work + (size_t)(lwork + 1) * es, &scr));
@@ -270,6 +324,8 @@ extern "C" int abft_panel_getrf(const abft_mat_t* mat, int32_t k, int64_t* ipiv,
   int32_t* piv_local = (int32_t*)(base + off_piv);
   int64_t* rows = (int64_t*)(base + off_rows);
   int32_t* nrows = (int32_t*)(base + off_nrows);
+  int32_t* src = (int32_t*)(base + off_src);
+  int32_t* tb = (int32_t*)(base + off_tb);
   if (ft)
     ABFT_CUDA_TRY(cudaMemcpy2DAsync(base, mk * es, panel, mat->lda * es, mk * es, nb, cudaMemcpyDeviceToDevice, s));
   {
@@ -284,9 +340,9 @@ extern "C" int abft_panel_getrf(const abft_mat_t* mat, int32_t k, int64_t* ipiv,
     if (st != CUSOLVER_STATUS_SUCCESS) return ABFT_E_CUSOLVER;
   }
   lu_pivots_kernel<<<1, 256, 0, s>>>(piv_local, ipiv, (int)nb, r0);
+  lu_perm_kernel<<<1, 1024, 0, s>>>(piv_local, (int)nb, r0, (int)nt, k, rows, src, tb, nrows);
   // c-14b: verify every trailing row a swap will move, fix before swapping
   if (ft && k < nt - 1) {
-    lu_swap_rows_kernel<<<1, 1024, 0, s>>>(piv_local, (int)nb, r0, rows, nrows);
     const int ncols = (int)(nt - k - 1);
     const int64_t items = 2 * nb * ncols;
     const bool use_mag = tol->kind == ABFT_TOL_MAGNITUDE && mat->rowmag;
@@ -306,21 +362,23 @@ extern "C" int abft_panel_getrf(const abft_mat_t* mat, int32_t k, int64_t* ipiv,
   }
   // swaps: data outside the panel + c deltas (panel: from the pre-PD copy)
   if (mat->dtype == ABFT_F64)
-    lu_swap_cols_kernel<double><<<blocks_for(n, 128), 128, 0, s>>>(
-        (double*)A, mat->lda, n, (int)nb, k, piv_local, (double*)base, mk, (double*)mat->colchk, mat->ldc,
-        (double*)mat->colmag, mat->ldcm);
+    lu_perm_cols_kernel<double><<<(unsigned)n, 256, 0, s>>>((double*)A, mat->lda, (int)nb, k, (int)nt, rows, src, tb,
+                                                            nrows, (const double*)base, mk, (double*)mat->colchk,
+                                                            mat->ldc, (double*)mat->colmag, mat->ldcm);
   else
-    lu_swap_cols_kernel<float><<<blocks_for(n, 128), 128, 0, s>>>((float*)A, mat->lda, n, (int)nb, k, piv_local,
-                                                                  (float*)base, mk, (float*)mat->colchk, mat->ldc,
-                                                                  (float*)mat->colmag, mat->ldcm);
+    lu_perm_cols_kernel<float><<<(unsigned)n, 256, 0, s>>>((float*)A, mat->lda, (int)nb, k, (int)nt, rows, src, tb,
+                                                           nrows, (const float*)base, mk, (float*)mat->colchk,
+                                                           mat->ldc, (float*)mat->colmag, mat->ldcm);
   ABFT_CUDA_TRY(cudaGetLastError());
   if (ft) {
     if (mat->dtype == ABFT_F64)
-      lu_swap_rowchk_kernel<double><<<1, 128, 0, s>>>((double*)mat->rowchk, mat->ldr, (double*)mat->rowmag,
-                                                       mat->ldrm, (int)nb, k, (int)nt, piv_local);
+      lu_perm_rowchk_kernel<double><<<(unsigned)(nt - k), 256, 0, s>>>((double*)mat->rowchk, mat->ldr,
+                                                                      (double*)mat->rowmag, mat->ldrm, k, rows, src,
+                                                                      nrows);
     else
-      lu_swap_rowchk_kernel<float><<<1, 128, 0, s>>>((float*)mat->rowchk, mat->ldr, (float*)mat->rowmag, mat->ldrm,
-                                                      (int)nb, k, (int)nt, piv_local);
+      lu_perm_rowchk_kernel<float><<<(unsigned)(nt - k), 256, 0, s>>>((float*)mat->rowchk, mat->ldr,
+                                                                     (float*)mat->rowmag, mat->ldrm, k, rows, src,
+                                                                     nrows);
     ABFT_CUDA_TRY(cudaGetLastError());
   }
   // inverses of the diagonal factors (reused by the PU) and the c-13 PD rules
