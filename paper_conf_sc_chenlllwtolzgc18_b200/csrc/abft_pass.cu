@@ -34,24 +34,35 @@ constexpr int kWarps = kThreads / 32;
 template <typename T, int NB>
 struct PassCfg {
   static constexpr int GC = NB < 64 ? NB : 64;  // group columns (slab granularity)
-  static constexpr int CC_RAW = (32 * 1024) / (NB * (int)sizeof(T));
-  static constexpr int CC = CC_RAW < GC ? CC_RAW : GC;      // columns per stage
+  static constexpr int COL_BYTES = NB * (int)sizeof(T);
+  // ~32 KiB stages, 16 KiB when a column is 8 KiB (nb = 1024 fp64) so that the
+  // ring still holds >= 4 stages within the 2-CTAs-per-SM budget
+  static constexpr int STAGE_TARGET = COL_BYTES >= 8192 ? 16 * 1024 : 32 * 1024;
+  static constexpr int CC_RAW = STAGE_TARGET / COL_BYTES;
+  static constexpr int CC = CC_RAW < GC ? (CC_RAW < 1 ? 1 : CC_RAW) : GC;  // columns per stage
   static constexpr int STAGE_ELEMS = CC * NB;
   static constexpr int STAGE_BYTES = STAGE_ELEMS * (int)sizeof(T);
-  static constexpr int RING_BYTES = NB >= 256 ? 96 * 1024 : 48 * 1024;
+  static constexpr int WPC = 1;  // one warp per column in phase A (columns rotate over warps)
+  // keep the whole CTA <= ~110 KiB (2 CTAs / SM): ring = budget - SYM area
+  static constexpr int SIDE_BYTES = NB * 3 * (int)sizeof(T);
+  static constexpr int RING_BYTES = NB >= 256 ? (96 * 1024 < 108 * 1024 - SIDE_BYTES ? 96 * 1024
+                                                                                        : 108 * 1024 - SIDE_BYTES)
+                                              : 48 * 1024;
   static constexpr int NSTAGE_RAW = RING_BYTES / STAGE_BYTES;
   static constexpr int NSTAGE = NSTAGE_RAW < 2 ? 2 : (NSTAGE_RAW > 8 ? 8 : NSTAGE_RAW);
-  static constexpr int WPC = CC >= kWarps ? 1 : kWarps / CC;  // warps per column (phase A)
   static constexpr int RH = NB / WPC;                         // rows per phase-A warp
   static constexpr int LPR = RH / 32;                         // rows per lane (phase A)
   static constexpr int RPT = NB >= kThreads ? NB / kThreads : 1;  // rows per thread (phase B)
   static constexpr int GROUPS = NB / GC;
+  // phase-A vector width: one 16-B shared load per lane when the column half
+  // spans >= 32 vectors
+  static constexpr int VEC = RH >= 32 * (16 / (int)sizeof(T)) ? 16 / (int)sizeof(T) : 1;
+  static constexpr int KV = RH / (32 * VEC);
   static constexpr size_t SMEM = (size_t)NSTAGE * STAGE_BYTES   // ring
                                  + (size_t)NB * 3 * sizeof(T)   // SYM column accumulators
-                                 + (size_t)WPC * CC * 3 * sizeof(T)  // phase-A partials
-                                 + NSTAGE * sizeof(uint64_t) + 64;
+                                 + 2 * NSTAGE * sizeof(uint64_t) + 64;  // full / empty barriers
   static_assert(CC >= 1 && GC % CC == 0, "stage must divide group");
-  static_assert(RH % 32 == 0, "column half must be a multiple of 32 rows");
+  static_assert(RH % 32 == 0, "a column must be a multiple of 32 rows");
 };
 
 struct PassArgs {
@@ -83,6 +94,23 @@ struct PassArgs {
   int* tflags;      // [ntiles] self-resetting
 };
 
+template <typename T, int VEC>
+__device__ __forceinline__ void load_vec(T (&x)[VEC], const T* p) {
+  if constexpr (VEC == 1) {
+    x[0] = p[0];
+  } else if constexpr (sizeof(T) == 8) {
+    const double2 v = *reinterpret_cast<const double2*>(p);
+    x[0] = v.x;
+    x[1] = v.y;
+  } else {
+    const float4 v = *reinterpret_cast<const float4*>(p);
+    x[0] = v.x;
+    x[1] = v.y;
+    x[2] = v.z;
+    x[3] = v.w;
+  }
+}
+
 template <typename T>
 struct Acc3 {
   T e, w, a;
@@ -103,14 +131,25 @@ __device__ __forceinline__ int check_pair(T me, T mw, T re, T rw, double m, doub
   return (fl ? 1 : 0) | (nf ? 2 : 0);
 }
 
+__device__ __forceinline__ void consumer_sync() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+// 8 consumer warps + 1 producer warp.  The producer's lane 0 streams the
+// unit's stages through the ring (full[] barriers count the TMA bytes); each
+// consumer warp releases a stage through empty[] as soon as it is done with
+// it, so warps never wait for each other inside the stage loop.
+constexpr int kBlock = kThreads + 32;
+
 template <typename T, int NB, bool VERIFY>
-__global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
+__global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
   using C = PassCfg<T, NB>;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   T* ring = reinterpret_cast<T*>(smem_raw);
   T* symacc = ring + (size_t)C::NSTAGE * C::STAGE_ELEMS;  // [3][NB]
-  T* cpart = symacc + 3 * NB;                               // [WPC][CC][3]
-  uint64_t* full = reinterpret_cast<uint64_t*>(cpart + C::WPC * C::CC * 3);
+  uint64_t* full = reinterpret_cast<uint64_t*>(symacc + 3 * NB);
+  uint64_t* empty = full + C::NSTAGE;
   __shared__ int s_colflags, s_ncols, s_nrows, s_last, s_rowflags;
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -139,26 +178,34 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
     s_nrows = 0;
     s_rowflags = 0;
     if (p.use_bulk) {
-      for (int s = 0; s < C::NSTAGE; ++s) mbar_init(&full[s], 1);
+      for (int s = 0; s < C::NSTAGE; ++s) {
+        mbar_init(&full[s], 1);
+        mbar_init(&empty[s], kWarps);
+      }
       mbar_fence_init();
     }
   }
   __syncthreads();
 
-  auto issue = [&](int s) {  // thread 0 only
-    int slot = s % C::NSTAGE;
-    T* dst = ring + (size_t)slot * C::STAGE_ELEMS;
-    fence_proxy_async();
-    mbar_arrive_expect_tx(&full[slot], C::STAGE_BYTES);
-    const T* src = tileA + (int64_t)(c0 + s * C::CC) * p.lda;
+  // ------------------------------------------------------------ producer --
+  if (warp == kWarps) {
+    if (p.use_bulk && lane == 0) {
+      for (int g = 0; g < nst; ++g) {
+        const int slot = g % C::NSTAGE;
+        if (g >= C::NSTAGE) mbar_wait(&empty[slot], (uint32_t)(((g / C::NSTAGE) - 1) & 1));
+        T* dst = ring + (size_t)slot * C::STAGE_ELEMS;
+        fence_proxy_async();
+        mbar_arrive_expect_tx(&full[slot], C::STAGE_BYTES);
+        const T* src = tileA + (int64_t)(c0 + g * C::CC) * p.lda;
 #pragma unroll 1
-    for (int cc = 0; cc < C::CC; ++cc)
-      bulk_g2s(dst + cc * NB, src + (int64_t)cc * p.lda, NB * sizeof(T), &full[slot]);
-  };
-  if (p.use_bulk && tid == 0) {
-    for (int s = 0; s < C::NSTAGE && s < nst; ++s) issue(s);
+        for (int cc = 0; cc < C::CC; ++cc)
+          bulk_g2s(dst + cc * NB, src + (int64_t)cc * p.lda, NB * sizeof(T), &full[slot]);
+      }
+    }
+    return;
   }
 
+  // ----------------------------------------------------------- consumers --
   Acc3<T> grp[C::RPT], tot[C::RPT];
 #pragma unroll
   for (int q = 0; q < C::RPT; ++q) {
@@ -181,7 +228,7 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
       symacc[NB + idx] = colchk[(int64_t)2 * I + 1 + gj * p.ldc];
       if (p.use_mag) symacc[2 * NB + idx] = colmag[I + gj * p.ldcm];
     }
-    __syncthreads();
+    consumer_sync();
   }
   // column finish: encode writes c (and m_c); verify compares (c-6, c-7)
   auto finish_col = [&](int jl, T pe, T pw, T pa) {
@@ -222,36 +269,44 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
     const int slot = s % C::NSTAGE;
     T* buf = ring + (size_t)slot * C::STAGE_ELEMS;
     if (p.use_bulk) {
-      mbar_wait(&full[slot], (s / C::NSTAGE) & 1);
+      mbar_wait(&full[slot], (uint32_t)((s / C::NSTAGE) & 1));
     } else {
+      consumer_sync();  // every warp is done with this slot's previous use
       const T* src = tileA + (int64_t)(c0 + s * C::CC) * p.lda;
       for (int idx = tid; idx < C::STAGE_ELEMS; idx += kThreads) {
         int cc = idx / NB, r = idx % NB;
         buf[idx] = src[(int64_t)cc * p.lda + r];
       }
-      __syncthreads();
+      consumer_sync();
     }
-    // ---------------- phase A: column sums -----------------------------
-    for (int u = warp; u < C::CC * C::WPC; u += kWarps) {
-      const int cc = u % C::CC, h = u / C::CC;
+    // ---------------- phase A: column sums (one warp per column) ----------
+#pragma unroll 1
+    for (int cc = 0; cc < C::CC; ++cc) {
+      if (((s * C::CC + cc) & (kWarps - 1)) != warp) continue;
       const int jl = c0 + s * C::CC + cc;  // tile-local column
-      const T* col = buf + cc * NB + h * C::RH;
+      const T* col = buf + cc * NB;
       T pe = T(0), pw = T(0), pa = T(0);
       if (viewA == ABFT_GENERAL) {
+        // sum_i (i+1) x_i with i = (32k + lane)*VEC + v
+        //   = (lane*VEC + 1) * S0 + sum_{k,v} (32*VEC*k + v) x   (compile-time weights)
+        T s1 = T(0);
 #pragma unroll
-        for (int k = 0; k < C::LPR; ++k) {
-          const int r = lane + 32 * k;
-          T x = col[r];
-          pe = fadd(pe, x);
-          pw = ffma(T(h * C::RH + r + 1), x, pw);
-          pa = fadd(pa, fabs(x));
+        for (int k = 0; k < C::KV; ++k) {
+          T xv[C::VEC];
+          load_vec<T, C::VEC>(xv, col + (32 * k + lane) * C::VEC);
+#pragma unroll
+          for (int v = 0; v < C::VEC; ++v) {
+            pe = fadd(pe, xv[v]);
+            s1 = ffma(T(32 * C::VEC * k + v), xv[v], s1);
+            pa = fadd(pa, fabs(xv[v]));
+          }
         }
+        pw = ffma(T(lane * C::VEC + 1), pe, s1);
       } else {
 #pragma unroll 4
-        for (int k = 0; k < C::LPR; ++k) {
-          const int r = lane + 32 * k;
-          const int i = h * C::RH + r;
-          T x = view_mask(viewA, i, jl, col[r]);
+        for (int k = 0; k < NB / 32; ++k) {
+          const int i = lane + 32 * k;
+          T x = view_mask(viewA, i, jl, col[i]);
           pe = fadd(pe, x);
           pw = ffma(T(i + 1), x, pw);
           pa = fadd(pa, fabs(x));
@@ -263,15 +318,7 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
         pw = fadd(pw, shfl_xor(pw, m));
         pa = fadd(pa, shfl_xor(pa, m));
       }
-      if (C::WPC > 1) {
-        if (lane == 0) {
-          cpart[(h * C::CC + cc) * 3 + 0] = pe;
-          cpart[(h * C::CC + cc) * 3 + 1] = pw;
-          cpart[(h * C::CC + cc) * 3 + 2] = pa;
-        }
-      } else if (lane == 0) {
-        finish_col(jl, pe, pw, pa);
-      }
+      if (lane == 0) finish_col(jl, pe, pw, pa);
     }
     // ---------------- phase B: row sums ---------------------------------
 #pragma unroll
@@ -279,14 +326,18 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
       const int r = tid + q * kThreads;
       if (r < NB) {
         if (view == ABFT_GENERAL) {
+          // sum_cc (jl+1) x with jl = c0 + s*CC + cc  =  (c0 + s*CC + 1) * S0 + sum_cc cc*x
+          T se = T(0), s1 = T(0), sa = T(0);
 #pragma unroll
           for (int cc = 0; cc < C::CC; ++cc) {
-            T x = buf[cc * NB + r];
-            const int jl = c0 + s * C::CC + cc;
-            grp[q].e = fadd(grp[q].e, x);
-            grp[q].w = ffma(T(jl + 1), x, grp[q].w);
-            grp[q].a = fadd(grp[q].a, fabs(x));
+            const T x = buf[cc * NB + r];
+            se = fadd(se, x);
+            s1 = ffma(T(cc), x, s1);
+            sa = fadd(sa, fabs(x));
           }
+          grp[q].e = fadd(grp[q].e, se);
+          grp[q].w = fadd(grp[q].w, ffma(T(c0 + s * C::CC + 1), se, s1));
+          grp[q].a = fadd(grp[q].a, sa);
         } else {
           for (int cc = 0; cc < C::CC; ++cc) {
             const int jl = c0 + s * C::CC + cc;
@@ -298,6 +349,11 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
           }
         }
       }
+    }
+    // stage consumed by this warp: release the slot to the producer
+    if (p.use_bulk) {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[slot]);
     }
     const bool group_end = (((s + 1) * C::CC) % C::GC) == 0;
     if (group_end) {
@@ -320,21 +376,6 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
         grp[q] = {T(0), T(0), T(0)};
       }
     }
-    __syncthreads();  // stage consumed (and cpart visible)
-    if (C::WPC > 1 && tid < C::CC) {
-      const int cc = tid;
-      const int jl = c0 + s * C::CC + cc;
-      T pe = cpart[cc * 3 + 0], pw = cpart[cc * 3 + 1], pa = cpart[cc * 3 + 2];
-#pragma unroll
-      for (int h = 1; h < C::WPC; ++h) {
-        pe = fadd(pe, cpart[(h * C::CC + cc) * 3 + 0]);
-        pw = fadd(pw, cpart[(h * C::CC + cc) * 3 + 1]);
-        pa = fadd(pa, cpart[(h * C::CC + cc) * 3 + 2]);
-      }
-      finish_col(jl, pe, pw, pa);
-    }
-    if (C::WPC > 1) __syncthreads();  // cpart reusable
-    if (p.use_bulk && tid == 0 && s + C::NSTAGE < nst) issue(s + C::NSTAGE);
   }
 
   // ---------------- column flags of this CTA ------------------------------
@@ -345,14 +386,14 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
   // ---------------- slab reduction: last CTA finishes the tile ------------
   if (nslab > 1) {
     __threadfence();
-    __syncthreads();
+    consumer_sync();
     if (tid == 0) {
       if (VERIFY && s_colflags) atomicOr(&p.tflags[tile], s_colflags);
       __threadfence();
       int old = atomicAdd(&p.ticket[tile], 1);
       s_last = (old == nslab - 1);
     }
-    __syncthreads();
+    consumer_sync();
     if (VERIFY && tid == 0 && s_ncols) atomicAdd(&p.counts[ABFT_CNT_COLS_FLAGGED], s_ncols);
     if (!s_last) return;
     __threadfence();
@@ -373,7 +414,7 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
       p.ticket[tile] = 0;
     }
   } else {
-    __syncthreads();
+    consumer_sync();
     if (VERIFY && tid == 0 && s_ncols) atomicAdd(&p.counts[ABFT_CNT_COLS_FLAGGED], s_ncols);
   }
 
@@ -457,7 +498,7 @@ __global__ void __launch_bounds__(kThreads) checksum_pass_kernel(PassArgs p) {
       atomicAdd(&s_ncols, my_symcols);
     }
   }
-  __syncthreads();
+  consumer_sync();
   if (tid == 0) {
     int cf = s_colflags, rf = s_rowflags;
     int st = ((cf & 1) ? ABFT_ST_COL : 0) | ((rf & 1) ? ABFT_ST_ROW : 0) | (((cf | rf) & 2) ? ABFT_ST_NONFINITE : 0);
@@ -504,7 +545,7 @@ static int launch_nb(PassArgs& a, int64_t ntiles, cudaStream_t s) {
     a.tflags = ctr + ntiles;
   }
   dim3 grid((unsigned)(ntiles * nslab));
-  kern<<<grid, kThreads, C::SMEM, s>>>(a);
+  kern<<<grid, kBlock, C::SMEM, s>>>(a);
   ABFT_CUDA_TRY(cudaGetLastError());
   return 0;
 }
