@@ -64,55 +64,75 @@ def ncu_traffic():
 
 
 class Clocks:
-    """nvidia-smi sampling during the timed region (B200_PROFILING.md)."""
+    """SM clock and clock-event (throttle) reasons sampled DURING the timed
+    region (B200_PROFILING.md clocks line) by an NVML polling thread (1 ms),
+    so even a ~20 ms timed region yields a few dozen samples; falls back to
+    one nvidia-smi query if NVML is unavailable."""
+
+    REASONS = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown", 0x4: "sw_power_cap"}
 
     def __init__(self, dev):
         self.dev = dev
-        self.proc = None
-        self.path = f"/tmp/bench_clocks_{os.getpid()}.csv"
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = False
+        self._t = None
+
+    def _nvml_index(self):
+        vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+        if vis:
+            ids = [v.strip() for v in vis.split(",") if v.strip()]
+            if self.dev < len(ids) and ids[self.dev].isdigit():
+                return int(ids[self.dev])
+        return self.dev
+
+    def _run(self):
+        import pynvml
+
+        h = pynvml.nvmlDeviceGetHandleByIndex(self._nvml_index())
+        self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+        get_reasons = getattr(pynvml, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+            pynvml.nvmlDeviceGetCurrentClocksThrottleReasons
+        while not self._stop:
+            self.samples.append(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM))
+            r = get_reasons(h)
+            for bit, name in self.REASONS.items():
+                if r & bit:
+                    self.reasons.add(name)
+            time.sleep(0.001)
 
     def __enter__(self):
-        q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
-             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-             "clocks_event_reasons.sw_power_cap")
+        import threading
+
         try:
-            self.f = open(self.path, "w")
-            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.dev), f"--query-gpu={q}",
-                                          "--format=csv,noheader,nounits", "-lms", "200"],
-                                         stdout=self.f, stderr=subprocess.DEVNULL)
+            import pynvml
+
+            pynvml.nvmlInit()
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+            t0 = time.time()
+            while not self.samples and time.time() - t0 < 2.0:  # sampler live before timing starts
+                time.sleep(0.001)
         except Exception:
-            self.proc = None
+            self._t = None
         return self
 
     def __exit__(self, *a):
-        if self.proc:
-            self.proc.terminate()
-            try:
-                self.proc.wait(timeout=5)
-            except Exception:
-                self.proc.kill()
-            self.f.close()
+        self._stop = True
+        if self._t:
+            self._t.join(timeout=2)
 
     def summary(self):
-        try:
-            rows = [r.split(",") for r in open(self.path).read().strip().splitlines()]
-        except Exception:
-            return None
-        sm, mx, reasons = [], 0.0, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for r in rows:
+        if not self.samples:
             try:
-                sm.append(float(r[0]))
-                mx = max(mx, float(r[1]))
-                for nm, v in zip(names, r[3:7]):
-                    if v.strip().lower() == "active":
-                        reasons.add(nm)
+                out = subprocess.run(["nvidia-smi", "-i", str(self.dev), "--query-gpu=clocks.sm,clocks.max.sm",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=10)
+                sm, mx = [float(x) for x in out.stdout.strip().split(",")[:2]]
+                return {"sm_mhz": sm, "sm_max_mhz": mx, "reasons": [], "samples": 1, "source": "nvidia-smi after"}
             except Exception:
-                continue
-        if not sm:
-            return None
-        sm.sort()
-        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+                return None
+        sm = sorted(self.samples)
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                "samples": len(sm), "source": "nvml 1 ms during the timed region"}
 
 
 # ------------------------------------------------------------- reference --
@@ -323,12 +343,12 @@ def potrf_overhead(abft, si, n, nb, reps):
     A = torch.empty_like(A0.t()).t()
     ctx = abft.Context()
 
-    def run(ft):
+    def run(ft, restart=True):
         A.copy_(A0)
         torch.cuda.synchronize()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record()
-        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft)
+        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart)
         b.record()
         torch.cuda.synchronize()
         assert rc == 0 and info == 0
@@ -336,15 +356,18 @@ def potrf_overhead(abft, si, n, nb, reps):
 
     run(True)
     run(False)
-    t_ft, t_plain = [], []
+    t_ft, t_plain, t_nors = [], [], []
     for _ in range(reps):
         t_plain.append(run(False)[0])
         t, st = run(True)
         t_ft.append(t)
         assert sum(st.counts) == 0
+        t_nors.append(run(True, restart=False)[0])
     t_ft.sort()
     t_plain.sort()
+    t_nors.sort()
     ft_ms, plain_ms = t_ft[len(t_ft) // 2], t_plain[len(t_plain) // 2]
+    nors_ms = t_nors[len(t_nors) // 2]
     # cuSOLVER dpotrf of the whole matrix (context)
     S = A0.t().contiguous()
     torch.backends.cuda.preferred_linalg_library("cusolver")
@@ -360,6 +383,7 @@ def potrf_overhead(abft, si, n, nb, reps):
     torch.cuda.empty_cache()
     return {"n": n, "nb": nb, "ms_ft": ft_ms, "ms_plain": plain_ms,
             "overhead_pct": 100.0 * (ft_ms - plain_ms) / plain_ms, "cusolver_potrf_ms": cus,
+            "ms_ft_no_restart": nors_ms, "overhead_pct_no_restart": 100.0 * (nors_ms - plain_ms) / plain_ms,
             "tflops_ft": n ** 3 / 3 / (ft_ms / 1e3) / 1e12, "reps": reps}
 
 

@@ -328,6 +328,9 @@ typedef struct {
   int32_t pu_gemm;       /* 1: PU as L21 = A21 * L_kk^-T (DGEMM with the PD's explicit inverse) in
                             both the protected and the unprotected driver; 0: cuBLAS DTRSM */
   int32_t refresh;       /* abft_tol_t.refresh for every check of the run (default 1) */
+  int32_t restart;       /* 1: local restart (L430): copy the PD / PU input with its checksums after the
+                            pre-op check; a 2D error left by the post-op check restores the copy and
+                            redoes the op once (one 8-byte read-back per check; ft_potrf) */
 } ft_opts_t;
 
 /* Host-side statistics, filled after the driver's final synchronisation. */
@@ -339,6 +342,7 @@ typedef struct {
   int32_t uncorrectable;        /* tiles left 2D (-> ABFT_E_UNCORRECTABLE) */
   int32_t n_checks;             /* verify calls issued */
   double ms_total;
+  int32_t restarts;             /* local restarts performed (f1) */
 } ft_stats_t;
 
 ABFT_API int ft_ctx_create(ft_ctx_t **ctx, int32_t device, abft_stream_t stream);

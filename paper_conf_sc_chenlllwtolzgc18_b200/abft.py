@@ -78,13 +78,13 @@ class ft_opts_t(C.Structure):
     _fields_ = [("nb", C.c_int64), ("abft", C.c_int32), ("tol_kind", C.c_int32), ("tol_scale", C.c_double),
                 ("fig4a_repair", C.c_int32), ("n_inject", C.c_int32), ("inject", C.POINTER(ft_inject_t)),
                 ("fix_log", C.c_void_p), ("fix_log_cap", C.c_int32), ("pu_gemm", C.c_int32),
-                ("refresh", C.c_int32)]
+                ("refresh", C.c_int32), ("restart", C.c_int32)]
 
 
 class ft_stats_t(C.Structure):
     _fields_ = [("counts", C.c_int32 * NCOUNTS), ("n_fixes", C.c_int32), ("repairs_applied", C.c_int32),
                 ("repairs_skipped", C.c_int32), ("uncorrectable", C.c_int32), ("n_checks", C.c_int32),
-                ("ms_total", C.c_double)]
+                ("ms_total", C.c_double), ("restarts", C.c_int32)]
 
 
 _L = _lib.load()
@@ -339,13 +339,13 @@ class Context:
             self._h = None
 
 
-def _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh=True):
+def _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh=True, restart=True):
     inj = (ft_inject_t * max(1, len(inject)))()
     for k, f in enumerate(inject):
         inj[k] = ft_inject_t(*f)
     opts = ft_opts_t(nb, int(abft), tol_kind, tol_scale, int(fig4a_repair), len(inject), inj,
                      _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES, int(pu_gemm),
-                     int(refresh))
+                     int(refresh), int(restart))
     return opts, inj
 
 
@@ -396,11 +396,11 @@ def ft_geqrf(ctx: Context, A: torch.Tensor, nb: int, tau: torch.Tensor, abft=Tru
 
 
 def ft_potrf(ctx: Context, A: torch.Tensor, nb: int, abft=True, tol_kind=TOL_MAGNITUDE, tol_scale=1.0,
-             fig4a_repair=True, inject=(), fix_log=None, pu_gemm=True, refresh=True):
+             fig4a_repair=True, inject=(), fix_log=None, pu_gemm=True, refresh=True, restart=True):
     """Fault-tolerant lower Cholesky in place on a column-major A.  Returns
     (rc, info, stats) with rc 0 or E_UNCORRECTABLE (other codes raise)."""
     n = A.shape[0]
-    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh)
+    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh, restart)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_potrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), C.byref(opts), C.byref(stats), C.byref(info))

@@ -31,38 +31,51 @@ namespace abft {
 constexpr int kThreads = 256;
 constexpr int kWarps = kThreads / 32;
 
-template <typename T, int NB>
+// NB = checksum tile; K = vertically adjacent tiles streamed by one CTA
+// (K > 1 for small tiles: one K*NB-row bulk copy per column and a K-times
+// longer CTA lifetime; GENERAL views only).
+template <typename T, int NB, int K>
 struct PassCfg {
+  static constexpr int RK = K * NB;              // rows per CTA
   static constexpr int GC = NB < 64 ? NB : 64;  // group columns (slab granularity)
-  static constexpr int COL_BYTES = NB * (int)sizeof(T);
-  // ~32 KiB stages, 16 KiB when a column is 8 KiB (nb = 1024 fp64) so that the
-  // ring still holds >= 4 stages within the 2-CTAs-per-SM budget
+  static constexpr int COL_BYTES = RK * (int)sizeof(T);
+  // ~32 KiB stages, 16 KiB when a column is 8 KiB so that the ring still
+  // holds >= 4 stages within the 2-CTAs-per-SM budget
   static constexpr int STAGE_TARGET = COL_BYTES >= 8192 ? 16 * 1024 : 32 * 1024;
   static constexpr int CC_RAW = STAGE_TARGET / COL_BYTES;
   static constexpr int CC = CC_RAW < GC ? (CC_RAW < 1 ? 1 : CC_RAW) : GC;  // columns per stage
-  static constexpr int STAGE_ELEMS = CC * NB;
+  static constexpr int STAGE_ELEMS = CC * RK;
   static constexpr int STAGE_BYTES = STAGE_ELEMS * (int)sizeof(T);
-  static constexpr int WPC = 1;  // one warp per column in phase A (columns rotate over warps)
-  // keep the whole CTA <= ~110 KiB (2 CTAs / SM): ring = budget - SYM area
-  static constexpr int SIDE_BYTES = NB * 3 * (int)sizeof(T);
-  static constexpr int RING_BYTES = NB >= 256 ? (96 * 1024 < 108 * 1024 - SIDE_BYTES ? 96 * 1024
+  // keep the whole CTA <= ~110 KiB (2 CTAs / SM): ring = budget - side area
+  static constexpr int SIDE_BYTES = RK * 3 * (int)sizeof(T);
+  static constexpr int RING_BYTES = RK >= 256 ? (96 * 1024 < 108 * 1024 - SIDE_BYTES ? 96 * 1024
                                                                                         : 108 * 1024 - SIDE_BYTES)
                                               : 48 * 1024;
   static constexpr int NSTAGE_RAW = RING_BYTES / STAGE_BYTES;
   static constexpr int NSTAGE = NSTAGE_RAW < 2 ? 2 : (NSTAGE_RAW > 8 ? 8 : NSTAGE_RAW);
-  static constexpr int RH = NB / WPC;                         // rows per phase-A warp
-  static constexpr int LPR = RH / 32;                         // rows per lane (phase A)
-  static constexpr int RPT = NB >= kThreads ? NB / kThreads : 1;  // rows per thread (phase B)
+  static constexpr int RPT = RK >= kThreads ? RK / kThreads : 1;  // rows per thread (phase B)
   static constexpr int GROUPS = NB / GC;
-  // phase-A vector width: one 16-B shared load per lane when the column half
-  // spans >= 32 vectors
-  static constexpr int VEC = RH >= 32 * (16 / (int)sizeof(T)) ? 16 / (int)sizeof(T) : 1;
-  static constexpr int KV = RH / (32 * VEC);
+  // phase-A vector width: one 16-B shared load per lane when a tile column
+  // spans >= 32 vectors (and a vector never straddles two tiles)
+  static constexpr int VEC = NB >= 32 * (16 / (int)sizeof(T)) ? 16 / (int)sizeof(T) : 1;
+  static constexpr int KV = RK / (32 * VEC);   // vector loads per lane per column
+  static constexpr int KPT = NB / (32 * VEC);  // ... of them per tile
+  // Canonical row-sum chunk: the stage width of the deepest stacking used for
+  // this (T, NB).  Row sums are accumulated per CQ-column chunk whatever K and
+  // CC are, so every launch shape gives bit-identical checksums.
+  static constexpr int KBIG_RAW = 4096 / (NB * (int)sizeof(T));
+  static constexpr int KBIG = KBIG_RAW < 1 ? 1 : (KBIG_RAW > 8 ? 8 : KBIG_RAW);
+  static constexpr int COLB_BIG = KBIG * NB * (int)sizeof(T);
+  static constexpr int CC_BIG_RAW = (COLB_BIG >= 8192 ? 16 * 1024 : 32 * 1024) / COLB_BIG;
+  static constexpr int CQ = CC_BIG_RAW < GC ? (CC_BIG_RAW < 1 ? 1 : CC_BIG_RAW) : GC;
+  static_assert(CC % CQ == 0, "row-sum chunk must divide the stage");
   static constexpr size_t SMEM = (size_t)NSTAGE * STAGE_BYTES   // ring
-                                 + (size_t)NB * 3 * sizeof(T)   // SYM column accumulators
+                                 + (size_t)RK * 3 * sizeof(T)   // SYM sums / maintained column checksums
                                  + 2 * NSTAGE * sizeof(uint64_t) + 64;  // full / empty barriers
   static_assert(CC >= 1 && GC % CC == 0, "stage must divide group");
-  static_assert(RH % 32 == 0, "a column must be a multiple of 32 rows");
+  static_assert(NB % 32 == 0, "a tile column must be a multiple of 32 rows");
+  static_assert(K == 1 || NB % (32 * VEC) == 0, "stacked tiles need whole vectors per tile");
+  static_assert(K <= 8, "at most 8 stacked tiles");
 };
 
 struct PassArgs {
@@ -88,9 +101,10 @@ struct PassArgs {
   void* dcol;
   void* drow;
   int32_t* counts;
-  void* part;       // [ntiles][GROUPS][NB][3] (slabbed tiles only)
+  int K;            // tiles per unit (vertical stack), see PassCfg
+  void* part;       // [nsuper][GROUPS][K*NB][3] (slabbed units only)
   void* symws;      // [ntiles][3][NB] SYM column sums of slabbed diagonal tiles
-  int* ticket;      // [ntiles] self-resetting
+  int* ticket;      // [nsuper] self-resetting
   int* tflags;      // [ntiles] self-resetting
 };
 
@@ -142,41 +156,57 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 // it, so warps never wait for each other inside the stage loop.
 constexpr int kBlock = kThreads + 32;
 
-template <typename T, int NB, bool VERIFY>
+// Unit decode: K == 1 follows the tile enumeration (lower_only aware); K > 1
+// stacks K consecutive tile rows of one tile column (rectangular ranges only).
+__device__ __forceinline__ void super_of(const abft_tiles_t& t, int K, int64_t su, int& Ib, int& J) {
+  if (K == 1) {
+    tile_of(t, su, Ib, J);
+    return;
+  }
+  const int64_t nIk = (t.I1 - t.I0) / K;
+  J = t.J0 + (int)(su / nIk);
+  Ib = t.I0 + (int)(su % nIk) * K;
+}
+
+template <typename T, int NB, int K, bool VERIFY>
 __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
-  using C = PassCfg<T, NB>;
+  using C = PassCfg<T, NB, K>;
+  constexpr int RK = C::RK;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   T* ring = reinterpret_cast<T*>(smem_raw);
-  T* symacc = ring + (size_t)C::NSTAGE * C::STAGE_ELEMS;  // [3][NB]
-  uint64_t* full = reinterpret_cast<uint64_t*>(symacc + 3 * NB);
+  T* symacc = ring + (size_t)C::NSTAGE * C::STAGE_ELEMS;  // [K][3][NB]
+  uint64_t* full = reinterpret_cast<uint64_t*>(symacc + 3 * RK);
   uint64_t* empty = full + C::NSTAGE;
-  __shared__ int s_colflags, s_ncols, s_nrows, s_last, s_rowflags;
+  __shared__ int s_colflags[K], s_ncols[K], s_nrows[K], s_rowflags[K];
+  __shared__ int s_last;
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int64_t unit = blockIdx.x;
-  const int64_t tile = unit / p.nslab;
+  const int64_t sup = unit / p.nslab;
   const int slab = (int)(unit % p.nslab);
-  int I, J;
-  tile_of(p.tiles, tile, I, J);
-  const int view = (I == J) ? p.tiles.diag_view : ABFT_GENERAL;
+  int Ib, J;
+  super_of(p.tiles, K, sup, Ib, J);
+  const int view = (K == 1 && Ib == J) ? p.tiles.diag_view : ABFT_GENERAL;
   const bool sym = view == ABFT_SYM_LOWER;
   const int nslab = p.nslab;
   // SYM column sums of a split tile go through the workspace (the finishing
   // CTA adds them to the row sums); an unsplit tile keeps them in smem
-  T* symcol = (sym && nslab > 1) ? reinterpret_cast<T*>(p.symws) + (size_t)tile * NB * 3 : symacc;
+  T* symcol = (sym && nslab > 1) ? reinterpret_cast<T*>(p.symws) + (size_t)sup * NB * 3 : symacc;
   const int cols = NB / nslab;
   const int c0 = slab * cols;
   const int nst = cols / C::CC;
   const T* A = reinterpret_cast<const T*>(p.A);
-  const T* tileA = A + (int64_t)J * NB * p.lda + (int64_t)I * NB;
+  const T* tileA = A + (int64_t)J * NB * p.lda + (int64_t)Ib * NB;
   // phase-A and phase-B masks: SYM uses LOWER for columns, strict lower for rows
   const int viewA = sym ? ABFT_LOWER : view;
 
   if (tid == 0) {
-    s_colflags = 0;
-    s_ncols = 0;
-    s_nrows = 0;
-    s_rowflags = 0;
+    for (int t = 0; t < K; ++t) {
+      s_colflags[t] = 0;
+      s_ncols[t] = 0;
+      s_nrows[t] = 0;
+      s_rowflags[t] = 0;
+    }
     if (p.use_bulk) {
       for (int s = 0; s < C::NSTAGE; ++s) {
         mbar_init(&full[s], 1);
@@ -199,7 +229,7 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
         const T* src = tileA + (int64_t)(c0 + g * C::CC) * p.lda;
 #pragma unroll 1
         for (int cc = 0; cc < C::CC; ++cc)
-          bulk_g2s(dst + cc * NB, src + (int64_t)cc * p.lda, NB * sizeof(T), &full[slot]);
+          bulk_g2s(dst + cc * RK, src + (int64_t)cc * p.lda, RK * sizeof(T), &full[slot]);
       }
     }
     return;
@@ -216,22 +246,29 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
   T* colchk = reinterpret_cast<T*>(p.colchk);
   T* colmag = reinterpret_cast<T*>(p.colmag);
   T* dcol = reinterpret_cast<T*>(p.dcol);
-  int my_colflags = 0, my_ncols = 0;
+  int my_colflags[K], my_ncols[K];
+#pragma unroll
+  for (int t = 0; t < K; ++t) {
+    my_colflags[t] = 0;
+    my_ncols[t] = 0;
+  }
   // verify: fetch the maintained column checksums (and magnitudes) of this
   // slab once, while the TMA prologue is in flight, instead of one dependent
   // strided load per column inside the stage loop.  For non-SYM tiles the
-  // SYM accumulator area is free and holds them: [e | w | mag] x cols.
+  // SYM area is free and holds them: per tile [e | w | mag] x cols.
   if (VERIFY && !sym && (p.which & ABFT_COL)) {
-    for (int idx = tid; idx < cols; idx += kThreads) {
-      const int64_t gj = (int64_t)J * NB + c0 + idx;
-      symacc[idx] = colchk[(int64_t)2 * I + gj * p.ldc];
-      symacc[NB + idx] = colchk[(int64_t)2 * I + 1 + gj * p.ldc];
-      if (p.use_mag) symacc[2 * NB + idx] = colmag[I + gj * p.ldcm];
+    for (int idx = tid; idx < K * cols; idx += kThreads) {
+      const int t = idx / cols, c = idx - t * cols;
+      const int64_t gj = (int64_t)J * NB + c0 + c;
+      T* sa = symacc + (size_t)t * 3 * NB;
+      sa[c] = colchk[(int64_t)2 * (Ib + t) + gj * p.ldc];
+      sa[NB + c] = colchk[(int64_t)2 * (Ib + t) + 1 + gj * p.ldc];
+      if (p.use_mag) sa[2 * NB + c] = colmag[(Ib + t) + gj * p.ldcm];
     }
     consumer_sync();
   }
-  // column finish: encode writes c (and m_c); verify compares (c-6, c-7)
-  auto finish_col = [&](int jl, T pe, T pw, T pa) {
+  // column finish of tile row Ib+t: encode writes c (and m_c); verify compares (c-6, c-7)
+  auto finish_col = [&](int t, int jl, T pe, T pw, T pa) {
     if (sym) {
       symcol[jl] = pe;
       symcol[NB + jl] = pw;
@@ -239,6 +276,7 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
       return;
     }
     if (!(p.which & ABFT_COL)) return;
+    const int I = Ib + t;
     const int64_t gj = (int64_t)J * NB + jl;
     if (!VERIFY) {
       T* cc2 = colchk + (int64_t)2 * I + gj * p.ldc;
@@ -247,15 +285,16 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
       if (colmag) colmag[I + gj * p.ldcm] = pa;
     } else {
       const int idx = jl - c0;
-      double m = p.use_mag ? (double)symacc[2 * NB + idx] : (double)pa;
+      const T* sa = symacc + (size_t)t * 3 * NB;
+      double m = p.use_mag ? (double)sa[2 * NB + idx] : (double)pa;
       T de, dw;
-      int f = check_pair<T>(symacc[idx], symacc[NB + idx], pe, pw, m, p.tau_fac, NB, &de, &dw);
+      int f = check_pair<T>(sa[idx], sa[NB + idx], pe, pw, m, p.tau_fac, NB, &de, &dw);
       if (dcol) {
         dcol[(int64_t)2 * I + gj * p.ldc] = de;
         dcol[(int64_t)2 * I + 1 + gj * p.ldc] = dw;
       }
-      my_colflags |= f;
-      my_ncols += f & 1;
+      my_colflags[t] |= f;
+      my_ncols[t] += f & 1;
       if (p.refresh && !(f & 1)) {
         T* cc2 = colchk + (int64_t)2 * I + gj * p.ldc;
         cc2[0] = pe;
@@ -274,7 +313,7 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
       consumer_sync();  // every warp is done with this slot's previous use
       const T* src = tileA + (int64_t)(c0 + s * C::CC) * p.lda;
       for (int idx = tid; idx < C::STAGE_ELEMS; idx += kThreads) {
-        int cc = idx / NB, r = idx % NB;
+        int cc = idx / RK, r = idx % RK;
         buf[idx] = src[(int64_t)cc * p.lda + r];
       }
       consumer_sync();
@@ -284,25 +323,41 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
     for (int cc = 0; cc < C::CC; ++cc) {
       if (((s * C::CC + cc) & (kWarps - 1)) != warp) continue;
       const int jl = c0 + s * C::CC + cc;  // tile-local column
-      const T* col = buf + cc * NB;
-      T pe = T(0), pw = T(0), pa = T(0);
+      const T* col = buf + cc * RK;
       if (viewA == ABFT_GENERAL) {
-        // sum_i (i+1) x_i with i = (32k + lane)*VEC + v
-        //   = (lane*VEC + 1) * S0 + sum_{k,v} (32*VEC*k + v) x   (compile-time weights)
-        T s1 = T(0);
+        // per tile t: sum_i (i+1) x_i with i = (32k' + lane)*VEC + v (k' = k - t*KPT)
+        //   = (lane*VEC + 1) * S0 + sum (32*VEC*k' + v) x   (compile-time weights)
+        T pe[K], s1[K], pa[K];
+#pragma unroll
+        for (int t = 0; t < K; ++t) pe[t] = s1[t] = pa[t] = T(0);
 #pragma unroll
         for (int k = 0; k < C::KV; ++k) {
+          constexpr int dummy = 0;
+          (void)dummy;
+          const int t = k / C::KPT;
+          const int kl = k - t * C::KPT;
           T xv[C::VEC];
           load_vec<T, C::VEC>(xv, col + (32 * k + lane) * C::VEC);
 #pragma unroll
           for (int v = 0; v < C::VEC; ++v) {
-            pe = fadd(pe, xv[v]);
-            s1 = ffma(T(32 * C::VEC * k + v), xv[v], s1);
-            pa = fadd(pa, fabs(xv[v]));
+            pe[t] = fadd(pe[t], xv[v]);
+            s1[t] = ffma(T(32 * C::VEC * kl + v), xv[v], s1[t]);
+            pa[t] = fadd(pa[t], fabs(xv[v]));
           }
         }
-        pw = ffma(T(lane * C::VEC + 1), pe, s1);
-      } else {
+#pragma unroll
+        for (int t = 0; t < K; ++t) {
+          T e = pe[t], w = ffma(T(lane * C::VEC + 1), pe[t], s1[t]), a2 = pa[t];
+#pragma unroll
+          for (int m = 16; m >= 1; m >>= 1) {
+            e = fadd(e, shfl_xor(e, m));
+            w = fadd(w, shfl_xor(w, m));
+            a2 = fadd(a2, shfl_xor(a2, m));
+          }
+          if (lane == t) finish_col(t, jl, e, w, a2);  // tiles finished by different lanes in parallel
+        }
+      } else {  // masked diagonal views (K == 1 only)
+        T pe = T(0), pw = T(0), pa = T(0);
 #pragma unroll 4
         for (int k = 0; k < NB / 32; ++k) {
           const int i = lane + 32 * k;
@@ -311,37 +366,40 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
           pw = ffma(T(i + 1), x, pw);
           pa = fadd(pa, fabs(x));
         }
-      }
 #pragma unroll
-      for (int m = 16; m >= 1; m >>= 1) {
-        pe = fadd(pe, shfl_xor(pe, m));
-        pw = fadd(pw, shfl_xor(pw, m));
-        pa = fadd(pa, shfl_xor(pa, m));
+        for (int m = 16; m >= 1; m >>= 1) {
+          pe = fadd(pe, shfl_xor(pe, m));
+          pw = fadd(pw, shfl_xor(pw, m));
+          pa = fadd(pa, shfl_xor(pa, m));
+        }
+        if (lane == 0) finish_col(0, jl, pe, pw, pa);
       }
-      if (lane == 0) finish_col(jl, pe, pw, pa);
     }
     // ---------------- phase B: row sums ---------------------------------
 #pragma unroll
     for (int q = 0; q < C::RPT; ++q) {
       const int r = tid + q * kThreads;
-      if (r < NB) {
+      if (r < RK) {
         if (view == ABFT_GENERAL) {
-          // sum_cc (jl+1) x with jl = c0 + s*CC + cc  =  (c0 + s*CC + 1) * S0 + sum_cc cc*x
-          T se = T(0), s1 = T(0), sa = T(0);
+          // per CQ-column chunk: sum (jl+1) x with jl = base + cq  =  (base + 1) * S0 + sum_cq cq*x
 #pragma unroll
-          for (int cc = 0; cc < C::CC; ++cc) {
-            const T x = buf[cc * NB + r];
-            se = fadd(se, x);
-            s1 = ffma(T(cc), x, s1);
-            sa = fadd(sa, fabs(x));
+          for (int ch = 0; ch < C::CC / C::CQ; ++ch) {
+            T se = T(0), s1 = T(0), sa = T(0);
+#pragma unroll
+            for (int cq = 0; cq < C::CQ; ++cq) {
+              const T x = buf[(ch * C::CQ + cq) * RK + r];
+              se = fadd(se, x);
+              s1 = ffma(T(cq), x, s1);
+              sa = fadd(sa, fabs(x));
+            }
+            grp[q].e = fadd(grp[q].e, se);
+            grp[q].w = fadd(grp[q].w, ffma(T(c0 + s * C::CC + ch * C::CQ + 1), se, s1));
+            grp[q].a = fadd(grp[q].a, sa);
           }
-          grp[q].e = fadd(grp[q].e, se);
-          grp[q].w = fadd(grp[q].w, ffma(T(c0 + s * C::CC + 1), se, s1));
-          grp[q].a = fadd(grp[q].a, sa);
         } else {
           for (int cc = 0; cc < C::CC; ++cc) {
             const int jl = c0 + s * C::CC + cc;
-            T x = buf[cc * NB + r];
+            T x = buf[cc * RK + r];
             x = sym ? (r > jl ? x : T(0)) : view_mask(view, r, jl, x);
             grp[q].e = fadd(grp[q].e, x);
             grp[q].w = ffma(T(jl + 1), x, grp[q].w);
@@ -361,13 +419,13 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
 #pragma unroll
       for (int q = 0; q < C::RPT; ++q) {
         const int r = tid + q * kThreads;
-        if (r < NB) {
+        if (r < RK) {
           if (nslab == 1) {
             tot[q].e = fadd(tot[q].e, grp[q].e);
             tot[q].w = fadd(tot[q].w, grp[q].w);
             tot[q].a = fadd(tot[q].a, grp[q].a);
           } else {
-            T* dst = partT + (((size_t)tile * C::GROUPS + g) * NB + r) * 3;
+            T* dst = partT + (((size_t)sup * C::GROUPS + g) * RK + r) * 3;
             dst[0] = grp[q].e;
             dst[1] = grp[q].w;
             dst[2] = grp[q].a;
@@ -379,30 +437,41 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
   }
 
   // ---------------- column flags of this CTA ------------------------------
-  if (VERIFY && (my_colflags | my_ncols)) {
-    atomicOr(&s_colflags, my_colflags);
-    atomicAdd(&s_ncols, my_ncols);
+  if (VERIFY) {
+#pragma unroll
+    for (int t = 0; t < K; ++t) {
+      const int f = __reduce_or_sync(0xffffffffu, my_colflags[t]);
+      const int nc = __reduce_add_sync(0xffffffffu, my_ncols[t]);
+      if (lane == 0 && (f | nc)) {
+        atomicOr(&s_colflags[t], f);
+        atomicAdd(&s_ncols[t], nc);
+      }
+    }
   }
-  // ---------------- slab reduction: last CTA finishes the tile ------------
+  // ---------------- slab reduction: last CTA finishes the unit ------------
   if (nslab > 1) {
     __threadfence();
     consumer_sync();
     if (tid == 0) {
-      if (VERIFY && s_colflags) atomicOr(&p.tflags[tile], s_colflags);
+      if (VERIFY)
+        for (int t = 0; t < K; ++t)
+          if (s_colflags[t]) atomicOr(&p.tflags[sup * K + t], s_colflags[t]);
       __threadfence();
-      int old = atomicAdd(&p.ticket[tile], 1);
+      int old = atomicAdd(&p.ticket[sup], 1);
       s_last = (old == nslab - 1);
     }
     consumer_sync();
-    if (VERIFY && tid == 0 && s_ncols) atomicAdd(&p.counts[ABFT_CNT_COLS_FLAGGED], s_ncols);
+    if (VERIFY && tid == 0)
+      for (int t = 0; t < K; ++t)
+        if (s_ncols[t]) atomicAdd(&p.counts[ABFT_CNT_COLS_FLAGGED], s_ncols[t]);
     if (!s_last) return;
     __threadfence();
 #pragma unroll
     for (int q = 0; q < C::RPT; ++q) {
       const int r = tid + q * kThreads;
-      if (r < NB) {
+      if (r < RK) {
         for (int g = 0; g < C::GROUPS; ++g) {
-          const T* src = partT + (((size_t)tile * C::GROUPS + g) * NB + r) * 3;
+          const T* src = partT + (((size_t)sup * C::GROUPS + g) * RK + r) * 3;
           tot[q].e = fadd(tot[q].e, __ldcg(src + 0));
           tot[q].w = fadd(tot[q].w, __ldcg(src + 1));
           tot[q].a = fadd(tot[q].a, __ldcg(src + 2));
@@ -410,23 +479,32 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
       }
     }
     if (tid == 0) {
-      if (VERIFY) s_colflags |= atomicExch(&p.tflags[tile], 0);
-      p.ticket[tile] = 0;
+      if (VERIFY)
+        for (int t = 0; t < K; ++t) {
+          s_colflags[t] |= atomicExch(&p.tflags[sup * K + t], 0);
+          s_ncols[t] = 0;  // already counted
+        }
+      p.ticket[sup] = 0;
     }
   } else {
     consumer_sync();
-    if (VERIFY && tid == 0 && s_ncols) atomicAdd(&p.counts[ABFT_CNT_COLS_FLAGGED], s_ncols);
+    if (VERIFY && tid == 0)
+      for (int t = 0; t < K; ++t) {
+        if (s_ncols[t]) atomicAdd(&p.counts[ABFT_CNT_COLS_FLAGGED], s_ncols[t]);
+        s_ncols[t] = 0;
+      }
   }
 
   // ---------------- finish rows (and SYM columns) -------------------------
   T* rowchk = reinterpret_cast<T*>(p.rowchk);
   T* rowmag = reinterpret_cast<T*>(p.rowmag);
   T* drow = reinterpret_cast<T*>(p.drow);
-  int my_rowflags = 0, my_nrows = 0, my_symcols = 0;
 #pragma unroll
   for (int q = 0; q < C::RPT; ++q) {
-    const int r = tid + q * kThreads;
-    if (r >= NB) continue;
+    const int rr = tid + q * kThreads;
+    if (rr >= RK) continue;
+    const int t = rr / NB, r = rr - t * NB;
+    const int I = Ib + t;
     T re = tot[q].e, rw = tot[q].w, ra = tot[q].a;
     if (sym) {  // c_sym[r] = colsum_lower[r] + rowsum_strict[r]; r_sym = c_sym^T
       if (nslab > 1) {
@@ -453,18 +531,17 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
         if (colmag) colmag[I + gj * p.ldcm] = ra;
       }
     } else {
+      int fr = 0, fc = 0;
       if (p.which & ABFT_ROW) {
         double m = p.use_mag ? (double)rowmag[gi + (int64_t)J * p.ldrm] : (double)ra;
         T de, dw;
-        int f = check_pair<T>(rowchk[gi + (int64_t)(2 * J) * p.ldr], rowchk[gi + (int64_t)(2 * J + 1) * p.ldr], re, rw,
-                              m, p.tau_fac, NB, &de, &dw);
+        fr = check_pair<T>(rowchk[gi + (int64_t)(2 * J) * p.ldr], rowchk[gi + (int64_t)(2 * J + 1) * p.ldr], re, rw,
+                           m, p.tau_fac, NB, &de, &dw);
         if (drow) {
           drow[gi + (int64_t)(2 * J) * p.ldr] = de;
           drow[gi + (int64_t)(2 * J + 1) * p.ldr] = dw;
         }
-        my_rowflags |= f;
-        my_nrows += f & 1;
-        if (p.refresh && !(f & 1)) {
+        if (p.refresh && !(fr & 1)) {
           rowchk[gi + (int64_t)(2 * J) * p.ldr] = re;
           rowchk[gi + (int64_t)(2 * J + 1) * p.ldr] = rw;
           if (rowmag) rowmag[gi + (int64_t)J * p.ldrm] = ra;
@@ -473,64 +550,65 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
       if (sym && (p.which & ABFT_COL)) {
         double m = p.use_mag ? (double)colmag[I + gj * p.ldcm] : (double)ra;
         T de, dw;
-        int f = check_pair<T>(colchk[(int64_t)2 * I + gj * p.ldc], colchk[(int64_t)2 * I + 1 + gj * p.ldc], re, rw, m,
-                              p.tau_fac, NB, &de, &dw);
+        fc = check_pair<T>(colchk[(int64_t)2 * I + gj * p.ldc], colchk[(int64_t)2 * I + 1 + gj * p.ldc], re, rw, m,
+                           p.tau_fac, NB, &de, &dw);
         if (dcol) {
           dcol[(int64_t)2 * I + gj * p.ldc] = de;
           dcol[(int64_t)2 * I + 1 + gj * p.ldc] = dw;
         }
-        my_colflags |= f;
-        my_symcols += f & 1;
-        if (p.refresh && !(f & 1)) {
+        if (p.refresh && !(fc & 1)) {
           colchk[(int64_t)2 * I + gj * p.ldc] = re;
           colchk[(int64_t)2 * I + 1 + gj * p.ldc] = rw;
           if (colmag) colmag[I + gj * p.ldcm] = ra;
         }
       }
+      if (fr) {
+        atomicOr(&s_rowflags[t], fr);
+        if (fr & 1) atomicAdd(&s_nrows[t], 1);
+      }
+      if (fc) {
+        atomicOr(&s_colflags[t], fc);
+        if (fc & 1) atomicAdd(&s_ncols[t], 1);
+      }
     }
   }
   if (!VERIFY) return;
-  if (my_rowflags | my_nrows | my_symcols) {
-    atomicOr(&s_rowflags, my_rowflags);
-    atomicAdd(&s_nrows, my_nrows);
-    if (my_symcols) {
-      atomicOr(&s_colflags, my_colflags);
-      atomicAdd(&s_ncols, my_symcols);
-    }
-  }
   consumer_sync();
-  if (tid == 0) {
-    int cf = s_colflags, rf = s_rowflags;
-    int st = ((cf & 1) ? ABFT_ST_COL : 0) | ((rf & 1) ? ABFT_ST_ROW : 0) | (((cf | rf) & 2) ? ABFT_ST_NONFINITE : 0);
+  if (tid < K) {
+    const int t = tid, I = Ib + t;
+    const int cf = s_colflags[t], rf = s_rowflags[t];
+    const int st = ((cf & 1) ? ABFT_ST_COL : 0) | ((rf & 1) ? ABFT_ST_ROW : 0) | (((cf | rf) & 2) ? ABFT_ST_NONFINITE : 0);
     p.status[I + (int64_t)J * p.ld_status] = st;
     if (st & (ABFT_ST_COL | ABFT_ST_ROW)) atomicAdd(&p.counts[ABFT_CNT_TILES_FLAGGED], 1);
     if (st & ABFT_ST_NONFINITE) atomicAdd(&p.counts[ABFT_CNT_NONFINITE], 1);
-    if (s_nrows) atomicAdd(&p.counts[ABFT_CNT_ROWS_FLAGGED], s_nrows);
-    if (sym && s_ncols) atomicAdd(&p.counts[ABFT_CNT_COLS_FLAGGED], s_ncols);
+    if (s_nrows[t]) atomicAdd(&p.counts[ABFT_CNT_ROWS_FLAGGED], s_nrows[t]);
+    if (s_ncols[t]) atomicAdd(&p.counts[ABFT_CNT_COLS_FLAGGED], s_ncols[t]);
   }
 }
 
 // ------------------------------------------------------------ launcher --
-template <typename T, int NB, bool VERIFY>
-static int launch_nb(PassArgs& a, int64_t ntiles, cudaStream_t s) {
-  using C = PassCfg<T, NB>;
-  auto kern = checksum_pass_kernel<T, NB, VERIFY>;
+template <typename T, int NB, int K, bool VERIFY>
+static int launch_k(PassArgs& a, int64_t ntiles, cudaStream_t s) {
+  using C = PassCfg<T, NB, K>;
+  auto kern = checksum_pass_kernel<T, NB, K, VERIFY>;
   static bool attr_done = false;  // per instantiation
   if (!attr_done) {
     ABFT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM));
     attr_done = true;
   }
-  // slabs: aim for >= 2 CTAs per SM when the tile count is small
   static int sms = 0;
   if (!sms) {
     int dev = 0;
     cudaGetDevice(&dev);
     if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms <= 0) sms = 148;
   }
+  const int64_t nsup = ntiles / K;
+  // slabs: aim for >= 2 CTAs per SM when the unit count is small
   int nslab = 1;
   const int max_slab = C::GROUPS;
-  while (nslab < max_slab && ntiles * nslab < 2LL * sms) nslab *= 2;
+  while (nslab < max_slab && nsup * nslab < 2LL * sms) nslab *= 2;
   a.nslab = nslab;
+  a.K = K;
   if (nslab > 1) {
     void* ws = nullptr;
     size_t bytes = (size_t)ntiles * (C::GROUPS + 1) * NB * 3 * sizeof(T);
@@ -544,10 +622,32 @@ static int launch_nb(PassArgs& a, int64_t ntiles, cudaStream_t s) {
     a.ticket = ctr;
     a.tflags = ctr + ntiles;
   }
-  dim3 grid((unsigned)(ntiles * nslab));
+  dim3 grid((unsigned)(nsup * nslab));
   kern<<<grid, kBlock, C::SMEM, s>>>(a);
   ABFT_CUDA_TRY(cudaGetLastError());
   return 0;
+}
+
+// Small tiles are streamed K at a time (K*NB*s >= 4 KiB per column copy)
+// when the range is rectangular, GENERAL everywhere and divisible by K.
+template <typename T, int NB, bool VERIFY>
+static int launch_nb(PassArgs& a, int64_t ntiles, cudaStream_t s) {
+  constexpr int KR = 4096 / (NB * (int)sizeof(T));
+  constexpr int KBIG = KR < 1 ? 1 : (KR > 8 ? 8 : KR);
+  constexpr int VEC = NB >= 32 * (16 / (int)sizeof(T)) ? 16 / (int)sizeof(T) : 1;
+  constexpr bool can = KBIG > 1 && NB % (32 * VEC) == 0;
+  if constexpr (can) {
+    const abft_tiles_t& t = a.tiles;
+    const bool touches_diag = t.I0 < t.J1 && t.J0 < t.I1;
+    const bool general = !t.lower_only && (t.diag_view == ABFT_GENERAL || !touches_diag);
+    if (general) {
+      int K = KBIG;
+      while (K > 1 && (t.I1 - t.I0) % K) K /= 2;
+      if (K == KBIG) return launch_k<T, NB, KBIG, VERIFY>(a, ntiles, s);
+      if (K >= 2 && KBIG >= 4 && K == KBIG / 2) return launch_k<T, NB, (KBIG >= 4 ? KBIG / 2 : 1), VERIFY>(a, ntiles, s);
+    }
+  }
+  return launch_k<T, NB, 1, VERIFY>(a, ntiles, s);
 }
 
 template <typename T, bool VERIFY>

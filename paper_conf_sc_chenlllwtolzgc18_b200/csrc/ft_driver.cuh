@@ -41,6 +41,9 @@ struct ft_ctx {
   size_t putmp_bytes = 0;
   void* aux = nullptr;  // driver-specific device scratch (LU pivots / swap rows)
   size_t aux_bytes = 0;
+  void* rsv = nullptr;  // local-restart copies (f1): PD tile + PU panel with checksums
+  size_t rsv_bytes = 0;
+  int32_t* hpin = nullptr;  // pinned host words for the restart read-back
 };
 
 namespace abft {
@@ -76,7 +79,8 @@ struct Driver {
   abft_report_t R{};
   abft_tol_t tol{};
   int32_t *status = nullptr, *counts = nullptr, *nfix = nullptr, *mark = nullptr, *info = nullptr, *rep = nullptr,
-          *info_total = nullptr;
+          *info_total = nullptr, *snap = nullptr;
+  int restarts = 0;
   std::vector<ft_inject_t> onchip_pending;
   int n_checks = 0;
 
@@ -110,6 +114,9 @@ struct Driver {
     info = mark + 1;
     rep = info + 1;
     info_total = rep + 2;
+    snap = info_total + 1;
+    if (o->abft && o->restart)
+      FT_TRY(grow_buffer(c->rsv, c->rsv_bytes, ((size_t)n * nb + (size_t)nb * nb + 3 * (size_t)nt * nb + 4 * nb) * es));
     ABFT_CUDA_TRY(cudaMemsetAsync(c->ints, 0, ints_need * sizeof(int32_t), s));
     char* st = (char*)c->state;
     M.dtype = dtype;
@@ -219,6 +226,7 @@ struct Driver {
       stats->repairs_skipped = h[12];
       stats->uncorrectable = h[ABFT_CNT_UNCORRECTABLE];
       stats->n_checks = n_checks;
+      stats->restarts = restarts;
       stats->ms_total = std::chrono::duration<double, std::milli>(t1 - t0).count();
     }
     return h[ABFT_CNT_UNCORRECTABLE] ? ABFT_E_UNCORRECTABLE : 0;

@@ -148,6 +148,11 @@ extern "C" int ft_ctx_create(ft_ctx_t** ctx, int32_t device, abft_stream_t strea
     delete c;
     return ABFT_E_NOMEM;
   }
+  if (cudaHostAlloc((void**)&c->hpin, 16 * sizeof(int32_t), cudaHostAllocDefault) != cudaSuccess) {
+    cudaFree(c->fixlog);
+    delete c;
+    return ABFT_E_NOMEM;
+  }
   *ctx = c;
   return 0;
 }
@@ -162,6 +167,8 @@ extern "C" int ft_ctx_destroy(ft_ctx_t* c) {
   if (c->uinv) cudaFree(c->uinv);
   if (c->putmp) cudaFree(c->putmp);
   if (c->aux) cudaFree(c->aux);
+  if (c->rsv) cudaFree(c->rsv);
+  if (c->hpin) cudaFreeHost(c->hpin);
   delete c;
   return 0;
 }
@@ -198,80 +205,145 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     // Alg. 2 lines 3-4: check the panel to be decomposed (diag tile, SYM view, both)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
     if (ft) FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_SYM_LOWER, ABFT_BOTH));
-    // line 5: PD (+ checksum rule c-12)
-    FT_TRY(d.inject_at(k, FT_AT_PRE_PD));
-    {
+    // Local restart (f1, L430): the PD input tile and the PU input panel are
+    // copied (with their checksums) right after their pre-op checks; a 2D
+    // error left by the post-op check restores the copy and redoes the op.
+    const bool rs = ft && o->restart;
+    const int64_t r0 = (int64_t)k * nb;
+    char* rbuf = (char*)c->rsv;
+    auto copy2d = [&](void* dst, int64_t ldd, const void* src, int64_t lds, int64_t rows, int64_t cols) -> int {
+      if (rows <= 0 || cols <= 0) return 0;
+      ABFT_CUDA_TRY(cudaMemcpy2DAsync(dst, ldd * d.es, src, lds * d.es, rows * d.es, cols, cudaMemcpyDeviceToDevice, s));
+      return 0;
+    };
+    // pd copy: A_kk (nb x nb) | c(A_kk) (2 x nb) | m_c (1 x nb);  pu copy: A21 | c(A21) | m_c(A21)
+    char* pd_a = rbuf;
+    char* pd_c = pd_a + (size_t)nb * nb * d.es;
+    char* pd_m = pd_c + (size_t)2 * nb * d.es;
+    char* pu_a = pd_m + (size_t)nb * d.es;
+    char* pu_c = pu_a + (size_t)nk * nb * d.es;
+    char* pu_m = pu_c + (size_t)m2 * nb * d.es;
+    auto uncorrectable_grew = [&](int32_t* snap) -> bool {  // 8-byte read-back into pinned memory
+      int32_t* h2 = c->hpin;
+      ABFT_CUDA_TRY(cudaMemcpyAsync(h2, snap, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+      ABFT_CUDA_TRY(cudaMemcpyAsync(h2 + 1, d.counts + ABFT_CNT_UNCORRECTABLE, sizeof(int32_t),
+                                    cudaMemcpyDeviceToHost, s));
+      if (cudaStreamSynchronize(s) != cudaSuccess) return false;
+      return h2[1] > h2[0];
+    };
+    if (rs) {
+      FT_TRY(copy2d(pd_a, nb, d.a_at(r0, r0), lda, nb, nb));
+      FT_TRY(copy2d(pd_c, 2, d.colchk_at(2 * k, r0), d.M.ldc, 2, nb));
+      FT_TRY(copy2d(pd_m, 1, d.colmag_at(k, r0), d.M.ldcm, 1, nb));
+    }
+    auto do_pd = [&]() -> int {
       abft_mat_t D{};
       D.dtype = dtype;
       D.m = D.n = D.nb = nb;
-      D.A = d.a_at(k * nb, k * nb);
+      D.A = d.a_at(r0, r0);
       D.lda = lda;
       if (ft) {
-        D.colchk = d.colchk_at(2 * k, k * nb);
+        D.colchk = d.colchk_at(2 * k, r0);
         D.ldc = d.M.ldc;
-        D.colmag = d.colmag_at(k, k * nb);
+        D.colmag = d.colmag_at(k, r0);
         D.ldcm = d.M.ldcm;
       }
       const bool need_inv = ft || o->pu_gemm;
       FT_TRY(abft_panel_potrf(&D, need_inv ? c->linv : nullptr, nb, d.info, as));
-      accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.info_total, (int64_t)k * nb);
-    }
+      accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.info_total, r0);
+      return 0;
+    };
+    // line 5: PD (+ checksum rule c-12)
+    FT_TRY(d.inject_at(k, FT_AT_PRE_PD));
+    FT_TRY(do_pd());
     FT_TRY(d.restore_onchip());
     FT_TRY(d.inject_at(k, FT_AT_POST_PD));
     // line 7: check the decomposed panel (LOWER view, c only; c-24)
-    if (ft) FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_LOWER, ABFT_COL));
+    if (ft) {
+      if (rs) ABFT_CUDA_TRY(cudaMemcpyAsync(d.snap, d.counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToDevice, s));
+      FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_LOWER, ABFT_COL));
+      if (rs && uncorrectable_grew(d.snap)) {
+        ++d.restarts;
+        ABFT_CUDA_TRY(cudaMemcpyAsync(d.counts + ABFT_CNT_UNCORRECTABLE, d.snap, 4, cudaMemcpyDeviceToDevice, s));
+        FT_TRY(copy2d(d.a_at(r0, r0), lda, pd_a, nb, nb, nb));
+        FT_TRY(copy2d(d.colchk_at(2 * k, r0), d.M.ldc, pd_c, 2, 2, nb));
+        FT_TRY(copy2d(d.colmag_at(k, r0), d.M.ldcm, pd_m, 1, 1, nb));
+        FT_TRY(do_pd());
+        FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_LOWER, ABFT_COL));
+      }
+    }
     if (k == nt - 1) break;
     // line 8: check the panel to be updated (both checksums)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PU_CHECK));
     if (ft) FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH));
+    if (rs) {
+      FT_TRY(copy2d(pu_a, nk, d.a_at(r1, r0), lda, nk, nb));
+      FT_TRY(copy2d(pu_c, m2, d.colchk_at(2 * (k + 1), r0), d.M.ldc, m2, nb));
+      FT_TRY(copy2d(pu_m, m2 / 2, d.colmag_at(k + 1, r0), d.M.ldcm, m2 / 2, nb));
+    }
     // line 9: PU  L_ik = A_ik L_kk^-T  (+ c(L_ik) = c(A_ik) L_kk^-T, c-12)
-    FT_TRY(d.inject_at(k, FT_AT_PRE_PU));
-    const bool refresh_inv = o->pu_gemm && d.diag_touched_before_pu(k);
-    if (refresh_inv) FT_TRY(abft_tri_inverse(dtype, 'L', 'N', nb, d.a_at(k * nb, k * nb), lda, c->linv, nb, as));
-    {
+    auto pu_data = [&]() -> int {
       cublasHandle_t h = blas_handle(s, lk);
       if (o->pu_gemm) {
         // L21 = A21 L_kk^-T as a DGEMM with the explicit inverse (tensor cores),
         // written to scratch and copied back
+        cublasStatus_t st;
         if (dtype == ABFT_F64) {
           const double one = 1.0, zero = 0.0;
-          if (cublasDgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)nk, (int)nb, (int)nb, &one, (const double*)d.a_at(r1, k * nb),
-                          (int)lda, (const double*)c->linv, (int)nb, &zero, (double*)c->putmp, (int)nk) !=
-              CUBLAS_STATUS_SUCCESS)
-            return ABFT_E_CUBLAS;
+          st = cublasDgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)nk, (int)nb, (int)nb, &one, (const double*)d.a_at(r1, r0),
+                           (int)lda, (const double*)c->linv, (int)nb, &zero, (double*)c->putmp, (int)nk);
         } else {
           const float one = 1.0f, zero = 0.0f;
-          if (cublasSgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)nk, (int)nb, (int)nb, &one, (const float*)d.a_at(r1, k * nb),
-                          (int)lda, (const float*)c->linv, (int)nb, &zero, (float*)c->putmp, (int)nk) !=
-              CUBLAS_STATUS_SUCCESS)
-            return ABFT_E_CUBLAS;
+          st = cublasSgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)nk, (int)nb, (int)nb, &one, (const float*)d.a_at(r1, r0),
+                           (int)lda, (const float*)c->linv, (int)nb, &zero, (float*)c->putmp, (int)nk);
         }
         lk.unlock();
-        ABFT_CUDA_TRY(cudaMemcpy2DAsync(d.a_at(r1, k * nb), lda * d.es, c->putmp, nk * d.es, nk * d.es, nb,
+        if (st != CUBLAS_STATUS_SUCCESS) return ABFT_E_CUBLAS;
+        ABFT_CUDA_TRY(cudaMemcpy2DAsync(d.a_at(r1, r0), lda * d.es, c->putmp, nk * d.es, nk * d.es, nb,
                                         cudaMemcpyDeviceToDevice, s));
-      } else if (dtype == ABFT_F64) {
-        const double one = 1.0;
-        if (cublasDtrsm(h, CUBLAS_SIDE_RIGHT, CUBLAS_FILL_MODE_LOWER, CUBLAS_OP_T, CUBLAS_DIAG_NON_UNIT, (int)nk,
-                        (int)nb, &one, (const double*)d.a_at(k * nb, k * nb), (int)lda, (double*)d.a_at(r1, k * nb),
-                        (int)lda) != CUBLAS_STATUS_SUCCESS)
-          return ABFT_E_CUBLAS;
       } else {
-        const float one = 1.0f;
-        if (cublasStrsm(h, CUBLAS_SIDE_RIGHT, CUBLAS_FILL_MODE_LOWER, CUBLAS_OP_T, CUBLAS_DIAG_NON_UNIT, (int)nk,
-                        (int)nb, &one, (const float*)d.a_at(k * nb, k * nb), (int)lda, (float*)d.a_at(r1, k * nb),
-                        (int)lda) != CUBLAS_STATUS_SUCCESS)
-          return ABFT_E_CUBLAS;
+        cublasStatus_t st;
+        if (dtype == ABFT_F64) {
+          const double one = 1.0;
+          st = cublasDtrsm(h, CUBLAS_SIDE_RIGHT, CUBLAS_FILL_MODE_LOWER, CUBLAS_OP_T, CUBLAS_DIAG_NON_UNIT, (int)nk,
+                           (int)nb, &one, (const double*)d.a_at(r0, r0), (int)lda, (double*)d.a_at(r1, r0), (int)lda);
+        } else {
+          const float one = 1.0f;
+          st = cublasStrsm(h, CUBLAS_SIDE_RIGHT, CUBLAS_FILL_MODE_LOWER, CUBLAS_OP_T, CUBLAS_DIAG_NON_UNIT, (int)nk,
+                           (int)nb, &one, (const float*)d.a_at(r0, r0), (int)lda, (float*)d.a_at(r1, r0), (int)lda);
+        }
+        lk.unlock();
+        if (st != CUBLAS_STATUS_SUCCESS) return ABFT_E_CUBLAS;
       }
-      if (lk.owns_lock()) lk.unlock();
-    }
+      return 0;
+    };
+    auto pu_chk = [&]() -> int {  // c(L_ik) = c(A_ik) L_kk^-T, m_c <- m_c |L_kk^-T| with the PD's inverse (c-12, c-6)
+      return abft_update_trsm_inv(dtype, 'R', 'T', nb, c->linv, nb, d.colchk_at(2 * (k + 1), r0), d.M.ldc, m2,
+                                  d.colmag_at(k + 1, r0), d.M.ldcm, m2 / 2, as);
+    };
+    FT_TRY(d.inject_at(k, FT_AT_PRE_PU));
+    const bool refresh_inv = o->pu_gemm && d.diag_touched_before_pu(k);
+    if (refresh_inv) FT_TRY(abft_tri_inverse(dtype, 'L', 'N', nb, d.a_at(r0, r0), lda, c->linv, nb, as));
+    FT_TRY(pu_data());
     FT_TRY(d.restore_onchip());  // on-chip flips hit the data step only (c-8)
-    if (refresh_inv) FT_TRY(abft_tri_inverse(dtype, 'L', 'N', nb, d.a_at(k * nb, k * nb), lda, c->linv, nb, as));
-    if (ft)  // c(L_ik) = c(A_ik) L_kk^-T, m_c <- m_c |L_kk^-T| with the PD's inverse (c-12, c-6)
-      FT_TRY(abft_update_trsm_inv(dtype, 'R', 'T', nb, c->linv, nb, d.colchk_at(2 * (k + 1), k * nb), d.M.ldc, m2,
-                                  d.colmag_at(k + 1, k * nb), d.M.ldcm, m2 / 2, as));
+    if (refresh_inv) FT_TRY(abft_tri_inverse(dtype, 'L', 'N', nb, d.a_at(r0, r0), lda, c->linv, nb, as));
+    if (ft) FT_TRY(pu_chk());
     FT_TRY(d.inject_at(k, FT_AT_POST_PU));
     // line 10: check the updated panel (c only; 1D_ROW fixable, 2D -> restart, L434)
-    if (ft) FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
+    if (ft) {
+      if (rs) ABFT_CUDA_TRY(cudaMemcpyAsync(d.snap, d.counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToDevice, s));
+      FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
+      if (rs && uncorrectable_grew(d.snap)) {
+        ++d.restarts;
+        ABFT_CUDA_TRY(cudaMemcpyAsync(d.counts + ABFT_CNT_UNCORRECTABLE, d.snap, 4, cudaMemcpyDeviceToDevice, s));
+        FT_TRY(copy2d(d.a_at(r1, r0), lda, pu_a, nk, nk, nb));
+        FT_TRY(copy2d(d.colchk_at(2 * (k + 1), r0), d.M.ldc, pu_c, m2, m2, nb));
+        FT_TRY(copy2d(d.colmag_at(k + 1, r0), d.M.ldcm, pu_m, m2 / 2, m2 / 2, nb));
+        FT_TRY(pu_data());
+        FT_TRY(pu_chk());
+        FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
+      }
+    }
     // line 12: TMU  A22 -= L21 L21^T (DSYRK on tensor cores) + checksum rules c-12
     FT_TRY(d.inject_at(k, FT_AT_PRE_TMU));
     {

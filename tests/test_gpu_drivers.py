@@ -65,6 +65,7 @@ def _compare(lib, ctx, A, nb, injects, fig4a=True):
     assert list(sg.counts) == so.counts, (list(sg.counts), so.counts)
     assert sorted((f[0], f[1], f[4], f[5]) for f in fg) == sorted((f.gi, f.gj, f.cls, f.kind) for f in so.fixes)
     assert sg.repairs_applied == so.repairs_applied and sg.repairs_skipped == so.repairs_skipped
+    assert sg.restarts == so.restarts
     assert (rc == lib.E_UNCORRECTABLE) == (so.uncorrectable > 0)
     if so.uncorrectable == 0:
         Lref = np.linalg.cholesky(A)
@@ -81,7 +82,8 @@ CASES = [
     (dr.AT_PRE_PU_CHECK, dr.KIND_PERSIST, 0, 200, 70, (60,)),
     (dr.AT_POST_PU, dr.KIND_PERSIST, 0, 150, 90, (63,)),
     (dr.AT_PRE_PU, dr.KIND_ONCHIP, 0, 130, 68, (58,)),
-    (dr.AT_PRE_PU, dr.KIND_ONCHIP, 0, 70, 66, (60,)),      # PU reference part -> 2D (R)
+    (dr.AT_PRE_PU, dr.KIND_ONCHIP, 0, 70, 66, (60,)),      # PU reference part -> 2D -> local restart
+    (dr.AT_PRE_PD, dr.KIND_PERSIST, 0, 70, 66, (57,)),     # consumed by the PD -> 2D -> local restart
     (dr.AT_PRE_TMU, dr.KIND_ONCHIP, 0, 140, 72, (57,)),
     (dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 170, 80, (54,)),    # Fig. 4a repair
     (dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 170, 80, (62,)),    # guarded: R

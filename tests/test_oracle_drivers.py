@@ -112,11 +112,29 @@ def test_fig4a_guard_huge_fault_detected_not_silent():
     assert ok or stats.uncorrectable >= 1
 
 
-def test_pu_reference_fault_is_2d():
-    # on-chip flip in L_kk while PU reads it: every panel row is wrong -> 2D (Table V)
+def test_pu_reference_fault_is_2d_and_restart_fixes_it():
+    # on-chip flip in L_kk while PU reads it: every panel row is wrong -> 2D
+    # (Table V); the local restart from the pre-PU copy (L430, f1) fixes it
     inj = [dr.Inject(2, dr.AT_PRE_PU, dr.KIND_ONCHIP, 0, 70, 66, (60,))]
-    _, _, _, stats = _run(256, 32, inj)
+    A = si.spd(256, seed=0)
+    _, stats = dr.ft_potrf(A, 32, inject=inj, restart=False)
     assert stats.uncorrectable >= 1
+    Lref, _ = dr.ft_potrf(A, 32)
+    L, stats = dr.ft_potrf(A, 32, inject=inj)
+    assert stats.uncorrectable == 0 and stats.restarts == 1
+    assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
+
+
+@pytest.mark.parametrize("bit", [53, 57, 60, 63])
+def test_pd_consumed_fault_restart(bit):
+    # DRAM fault in A_kk between the pre-PD check and the PD: the PD consumes
+    # it (2D in L_kk); the restart from the pre-PD copy gives the right factor
+    inj = [dr.Inject(3, dr.AT_PRE_PD, dr.KIND_PERSIST, 0, 100, 99, (bit,))]
+    A = si.spd(256, seed=1)
+    Lref, _ = dr.ft_potrf(A, 32)
+    L, stats = dr.ft_potrf(A, 32, inject=inj)
+    assert stats.uncorrectable == 0 and stats.restarts == 1
+    assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
 
 
 def test_checksum_memory_fault_repaired():
