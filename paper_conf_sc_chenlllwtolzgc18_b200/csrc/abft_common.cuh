@@ -133,4 +133,7 @@ struct Workspace {
 int workspace_get(cudaStream_t s, size_t bytes, void** out);
 // Per-stream zero-initialised counter area (self-resetting kernels use it).
 int counters_get(cudaStream_t s, size_t n_ints, int** out);
+// Device-to-device 2-D copy (pitches and width in bytes) with an SM kernel:
+// cudaMemcpy2DAsync D2D of column panels runs far below HBM bandwidth.
+int copy2d(void* dst, size_t dpitch, const void* src, size_t spitch, size_t width, size_t height, cudaStream_t s);
 }  // namespace abft

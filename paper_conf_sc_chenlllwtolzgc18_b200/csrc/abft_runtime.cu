@@ -1,4 +1,5 @@
 // abft_runtime.cu — per-stream workspace / counter pools and the inject hook.
+#include <algorithm>
 #include <mutex>
 #include <unordered_map>
 
@@ -65,6 +66,37 @@ int counters_get(cudaStream_t s, size_t n, int** out) {
     p.ctr_n = nn;
   }
   *out = p.ctr;
+  return 0;
+}
+
+template <typename V>
+__global__ void __launch_bounds__(256) copy2d_kernel(char* __restrict__ dst, size_t dpitch, const char* __restrict__ src,
+                                                     size_t spitch, size_t wv, size_t height) {
+  for (size_t c = blockIdx.y; c < height; c += gridDim.y) {
+    const V* sc = reinterpret_cast<const V*>(src + c * spitch);
+    V* dc = reinterpret_cast<V*>(dst + c * dpitch);
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < wv; i += (size_t)gridDim.x * blockDim.x)
+      dc[i] = sc[i];
+  }
+}
+
+int copy2d(void* dst, size_t dpitch, const void* src, size_t spitch, size_t width, size_t height, cudaStream_t s) {
+  if (width == 0 || height == 0) return 0;
+  const uintptr_t al = (uintptr_t)dst | (uintptr_t)src | dpitch | spitch | width;
+  const int vb = (al % 16 == 0) ? 16 : (al % 8 == 0) ? 8 : (al % 4 == 0) ? 4 : 1;
+  const size_t wv = width / vb;
+  const unsigned gx = (unsigned)std::min<size_t>((wv + 255) / 256, 1024);
+  const unsigned gy = (unsigned)std::min<size_t>(height, std::max<size_t>(1, 8 * 148 / gx + 1));
+  dim3 g(gx, std::min<unsigned>(gy, 65535u));
+  char* d = (char*)dst;
+  const char* r = (const char*)src;
+  switch (vb) {
+    case 16: copy2d_kernel<int4><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height); break;
+    case 8: copy2d_kernel<int2><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height); break;
+    case 4: copy2d_kernel<int><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height); break;
+    default: copy2d_kernel<char><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height); break;
+  }
+  ABFT_CUDA_TRY(cudaGetLastError());
   return 0;
 }
 

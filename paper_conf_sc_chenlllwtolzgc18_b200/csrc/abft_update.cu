@@ -290,9 +290,7 @@ int tri_inverse_t(char uplo, char diag, int nb, const T* Tm, int ldt, T* W, int 
 // out (rows x cols, ld ldo) <- tmp (ld rows): stream-ordered copy back
 template <typename T>
 static int copy_back(T* out, int64_t ldo, const T* tmp, int64_t rows, int64_t cols, cudaStream_t s) {
-  ABFT_CUDA_TRY(cudaMemcpy2DAsync(out, ldo * sizeof(T), tmp, rows * sizeof(T), rows * sizeof(T), cols,
-                                  cudaMemcpyDeviceToDevice, s));
-  return 0;
+  return abft::copy2d(out, ldo * sizeof(T), tmp, rows * sizeof(T), rows * sizeof(T), cols, s);
 }
 
 // a5 with a precomputed inverse W = T^-1:

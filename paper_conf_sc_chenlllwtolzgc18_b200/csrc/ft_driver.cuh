@@ -44,6 +44,7 @@ struct ft_ctx {
   void* rsv = nullptr;  // local-restart copies (f1): PD tile + PU panel with checksums
   size_t rsv_bytes = 0;
   int32_t* hpin = nullptr;  // pinned host words for the restart read-back
+  cudaEvent_t ev = nullptr;  // marks the PD-check read-back (restart decision)
 };
 
 namespace abft {
@@ -176,6 +177,11 @@ struct Driver {
         onchip_pending.push_back(f);
     }
     return 0;
+  }
+  bool has_inject(int k, int point) const {
+    for (int t = 0; t < o->n_inject; ++t)
+      if (o->inject[t].iter == k && o->inject[t].point == point) return true;
+    return false;
   }
   // Fault-injection runs only: does the plan touch the diagonal tile between
   // the PD (which produced the inverse the GEMM-based PU reads) and the PU?

@@ -196,8 +196,7 @@ static int panel_geqrf_t(const abft_mat_t* mat, int k, T* tau, T* Vbuf, T* Tout,
   T* A = reinterpret_cast<T*>(mat->A);
   T* panel = A + r0 + r0 * mat->lda;
   if (ft)
-    ABFT_CUDA_TRY(cudaMemcpy2DAsync(P0, mk * sizeof(T), panel, mat->lda * sizeof(T), mk * sizeof(T), nb,
-                                    cudaMemcpyDeviceToDevice, s));
+    FT_TRY(abft::copy2d(P0, mk * sizeof(T), panel, mat->lda * sizeof(T), mk * sizeof(T), nb, s));
   {
     std::unique_lock<std::mutex> lk;
     cusolverDnHandle_t h = solver_handle(s, lk);

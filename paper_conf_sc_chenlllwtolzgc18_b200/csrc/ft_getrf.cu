@@ -327,7 +327,7 @@ extern "C" int abft_panel_getrf(const abft_mat_t* mat, int32_t k, int64_t* ipiv,
   int32_t* src = (int32_t*)(base + off_src);
   int32_t* tb = (int32_t*)(base + off_tb);
   if (ft)
-    ABFT_CUDA_TRY(cudaMemcpy2DAsync(base, mk * es, panel, mat->lda * es, mk * es, nb, cudaMemcpyDeviceToDevice, s));
+    FT_TRY(abft::copy2d(base, mk * es, panel, mat->lda * es, mk * es, nb, s));
   {
     std::unique_lock<std::mutex> lk;
     cusolverDnHandle_t h = solver_handle(s, lk);
@@ -464,8 +464,7 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       }
       lk.unlock();
       if (st != CUBLAS_STATUS_SUCCESS) return ABFT_E_CUBLAS;
-      ABFT_CUDA_TRY(cudaMemcpy2DAsync(d.a_at(r0, r1), lda * d.es, c->putmp, nb * d.es, nb * d.es, nk,
-                                      cudaMemcpyDeviceToDevice, s));
+      FT_TRY(abft::copy2d(d.a_at(r0, r1), lda * d.es, c->putmp, nb * d.es, nb * d.es, nk, s));
     }
     FT_TRY(d.restore_onchip());
     if (refresh) FT_TRY(abft_tri_inverse(dtype, 'L', 'U', nb, d.a_at(r0, r0), lda, c->linv, nb, as));

@@ -137,6 +137,10 @@ __global__ void fig4a_repair_kernel(RepairArgs r) {
 }  // namespace abft
 
 // ----------------------------------------------------------------- driver --
+namespace abft {
+__global__ void add_i32_kernel(int32_t* p, int32_t v) { *p += v; }
+}  // namespace abft
+
 extern "C" int ft_ctx_create(ft_ctx_t** ctx, int32_t device, abft_stream_t stream) {
   if (!ctx) return -1;
   ABFT_CUDA_TRY(cudaSetDevice(device));
@@ -148,8 +152,10 @@ extern "C" int ft_ctx_create(ft_ctx_t** ctx, int32_t device, abft_stream_t strea
     delete c;
     return ABFT_E_NOMEM;
   }
-  if (cudaHostAlloc((void**)&c->hpin, 16 * sizeof(int32_t), cudaHostAllocDefault) != cudaSuccess) {
+  if (cudaHostAlloc((void**)&c->hpin, 16 * sizeof(int32_t), cudaHostAllocDefault) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev, cudaEventDisableTiming) != cudaSuccess) {
     cudaFree(c->fixlog);
+    if (c->hpin) cudaFreeHost(c->hpin);
     delete c;
     return ABFT_E_NOMEM;
   }
@@ -169,6 +175,7 @@ extern "C" int ft_ctx_destroy(ft_ctx_t* c) {
   if (c->aux) cudaFree(c->aux);
   if (c->rsv) cudaFree(c->rsv);
   if (c->hpin) cudaFreeHost(c->hpin);
+  if (c->ev) cudaEventDestroy(c->ev);
   delete c;
   return 0;
 }
@@ -213,7 +220,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     char* rbuf = (char*)c->rsv;
     auto copy2d = [&](void* dst, int64_t ldd, const void* src, int64_t lds, int64_t rows, int64_t cols) -> int {
       if (rows <= 0 || cols <= 0) return 0;
-      ABFT_CUDA_TRY(cudaMemcpy2DAsync(dst, ldd * d.es, src, lds * d.es, rows * d.es, cols, cudaMemcpyDeviceToDevice, s));
+      FT_TRY(abft::copy2d(dst, ldd * d.es, src, lds * d.es, rows * d.es, cols, s));
       return 0;
     };
     // pd copy: A_kk (nb x nb) | c(A_kk) (2 x nb) | m_c (1 x nb);  pu copy: A21 | c(A21) | m_c(A21)
@@ -223,13 +230,21 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     char* pu_a = pd_m + (size_t)nb * d.es;
     char* pu_c = pu_a + (size_t)nk * nb * d.es;
     char* pu_m = pu_c + (size_t)m2 * nb * d.es;
-    auto uncorrectable_grew = [&](int32_t* snap) -> bool {  // 8-byte read-back into pinned memory
-      int32_t* h2 = c->hpin;
-      ABFT_CUDA_TRY(cudaMemcpyAsync(h2, snap, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-      ABFT_CUDA_TRY(cudaMemcpyAsync(h2 + 1, d.counts + ABFT_CNT_UNCORRECTABLE, sizeof(int32_t),
+    // restart decision: snapshot the uncorrectable count before a check, read
+    // both words back into pinned memory after it (8 bytes, one event)
+    auto post_readback = [&](int32_t* snap) -> int {
+      ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin, snap, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+      ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin + 1, d.counts + ABFT_CNT_UNCORRECTABLE, sizeof(int32_t),
                                     cudaMemcpyDeviceToHost, s));
-      if (cudaStreamSynchronize(s) != cudaSuccess) return false;
-      return h2[1] > h2[0];
+      ABFT_CUDA_TRY(cudaEventRecord(c->ev, s));
+      return 0;
+    };
+    static const bool dbg_nosync = getenv("ABFT_DBG_RESTART_NOSYNC") != nullptr;
+    auto readback_delta = [&](int* delta) -> int {  // uncorrectable errors the check added
+      if (dbg_nosync) { *delta = 0; return 0; }
+      ABFT_CUDA_TRY(cudaEventSynchronize(c->ev));
+      *delta = c->hpin[1] - c->hpin[0];
+      return 0;
     };
     if (rs) {
       FT_TRY(copy2d(pd_a, nb, d.a_at(r0, r0), lda, nb, nb));
@@ -262,16 +277,26 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft) {
       if (rs) ABFT_CUDA_TRY(cudaMemcpyAsync(d.snap, d.counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToDevice, s));
       FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_LOWER, ABFT_COL));
-      if (rs && uncorrectable_grew(d.snap)) {
-        ++d.restarts;
-        ABFT_CUDA_TRY(cudaMemcpyAsync(d.counts + ABFT_CNT_UNCORRECTABLE, d.snap, 4, cudaMemcpyDeviceToDevice, s));
-        FT_TRY(copy2d(d.a_at(r0, r0), lda, pd_a, nb, nb, nb));
-        FT_TRY(copy2d(d.colchk_at(2 * k, r0), d.M.ldc, pd_c, 2, 2, nb));
-        FT_TRY(copy2d(d.colmag_at(k, r0), d.M.ldcm, pd_m, 1, 1, nb));
-        FT_TRY(do_pd());
-        FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_LOWER, ABFT_COL));
-      }
+      if (rs) FT_TRY(post_readback(d.snap));
     }
+    // The PD restart decision is taken after the pre-PU check has been queued
+    // (that check reads only the panel below A_kk), so the host waits on the
+    // read-back while the device is busy.  Not when the fault plan injects at
+    // the pre-PU-check point: then the paper's order is kept exactly.
+    const bool defer_pd = rs && k < nt - 1 && !d.has_inject(k, FT_AT_PRE_PU_CHECK);
+    auto pd_restart = [&]() -> int {
+      int delta = 0;
+      FT_TRY(readback_delta(&delta));
+      if (delta <= 0) return 0;
+      ++d.restarts;
+      add_i32_kernel<<<1, 1, 0, s>>>(d.counts + ABFT_CNT_UNCORRECTABLE, -delta);
+      FT_TRY(copy2d(d.a_at(r0, r0), lda, pd_a, nb, nb, nb));
+      FT_TRY(copy2d(d.colchk_at(2 * k, r0), d.M.ldc, pd_c, 2, 2, nb));
+      FT_TRY(copy2d(d.colmag_at(k, r0), d.M.ldcm, pd_m, 1, 1, nb));
+      FT_TRY(do_pd());
+      return d.check(k, k + 1, k, k + 1, ABFT_LOWER, ABFT_COL);
+    };
+    if (rs && !defer_pd) FT_TRY(pd_restart());
     if (k == nt - 1) break;
     // line 8: check the panel to be updated (both checksums)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PU_CHECK));
@@ -281,6 +306,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       FT_TRY(copy2d(pu_c, m2, d.colchk_at(2 * (k + 1), r0), d.M.ldc, m2, nb));
       FT_TRY(copy2d(pu_m, m2 / 2, d.colmag_at(k + 1, r0), d.M.ldcm, m2 / 2, nb));
     }
+    if (defer_pd) FT_TRY(pd_restart());
     // line 9: PU  L_ik = A_ik L_kk^-T  (+ c(L_ik) = c(A_ik) L_kk^-T, c-12)
     auto pu_data = [&]() -> int {
       cublasHandle_t h = blas_handle(s, lk);
@@ -299,8 +325,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
         }
         lk.unlock();
         if (st != CUBLAS_STATUS_SUCCESS) return ABFT_E_CUBLAS;
-        ABFT_CUDA_TRY(cudaMemcpy2DAsync(d.a_at(r1, r0), lda * d.es, c->putmp, nk * d.es, nk * d.es, nb,
-                                        cudaMemcpyDeviceToDevice, s));
+        FT_TRY(abft::copy2d(d.a_at(r1, r0), lda * d.es, c->putmp, nk * d.es, nk * d.es, nb, s));
       } else {
         cublasStatus_t st;
         if (dtype == ABFT_F64) {
@@ -333,9 +358,14 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft) {
       if (rs) ABFT_CUDA_TRY(cudaMemcpyAsync(d.snap, d.counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToDevice, s));
       FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
-      if (rs && uncorrectable_grew(d.snap)) {
+      int delta = 0;
+      if (rs) {
+        FT_TRY(post_readback(d.snap));
+        FT_TRY(readback_delta(&delta));
+      }
+      if (delta > 0) {
         ++d.restarts;
-        ABFT_CUDA_TRY(cudaMemcpyAsync(d.counts + ABFT_CNT_UNCORRECTABLE, d.snap, 4, cudaMemcpyDeviceToDevice, s));
+        add_i32_kernel<<<1, 1, 0, s>>>(d.counts + ABFT_CNT_UNCORRECTABLE, -delta);
         FT_TRY(copy2d(d.a_at(r1, r0), lda, pu_a, nk, nk, nb));
         FT_TRY(copy2d(d.colchk_at(2 * (k + 1), r0), d.M.ldc, pu_c, m2, m2, nb));
         FT_TRY(copy2d(d.colmag_at(k + 1, r0), d.M.ldcm, pu_m, m2 / 2, m2 / 2, nb));
