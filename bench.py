@@ -302,6 +302,13 @@ def run_ours(args):
                "d2h_bytes_per_step": int(counts_h.numel() * 4 + status_h.numel() * 4), "ms_per_step": ems}
         del hostA
 
+    del A, mat
+    torch.cuda.empty_cache()
+    # ---- BASELINE configs[4]: distributed ft_potrf on all ranks (row e) ----
+    mg = None
+    if not args.no_mgpu:
+        mg = mgpu_overhead(si, args.mgpu_n, nb, args.mgpu_reps, world, rank)
+
     # ---- ft_potrf overhead at n=30720 (the metric's second half) ----
     ftp = lq = None
     if not args.no_potrf and rank == 0:
@@ -309,8 +316,6 @@ def run_ours(args):
     if not args.no_lu_qr and rank == 0:
         lq = lu_qr_overhead(abft, si, args.lu_qr_n, nb, args.lu_qr_reps)
 
-    del A, mat
-    torch.cuda.empty_cache()
     cpu = cpu_baseline_sample(args.cpu_seconds) if (rank == 0 and world == 1 and not args.no_cpu) else None
     if rank == 0:
         line = {
@@ -327,7 +332,7 @@ def run_ours(args):
                          "encode_GBs": pass_bytes / (enc_ms / 1e3) / 1e9,
                          "verify_GBs": pass_bytes / (ver_ms / 1e3) / 1e9},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": 3 * args.steps, "clocks": clk.summary(),
-            "ft_potrf": ftp, "ft_getrf_geqrf": lq,
+            "ft_potrf": ftp, "ft_getrf_geqrf": lq, "ft_potrf_mgpu": mg,
         }
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -385,6 +390,53 @@ def potrf_overhead(abft, si, n, nb, reps):
             "overhead_pct": 100.0 * (ft_ms - plain_ms) / plain_ms, "cusolver_potrf_ms": cus,
             "ms_ft_no_restart": nors_ms, "overhead_pct_no_restart": 100.0 * (nors_ms - plain_ms) / plain_ms,
             "tflops_ft": n ** 3 / 3 / (ft_ms / 1e3) / 1e12, "reps": reps}
+
+
+def mgpu_overhead(si, n, nb, reps, world, rank):
+    """BASELINE configs[4]: ft_potrf_mgpu (2D block-cyclic over the ranks,
+    NCCL panel broadcasts + error-report all-reduce) at n=61440, ABFT on vs
+    off; device time per rank between barriers, max over ranks."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_chenlllwtolzgc18_b200 import dist as D
+    from paper_conf_sc_chenlllwtolzgc18_b200 import mgpu
+
+    P, Q = D.grid_shape(world)
+    lay = mgpu.Layout(n, nb, P, Q, rank)
+    A0 = si.spd_block_cyclic_device(n, nb, P, Q, rank, seed=61440)
+    A = torch.empty_like(A0.t()).t()
+
+    def run(ft):
+        A.copy_(A0)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        rc, st = mgpu.ft_potrf_mgpu(A, lay, abft_on=ft)
+        b.record()
+        torch.cuda.synchronize()
+        ms = a.elapsed_time(b)
+        if world > 1:
+            t = torch.tensor([ms], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+        assert rc == 0 and st.info == 0 and sum(st.counts) == 0 and sum(st.bcast_counts) == 0
+        return ms
+
+    run(True)  # warm-up (allocator, cuBLAS / cuSOLVER handles, NCCL)
+    t_ft, t_plain = [], []
+    for _ in range(reps):
+        t_plain.append(run(False))
+        t_ft.append(run(True))
+    del A, A0
+    torch.cuda.empty_cache()
+    ft_ms, plain_ms = min(t_ft), min(t_plain)
+    return {"n": n, "nb": nb, "grid": [P, Q], "ms_ft": ft_ms, "ms_plain": plain_ms,
+            "overhead_pct": 100.0 * (ft_ms - plain_ms) / plain_ms,
+            "tflops_ft": n ** 3 / 3 / (ft_ms / 1e3) / 1e12, "reps": reps, "timing": "min over reps, max over ranks",
+            "comm": "NCCL broadcast of L_kk and of each process row's panel piece; int32 report all-reduce"}
 
 
 def lu_qr_overhead(abft, si, n, nb, reps):
@@ -450,6 +502,9 @@ def main():
     ap.add_argument("--lu-qr-n", type=int, default=20480)
     ap.add_argument("--lu-qr-reps", type=int, default=1)
     ap.add_argument("--no-lu-qr", action="store_true")
+    ap.add_argument("--mgpu-n", type=int, default=61440)
+    ap.add_argument("--mgpu-reps", type=int, default=1)
+    ap.add_argument("--no-mgpu", action="store_true")
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args)

@@ -185,7 +185,7 @@ class MgpuStats:
 
 
 def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0, inject=(), group=None,
-                  tmu_groups=8):
+                  tmu_groups=32):
     """Fault-tolerant lower Cholesky of the distributed matrix in place.
     A_loc: this rank's local column-major matrix (from scatter_tiles).
     inject: (iter, point, gi, gj, xor_mask, rank) with global (gi, gj);
@@ -348,27 +348,27 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
                 Lcol.mu.index_copy_(1, dst_idx, pieces[pp].mu.index_select(1, src_idx))
             hook(k, abft.AT_PRE_TMU)
             jl0 = lay.col_first(k + 1)
+            # data: tile-column groups, rows from the group's first diagonal
+            # tile (the upper tiles inside a group are computed and unused:
+            # <= 1/tmu_groups of the flops)
             g = max(1, math.ceil(ncol / max(1, tmu_groups)))
             for ta in range(0, ncol, g):
                 tb = min(ncol, ta + g)
-                Jf = (jl0 + ta) * Q + q
-                ia = lay.row_first(Jf)
+                ia = lay.row_first((jl0 + ta) * Q + q)
                 rows = lay.mt_loc - ia
                 if rows <= 0:
                     continue
                 s0 = ia - ir0  # first Lrow tile used
-                c0, c1 = (jl0 + ta) * nb, (jl0 + tb) * nb
-                X = Lrow.L[s0 * nb:, :]
-                Y = Lcol.L[ta * nb:tb * nb, :]
-                abft.abft_update_gemm(abft.COL, "N", "T", -1.0, X, Y, A_loc[ia * nb:, c0:c1], rows * nb,
-                                      (tb - ta) * nb, nb)
-                if abft_on:
-                    abft.abft_update_gemm(abft.COL, "N", "T", -1.0, Lrow.c[2 * s0:, :], Y, mat.colchk[2 * ia:, c0:c1],
-                                          2 * rows, (tb - ta) * nb, nb, Lrow.m[s0:, :], mat.colmag[ia:, c0:c1])
-                    abft.abft_update_gemm(abft.ROW, "T", "N", -1.0, Lcol.c[2 * ta:2 * tb, :], X,
-                                          mat.rowchk[ia * nb:, 2 * (jl0 + ta):2 * (jl0 + tb)], 2 * (tb - ta),
-                                          rows * nb, nb, Lcol.m[ta:tb, :],
-                                          mat.rowmag[ia * nb:, jl0 + ta:jl0 + tb])
+                abft.abft_update_gemm(abft.COL, "N", "T", -1.0, Lrow.L[s0 * nb:, :], Lcol.L[ta * nb:tb * nb, :],
+                                      A_loc[ia * nb:, (jl0 + ta) * nb:(jl0 + tb) * nb], rows * nb, (tb - ta) * nb, nb)
+            if abft_on:
+                # checksums of the whole local trailing block, one product per
+                # side (entries of upper tiles are updated and never read):
+                # c(A_IJ) -= c(L_ik) L_jk^T,  r(A_IJ) -= L_ik c(L_jk)^T  (c-12)
+                abft.abft_update_gemm(abft.COL, "N", "T", -1.0, Lrow.c, Lcol.L, mat.colchk[2 * ir0:, jl0 * nb:],
+                                      2 * cnt, ncol * nb, nb, Lrow.m, mat.colmag[ir0:, jl0 * nb:])
+                abft.abft_update_gemm(abft.ROW, "T", "N", -1.0, Lcol.c, Lrow.L, mat.rowchk[ir0 * nb:, 2 * jl0:],
+                                      2 * ncol, cnt * nb, nb, Lcol.m, mat.rowmag[ir0 * nb:, jl0:])
             hook(k, abft.AT_POST_TMU)
             # ---- 6. Fig. 4a re-check of the panel copies the update read
             if abft_on:

@@ -111,3 +111,32 @@ def spd_device(n: int, seed: int = 0, dtype=None, device="cuda"):
     S.mul_(0.5)
     S.diagonal().add_(float(n))
     return S.t()
+
+
+def spd_block_cyclic_device(n: int, nb: int, P: int, Q: int, rank: int, seed: int = 0, dtype=None, device="cuda"):
+    """This rank's tiles of the SPD matrix S = (M + M^T)/2 + n*I under the 2D
+    block-cyclic layout (tile (I, J) on rank (I mod P)*Q + J mod Q), as one
+    column-major local matrix.  Tile M_IJ ~ U(-1,1) is drawn from its own
+    seed (seed, I, J), so every rank builds its tiles without the full
+    matrix; the distribution is the one of `spd`/`spd_device`."""
+    import torch
+
+    dtype = dtype or torch.float64
+    nt = n // nb
+    p, q = divmod(rank, Q)
+    rows, cols = list(range(p, nt, P)), list(range(q, nt, Q))
+    buf = torch.empty((len(cols) * nb, len(rows) * nb), dtype=dtype, device=device)  # col-major storage
+    g = torch.Generator(device=device)
+
+    def tile(I, J):
+        g.manual_seed(seed * 1_000_003 + I * nt + J)
+        return torch.rand((nb, nb), generator=g, dtype=dtype, device=device).mul_(2.0).sub_(1.0)
+
+    for jl, J in enumerate(cols):
+        for il, I in enumerate(rows):
+            S = tile(I, J)
+            S.add_(tile(J, I).t()).mul_(0.5)
+            if I == J:
+                S.diagonal().add_(float(n))
+            buf[jl * nb:(jl + 1) * nb, il * nb:(il + 1) * nb] = S.t()
+    return buf.t()
