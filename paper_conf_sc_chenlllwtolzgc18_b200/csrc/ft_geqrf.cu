@@ -63,66 +63,89 @@ __global__ void qr_fix_zero_tau_kernel(T* Tm, const T* tau, int nb) {
   }
 }
 
-// Alg. 1 checksum replay, one warp per checksum row rho of the panel's
-// colchk block (2 (nt-k) rows); tile row 0 of the block is the diagonal tile.
-// The row (and its magnitude row) lives in shared memory for the whole
-// recurrence; ZT = Z^T so step j reads row j of Z contiguously.
-constexpr int kReplayWarps = 4;
-
+// Alg. 1 checksum replay as a triangular solve.  Per checksum row x of the
+// panel's colchk block (2 (nt-k) rows; tile row 0 = the diagonal tile, with
+// weights w = 1 / (i+1), w = 0 elsewhere) Alg. 1 runs, for j = 0..nb-1,
+//   y_j = (x_j - acc_j - beta_j w_j) / den_j,   x_c -= y_j Z[j,c]  (c > j)
+// with den_j = -tau_j beta_j, beta_j = R[j,j], acc_j = sum_{i<j} w_i R[i,j]
+// and Z = T^T V^T P0 (row j = tau_j v_j^T P^(j-1)).  That recurrence is the
+// forward substitution of  y (D + striu(Z)) = b,  b_j = x_j - acc_j - beta_j w_j,
+// so all rows are solved at once as  Y = B (D + striu(Z))^-1  (explicit
+// triangular inverse + one DGEMM) instead of nb dependent steps per row.
+// tau_j = 0 (identity reflector): y_j = w_j and step j changes nothing, i.e.
+// row and column j of the off-diagonal part vanish and D_j = 1, b_j = w_j.
+// Magnitudes (c-6): mv_j = (m_j + |beta_j| [I=0]) / |den_j|, m_c += mv_j |Z[j,c]|
+//   <=>  mv (|D| - striu(|Z|)) = m + |beta| [I=0]  (an M-matrix, inverse >= 0).
 template <typename T>
-__global__ void __launch_bounds__(32 * kReplayWarps) qr_replay_kernel(T* ck, int64_t ldc, T* mck, int64_t ldcm,
-                                                                      int nrows, const T* panel, int64_t lda,
-                                                                      const T* tau, const T* ZT, int nb) {
-  extern __shared__ __align__(16) unsigned char rp_sm[];
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  const int rho = blockIdx.x * kReplayWarps + wid;
-  if (rho >= nrows) return;
-  T* row = reinterpret_cast<T*>(rp_sm) + (size_t)wid * 2 * nb;
-  T* mrow = row + nb;
-  const int I = rho / 2, wt = rho % 2;  // tile row (0 = diagonal tile), weight v1 / v2
-  const bool emag = mck && wt == 0;
-  T* ckr = ck + rho;  // ck[rho, c] = ckr[c * ldc]
-  T* mr = emag ? mck + I : nullptr;
-  for (int c = lane; c < nb; c += 32) {
-    row[c] = ckr[(int64_t)c * ldc];
-    mrow[c] = emag ? mr[(int64_t)c * ldcm] : T(0);
-  }
-  __syncwarp();
-  for (int j = 0; j < nb; ++j) {
-    // c_x = ck[rho, j] - W[rho, :j] R[:j, j]  (rows above j are in the diagonal tile)
-    T acc = T(0);
-    if (I == 0)
-      for (int i = lane; i < j; i += 32) acc = ffma(wt ? T(i + 1) : T(1), panel[i + (int64_t)j * lda], acc);
-    for (int m = 16; m >= 1; m >>= 1) acc = fadd(acc, shfl_xor(acc, m));
-    const T beta = panel[j + (int64_t)j * lda];
-    const T t = tau[j];
-    const T wj = I == 0 ? (wt ? T(j + 1) : T(1)) : T(0);
-    T vck, mv = T(0);
-    if (t == T(0)) {
-      vck = wj;
-      if (emag) mv = I == 0 ? T(1) : T(0);
-    } else {
-      const T cx = row[j] - acc;
-      const T den = -t * beta;  // x1 - beta
-      vck = (cx - beta * wj) / den;
-      if (emag) mv = (mrow[j] + fabs(beta) * (I == 0 ? T(1) : T(0))) / fabs(den);
-      const T* zr = ZT + (int64_t)j * nb;
-      for (int c = j + 1 + lane; c < nb; c += 32) {
-        const T z = zr[c];
-        row[c] -= vck * z;
-        if (emag) mrow[c] += mv * fabs(z);
+__global__ void qr_replay_mats_kernel(T* Tm, T* Mm, const T* ZT, const T* panel, int64_t lda, const T* tau, int nb) {
+  const int64_t total = (int64_t)nb * nb;
+  for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+       idx += (int64_t)gridDim.x * blockDim.x) {
+    const int c = (int)(idx / nb), i = (int)(idx - (int64_t)c * nb);
+    T t = T(0), m = T(0);
+    if (i < c) {
+      if (tau[i] != T(0) && tau[c] != T(0)) {
+        const T z = ZT[c + (int64_t)i * nb];  // Z[i, c]
+        t = z;
+        m = -fabs(z);
+      }
+    } else if (i == c) {
+      if (tau[c] != T(0)) {
+        const T den = -tau[c] * panel[c + (int64_t)c * lda];
+        t = den;
+        m = fabs(den);
+      } else {
+        t = m = T(1);
       }
     }
-    __syncwarp();
-    if (lane == 0) {
-      row[j] = vck;
-      mrow[j] = mv;
-    }
-    __syncwarp();
+    Tm[idx] = t;
+    Mm[idx] = m;
   }
-  for (int c = lane; c < nb; c += 32) {
-    ckr[(int64_t)c * ldc] = row[c];
-    if (emag) mr[(int64_t)c * ldcm] = mrow[c];
+}
+
+// right-hand sides in place: rows 0/1 (diagonal tile) get -acc_j - beta_j w_j;
+// a tau_j = 0 column becomes w_j in every row (0 below the diagonal tile);
+// magnitude row 0 gets +|beta_j|, a tau_j = 0 column becomes [I = 0].
+template <typename T>
+__global__ void qr_replay_rhs_kernel(T* ck, int64_t ldc, T* mck, int64_t ldcm, int nrows, const T* panel, int64_t lda,
+                                     const T* tau, int nb) {
+  const int j = blockIdx.x;
+  T ae = T(0), aw = T(0);
+  for (int i = threadIdx.x; i < j; i += blockDim.x) {
+    const T r = panel[i + (int64_t)j * lda];
+    ae = fadd(ae, r);
+    aw = ffma(T(i + 1), r, aw);
+  }
+  __shared__ T se[32], sw[32];
+  for (int m = 16; m >= 1; m >>= 1) {
+    ae = fadd(ae, shfl_xor(ae, m));
+    aw = fadd(aw, shfl_xor(aw, m));
+  }
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if (lane == 0) {
+    se[wid] = ae;
+    sw[wid] = aw;
+  }
+  __syncthreads();
+  const T t = tau[j];
+  const T beta = panel[j + (int64_t)j * lda];
+  T* col = ck + (int64_t)j * ldc;
+  T* mcol = mck ? mck + (int64_t)j * ldcm : nullptr;
+  if (t == T(0)) {
+    for (int r = threadIdx.x; r < nrows; r += blockDim.x) col[r] = r == 0 ? T(1) : (r == 1 ? T(j + 1) : T(0));
+    if (mcol)
+      for (int r = threadIdx.x; r < nrows / 2; r += blockDim.x) mcol[r] = r == 0 ? T(1) : T(0);
+    return;
+  }
+  if (threadIdx.x == 0) {
+    T e = T(0), w = T(0);
+    for (int q = 0; q < (int)(blockDim.x >> 5); ++q) {
+      e = fadd(e, se[q]);
+      w = fadd(w, sw[q]);
+    }
+    col[0] = col[0] - e - beta;
+    col[1] = col[1] - w - beta * T(j + 1);
+    if (mcol) mcol[0] = mcol[0] + fabs(beta);
   }
 }
 
@@ -247,15 +270,24 @@ static int panel_geqrf_t(const abft_mat_t* mat, int k, T* tau, T* Vbuf, T* Tout,
   const int nrows = (int)(2 * (nt - k));
   T* ck = reinterpret_cast<T*>(mat->colchk) + 2 * k + r0 * mat->ldc;
   T* mck = mat->colmag ? reinterpret_cast<T*>(mat->colmag) + k + r0 * mat->ldcm : nullptr;
-  const size_t rsm = (size_t)kReplayWarps * 2 * nb * sizeof(T);
-  static bool rattr = false;
-  if (!rattr) {
-    ABFT_CUDA_TRY(cudaFuncSetAttribute(qr_replay_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024));
-    rattr = true;
-  }
-  qr_replay_kernel<T><<<(unsigned)((nrows + kReplayWarps - 1) / kReplayWarps), 32 * kReplayWarps, rsm, s>>>(
-      ck, mat->ldc, mck, mat->ldcm, nrows, panel, mat->lda, tau, ZT, (int)nb);
+  T* Tm = Ti;  // free again: D + striu(Z)
+  T* Mm = G;   // |D| - striu(|Z|)
+  void* wv = nullptr;
+  FT_TRY(scratch(s, 16, (size_t)nb * nb * 2 * sizeof(T), &wv));
+  T* W1 = reinterpret_cast<T*>(wv);
+  T* W2 = W1 + (size_t)nb * nb;
+  qr_replay_mats_kernel<T><<<blocks_of(nb * nb), 256, 0, s>>>(Tm, Mm, ZT, panel, mat->lda, tau, (int)nb);
+  qr_replay_rhs_kernel<T><<<(unsigned)nb, 128, 0, s>>>(ck, mat->ldc, mck, mat->ldcm, nrows, panel, mat->lda, tau,
+                                                        (int)nb);
   ABFT_CUDA_TRY(cudaGetLastError());
+  FT_TRY(abft_tri_inverse(mat->dtype, 'U', 'N', nb, Tm, nb, W1, nb, (abft_stream_t)s));
+  FT_TRY(abft_update_trsm_inv(mat->dtype, 'R', 'N', nb, W1, nb, ck, mat->ldc, nrows, nullptr, 0, 0,
+                              (abft_stream_t)s));
+  if (mck) {
+    FT_TRY(abft_tri_inverse(mat->dtype, 'U', 'N', nb, Mm, nb, W2, nb, (abft_stream_t)s));
+    FT_TRY(abft_update_trsm_inv(mat->dtype, 'R', 'N', nb, W2, nb, mck, mat->ldcm, nrows / 2, nullptr, 0, 0,
+                                (abft_stream_t)s));
+  }
   // r(R): r(P) <- Q^T r(P) for the panel's row checksums (m_k x 2)
   {
     std::unique_lock<std::mutex> lk;
