@@ -20,7 +20,7 @@ __global__ void lu_pivots_kernel(const int32_t* piv_local, int64_t* ipiv_global,
 // distinct moved rows), src[s] = slot in S of the row whose value ends at
 // S[s] after all nb swaps, tb[T - k] = first slot in tile row T (T = k..nt).
 // One CTA of 1024 threads: bitonic sort in shared memory, then the nb swaps
-// replayed on slot contents by one thread (binary search row -> slot).
+// replayed on slot contents by one thread (row -> slot found in parallel).
 __global__ void __launch_bounds__(1024) lu_perm_kernel(const int32_t* piv_local, int nb, int64_t r0, int nt, int k,
                                                        int64_t* S, int32_t* src, int32_t* tb, int32_t* nrows) {
   __shared__ int64_t key[2048];
@@ -51,27 +51,74 @@ __global__ void __launch_bounds__(1024) lu_perm_kernel(const int32_t* piv_local,
       }
       __syncthreads();
     }
-  if (tid == 0) {  // unique + permutation replay (serial, <= 2 nb entries)
-    int n = 0;
-    for (int i = 0; i < 2048 && key[i] != INT64_MAX; ++i)
-      if (n == 0 || key[i] != key[n - 1]) key[n++] = key[i];
-    cnt = n;
-    for (int i = 0; i < n; ++i) content[i] = i;
-    auto slot = [&](int64_t r) {
-      int lo = 0, hi = n - 1;
+  // unique: keep key[i] if it differs from key[i-1] (block scan of the flags)
+  __shared__ int32_t wsum[32];
+  __shared__ int64_t ukey[2048];
+  __shared__ int16_t slotp[1024], slotq[1024];
+  {
+    const int i0 = 2 * tid, i1 = 2 * tid + 1;  // 1024 threads x 2 entries
+    const int f0 = key[i0] != INT64_MAX && (i0 == 0 || key[i0] != key[i0 - 1]);
+    const int f1 = key[i1] != INT64_MAX && key[i1] != key[i1 - 1];
+    int v = f0 + f1, incl = v;
+    const int lane = tid & 31, wid = tid >> 5;
+    for (int m = 1; m < 32; m <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, incl, m);
+      if (lane >= m) incl += y;
+    }
+    if (lane == 31) wsum[wid] = incl;
+    __syncthreads();
+    if (wid == 0) {
+      int w = wsum[lane], wi = w;
+      for (int m = 1; m < 32; m <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, wi, m);
+        if (lane >= m) wi += y;
+      }
+      wsum[lane] = wi - w;  // exclusive warp offsets
+      if (lane == 31) cnt = wi;
+    }
+    __syncthreads();
+    const int excl = wsum[wid] + incl - v;
+    if (f0) ukey[excl] = key[i0];
+    if (f1) ukey[excl + f0] = key[i1];
+  }
+  __syncthreads();
+  const int nu = cnt;
+  for (int i = tid; i < 2048; i += blockDim.x) {
+    key[i] = i < nu ? ukey[i] : INT64_MAX;
+    content[i] = i;
+  }
+  __syncthreads();
+  // row -> slot for both rows of every swap (parallel binary searches)
+  for (int j = tid; j < nb; j += blockDim.x) {
+    const int64_t p = r0 + j, q = r0 + piv_local[j] - 1;
+    int sp = -1, sq = -1;
+    if (p != q) {
+      int lo = 0, hi = nu - 1;
       while (lo < hi) {
         const int mid = (lo + hi) >> 1;
-        if (key[mid] < r) lo = mid + 1; else hi = mid;
+        if (key[mid] < p) lo = mid + 1; else hi = mid;
       }
-      return lo;
-    };
+      sp = lo;
+      lo = 0;
+      hi = nu - 1;
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (key[mid] < q) lo = mid + 1; else hi = mid;
+      }
+      sq = lo;
+    }
+    slotp[j] = (int16_t)sp;
+    slotq[j] = (int16_t)sq;
+  }
+  __syncthreads();
+  if (tid == 0) {  // the nb swaps in LAPACK order on slot contents (serial)
     for (int j = 0; j < nb; ++j) {
-      const int64_t p = r0 + j, q = r0 + piv_local[j] - 1;
-      if (p == q) continue;
-      const int a = slot(p), b = slot(q);
-      const int t = content[a];
-      content[a] = content[b];
-      content[b] = t;
+      const int a2 = slotp[j];
+      if (a2 < 0) continue;
+      const int b2 = slotq[j];
+      const int t = content[a2];
+      content[a2] = content[b2];
+      content[b2] = t;
     }
   }
   __syncthreads();
@@ -136,7 +183,8 @@ __global__ void lu_row_check_kernel(const T* A, int64_t lda, const T* rowchk, in
 // the c-14 column-checksum deltas, applied as the net permutation of the moved
 // rows: one CTA per column gathers the moved values into shared memory, the
 // thread of each tile row sums its deltas in slot order (deterministic), then
-// the permuted values are written back.  Panel columns only update their
+// the permuted values are written back.  (Warp per tile row, lanes strided
+// over its slots, butterfly reduction: a fixed order, so deterministic.)  Panel columns only update their
 // checksums, with values from the pre-PD copy (L430).  Equal to the sequential
 // swap rule in exact arithmetic.
 template <typename T>
@@ -153,23 +201,31 @@ __global__ void __launch_bounds__(256) lu_perm_cols_kernel(T* A, int64_t lda, in
   const T* col = panel ? pcopy + (c - r0) * ldp - r0 : A + c * lda;
   for (int s = threadIdx.x; s < n; s += blockDim.x) xs[s] = col[S[s]];
   __syncthreads();
-  if (colchk) {
-    for (int T0 = threadIdx.x; T0 < nt - k; T0 += blockDim.x) {
+  if (colchk) {  // one warp per tile row: lane-strided slots, butterfly sum
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    for (int T0 = wid; T0 < nt - k; T0 += nw) {
       const int b = tb[T0], e = tb[T0 + 1];
       if (b == e) continue;
       const int64_t base = (int64_t)(k + T0) * nb;
       T de = T(0), dw = T(0), da = T(0);
-      for (int s = b; s < e; ++s) {
+      for (int s = b + lane; s < e; s += 32) {
         const T xn = xs[src[s]], xo = xs[s];
         const T d = xn - xo;
         de += d;
         dw += T(S[s] - base + 1) * d;
         da += fabs(xn) - fabs(xo);
       }
-      const int64_t P = k + T0;
-      colchk[2 * P + c * ldc] += de;
-      colchk[2 * P + 1 + c * ldc] += dw;
-      if (colmag) colmag[P + c * ldcm] += da;
+      for (int m = 16; m >= 1; m >>= 1) {
+        de += shfl_xor(de, m);
+        dw += shfl_xor(dw, m);
+        da += shfl_xor(da, m);
+      }
+      if (lane == 0) {
+        const int64_t P = k + T0;
+        colchk[2 * P + c * ldc] += de;
+        colchk[2 * P + 1 + c * ldc] += dw;
+        if (colmag) colmag[P + c * ldcm] += da;
+      }
     }
   }
   if (panel) return;  // getrf already permuted the panel data
