@@ -312,9 +312,9 @@ def run_ours(args):
     # ---- ft_potrf overhead at n=30720 (the metric's second half) ----
     ftp = lq = None
     if not args.no_potrf and rank == 0:
-        ftp = potrf_overhead(abft, si, args.potrf_n, nb, args.potrf_reps)
+        ftp = potrf_overhead(abft, si, args.potrf_n, nb, args.potrf_reps, host_pd=not args.no_host_pd)
     if not args.no_lu_qr and rank == 0:
-        lq = lu_qr_overhead(abft, si, args.lu_qr_n, nb, args.lu_qr_reps)
+        lq = lu_qr_overhead(abft, si, args.lu_qr_n, nb, args.lu_qr_reps, host_pd=not args.no_host_pd)
 
     cpu = cpu_baseline_sample(args.cpu_seconds) if (rank == 0 and world == 1 and not args.no_cpu) else None
     if rank == 0:
@@ -339,7 +339,7 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
-def potrf_overhead(abft, si, n, nb, reps):
+def potrf_overhead(abft, si, n, nb, reps, host_pd=True):
     """T_ft vs T_plain of the same blocked driver, plus cuSOLVER
     potrf as context; ms are CUDA-event times on the driver's stream."""
     import torch
@@ -348,12 +348,12 @@ def potrf_overhead(abft, si, n, nb, reps):
     A = torch.empty_like(A0.t()).t()
     ctx = abft.Context()
 
-    def run(ft, restart=True):
+    def run(ft, restart=True, pd=abft.PD_DEVICE):
         A.copy_(A0)
         torch.cuda.synchronize()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record()
-        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart)
+        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart, pd_location=pd)
         b.record()
         torch.cuda.synchronize()
         assert rc == 0 and info == 0
@@ -373,6 +373,16 @@ def potrf_overhead(abft, si, n, nb, reps):
     t_nors.sort()
     ft_ms, plain_ms = t_ft[len(t_ft) // 2], t_plain[len(t_plain) // 2]
     nors_ms = t_nors[len(t_nors) // 2]
+    host = None
+    if host_pd:  # Alg. 2 lines 3-7 with the PD on the host (FT_PD_HOST)
+        import os
+
+        ctx.set_host_lapack()
+        run(True, pd=abft.PD_HOST)
+        hf, hst = run(True, pd=abft.PD_HOST)
+        hp = run(False, pd=abft.PD_HOST)[0]
+        host = {"ms_ft": hf, "ms_plain": hp, "overhead_pct": 100.0 * (hf - hp) / hp, "ms_host_pd": hst.ms_host_pd,
+                "host_cores": len(os.sched_getaffinity(0)), "lapack": os.path.basename(ctx.host_lapack)}
     # cuSOLVER dpotrf of the whole matrix (context)
     S = A0.t().contiguous()
     torch.backends.cuda.preferred_linalg_library("cusolver")
@@ -389,7 +399,7 @@ def potrf_overhead(abft, si, n, nb, reps):
     return {"n": n, "nb": nb, "ms_ft": ft_ms, "ms_plain": plain_ms,
             "overhead_pct": 100.0 * (ft_ms - plain_ms) / plain_ms, "cusolver_potrf_ms": cus,
             "ms_ft_no_restart": nors_ms, "overhead_pct_no_restart": 100.0 * (nors_ms - plain_ms) / plain_ms,
-            "tflops_ft": n ** 3 / 3 / (ft_ms / 1e3) / 1e12, "reps": reps}
+            "tflops_ft": n ** 3 / 3 / (ft_ms / 1e3) / 1e12, "reps": reps, "host_pd": host}
 
 
 def mgpu_overhead(si, n, nb, reps, world, rank):
@@ -439,14 +449,19 @@ def mgpu_overhead(si, n, nb, reps, world, rank):
             "comm": "NCCL broadcast of L_kk and of each process row's panel piece; int32 report all-reduce"}
 
 
-def lu_qr_overhead(abft, si, n, nb, reps):
+def lu_qr_overhead(abft, si, n, nb, reps, host_pd=True):
     """BASELINE configs[2]: ft_getrf / ft_geqrf at n=20480 nb=512, ABFT on vs
-    the same driver with ABFT off; cuSOLVER getrf / geqrf as context."""
+    the same driver with ABFT off; cuSOLVER getrf / geqrf as context.  With
+    host_pd, also the FT_PD_HOST drivers (Alg. 2 lines 3-7: guarded panel
+    round trip through pinned host memory around the host LAPACK, the
+    configuration's 'panel/PCIe-transfer verification'), ABFT on vs off."""
     import torch
 
     A0 = si.general_device(n, seed=21)
     A = torch.empty_like(A0.t()).t()
     ctx = abft.Context()
+    if host_pd:
+        ctx.set_host_lapack()
     ipiv = torch.zeros(n, dtype=torch.int64, device="cuda")
     tau = torch.zeros(n, dtype=torch.float64, device="cuda")
     out = {"n": n, "nb": nb, "reps": reps}
@@ -470,6 +485,17 @@ def lu_qr_overhead(abft, si, n, nb, reps):
         tp = sorted(run(fn, False) for _ in range(reps))[reps // 2]
         out[name] = {"ms_ft": tf, "ms_plain": tp, "overhead_pct": 100.0 * (tf - tp) / tp,
                      "tflops_ft": flops / (tf / 1e3) / 1e12}
+    if host_pd:
+        import os
+
+        for name, fn in [("getrf", lambda ft: abft.ft_getrf(ctx, A, nb, ipiv, abft=ft, pd_location=abft.PD_HOST)),
+                         ("geqrf", lambda ft: abft.ft_geqrf(ctx, A, nb, tau, abft=ft, pd_location=abft.PD_HOST))]:
+            run(fn, True)
+            tf = run(fn, True)
+            tp = run(fn, False)
+            out[name]["host_pd"] = {"ms_ft": tf, "ms_plain": tp, "overhead_pct": 100.0 * (tf - tp) / tp,
+                                    "host_cores": len(os.sched_getaffinity(0)),
+                                    "lapack": os.path.basename(ctx.host_lapack)}
     torch.backends.cuda.preferred_linalg_library("cusolver")
     G = A0.t().contiguous()
     for name, fn in [("getrf", lambda: torch.linalg.lu_factor(G)), ("geqrf", lambda: torch.geqrf(G))]:
@@ -502,6 +528,7 @@ def main():
     ap.add_argument("--lu-qr-n", type=int, default=20480)
     ap.add_argument("--lu-qr-reps", type=int, default=1)
     ap.add_argument("--no-lu-qr", action="store_true")
+    ap.add_argument("--no-host-pd", action="store_true")
     ap.add_argument("--mgpu-n", type=int, default=61440)
     ap.add_argument("--mgpu-reps", type=int, default=1)
     ap.add_argument("--no-mgpu", action="store_true")

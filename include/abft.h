@@ -306,8 +306,15 @@ typedef struct ft_ctx ft_ctx_t;
  * target: 0 = A, 1 = colchk, 2 = rowchk; (gi, gj) element of that array. */
 enum {
   FT_AT_PRE_PD_CHECK = 0, FT_AT_PRE_PD = 1, FT_AT_POST_PD = 2, FT_AT_PRE_PU_CHECK = 3,
-  FT_AT_PRE_PU = 4, FT_AT_POST_PU = 5, FT_AT_PRE_TMU = 6, FT_AT_POST_TMU = 7
+  FT_AT_PRE_PU = 4, FT_AT_POST_PU = 5, FT_AT_PRE_TMU = 6, FT_AT_POST_TMU = 7,
+  /* pd_location = FT_PD_HOST only (Alg. 2 lines 3 and 6): a flip in the host
+   * copy right after the device-to-host transfer of iteration iter's panel,
+   * or in the device panel right after the host-to-device transfer of the
+   * factored panel (target must be 0 = A; first trip of the iteration only) */
+  FT_AT_D2H = 8, FT_AT_H2D = 9
 };
+/* Where the panel decomposition runs (ft_opts_t.pd_location). */
+enum { FT_PD_DEVICE = 0, FT_PD_HOST = 1 };
 enum { FT_KIND_PERSIST = 0, FT_KIND_ONCHIP = 1 };
 typedef struct {
   int32_t iter, point, kind, target;
@@ -331,6 +338,16 @@ typedef struct {
   int32_t restart;       /* 1: local restart (L430): copy the PD / PU input with its checksums after the
                             pre-op check; a 2D error left by the post-op check restores the copy and
                             redoes the op once (one 8-byte read-back per check; ft_potrf) */
+  int32_t pd_location;   /* FT_PD_DEVICE (default): PD by cuSOLVER on the device.  FT_PD_HOST: Alg. 2
+                            lines 3-7 as the paper runs them (L364-L372, L61): the panel (Cholesky:
+                            A_kk; LU/QR: the m_k x nb column panel) goes to pinned host memory, is
+                            factored there by the host LAPACK set with ft_ctx_set_host_lapack, and
+                            comes back; with abft, both transfers carry a fresh column-checksum
+                            guard (reading c-28): the host checks what it received (locate/correct,
+                            else re-transfer), the device verifies + corrects the factored panel
+                            (abft_verify / abft_locate_correct; uncorrectable -> re-send), then the
+                            PD checksum rule and the post-PD check run on the device as usual.
+                            The host waits for the device once per iteration. */
 } ft_opts_t;
 
 /* Host-side statistics, filled after the driver's final synchronisation. */
@@ -343,10 +360,27 @@ typedef struct {
   int32_t n_checks;             /* verify calls issued */
   double ms_total;
   int32_t restarts;             /* local restarts performed (f1) */
+  /* FT_PD_HOST transfer guard (reading c-28) */
+  int32_t xfer_d2h_flagged;     /* host check: columns whose guard residual was flagged */
+  int32_t xfer_d2h_fixed;       /* host check: elements corrected */
+  int32_t xfer_retransfers;     /* device-to-host transfers repeated */
+  int32_t xfer_h2d_flagged;     /* device check: flagged columns */
+  int32_t xfer_h2d_fixed;       /* device check: elements corrected (also in the fix log) */
+  int32_t xfer_resends;         /* host-to-device transfers repeated */
+  int32_t xfer_uncorrectable;   /* transfers still wrong after 2 repeats (-> uncorrectable) */
+  double ms_host_pd;            /* wall time of the host round trips (transfers + host PD) */
 } ft_stats_t;
 
 ABFT_API int ft_ctx_create(ft_ctx_t **ctx, int32_t device, abft_stream_t stream);
 ABFT_API int ft_ctx_destroy(ft_ctx_t *ctx);
+
+/* Host LAPACK for pd_location = FT_PD_HOST: `path` is a shared library with
+ * the LP64 (int32) Fortran LAPACK symbols dpotrf_/spotrf_, dgetrf_/sgetrf_,
+ * dgeqrf_/sgeqrf_, plain or with the "scipy_" prefix (the OpenBLAS bundled with
+ * SciPy).  Host pointer; the library is dlopen'ed and kept until
+ * ft_ctx_destroy.  Returns ABFT_E_UNSUPPORTED when it cannot be loaded or a
+ * symbol is missing. */
+ABFT_API int ft_ctx_set_host_lapack(ft_ctx_t *ctx, const char *path);
 
 /* ft_potrf — fault-tolerant lower Cholesky A = L L^T of the n x n SPD matrix
  * dA (device, lda >= n, n % nb == 0), right-looking blocked, Alg. 2 order

@@ -32,7 +32,9 @@ NCOUNTS = 8
 E_UNCORRECTABLE = 5
 AT_PRE_PD_CHECK, AT_PRE_PD, AT_POST_PD, AT_PRE_PU_CHECK = 0, 1, 2, 3
 AT_PRE_PU, AT_POST_PU, AT_PRE_TMU, AT_POST_TMU = 4, 5, 6, 7
+AT_D2H, AT_H2D = 8, 9
 KIND_PERSIST, KIND_ONCHIP = 0, 1
+PD_DEVICE, PD_HOST = 0, 1
 
 
 # ------------------------------------------------------------- structs ----
@@ -78,13 +80,16 @@ class ft_opts_t(C.Structure):
     _fields_ = [("nb", C.c_int64), ("abft", C.c_int32), ("tol_kind", C.c_int32), ("tol_scale", C.c_double),
                 ("fig4a_repair", C.c_int32), ("n_inject", C.c_int32), ("inject", C.POINTER(ft_inject_t)),
                 ("fix_log", C.c_void_p), ("fix_log_cap", C.c_int32), ("pu_gemm", C.c_int32),
-                ("refresh", C.c_int32), ("restart", C.c_int32)]
+                ("refresh", C.c_int32), ("restart", C.c_int32), ("pd_location", C.c_int32)]
 
 
 class ft_stats_t(C.Structure):
     _fields_ = [("counts", C.c_int32 * NCOUNTS), ("n_fixes", C.c_int32), ("repairs_applied", C.c_int32),
                 ("repairs_skipped", C.c_int32), ("uncorrectable", C.c_int32), ("n_checks", C.c_int32),
-                ("ms_total", C.c_double), ("restarts", C.c_int32)]
+                ("ms_total", C.c_double), ("restarts", C.c_int32),
+                ("xfer_d2h_flagged", C.c_int32), ("xfer_d2h_fixed", C.c_int32), ("xfer_retransfers", C.c_int32),
+                ("xfer_h2d_flagged", C.c_int32), ("xfer_h2d_fixed", C.c_int32), ("xfer_resends", C.c_int32),
+                ("xfer_uncorrectable", C.c_int32), ("ms_host_pd", C.c_double)]
 
 
 _L = _lib.load()
@@ -112,6 +117,7 @@ _sig = {
     "ft_ctx_create": [_P(_vp), _i32, _vp],
     "ft_ctx_destroy": [_vp],
     "ft_potrf": [_vp, _i32, _i64, _vp, _i64, _P(ft_opts_t), _P(ft_stats_t), _P(_i64)],
+    "ft_ctx_set_host_lapack": [_vp, C.c_char_p],
 }
 for _name, _args in _sig.items():
     _f = getattr(_L, _name)
@@ -332,6 +338,15 @@ class Context:
         self._h = C.c_void_p()
         _check("ft_ctx_create", _L.ft_ctx_create(C.byref(self._h), dev, _stream(stream)))
 
+    def set_host_lapack(self, path=None):
+        """Host LAPACK for pd_location=PD_HOST (Alg. 2's CPU panel, L61):
+        `path` to a shared library with LP64 dpotrf_/dgetrf_/dgeqrf_ (and the
+        s-variants); default: the OpenBLAS bundled with SciPy."""
+        if path is None:
+            path = host_lapack_path()
+        _check("ft_ctx_set_host_lapack", _L.ft_ctx_set_host_lapack(self._h, path.encode()))
+        self.host_lapack = path
+
     def __del__(self):
         h = getattr(self, "_h", None)
         if h is not None and h.value and _L is not None:
@@ -339,13 +354,27 @@ class Context:
             self._h = None
 
 
-def _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh=True, restart=True):
+def host_lapack_path():
+    """The LP64 OpenBLAS shipped in scipy.libs (exports scipy_dpotrf_ etc.)."""
+    import glob
+
+    import scipy
+
+    libs = os.path.join(os.path.dirname(os.path.dirname(scipy.__file__)), "scipy.libs")
+    cands = sorted(glob.glob(os.path.join(libs, "libscipy_openblas-*.so")))
+    if not cands:
+        raise FileNotFoundError(f"no libscipy_openblas-*.so under {libs}")
+    return cands[0]
+
+
+def _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh=True, restart=True,
+          pd_location=PD_DEVICE):
     inj = (ft_inject_t * max(1, len(inject)))()
     for k, f in enumerate(inject):
         inj[k] = ft_inject_t(*f)
     opts = ft_opts_t(nb, int(abft), tol_kind, tol_scale, int(fig4a_repair), len(inject), inj,
                      _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES, int(pu_gemm),
-                     int(refresh), int(restart))
+                     int(refresh), int(restart), int(pd_location))
     return opts, inj
 
 
@@ -361,11 +390,12 @@ def abft_panel_getrf(mat: Mat, k: int, ipiv: torch.Tensor, Linv: torch.Tensor, U
 
 
 def ft_getrf(ctx: Context, A: torch.Tensor, nb: int, ipiv: torch.Tensor, abft=True, tol_kind=TOL_MAGNITUDE,
-             tol_scale=1.0, fig4a_repair=True, inject=(), fix_log=None):
+             tol_scale=1.0, fig4a_repair=True, inject=(), fix_log=None, pd_location=PD_DEVICE):
     """Fault-tolerant LU with partial pivoting in place on a column-major A;
     ipiv: int64 device tensor (n), receives 1-based global pivots."""
     n = A.shape[0]
-    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, True)
+    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, True,
+                       pd_location=pd_location)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_getrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), _ptr(ipiv), C.byref(opts), C.byref(stats),
@@ -382,11 +412,11 @@ def abft_panel_geqrf(mat: Mat, k: int, tau: torch.Tensor, V: torch.Tensor, T: to
 
 
 def ft_geqrf(ctx: Context, A: torch.Tensor, nb: int, tau: torch.Tensor, abft=True, tol_kind=TOL_MAGNITUDE,
-             tol_scale=1.0, inject=(), fix_log=None):
+             tol_scale=1.0, inject=(), fix_log=None, pd_location=PD_DEVICE):
     """Fault-tolerant Householder QR in place on a column-major A (LAPACK
     dgeqrf storage); tau: device tensor (n) of A's dtype."""
     n = A.shape[0]
-    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, True, inject, fix_log, True)
+    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, True, inject, fix_log, True, pd_location=pd_location)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_geqrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), _ptr(tau), C.byref(opts), C.byref(stats),
@@ -396,11 +426,14 @@ def ft_geqrf(ctx: Context, A: torch.Tensor, nb: int, tau: torch.Tensor, abft=Tru
 
 
 def ft_potrf(ctx: Context, A: torch.Tensor, nb: int, abft=True, tol_kind=TOL_MAGNITUDE, tol_scale=1.0,
-             fig4a_repair=True, inject=(), fix_log=None, pu_gemm=True, refresh=True, restart=True):
+             fig4a_repair=True, inject=(), fix_log=None, pu_gemm=True, refresh=True, restart=True,
+             pd_location=PD_DEVICE):
     """Fault-tolerant lower Cholesky in place on a column-major A.  Returns
-    (rc, info, stats) with rc 0 or E_UNCORRECTABLE (other codes raise)."""
+    (rc, info, stats) with rc 0 or E_UNCORRECTABLE (other codes raise).
+    pd_location=PD_HOST needs ctx.set_host_lapack() first."""
     n = A.shape[0]
-    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh, restart)
+    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh, restart,
+                       pd_location)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_potrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), C.byref(opts), C.byref(stats), C.byref(info))

@@ -7,7 +7,9 @@
 
 #include <algorithm>
 #include <chrono>
+#include <cstring>
 #include <mutex>
+#include <string>
 #include <vector>
 
 #include "abft_common.cuh"
@@ -45,6 +47,13 @@ struct ft_ctx {
   size_t rsv_bytes = 0;
   int32_t* hpin = nullptr;  // pinned host words for the restart read-back
   cudaEvent_t ev = nullptr;  // marks the PD-check read-back (restart decision)
+  // FT_PD_HOST (ft_host.cu): host LAPACK, pinned panel staging, device guard
+  void* lapack = nullptr;  // dlopen handle
+  void* lp[6] = {};        // dpotrf spotrf dgetrf sgetrf dgeqrf sgeqrf
+  char* hstage = nullptr;  // pinned: panel | guard | tau | ipiv | counts | work
+  size_t hstage_bytes = 0;
+  void* dguard = nullptr;  // device transfer guard
+  size_t dguard_bytes = 0;
 };
 
 namespace abft {
@@ -84,6 +93,12 @@ struct Driver {
   int restarts = 0;
   std::vector<ft_inject_t> onchip_pending;
   int n_checks = 0;
+  // FT_PD_HOST bookkeeping (ft_host.cu)
+  int32_t* xcounts = nullptr;          // device int32[8]: counts of one H2D guard check
+  int32_t* mark2 = nullptr;            // device: fix-log position before an H2D guard check
+  int xs[7] = {};                      // ft_stats_t.xfer_* accumulators
+  double ms_host = 0.0;
+  std::vector<std::pair<int, int>> xfer_used;  // (iter, point) transfer faults already applied
 
   int setup(ft_ctx* ctx, int32_t dt, int64_t n_, int64_t nb_, void* dA, int64_t lda_, const ft_opts_t* opts,
             bool is_lu) {
@@ -101,7 +116,9 @@ struct Driver {
     const bool ft = o->abft != 0;
     size_t need = ft ? (size_t)(2 * nt * n + n * 2 * nt + nt * n + n * nt) * es : 0;
     FT_TRY(grow_buffer(c->state, c->state_bytes, need));
-    size_t ints_need = (size_t)nt * nt + 8 + 8;
+    if (o->pd_location == FT_PD_HOST && !c->lapack) return ABFT_E_UNSUPPORTED;
+    if (o->pd_location != FT_PD_DEVICE && o->pd_location != FT_PD_HOST) return ABFT_E_UNSUPPORTED;
+    size_t ints_need = (size_t)nt * nt + 8 + 8 + 8;
     void* ip = c->ints;
     FT_TRY(grow_buffer(ip, c->ints_n, ints_need * sizeof(int32_t)));
     c->ints = reinterpret_cast<int32_t*>(ip);
@@ -116,6 +133,8 @@ struct Driver {
     rep = info + 1;
     info_total = rep + 2;
     snap = info_total + 1;
+    mark2 = snap + 1;
+    xcounts = counts + 16;
     if (o->abft && o->restart)
       FT_TRY(grow_buffer(c->rsv, c->rsv_bytes, ((size_t)n * nb + (size_t)nb * nb + 3 * (size_t)nt * nb + 4 * nb) * es));
     ABFT_CUDA_TRY(cudaMemsetAsync(c->ints, 0, ints_need * sizeof(int32_t), s));
@@ -195,6 +214,9 @@ struct Driver {
     }
     return false;
   }
+  int inject_at_elem(const ft_inject_t& f) {  // one planned flip, now (transfer hooks)
+    return abft_inject(elem(f.target, f.gi, f.gj), dtype, 0, f.xor_mask, (abft_stream_t)s);
+  }
   int restore_onchip() {  // after the op's data step: undo on-chip flips (the stored value was never wrong)
     for (auto& f : onchip_pending)
       FT_TRY(abft_inject(elem(f.target, f.gi, f.gj), dtype, 0, f.xor_mask, (abft_stream_t)s));
@@ -234,9 +256,21 @@ struct Driver {
       stats->n_checks = n_checks;
       stats->restarts = restarts;
       stats->ms_total = std::chrono::duration<double, std::milli>(t1 - t0).count();
+      int32_t* x = &stats->xfer_d2h_flagged;
+      for (int i = 0; i < 7; ++i) x[i] = xs[i];
+      stats->ms_host_pd = ms_host;
     }
     return h[ABFT_CNT_UNCORRECTABLE] ? ABFT_E_UNCORRECTABLE : 0;
   }
 };
+
+// FT_PD_HOST (ft_host.cu): Alg. 2 lines 3-7 for the panel of iteration k,
+// rows x nb at (row0, col0) of A: guarded D2H, host check, host LAPACK
+// factorization (kind), guarded H2D, device check.  Writes the LAPACK info to
+// info_dev (device int32), the 1-based local pivots to piv_dev (GETRF) and
+// tau to tau_dev (GEQRF).
+enum { HOST_POTRF = 0, HOST_GETRF = 1, HOST_GEQRF = 2 };
+int host_panel_pd(Driver& d, int k, int kind, int64_t row0, int64_t col0, int64_t rows, int32_t* piv_dev,
+                  void* tau_dev, int32_t* info_dev);
 
 }  // namespace abft

@@ -213,14 +213,16 @@ static int qr_rows_rule(cublasHandle_t h, cudaStream_t s, int64_t mk, int nb, in
 
 template <typename T>
 static int panel_geqrf_t(const abft_mat_t* mat, int k, T* tau, T* Vbuf, T* Tout, T* P0, int32_t* info,
-                         cudaStream_t s) {
+                         cudaStream_t s, Driver* host = nullptr) {
   const int64_t nb = mat->nb, n = mat->n, nt = n / nb, r0 = k * nb, mk = n - r0;
   const bool ft = mat->colchk != nullptr;
   T* A = reinterpret_cast<T*>(mat->A);
   T* panel = A + r0 + r0 * mat->lda;
   if (ft)
     FT_TRY(abft::copy2d(P0, mk * sizeof(T), panel, mat->lda * sizeof(T), mk * sizeof(T), nb, s));
-  {
+  if (host) {  // FT_PD_HOST: Alg. 2 lines 3-7 around the host dgeqrf (ft_host.cu)
+    FT_TRY(host_panel_pd(*host, k, HOST_GEQRF, r0, r0, mk, nullptr, tau, info));
+  } else {
     std::unique_lock<std::mutex> lk;
     cusolverDnHandle_t h = solver_handle(s, lk);
     int lwork = 0;
@@ -346,7 +348,10 @@ static int geqrf_driver(Driver& d, ft_ctx* c, T* tau_all) {
     if (ft) FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH));
     // line 5: PD (Alg. 1: V with c(V), R_kk with r(R)) + CTF
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD));
-    FT_TRY(abft_panel_geqrf(&d.M, k, tau_all + r0, Vbuf, Tm, P0, d.info, as));
+    if (d.o->pd_location == FT_PD_HOST)
+      FT_TRY(panel_geqrf_t<T>(&d.M, k, tau_all + r0, Vbuf, Tm, P0, d.info, s, &d));
+    else
+      FT_TRY(abft_panel_geqrf(&d.M, k, tau_all + r0, Vbuf, Tm, P0, d.info, as));
     accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.info_total, r0);
     FT_TRY(d.restore_onchip());
     FT_TRY(d.inject_at(k, FT_AT_POST_PD));

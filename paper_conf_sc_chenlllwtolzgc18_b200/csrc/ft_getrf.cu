@@ -337,9 +337,22 @@ static unsigned blocks_for(int64_t work, int per) {
 }  // namespace abft
 
 // ------------------------------------------------------------ panel getrf --
+// host != nullptr: the panel factorization is the FT_PD_HOST round trip
+// (Alg. 2 lines 3-7, ft_host.cu) instead of cuSOLVER; everything else is the
+// same device work.
+static int panel_getrf_impl(const abft_mat_t* mat, int32_t k, int64_t* ipiv, const abft_tol_t* tol,
+                            const abft_report_t* rep, abft_fix_t* fixes, int32_t max_fixes, int32_t* n_fixes,
+                            void* Linv, void* Uinv, int32_t* info, abft_stream_t stream, abft::Driver* host);
+
 extern "C" int abft_panel_getrf(const abft_mat_t* mat, int32_t k, int64_t* ipiv, const abft_tol_t* tol,
                                 const abft_report_t* rep, abft_fix_t* fixes, int32_t max_fixes, int32_t* n_fixes,
                                 void* Linv, void* Uinv, int32_t* info, abft_stream_t stream) {
+  return panel_getrf_impl(mat, k, ipiv, tol, rep, fixes, max_fixes, n_fixes, Linv, Uinv, info, stream, nullptr);
+}
+
+static int panel_getrf_impl(const abft_mat_t* mat, int32_t k, int64_t* ipiv, const abft_tol_t* tol,
+                            const abft_report_t* rep, abft_fix_t* fixes, int32_t max_fixes, int32_t* n_fixes,
+                            void* Linv, void* Uinv, int32_t* info, abft_stream_t stream, abft::Driver* host) {
   using namespace abft;
   if (!mat || mat->m != mat->n || mat->nb < 32 || mat->nb > 1024 || (mat->nb & (mat->nb - 1)) ||
       mat->n % mat->nb || !mat->A || mat->lda < mat->m)
@@ -359,7 +372,7 @@ extern "C" int abft_panel_getrf(const abft_mat_t* mat, int32_t k, int64_t* ipiv,
   char* panel = A + (r0 + r0 * mat->lda) * es;
   // scratch: pre-PD panel copy | local pivots | swap rows | nrows | getrf work
   int lwork = 0;
-  {
+  if (!host) {
     std::unique_lock<std::mutex> lk;
     cusolverDnHandle_t h = solver_handle(s, lk);
     cusolverStatus_t st = mat->dtype == ABFT_F64
@@ -384,7 +397,9 @@ extern "C" int abft_panel_getrf(const abft_mat_t* mat, int32_t k, int64_t* ipiv,
   int32_t* tb = (int32_t*)(base + off_tb);
   if (ft)
     FT_TRY(abft::copy2d(base, mk * es, panel, mat->lda * es, mk * es, nb, s));
-  {
+  if (host) {
+    FT_TRY(host_panel_pd(*host, k, HOST_GETRF, r0, r0, mk, piv_local, nullptr, info));
+  } else {
     std::unique_lock<std::mutex> lk;
     cusolverDnHandle_t h = solver_handle(s, lk);
     cusolverStatus_t st =
@@ -487,8 +502,8 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft) FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH));
     // line 5: PD with pivoting, swap rule, c(L), r(U_kk)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD));
-    FT_TRY(abft_panel_getrf(&d.M, k, ipiv + r0, ft ? &d.tol : nullptr, ft ? &d.R : nullptr, c->fixlog, c->fixcap,
-                            d.nfix, c->linv, c->uinv, d.info, as));
+    FT_TRY(panel_getrf_impl(&d.M, k, ipiv + r0, ft ? &d.tol : nullptr, ft ? &d.R : nullptr, c->fixlog, c->fixcap,
+                            d.nfix, c->linv, c->uinv, d.info, as, o->pd_location == FT_PD_HOST ? &d : nullptr));
     if (ft && k < nt - 1) ++d.n_checks;  // the pre-swap row check (c-14b)
     accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.info_total, r0);
     FT_TRY(d.restore_onchip());

@@ -1,0 +1,389 @@
+// ft_host.cu — pd_location = FT_PD_HOST: Alg. 2 lines 3-7 as the paper runs
+// them (L364-L372; MAGMA's CPU panel, L61).  Per iteration the panel goes to
+// pinned host memory, is factored there by the host LAPACK, and comes back.
+//
+// Transfer protection (reading c-28): each direction carries a
+// fresh column-checksum guard c(X) = [v1 v2]^T X per nb-row tile (L111/L446)
+// encoded by the sender right before the copy.
+//   D2H: abft_encode on the device -> copy -> host recomputes and compares
+//        (tau = 2 gamma_nb e^T|x|), locates each flagged column by the ratio
+//        rule (c-5) or the c-7 candidate, corrects by c-4 and re-checks the
+//        column; anything left -> fetch again (the device copy is intact),
+//        at most 2 repeats.
+//   H2D: host guard of the factored panel -> copy -> abft_verify +
+//        abft_locate_correct on the device (GENERAL, COL, posteriori tau);
+//        an uncorrectable tile -> send again, at most 2 repeats.
+// The maintained checksums were checked on the device before line 3 (the
+// pre-PD check) and the PD checksum rule + post-PD check follow on the
+// device, so the guard covers exactly the two transfers.
+#include <dlfcn.h>
+#include <math.h>
+
+#include <thread>
+
+#include "ft_driver.cuh"
+
+namespace abft {
+namespace {
+
+typedef void (*potrf_d_t)(const char*, const int*, double*, const int*, int*, size_t);
+typedef void (*potrf_s_t)(const char*, const int*, float*, const int*, int*, size_t);
+typedef void (*getrf_d_t)(const int*, const int*, double*, const int*, int*, int*);
+typedef void (*getrf_s_t)(const int*, const int*, float*, const int*, int*, int*);
+typedef void (*geqrf_d_t)(const int*, const int*, double*, const int*, double*, double*, const int*, int*);
+typedef void (*geqrf_s_t)(const int*, const int*, float*, const int*, float*, float*, const int*, int*);
+
+// Columns of a panel split over the host's cores (plain threads: the process
+// already hosts torch's OpenMP runtime, a second one is not linked in).
+template <typename F>
+void parallel_cols(int64_t w, F f) {
+  const int64_t nth = std::max<int64_t>(1, std::min<int64_t>((int64_t)std::thread::hardware_concurrency(), w / 8));
+  if (nth == 1) {
+    f(0, w);
+    return;
+  }
+  std::vector<std::thread> th;
+  const int64_t per = (w + nth - 1) / nth;
+  for (int64_t t = 0; t < nth; ++t) {
+    const int64_t a = t * per, b = std::min<int64_t>(w, a + per);
+    if (a < b) th.emplace_back([=] { f(a, b); });
+  }
+  for (auto& x : th) x.join();
+}
+
+__global__ void add_counter_kernel(int32_t* p, int32_t v) { *p += v; }
+
+// Fix records of a guard check are relative to the panel; make them global.
+__global__ void offset_fixes_kernel(abft_fix_t* fixes, int cap, const int32_t* from, const int32_t* to, int64_t row0,
+                                    int64_t col0, int64_t nb) {
+  const int n0 = *from, n1 = min(*to, cap);
+  for (int f = n0 + (int)threadIdx.x; f < n1; f += blockDim.x) {
+    abft_fix_t& x = fixes[f];
+    if (x.kind == ABFT_FIX_COLCHK) {
+      x.gi += row0 / nb;
+      x.gj += col0;
+    } else if (x.kind == ABFT_FIX_ROWCHK) {
+      x.gi += row0;
+      x.gj += col0 / nb;
+    } else {
+      x.gi += row0;
+      x.gj += col0;
+    }
+  }
+}
+
+// Host guard: G[2I + 2mt*j] = sum_i x, G[2I+1 + 2mt*j] = sum_i (i+1) x of
+// every nb-row tile I of column j (column-major panel, ld = rows).
+template <typename T>
+void host_guard(const T* P, int64_t rows, int64_t nb, int64_t w, T* G) {
+  const int64_t mt = rows / nb;
+  parallel_cols(w, [=](int64_t j0, int64_t j1) {
+    for (int64_t j = j0; j < j1; ++j)
+      for (int64_t I = 0; I < mt; ++I) {
+        const T* x = P + I * nb + j * rows;
+        double se = 0.0, sw = 0.0;
+        for (int64_t i = 0; i < nb; ++i) {
+          se += (double)x[i];
+          sw += (double)(i + 1) * (double)x[i];
+        }
+        G[2 * I + j * 2 * mt] = (T)se;
+        G[2 * I + 1 + j * 2 * mt] = (T)sw;
+      }
+  });
+}
+
+struct ColResid {
+  double de, dw, te;
+  bool bad;
+};
+
+template <typename T>
+ColResid col_resid(const T* x, int64_t nb, double ge, double gw, double gam) {
+  double se = 0.0, sw = 0.0, sa = 0.0;
+  for (int64_t i = 0; i < nb; ++i) {
+    const double v = (double)x[i];
+    se += v;
+    sw += (double)(i + 1) * v;
+    sa += fabs(v);
+  }
+  ColResid r;
+  r.de = ge - se;
+  r.dw = gw - sw;
+  r.te = 2.0 * gam * sa;
+  r.bad = !isfinite(r.de) || !isfinite(r.dw) || fabs(r.de) > r.te || fabs(r.dw) > (double)nb * r.te;
+  return r;
+}
+
+// c-5: q = dw/de, j = rint(q) accepted iff finite, |q-j| <= 0.25, 1 <= j <= nb,
+// |dw - j de| <= tw + j te.  Returns the 0-based row or -1.
+int locate_ratio(double de, double dw, double te, double tw, int64_t nb) {
+  if (!isfinite(de) || !isfinite(dw) || de == 0.0) return -1;
+  const double q = dw / de;
+  if (!isfinite(q)) return -1;
+  const double j = rint(q);
+  if (fabs(q - j) > 0.25 || j < 1.0 || j > (double)nb) return -1;
+  if (!(fabs(dw - j * de) <= tw + j * te)) return -1;
+  return (int)j - 1;
+}
+
+// Line 4 (host check of the received panel, in place).  Returns 1 if every
+// flagged column was located and corrected, 0 if the panel must be fetched
+// again; accumulates flagged columns / fixed elements.
+template <typename T>
+int host_check(T* P, int64_t rows, int64_t nb, int64_t w, const T* G, int* flagged, int* fixed) {
+  const int64_t mt = rows / nb;
+  const double gam = (double)nb * Prec<T>::u / (1.0 - (double)nb * Prec<T>::u);
+  std::vector<int> fl_c(w, 0), fx_c(w, 0), ok_c(w, 1);
+  parallel_cols(w, [&](int64_t j0, int64_t j1) {
+  for (int64_t j = j0; j < j1; ++j) {
+    int& fl = fl_c[j];
+    int& fx = fx_c[j];
+    int& ok = ok_c[j];
+    for (int64_t I = 0; I < mt; ++I) {
+      T* x = P + I * nb + j * rows;
+      const double ge = (double)G[2 * I + j * 2 * mt], gw = (double)G[2 * I + 1 + j * 2 * mt];
+      ColResid r = col_resid(x, nb, ge, gw, gam);
+      if (!r.bad) continue;
+      ++fl;
+      int i = locate_ratio(r.de, r.dw, r.te, (double)nb * r.te, nb);
+      if (i < 0) {  // c-7 candidate: the unique non-finite element, else the largest |x|
+        int nf = 0, inf_at = -1, big_at = -1;
+        double big = -1.0;
+        for (int64_t a = 0; a < nb; ++a) {
+          const double v = (double)x[a];
+          if (!isfinite(v)) {
+            ++nf;
+            inf_at = (int)a;
+          } else if (fabs(v) > big) {
+            big = fabs(v);
+            big_at = (int)a;
+          }
+        }
+        i = nf == 1 ? inf_at : big_at;
+      }
+      if (i < 0) {
+        ok = 0;
+        continue;
+      }
+      double rest = 0.0;  // c-4: x_i <- c_e - sum_{r != i} x_r
+      for (int64_t a = 0; a < nb; ++a)
+        if (a != i) rest += (double)x[a];
+      const T before = x[i];
+      x[i] = (T)(ge - rest);
+      if (col_resid(x, nb, ge, gw, gam).bad) {
+        x[i] = before;
+        ok = 0;
+        continue;
+      }
+      ++fx;
+    }
+  }
+  });
+  int ok = 1;
+  for (int64_t j = 0; j < w; ++j) {
+    *flagged += fl_c[j];
+    *fixed += fx_c[j];
+    ok &= ok_c[j];
+  }
+  return ok;
+}
+
+int lapack_info_potrf(ft_ctx* c, int dt, int n, void* a, int lda) {
+  int info = 0;
+  if (dt == ABFT_F64)
+    ((potrf_d_t)c->lp[0])("L", &n, (double*)a, &lda, &info, 1);
+  else
+    ((potrf_s_t)c->lp[1])("L", &n, (float*)a, &lda, &info, 1);
+  return info;
+}
+
+}  // namespace
+
+template <typename T>
+static int host_pd_t(Driver& d, int k, int kind, int64_t row0, int64_t col0, int64_t rows, int32_t* piv_dev,
+                     T* tau_dev, int32_t* info_dev) {
+  ft_ctx* c = d.c;
+  cudaStream_t s = d.s;
+  const abft_stream_t as = (abft_stream_t)s;
+  const int64_t nb = d.nb, mt = rows / nb, es = sizeof(T);
+  const bool ft = d.o->abft != 0;
+  const auto t0 = std::chrono::steady_clock::now();
+  // staging: panel | guard | tau | ipiv | counts | work
+  int lwork = 0;
+  if (kind == HOST_GEQRF) {
+    int m = (int)rows, n = (int)nb, ld = (int)rows, q = -1, info = 0;
+    T wq = 0;
+    if (sizeof(T) == 8)
+      ((geqrf_d_t)c->lp[4])(&m, &n, nullptr, &ld, nullptr, (double*)&wq, &q, &info);
+    else
+      ((geqrf_s_t)c->lp[5])(&m, &n, nullptr, &ld, nullptr, (float*)&wq, &q, &info);
+    lwork = std::max<int>((int)wq, (int)nb);
+  }
+  const size_t off_guard = ((size_t)rows * nb * es + 255) / 256 * 256;
+  const size_t off_tau = off_guard + ((size_t)2 * mt * nb * es + 255) / 256 * 256;
+  const size_t off_piv = off_tau + ((size_t)nb * es + 255) / 256 * 256;
+  const size_t off_cnt = off_piv + ((size_t)nb * 4 + 255) / 256 * 256;
+  const size_t off_work = off_cnt + 256;
+  const size_t need = off_work + (size_t)(lwork + 1) * es;
+  if (c->hstage_bytes < need) {
+    if (c->hstage) cudaFreeHost(c->hstage);
+    c->hstage = nullptr;
+    c->hstage_bytes = 0;
+    if (cudaHostAlloc((void**)&c->hstage, need, cudaHostAllocDefault) != cudaSuccess) return ABFT_E_NOMEM;
+    c->hstage_bytes = need;
+  }
+  FT_TRY(grow_buffer(c->dguard, c->dguard_bytes, (size_t)2 * mt * nb * es));
+  T* hp = reinterpret_cast<T*>(c->hstage);
+  T* hg = reinterpret_cast<T*>(c->hstage + off_guard);
+  T* htau = reinterpret_cast<T*>(c->hstage + off_tau);
+  int* hpiv = reinterpret_cast<int*>(c->hstage + off_piv);
+  int32_t* hcnt = reinterpret_cast<int32_t*>(c->hstage + off_cnt);
+  T* hwork = reinterpret_cast<T*>(c->hstage + off_work);
+  T* panel = reinterpret_cast<T*>(d.a_at(row0, col0));
+
+  abft_mat_t P{};
+  P.dtype = d.dtype;
+  P.m = rows;
+  P.n = nb;
+  P.nb = nb;
+  P.A = panel;
+  P.lda = d.lda;
+  P.colchk = c->dguard;
+  P.ldc = 2 * mt;
+  abft_tiles_t all{0, (int)mt, 0, 1, 0, ABFT_GENERAL};
+  auto faults = [&](int point) {
+    std::vector<ft_inject_t> v;
+    for (auto& u : d.xfer_used)
+      if (u.first == k && u.second == point) return v;
+    d.xfer_used.push_back({k, point});
+    for (int t = 0; t < d.o->n_inject; ++t) {
+      const ft_inject_t& f = d.o->inject[t];
+      if (f.iter == k && f.point == point && f.target == 0) v.push_back(f);
+    }
+    return v;
+  };
+
+  // lines 3-4: guarded D2H + host check
+  if (ft) FT_TRY(abft_encode(&P, &all, ABFT_COL, as));
+  const auto d2h_faults = faults(FT_AT_D2H);
+  for (int attempt = 0; attempt < 3; ++attempt) {
+    ABFT_CUDA_TRY(cudaMemcpy2DAsync(hp, rows * es, panel, d.lda * es, rows * es, nb, cudaMemcpyDeviceToHost, s));
+    if (ft) ABFT_CUDA_TRY(cudaMemcpyAsync(hg, c->dguard, (size_t)2 * mt * nb * es, cudaMemcpyDeviceToHost, s));
+    ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+    if (attempt == 0)
+      for (auto& f : d2h_faults) {
+        T* e = hp + (f.gi - row0) + (f.gj - col0) * rows;
+        if (sizeof(T) == 8) {
+          uint64_t b;
+          memcpy(&b, e, 8);
+          b ^= f.xor_mask;
+          memcpy(e, &b, 8);
+        } else {
+          uint32_t b;
+          memcpy(&b, e, 4);
+          b ^= (uint32_t)f.xor_mask;
+          memcpy(e, &b, 4);
+        }
+      }
+    if (!ft) break;
+    if (host_check<T>(hp, rows, nb, nb, hg, &d.xs[0], &d.xs[1])) break;
+    if (attempt < 2) {
+      ++d.xs[2];
+    } else {
+      ++d.xs[6];
+      add_counter_kernel<<<1, 1, 0, s>>>(d.counts + ABFT_CNT_UNCORRECTABLE, 1);
+    }
+  }
+
+  // line 5: host PD
+  int info = 0;
+  {
+    int m = (int)rows, n = (int)nb, ld = (int)rows;
+    if (kind == HOST_POTRF) {
+      info = lapack_info_potrf(c, d.dtype, n, hp, ld);
+    } else if (kind == HOST_GETRF) {
+      if (sizeof(T) == 8)
+        ((getrf_d_t)c->lp[2])(&m, &n, (double*)hp, &ld, hpiv, &info);
+      else
+        ((getrf_s_t)c->lp[3])(&m, &n, (float*)hp, &ld, hpiv, &info);
+    } else {
+      if (sizeof(T) == 8)
+        ((geqrf_d_t)c->lp[4])(&m, &n, (double*)hp, &ld, (double*)htau, (double*)hwork, &lwork, &info);
+      else
+        ((geqrf_s_t)c->lp[5])(&m, &n, (float*)hp, &ld, (float*)htau, (float*)hwork, &lwork, &info);
+    }
+  }
+  hcnt[8] = info > 0 ? info : 0;
+  if (ft) host_guard<T>(hp, rows, nb, nb, hg);
+
+  // lines 6-7: guarded H2D + device check
+  const auto h2d_faults = faults(FT_AT_H2D);
+  for (int attempt = 0; attempt < 3; ++attempt) {
+    ABFT_CUDA_TRY(cudaMemcpy2DAsync(panel, d.lda * es, hp, rows * es, rows * es, nb, cudaMemcpyHostToDevice, s));
+    if (attempt == 0) {
+      ABFT_CUDA_TRY(cudaMemcpyAsync(info_dev, hcnt + 8, 4, cudaMemcpyHostToDevice, s));
+      if (kind == HOST_GETRF) ABFT_CUDA_TRY(cudaMemcpyAsync(piv_dev, hpiv, nb * 4, cudaMemcpyHostToDevice, s));
+      if (kind == HOST_GEQRF) ABFT_CUDA_TRY(cudaMemcpyAsync(tau_dev, htau, nb * es, cudaMemcpyHostToDevice, s));
+      for (auto& f : h2d_faults) FT_TRY(d.inject_at_elem(f));
+    }
+    if (!ft) break;
+    ABFT_CUDA_TRY(cudaMemcpyAsync(c->dguard, hg, (size_t)2 * mt * nb * es, cudaMemcpyHostToDevice, s));
+    ABFT_CUDA_TRY(cudaMemsetAsync(d.xcounts, 0, 8 * sizeof(int32_t), s));
+    ABFT_CUDA_TRY(cudaMemcpyAsync(d.mark2, d.nfix, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
+    abft_tol_t tol{ABFT_TOL_POSTERIORI, 1.0, 0};
+    abft_report_t R{d.status, d.nt, nullptr, nullptr, d.xcounts};
+    FT_TRY(abft_verify(&P, &all, ABFT_COL, &tol, &R, as));
+    FT_TRY(abft_locate_correct(&P, &all, ABFT_COL, &tol, &R, c->fixlog, c->fixcap, d.nfix, as));
+    offset_fixes_kernel<<<1, 128, 0, s>>>(c->fixlog, c->fixcap, d.mark2, d.nfix, row0, col0, nb);
+    ABFT_CUDA_TRY(cudaMemcpyAsync(hcnt, d.xcounts, 8 * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+    ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+    d.xs[3] += hcnt[ABFT_CNT_COLS_FLAGGED];
+    d.xs[4] += hcnt[ABFT_CNT_ELEMS_FIXED];
+    if (hcnt[ABFT_CNT_UNCORRECTABLE] == 0) break;
+    if (attempt < 2) {
+      ++d.xs[5];
+    } else {
+      ++d.xs[6];
+      add_counter_kernel<<<1, 1, 0, s>>>(d.counts + ABFT_CNT_UNCORRECTABLE, 1);
+    }
+  }
+  ABFT_CUDA_TRY(cudaGetLastError());
+  d.ms_host += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return 0;
+}
+
+int host_panel_pd(Driver& d, int k, int kind, int64_t row0, int64_t col0, int64_t rows, int32_t* piv_dev,
+                  void* tau_dev, int32_t* info_dev) {
+  if (!d.c->lapack) return ABFT_E_UNSUPPORTED;
+  return d.dtype == ABFT_F64
+             ? host_pd_t<double>(d, k, kind, row0, col0, rows, piv_dev, (double*)tau_dev, info_dev)
+             : host_pd_t<float>(d, k, kind, row0, col0, rows, piv_dev, (float*)tau_dev, info_dev);
+}
+
+}  // namespace abft
+
+extern "C" int ft_ctx_set_host_lapack(ft_ctx_t* c, const char* path) {
+  if (!c) return -1;
+  if (!path) return -2;
+  void* h = dlopen(path, RTLD_NOW | RTLD_LOCAL);
+  if (!h) {
+    fprintf(stderr, "[abft] dlopen(%s): %s\n", path, dlerror());
+    return ABFT_E_UNSUPPORTED;
+  }
+  static const char* names[6] = {"dpotrf_", "spotrf_", "dgetrf_", "sgetrf_", "dgeqrf_", "sgeqrf_"};
+  void* f[6];
+  for (int i = 0; i < 6; ++i) {
+    std::string scipy = std::string("scipy_") + names[i];
+    f[i] = dlsym(h, scipy.c_str());
+    if (!f[i]) f[i] = dlsym(h, names[i]);
+    if (!f[i]) {
+      fprintf(stderr, "[abft] %s: no %s\n", path, names[i]);
+      dlclose(h);
+      return ABFT_E_UNSUPPORTED;
+    }
+  }
+  if (c->lapack) dlclose(c->lapack);
+  c->lapack = h;
+  for (int i = 0; i < 6; ++i) c->lp[i] = f[i];
+  return 0;
+}

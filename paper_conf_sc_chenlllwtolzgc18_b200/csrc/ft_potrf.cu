@@ -6,6 +6,8 @@
 // PD on the CPU in MAGMA (L61) — here the PD runs on the device (cuSOLVER),
 // DESIGN.md §7 explains why.  Readings: c-12 (Cholesky rules), c-24 (views
 // before/after PD), c-25 (guarded Fig. 4a trailing repair), c-8 (fault hooks).
+#include <dlfcn.h>
+
 #include "ft_driver.cuh"
 
 // ------------------------------------------------------------ panel potrf --
@@ -32,6 +34,12 @@ static int potrf_tile(const abft_mat_t* d, int32_t* info, cudaStream_t s) {
 }
 }  // namespace abft
 
+namespace abft {
+// The device part of the PD after the factorization (c-12): L_kk^-1 and the
+// checksum rule.  Shared by abft_panel_potrf and the FT_PD_HOST driver path.
+int panel_potrf_rules(const abft_mat_t* d, void* Linv, int64_t ldw, abft_stream_t stream);
+}  // namespace abft
+
 extern "C" int abft_panel_potrf(const abft_mat_t* d, void* Linv, int64_t ldw, int32_t* info, abft_stream_t stream) {
   if (!d || d->m != d->nb || d->n != d->nb || !d->A || d->lda < d->nb) return -1;
   if (Linv && ldw < d->nb) return -3;
@@ -40,6 +48,11 @@ extern "C" int abft_panel_potrf(const abft_mat_t* d, void* Linv, int64_t ldw, in
   cudaStream_t s = (cudaStream_t)stream;
   int rc = d->dtype == ABFT_F64 ? abft::potrf_tile<double>(d, info, s) : abft::potrf_tile<float>(d, info, s);
   if (rc) return rc;
+  return abft::panel_potrf_rules(d, Linv, ldw, stream);
+}
+
+int abft::panel_potrf_rules(const abft_mat_t* d, void* Linv, int64_t ldw, abft_stream_t stream) {
+  cudaStream_t s = (cudaStream_t)stream;
   if (!d->colchk && !Linv) return 0;
   // L_kk^-1 once (reused by the caller for the PU when Linv is given)
   void* W = Linv;
@@ -176,6 +189,9 @@ extern "C" int ft_ctx_destroy(ft_ctx_t* c) {
   if (c->rsv) cudaFree(c->rsv);
   if (c->hpin) cudaFreeHost(c->hpin);
   if (c->ev) cudaEventDestroy(c->ev);
+  if (c->hstage) cudaFreeHost(c->hstage);
+  if (c->dguard) cudaFree(c->dguard);
+  if (c->lapack) dlclose(c->lapack);
   delete c;
   return 0;
 }
@@ -264,7 +280,12 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
         D.ldcm = d.M.ldcm;
       }
       const bool need_inv = ft || o->pu_gemm;
-      FT_TRY(abft_panel_potrf(&D, need_inv ? c->linv : nullptr, nb, d.info, as));
+      if (o->pd_location == FT_PD_HOST) {  // Alg. 2 lines 3-7 with the PD on the host (c-28)
+        FT_TRY(host_panel_pd(d, k, HOST_POTRF, r0, r0, nb, nullptr, nullptr, d.info));
+        FT_TRY(panel_potrf_rules(&D, need_inv ? c->linv : nullptr, nb, as));
+      } else {
+        FT_TRY(abft_panel_potrf(&D, need_inv ? c->linv : nullptr, nb, d.info, as));
+      }
       accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.info_total, r0);
       return 0;
     };

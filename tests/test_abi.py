@@ -48,3 +48,17 @@ def test_illegal_arguments_rejected_without_gpu():
     # null matrix pointer -> -1 (xerbla style); no device work is attempted
     assert lib.abft_encode(None, None, 3, None) == -1
     assert lib.abft_sizes(10, 10, 3, None, None, None, None) == -3
+
+
+def test_host_lapack_for_the_host_pd_mode():
+    # FT_PD_HOST (Alg. 2's CPU panel, L61) loads the OpenBLAS bundled with
+    # SciPy; it must exist and export the LP64 symbols the library looks up
+    import ctypes
+
+    from paper_conf_sc_chenlllwtolzgc18_b200 import abft
+
+    path = abft.host_lapack_path()
+    lapack = ctypes.CDLL(path)
+    for name in ("dpotrf_", "spotrf_", "dgetrf_", "sgetrf_", "dgeqrf_", "sgeqrf_"):
+        assert hasattr(lapack, "scipy_" + name) or hasattr(lapack, name), name
+    assert abft._L.ft_ctx_set_host_lapack(None, path.encode()) == -1
