@@ -422,6 +422,28 @@ def qr_T(V, tau):
     return T
 
 
+def qr_ctf_check(V, T, prec="f64", scale=1.0):
+    """f2, the CTF check (L263: "Error in T can be detected by verifying the
+    orthogonality of (I − V T V^T) ... recover the corrupted T by re-computing
+    it using V").  Q = I − V T V^T is orthogonal iff V (T + T^T − T^T V^T V T) V^T
+    = 0, i.e. for V of full column rank iff E = T^T (V^T V) T − T − T^T = 0.
+    Reading c-29: flag iff some |E_ij| > scale·4·γ_{m+nb}·(a_i a_j + |T_ij| +
+    |T_ji|) with a = |T|^T ‖v‖ (‖v_k‖ = column norms of V, so that
+    |V|^T |V| ≤ ‖v‖ ‖v‖^T bounds the rounding of V^T V; the |T| terms cover
+    2/τ_j vs v_j^T v_j); a non-finite E_ij or bound is flagged.  Returns
+    (flagged entries, E)."""
+    m, nb = V.shape
+    S = V.T @ V
+    E = T.T @ S @ T - T - T.T
+    a = np.abs(T).T @ np.sqrt(np.diag(S))
+    u = 2.0 ** -53 if prec == "f64" else 2.0 ** -24
+    g = (m + nb) * u / (1.0 - (m + nb) * u)
+    bound = scale * 4.0 * g * (np.outer(a, a) + np.abs(T) + np.abs(T).T)
+    with np.errstate(invalid="ignore"):
+        bad = ~np.isfinite(E) | ~np.isfinite(bound) | ~(np.abs(E) <= bound)
+    return int(np.count_nonzero(bad)), E
+
+
 def qr_tmu_data(st: State, k: int, V, T):
     """QR TMU data step (Table III): A2 ← (I − V T V^T)^T A2 = A2 − V (T^T V^T A2)
     for A2 = A[k·nb:, (k+1)·nb:] (its first nb rows become R12)."""
