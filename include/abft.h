@@ -303,7 +303,9 @@ typedef struct ft_ctx ft_ctx_t;
  * kind:  FT_KIND_PERSIST (computation / DRAM / communication: the flipped
  *        value stays) or FT_KIND_ONCHIP (flipped before the op that follows
  *        `point` and restored right after it, before any check).
- * target: 0 = A, 1 = colchk, 2 = rowchk; (gi, gj) element of that array. */
+ * target: 0 = A, 1 = colchk, 2 = rowchk, 3 = the CTF T of ft_geqrf (nb x nb,
+ *         local (gi, gj); points FT_AT_POST_PD / FT_AT_PRE_TMU of iterations
+ *         k < n/nb - 1); (gi, gj) element of that array. */
 enum {
   FT_AT_PRE_PD_CHECK = 0, FT_AT_PRE_PD = 1, FT_AT_POST_PD = 2, FT_AT_PRE_PU_CHECK = 3,
   FT_AT_PRE_PU = 4, FT_AT_POST_PU = 5, FT_AT_PRE_TMU = 6, FT_AT_POST_TMU = 7,
@@ -369,6 +371,9 @@ typedef struct {
   int32_t xfer_resends;         /* host-to-device transfers repeated */
   int32_t xfer_uncorrectable;   /* transfers still wrong after 2 repeats (-> uncorrectable) */
   double ms_host_pd;            /* wall time of the host round trips (transfers + host PD) */
+  /* ft_geqrf CTF check (row f2, L263; reading c-29) */
+  int32_t ctf_flagged;          /* checks whose E = T^T V^T V T - T - T^T exceeded the bound */
+  int32_t ctf_recomputed;       /* T recomputed from V after a flagged check */
 } ft_stats_t;
 
 ABFT_API int ft_ctx_create(ft_ctx_t **ctx, int32_t device, abft_stream_t stream);
@@ -411,7 +416,10 @@ ABFT_API int ft_getrf(ft_ctx_t *ctx, int32_t dtype, int64_t n, void *dA, int64_t
  * (device, lda >= n, n % nb == 0) with full checksums (Table III): per
  * iteration k — check the column panel (c+r) -> abft_panel_geqrf -> check V
  * (UNIT_LOWER, c) and R_kk (UPPER, r) -> TMU A2 <- Q^T A2 (three DGEMMs) with
- * c(A2) -= c(V) W, r(A2) -= V T^T V^T r(A2) -> re-check V (a V correction
+ * c(A2) -= c(V) W, r(A2) -= V T^T V^T r(A2), preceded by the check of A2
+ * (c+r, c-25q) and the CTF check of T (f2, L263: E = T^T V^T V T - T - T^T
+ * against the c-29 bound, recompute T from V when flagged; one host
+ * read-back per iteration) -> re-check V (a V correction
  * after the TMU consumed it is outcome R) and R12 (r).  Output as LAPACK
  * dgeqrf (R and V in dA, tau: device array of n).  Returns
  * ABFT_E_UNCORRECTABLE if a 2D / consumed error remained. */

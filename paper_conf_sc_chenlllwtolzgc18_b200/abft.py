@@ -89,7 +89,8 @@ class ft_stats_t(C.Structure):
                 ("ms_total", C.c_double), ("restarts", C.c_int32),
                 ("xfer_d2h_flagged", C.c_int32), ("xfer_d2h_fixed", C.c_int32), ("xfer_retransfers", C.c_int32),
                 ("xfer_h2d_flagged", C.c_int32), ("xfer_h2d_fixed", C.c_int32), ("xfer_resends", C.c_int32),
-                ("xfer_uncorrectable", C.c_int32), ("ms_host_pd", C.c_double)]
+                ("xfer_uncorrectable", C.c_int32), ("ms_host_pd", C.c_double),
+                ("ctf_flagged", C.c_int32), ("ctf_recomputed", C.c_int32)]
 
 
 _L = _lib.load()

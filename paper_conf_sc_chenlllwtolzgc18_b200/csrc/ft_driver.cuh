@@ -98,6 +98,9 @@ struct Driver {
   int32_t* mark2 = nullptr;            // device: fix-log position before an H2D guard check
   int xs[7] = {};                      // ft_stats_t.xfer_* accumulators
   double ms_host = 0.0;
+  double host_phase[4] = {};           // ABFT_HOST_TIMING=1: per-phase host ms (stderr at the end)
+  int32_t* ctf_cnt = nullptr;          // device: flagged entries of one CTF check (QR, f2)
+  int ctf_flagged = 0, ctf_recomputed = 0;
   std::vector<std::pair<int, int>> xfer_used;  // (iter, point) transfer faults already applied
 
   int setup(ft_ctx* ctx, int32_t dt, int64_t n_, int64_t nb_, void* dA, int64_t lda_, const ft_opts_t* opts,
@@ -118,7 +121,7 @@ struct Driver {
     FT_TRY(grow_buffer(c->state, c->state_bytes, need));
     if (o->pd_location == FT_PD_HOST && !c->lapack) return ABFT_E_UNSUPPORTED;
     if (o->pd_location != FT_PD_DEVICE && o->pd_location != FT_PD_HOST) return ABFT_E_UNSUPPORTED;
-    size_t ints_need = (size_t)nt * nt + 8 + 8 + 8;
+    size_t ints_need = (size_t)nt * nt + 8 + 8 + 8 + 8;
     void* ip = c->ints;
     FT_TRY(grow_buffer(ip, c->ints_n, ints_need * sizeof(int32_t)));
     c->ints = reinterpret_cast<int32_t*>(ip);
@@ -135,6 +138,7 @@ struct Driver {
     snap = info_total + 1;
     mark2 = snap + 1;
     xcounts = counts + 16;
+    ctf_cnt = counts + 24;
     if (o->abft && o->restart)
       FT_TRY(grow_buffer(c->rsv, c->rsv_bytes, ((size_t)n * nb + (size_t)nb * nb + 3 * (size_t)nt * nb + 4 * nb) * es));
     ABFT_CUDA_TRY(cudaMemsetAsync(c->ints, 0, ints_need * sizeof(int32_t), s));
@@ -170,6 +174,7 @@ struct Driver {
   char* elem(int target, int64_t gi, int64_t gj) {
     if (target == 1) return (char*)M.colchk + (gi + gj * M.ldc) * es;
     if (target == 2) return (char*)M.rowchk + (gi + gj * M.ldr) * es;
+    if (target == 3) return (char*)c->linv + (gi + gj * nb) * es;  // ft_geqrf: the CTF T (nb x nb)
     return (char*)A + (gi + gj * lda) * es;
   }
   // Elements the op after `point` overwrites: an on-chip flip there cannot be
@@ -259,6 +264,11 @@ struct Driver {
       int32_t* x = &stats->xfer_d2h_flagged;
       for (int i = 0; i < 7; ++i) x[i] = xs[i];
       stats->ms_host_pd = ms_host;
+      if (ms_host > 0 && getenv("ABFT_HOST_TIMING"))
+        fprintf(stderr, "[abft] host PD ms: d2h+check %.1f lapack %.1f guard %.1f h2d+check %.1f\n", host_phase[0],
+                host_phase[1], host_phase[2], host_phase[3]);
+      stats->ctf_flagged = ctf_flagged;
+      stats->ctf_recomputed = ctf_recomputed;
     }
     return h[ABFT_CNT_UNCORRECTABLE] ? ABFT_E_UNCORRECTABLE : 0;
   }

@@ -18,9 +18,15 @@
 // tau_j y_j of the interleaved algorithm), one warp per checksum row, instead
 // of interleaving two checksum rows into a memory-bound unblocked panel
 // factorization.  r(R) follows from r(P) by Q^T = I - V T^T V^T (GEMMs).
+//
+// CTF check (row f2, L263; reading c-29): before the TMU, with V as it is in
+// memory, E = T^T (V^T V) T - T - T^T must vanish (orthogonality of
+// I - V T V^T); a flagged T is recomputed from V and checked again.
 #include "ft_driver.cuh"
 
 namespace abft {
+
+__global__ void add_i32_kernel_qr(int32_t* p, int32_t v) { *p += v; }
 
 // Vbuf (mk x nb, ld mk) = unit lower trapezoidal V of the factored panel.
 template <typename T>
@@ -321,6 +327,100 @@ extern "C" int abft_panel_geqrf(const abft_mat_t* mat, int32_t k, void* tau, voi
              : panel_geqrf_t<float>(mat, k, (float*)tau, (float*)V, (float*)T, (float*)panel_copy, info, s);
 }
 
+// ---------------------------------------------------------- CTF check (f2) --
+namespace abft {
+// a_i = sum_k |T_ki| sqrt(S_kk): |T|^T ||v|| (c-29 bound)
+template <typename T>
+__global__ void ctf_a_kernel(T* a, const T* Tm, const T* S, int nb) {
+  const int i = blockIdx.x;
+  double acc = 0.0;
+  for (int k = threadIdx.x; k < nb; k += blockDim.x)
+    acc += fabs((double)Tm[k + (int64_t)i * nb]) * sqrt(fabs((double)S[k + (int64_t)k * nb]));
+  for (int m = 16; m >= 1; m >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, m);
+  __shared__ double part[32];
+  if ((threadIdx.x & 31) == 0) part[threadIdx.x >> 5] = acc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += part[w];
+    a[i] = (T)t;
+  }
+}
+
+// E = T^T S T (precomputed) ; flag (i, j) iff E_ij - T_ij - T_ji is non-finite
+// or exceeds g4 (a_i a_j + |T_ij| + |T_ji|)
+template <typename T>
+__global__ void ctf_flag_kernel(const T* TST, const T* Tm, const T* a, int nb, double g4, int32_t* cnt) {
+  const int64_t total = (int64_t)nb * nb;
+  int bad = 0;
+  for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+       idx += (int64_t)gridDim.x * blockDim.x) {
+    const int j = (int)(idx / nb), i = (int)(idx - (int64_t)j * nb);
+    const double tij = (double)Tm[idx], tji = (double)Tm[j + (int64_t)i * nb];
+    const double e = (double)TST[idx] - tij - tji;
+    const double b = g4 * ((double)a[i] * (double)a[j] + fabs(tij) + fabs(tji));
+    if (!isfinite(e) || !isfinite(b) || !(fabs(e) <= b)) ++bad;
+  }
+  for (int m = 16; m >= 1; m >>= 1) bad += __shfl_xor_sync(0xffffffffu, bad, m);
+  if ((threadIdx.x & 31) == 0 && bad) atomicAdd(cnt, bad);
+}
+
+// One CTF check of T (nb x nb) against the V in Vbuf (mk x nb): S = V^T V,
+// TST = T^T (S T), flags -> *cnt (device).  S stays in `S` for a recompute.
+template <typename T>
+static int ctf_eval(cudaStream_t s, int64_t mk, int nb, const T* Vbuf, const T* Tm, T* S, T* W, T* TST, T* a,
+                    double g4, int32_t* cnt) {
+  {
+    std::unique_lock<std::mutex> lk;
+    cublasHandle_t h = blas_handle(s, lk);
+    if (gemmT<T>(h, CUBLAS_OP_T, CUBLAS_OP_N, nb, nb, (int)mk, T(1), Vbuf, (int)mk, Vbuf, (int)mk, T(0), S, nb) ||
+        gemmT<T>(h, CUBLAS_OP_N, CUBLAS_OP_N, nb, nb, nb, T(1), S, nb, Tm, nb, T(0), W, nb) ||
+        gemmT<T>(h, CUBLAS_OP_T, CUBLAS_OP_N, nb, nb, nb, T(1), Tm, nb, W, nb, T(0), TST, nb))
+      return ABFT_E_CUBLAS;
+  }
+  ABFT_CUDA_TRY(cudaMemsetAsync(cnt, 0, sizeof(int32_t), s));
+  ctf_a_kernel<T><<<(unsigned)nb, 128, 0, s>>>(a, Tm, S, nb);
+  ctf_flag_kernel<T><<<blocks_of((int64_t)nb * nb), 256, 0, s>>>(TST, Tm, a, nb, g4, cnt);
+  ABFT_CUDA_TRY(cudaGetLastError());
+  return 0;
+}
+
+// f2 for iteration k: check T, recompute it from V (the CTF of
+// panel_geqrf_t: T = (striu(V^T V) + diag(1/tau))^-1) if flagged, check again;
+// a T still flagged is uncorrectable.  One host read-back per call.
+template <typename T>
+static int ctf_check(Driver& d, ft_ctx* c, int64_t mk, T* Vbuf, T* Tm, const T* tau) {
+  cudaStream_t s = d.s;
+  const int nb = (int)d.nb;
+  void* sv = nullptr;
+  FT_TRY(scratch(s, 17, ((size_t)nb * nb * 4 + nb) * sizeof(T), &sv));
+  T* S = reinterpret_cast<T*>(sv);
+  T* W = S + (size_t)nb * nb;
+  T* TST = W + (size_t)nb * nb;
+  T* Ti = TST + (size_t)nb * nb;
+  T* a = Ti + (size_t)nb * nb;
+  const double m = (double)(mk + nb), u = Prec<T>::u;
+  const double g4 = 4.0 * d.tol.scale * m * u / (1.0 - m * u);
+  int32_t* cnt = d.ctf_cnt;
+  qr_build_v_kernel<T><<<blocks_of(mk * nb), 256, 0, s>>>(Vbuf, mk, nb, reinterpret_cast<T*>(d.a_at(d.n - mk, d.n - mk)),
+                                                         d.lda);
+  FT_TRY(ctf_eval<T>(s, mk, nb, Vbuf, Tm, S, W, TST, a, g4, cnt));
+  ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin + 4, cnt, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+  ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+  if (c->hpin[4] == 0) return 0;
+  ++d.ctf_flagged;
+  qr_tinv_kernel<T><<<blocks_of((int64_t)nb * nb), 256, 0, s>>>(Ti, S, tau, nb);
+  FT_TRY(abft_tri_inverse(d.dtype, 'U', 'N', nb, Ti, nb, Tm, nb, (abft_stream_t)s));
+  qr_fix_zero_tau_kernel<T><<<(unsigned)nb, 128, 0, s>>>(Tm, tau, nb);
+  ++d.ctf_recomputed;
+  FT_TRY(ctf_eval<T>(s, mk, nb, Vbuf, Tm, S, W, TST, a, g4, cnt));
+  ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin + 4, cnt, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+  ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+  if (c->hpin[4] != 0) add_i32_kernel_qr<<<1, 1, 0, s>>>(d.counts + ABFT_CNT_UNCORRECTABLE, 1);
+  return 0;
+}
+}  // namespace abft
+
 // ----------------------------------------------------------------- driver --
 namespace abft {
 template <typename T>
@@ -364,6 +464,8 @@ static int geqrf_driver(Driver& d, ft_ctx* c, T* tau_all) {
     // QR's TMU reads all of A2 (W = T^T V^T A2): A2 is a reference part, so it
     // is checked before the TMU (Alg. 2 line 8 for QR, reading c-25q)
     if (ft) FT_TRY(d.check(k, (int)nt, k + 1, (int)nt, ABFT_GENERAL, ABFT_BOTH));
+    // f2 (L263): T carries no checksum; verify the orthogonality of I - V T V^T
+    if (ft) FT_TRY(ctf_check<T>(d, c, mk, Vbuf, Tm, tau_all + r0));
     // line 12: TMU  A2 <- (I - V T V^T)^T A2 = A2 - V W,  W = T^T V^T A2
     FT_TRY(d.inject_at(k, FT_AT_PRE_TMU));
     const bool touched = d.o->n_inject > 0;  // V re-read from memory after hooks

@@ -18,6 +18,7 @@
 // device, so the guard covers exactly the two transfers.
 #include <dlfcn.h>
 #include <math.h>
+#include <sched.h>
 
 #include <thread>
 
@@ -33,11 +34,20 @@ typedef void (*getrf_s_t)(const int*, const int*, float*, const int*, int*, int*
 typedef void (*geqrf_d_t)(const int*, const int*, double*, const int*, double*, double*, const int*, int*);
 typedef void (*geqrf_s_t)(const int*, const int*, float*, const int*, float*, float*, const int*, int*);
 
+// Host cores for the guard / check loops: the half of the process's cores
+// that ft_ctx_set_host_lapack leaves to us (OpenBLAS gets the other half: its
+// idle threads spin, so sharing all cores slows both sides down).
+int64_t g_host_threads = 8;
+
 // Columns of a panel split over the host's cores (plain threads: the process
 // already hosts torch's OpenMP runtime, a second one is not linked in).
 template <typename F>
-void parallel_cols(int64_t w, F f) {
-  const int64_t nth = std::max<int64_t>(1, std::min<int64_t>((int64_t)std::thread::hardware_concurrency(), w / 8));
+void parallel_cols(int64_t w, int64_t rows, F f) {
+  // one thread per >= 256K elements, at most 16 (thread start-up is ~20 us)
+  const int64_t by_work = (w * rows) >> 18;
+  const int64_t cap = g_host_threads;
+  const int64_t nth =
+      std::max<int64_t>(1, std::min<int64_t>({(int64_t)std::thread::hardware_concurrency(), cap, by_work, w}));
   if (nth == 1) {
     f(0, w);
     return;
@@ -72,20 +82,34 @@ __global__ void offset_fixes_kernel(abft_fix_t* fixes, int cap, const int32_t* f
   }
 }
 
+// sum x, sum (i+1) x, sum |x| of one nb-element column segment: four
+// interleaved partial sums per quantity (fixed order, so deterministic; nb is
+// a power of two >= 32), added pairwise at the end.
+template <typename T>
+inline void col_sums(const T* x, int64_t nb, double& se, double& sw, double& sa) {
+  double e[4] = {0, 0, 0, 0}, w[4] = {0, 0, 0, 0}, a[4] = {0, 0, 0, 0};
+  for (int64_t i = 0; i < nb; i += 4)
+    for (int q = 0; q < 4; ++q) {
+      const double v = (double)x[i + q];
+      e[q] += v;
+      w[q] += (double)(i + q + 1) * v;
+      a[q] += fabs(v);
+    }
+  se = (e[0] + e[1]) + (e[2] + e[3]);
+  sw = (w[0] + w[1]) + (w[2] + w[3]);
+  sa = (a[0] + a[1]) + (a[2] + a[3]);
+}
+
 // Host guard: G[2I + 2mt*j] = sum_i x, G[2I+1 + 2mt*j] = sum_i (i+1) x of
 // every nb-row tile I of column j (column-major panel, ld = rows).
 template <typename T>
 void host_guard(const T* P, int64_t rows, int64_t nb, int64_t w, T* G) {
   const int64_t mt = rows / nb;
-  parallel_cols(w, [=](int64_t j0, int64_t j1) {
+  parallel_cols(w, rows, [=](int64_t j0, int64_t j1) {
     for (int64_t j = j0; j < j1; ++j)
       for (int64_t I = 0; I < mt; ++I) {
-        const T* x = P + I * nb + j * rows;
-        double se = 0.0, sw = 0.0;
-        for (int64_t i = 0; i < nb; ++i) {
-          se += (double)x[i];
-          sw += (double)(i + 1) * (double)x[i];
-        }
+        double se, sw, sa;
+        col_sums(P + I * nb + j * rows, nb, se, sw, sa);
         G[2 * I + j * 2 * mt] = (T)se;
         G[2 * I + 1 + j * 2 * mt] = (T)sw;
       }
@@ -99,13 +123,8 @@ struct ColResid {
 
 template <typename T>
 ColResid col_resid(const T* x, int64_t nb, double ge, double gw, double gam) {
-  double se = 0.0, sw = 0.0, sa = 0.0;
-  for (int64_t i = 0; i < nb; ++i) {
-    const double v = (double)x[i];
-    se += v;
-    sw += (double)(i + 1) * v;
-    sa += fabs(v);
-  }
+  double se, sw, sa;
+  col_sums(x, nb, se, sw, sa);
   ColResid r;
   r.de = ge - se;
   r.dw = gw - sw;
@@ -134,7 +153,7 @@ int host_check(T* P, int64_t rows, int64_t nb, int64_t w, const T* G, int* flagg
   const int64_t mt = rows / nb;
   const double gam = (double)nb * Prec<T>::u / (1.0 - (double)nb * Prec<T>::u);
   std::vector<int> fl_c(w, 0), fx_c(w, 0), ok_c(w, 1);
-  parallel_cols(w, [&](int64_t j0, int64_t j1) {
+  parallel_cols(w, rows, [&](int64_t j0, int64_t j1) {
   for (int64_t j = j0; j < j1; ++j) {
     int& fl = fl_c[j];
     int& fx = fx_c[j];
@@ -295,6 +314,7 @@ static int host_pd_t(Driver& d, int k, int kind, int64_t row0, int64_t col0, int
     }
   }
 
+  const auto t1 = std::chrono::steady_clock::now();
   // line 5: host PD
   int info = 0;
   {
@@ -314,7 +334,9 @@ static int host_pd_t(Driver& d, int k, int kind, int64_t row0, int64_t col0, int
     }
   }
   hcnt[8] = info > 0 ? info : 0;
+  const auto t2 = std::chrono::steady_clock::now();
   if (ft) host_guard<T>(hp, rows, nb, nb, hg);
+  const auto t3 = std::chrono::steady_clock::now();
 
   // lines 6-7: guarded H2D + device check
   const auto h2d_faults = faults(FT_AT_H2D);
@@ -348,7 +370,15 @@ static int host_pd_t(Driver& d, int k, int kind, int64_t row0, int64_t col0, int
     }
   }
   ABFT_CUDA_TRY(cudaGetLastError());
-  d.ms_host += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  const auto t4 = std::chrono::steady_clock::now();
+  auto ms = [](std::chrono::steady_clock::time_point a, std::chrono::steady_clock::time_point b) {
+    return std::chrono::duration<double, std::milli>(b - a).count();
+  };
+  d.ms_host += ms(t0, t4);
+  d.host_phase[0] += ms(t0, t1);  // guard encode + D2H (+ waiting for the device) + host check
+  d.host_phase[1] += ms(t1, t2);  // host LAPACK
+  d.host_phase[2] += ms(t2, t3);  // host guard
+  d.host_phase[3] += ms(t3, t4);  // H2D + device check + read-back
   return 0;
 }
 
@@ -382,6 +412,17 @@ extern "C" int ft_ctx_set_host_lapack(ft_ctx_t* c, const char* path) {
       return ABFT_E_UNSUPPORTED;
     }
   }
+  // split the cores between OpenBLAS and the guard loops (see g_host_threads)
+  cpu_set_t cs;
+  int cores = 16;
+  if (sched_getaffinity(0, sizeof(cs), &cs) == 0) cores = CPU_COUNT(&cs);
+  const int half = cores > 1 ? cores / 2 : 1;
+  typedef void (*set_threads_t)(int);
+  set_threads_t st = (set_threads_t)dlsym(h, "scipy_openblas_set_num_threads");
+  if (!st) st = (set_threads_t)dlsym(h, "openblas_set_num_threads");
+  if (st) st(half);
+  abft::g_host_threads = st ? std::max(1, cores - half) : std::max(1, cores);
+  if (getenv("ABFT_HOST_THREADS")) abft::g_host_threads = atoi(getenv("ABFT_HOST_THREADS"));
   if (c->lapack) dlclose(c->lapack);
   c->lapack = h;
   for (int i = 0; i < 6; ++i) c->lp[i] = f[i];

@@ -55,6 +55,7 @@ def _compare(lib, ctx, A, nb, injects):
     assert list(sg.counts) == so.counts, (list(sg.counts), so.counts)
     assert sorted((f[0], f[1], f[4], f[5]) for f in fg) == sorted((f.gi, f.gj, f.cls, f.kind) for f in so.fixes)
     assert sg.n_checks == so.n_checks
+    assert (sg.ctf_flagged, sg.ctf_recomputed) == (so.ctf_flagged, so.ctf_recomputed)
     h, t = np.linalg.qr(A, mode="raw")
     assert np.abs(Hg - h.T).max() <= 1e-12 * np.abs(h).max()
     return so, sg
@@ -69,6 +70,9 @@ QR_CASES = [
     (2, dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 170, 80, (54,)),     # consumed V fault -> R
     (2, dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 1, 9, 75, (61,)),  # column-checksum memory fault
     (2, dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 2, 100, 5, (61,)),  # row-checksum memory fault
+    (2, dr.AT_POST_PD, dr.KIND_PERSIST, 3, 4, 17, (61,)),     # CTF T, upper part (f2: recompute)
+    (3, dr.AT_POST_PD, dr.KIND_PERSIST, 3, 20, 20, (55,)),    # CTF T, diagonal
+    (1, dr.AT_POST_PD, dr.KIND_PERSIST, 3, 30, 2, (62,)),     # CTF T, a zero below the diagonal
 ]
 
 
@@ -110,3 +114,18 @@ def test_config3_shape_error_free(lib, ctx):
     R = torch.triu(A)[:, cols]
     res = (A0[:, cols] - Q @ R).abs().max().item()
     assert res <= 1e-10 * A0.abs().max().item() * n ** 0.5
+
+
+@pytest.mark.parametrize("n,nb", [(1024, 128), (2048, 512), (4096, 256)])
+def test_ctf_check_silent_when_error_free(lib, ctx, n, nb):
+    A = si.general(n, seed=n + nb)
+    *_, rc, info, stats, fixes = _gpu_geqrf(lib, ctx, A, nb)
+    assert rc == 0 and (stats.ctf_flagged, stats.ctf_recomputed) == (0, 0)
+
+
+def test_ctf_fault_without_check_is_silent(lib, ctx):
+    A = si.general(256, seed=0)
+    inj = [dr.Inject(2, dr.AT_POST_PD, dr.KIND_PERSIST, 3, 4, 17, (61,))]
+    H, *_ = _gpu_geqrf(lib, ctx, A, 32, inject=inj, abft=False)
+    h, _ = np.linalg.qr(A, mode="raw")
+    assert not np.abs(H - h.T).max() <= 1e-6
