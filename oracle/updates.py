@@ -229,6 +229,31 @@ def lu_pd_apply(st: State, k: int, lu, ipiv, P0):
         st.rowmag[r0:r1, k] = np.abs(Linv) @ st.rowmag[r0:r1, k]
 
 
+def lu_pd_undo(st: State, k: int, ipiv):
+    """f1 (L430) for LU: take back the row swaps a PD applied outside its
+    panel — the same transpositions in reverse order (a transposition is its
+    own inverse), with the c-14 swap rule on the left and right columns and
+    the row checksums of tile columns > k moving back with their rows.  The
+    panel itself and its checksums are restored from the pre-PD copy by the
+    caller."""
+    nb, n = st.nb, st.A.shape[0]
+    nt = n // nb
+    r0, r1 = k * nb, (k + 1) * nb
+    left_cols = np.arange(0, r0)
+    right_cols = np.arange(r1, n)
+    for j in reversed(range(nb)):
+        p, q = r0 + j, int(ipiv[j])
+        if p == q:
+            continue
+        if r0 > 0:
+            lu_swap_rule(st, p, q, left_cols, st.A[p, :r0].copy(), st.A[q, :r0].copy())
+        if r1 < n:
+            lu_swap_rule(st, p, q, right_cols, st.A[p, r1:].copy(), st.A[q, r1:].copy(),
+                         row_chk_cols=range(k + 1, nt))
+        st.A[[p, q], :r0] = st.A[[q, p], :r0]
+        st.A[[p, q], r1:] = st.A[[q, p], r1:]
+
+
 def lu_pd(st: State, k: int):
     """Factor + apply (no pre-swap check): returns (ipiv_global, info)."""
     lu, ipiv, info, P0 = lu_panel_getrf(st, k)

@@ -9,6 +9,7 @@ import pytest
 import synth_inputs as si
 from oracle import checksum as ck
 from oracle import drivers as dr
+from oracle import updates as up
 
 
 def _invariant(st, k, phase):
@@ -294,3 +295,61 @@ def test_qr_tmu_reference_fault_detected():
     A = si.general(256, seed=0)
     _, _, stats = dr.ft_geqrf(A, 32, inject=[dr.Inject(2, dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 170, 80, (54,))])
     assert stats.uncorrectable >= 1 and stats.repairs_skipped == 1
+
+
+# ---- f1 local restart for LU and QR (L430) ---------------------------------
+@pytest.mark.parametrize("bit,gi,gj", [(62, 200, 66), (60, 130, 70), (55, 64, 64)])
+def test_lu_pd_consumed_fault_restart(bit, gi, gj):
+    # a DRAM flip in the column panel between the pre-PD check and the PD is
+    # consumed by getrf (2D, possibly other pivots); the restart takes back the
+    # swaps outside the panel, restores the pre-PD copy and redoes the PD
+    A = si.general(256, seed=31)
+    ref, pref, _ = dr.ft_getrf(A, 64)
+    inj = [dr.Inject(1, dr.AT_PRE_PD, dr.KIND_PERSIST, 0, gi, gj, (bit,))]
+    _, _, s0 = dr.ft_getrf(A, 64, inject=inj, restart=False)
+    assert s0.uncorrectable >= 1
+    lu, piv, st = dr.ft_getrf(A, 64, inject=inj)
+    assert st.uncorrectable == 0 and st.restarts == 1
+    assert np.array_equal(piv, pref)
+    assert np.abs(lu - ref).max() <= 1e-12 * np.abs(ref).max()
+
+
+def test_lu_pd_undo_is_the_inverse_of_the_swaps():
+    # lu_pd_undo after lu_pd_apply restores every row outside the panel and
+    # the checksums (to rounding), whatever the pivots
+    n, nb, k = 256, 32, 2
+    st = ck.State.alloc(si.general(n, seed=32), nb)
+    ck.encode(st, ck.Tiles(0, n // nb, 0, n // nb), ck.BOTH)
+    before = st.copy()
+    lu, piv, _, P0 = up.lu_panel_getrf(st, k)
+    assert (piv != np.arange(k * nb, (k + 1) * nb)).sum() > 10
+    up.lu_pd_apply(st, k, lu, piv, P0)
+    up.lu_pd_undo(st, k, piv)
+    out = np.r_[0:k * nb, (k + 1) * nb:n]
+    assert np.array_equal(st.A[:, out], before.A[:, out])
+    assert np.abs(st.colchk[:, out] - before.colchk[:, out]).max() <= 1e-12 * np.abs(before.colchk).max()
+    assert np.array_equal(st.rowchk[:, 2 * (k + 1):], before.rowchk[:, 2 * (k + 1):])
+
+
+def test_lu_pu_reference_fault_restart():
+    # on-chip flip in L_kk while the PU reads it: U12 is 2D-wrong; restart
+    A = si.general(256, seed=33)
+    ref, _, _ = dr.ft_getrf(A, 32)
+    inj = [dr.Inject(2, dr.AT_PRE_PU, dr.KIND_ONCHIP, 0, 70, 66, (60,))]
+    _, _, s0 = dr.ft_getrf(A, 32, inject=inj, restart=False)
+    assert s0.uncorrectable >= 1
+    lu, _, st = dr.ft_getrf(A, 32, inject=inj)
+    assert st.uncorrectable == 0 and st.restarts == 1
+    assert np.abs(lu - ref).max() <= 1e-12 * np.abs(ref).max()
+
+
+@pytest.mark.parametrize("bit,gi,gj", [(62, 200, 66), (57, 70, 70)])
+def test_qr_pd_consumed_fault_restart(bit, gi, gj):
+    A = si.general(256, seed=34)
+    ref, tref, _ = dr.ft_geqrf(A, 64)
+    inj = [dr.Inject(1, dr.AT_PRE_PD, dr.KIND_PERSIST, 0, gi, gj, (bit,))]
+    _, _, s0 = dr.ft_geqrf(A, 64, inject=inj, restart=False)
+    assert s0.uncorrectable >= 1
+    qr, tau, st = dr.ft_geqrf(A, 64, inject=inj)
+    assert st.uncorrectable == 0 and st.restarts == 1
+    assert np.abs(qr - ref).max() <= 1e-12 * np.abs(ref).max() and np.abs(tau - tref).max() <= 1e-12
