@@ -391,11 +391,11 @@ def abft_panel_getrf(mat: Mat, k: int, ipiv: torch.Tensor, Linv: torch.Tensor, U
 
 
 def ft_getrf(ctx: Context, A: torch.Tensor, nb: int, ipiv: torch.Tensor, abft=True, tol_kind=TOL_MAGNITUDE,
-             tol_scale=1.0, fig4a_repair=True, inject=(), fix_log=None, pd_location=PD_DEVICE):
+             tol_scale=1.0, fig4a_repair=True, inject=(), fix_log=None, pd_location=PD_DEVICE, restart=True):
     """Fault-tolerant LU with partial pivoting in place on a column-major A;
     ipiv: int64 device tensor (n), receives 1-based global pivots."""
     n = A.shape[0]
-    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, True,
+    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, True, restart=restart,
                        pd_location=pd_location)
     stats = ft_stats_t()
     info = C.c_int64()
@@ -413,11 +413,12 @@ def abft_panel_geqrf(mat: Mat, k: int, tau: torch.Tensor, V: torch.Tensor, T: to
 
 
 def ft_geqrf(ctx: Context, A: torch.Tensor, nb: int, tau: torch.Tensor, abft=True, tol_kind=TOL_MAGNITUDE,
-             tol_scale=1.0, inject=(), fix_log=None, pd_location=PD_DEVICE):
+             tol_scale=1.0, inject=(), fix_log=None, pd_location=PD_DEVICE, restart=True):
     """Fault-tolerant Householder QR in place on a column-major A (LAPACK
     dgeqrf storage); tau: device tensor (n) of A's dtype."""
     n = A.shape[0]
-    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, True, inject, fix_log, True, pd_location=pd_location)
+    opts, _inj = _opts(nb, abft, tol_kind, tol_scale, True, inject, fix_log, True, restart=restart,
+                       pd_location=pd_location)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_geqrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), _ptr(tau), C.byref(opts), C.byref(stats),

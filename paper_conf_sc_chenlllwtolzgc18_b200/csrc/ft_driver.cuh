@@ -70,6 +70,8 @@ inline int grow_buffer(void*& p, size_t& have, size_t need) {
 
 // LAPACK info of the whole factorization: first failing panel's local value
 // offset by the panel origin.
+static __global__ void drv_add_i32_kernel(int32_t* p, int32_t v) { *p += v; }
+
 static __global__ void accum_info_kernel(int32_t* tile_info, int32_t* total, int64_t offset) {
   if (*tile_info != 0 && *total == 0) *total = (int32_t)(*tile_info + offset);
   *tile_info = 0;
@@ -140,7 +142,8 @@ struct Driver {
     xcounts = counts + 16;
     ctf_cnt = counts + 24;
     if (o->abft && o->restart)
-      FT_TRY(grow_buffer(c->rsv, c->rsv_bytes, ((size_t)n * nb + (size_t)nb * nb + 3 * (size_t)nt * nb + 4 * nb) * es));
+      FT_TRY(grow_buffer(c->rsv, c->rsv_bytes,
+                         ((size_t)n * nb + (size_t)nb * nb + 3 * (size_t)nt * nb + 4 * nb + 3 * (size_t)n) * es));
     ABFT_CUDA_TRY(cudaMemsetAsync(c->ints, 0, ints_need * sizeof(int32_t), s));
     char* st = (char*)c->state;
     M.dtype = dtype;
@@ -234,6 +237,31 @@ struct Driver {
     FT_TRY(abft_locate_correct(&M, &t, which, &tol, &R, c->fixlog, c->fixcap, nfix, (abft_stream_t)s));
     ++n_checks;
     return 0;
+  }
+  // Local restart (f1, L430) bookkeeping: snapshot the uncorrectable counter
+  // before a post-op check, read back how many 2D errors that check added
+  // (one host wait), and take them back when the op is redone.
+  int snap_uncorrectable() {
+    ABFT_CUDA_TRY(cudaMemcpyAsync(snap, counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToDevice, s));
+    return 0;
+  }
+  int uncorrectable_added(int* delta) {
+    ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin, snap, 4, cudaMemcpyDeviceToHost, s));
+    ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin + 1, counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToHost, s));
+    ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+    *delta = c->hpin[1] - c->hpin[0];
+    return 0;
+  }
+  int take_back_uncorrectable(int delta) {
+    ++restarts;
+    drv_add_i32_kernel<<<1, 1, 0, s>>>(counts + ABFT_CNT_UNCORRECTABLE, -delta);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    return 0;
+  }
+  // 2-D copy of rows x cols elements between column-major arrays (SM kernel)
+  int copy(void* dst, int64_t ldd, const void* src, int64_t lds, int64_t rows, int64_t cols) {
+    if (rows <= 0 || cols <= 0) return 0;
+    return abft::copy2d(dst, ldd * es, src, lds * es, rows * es, cols, s);
   }
   void* colchk_at(int64_t r, int64_t col) { return (char*)M.colchk + (r + col * M.ldc) * es; }
   void* colmag_at(int64_t r, int64_t col) { return (char*)M.colmag + (r + col * M.ldcm) * es; }

@@ -446,19 +446,56 @@ static int geqrf_driver(Driver& d, ft_ctx* c, T* tau_all) {
     // Alg. 2 lines 3-4: check the column panel to be decomposed (c + r)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
     if (ft) FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH));
+    // Local restart (f1, L430): copy of the column panel with its checksums
+    // (rsv: panel | c | m_c | r | m_r) after its pre-op check
+    const bool rs = ft && d.o->restart;
+    const int ntk = (int)(nt - k);
+    char* cp_a = (char*)c->rsv;
+    char* cp_c = cp_a + (size_t)mk * nb * d.es;
+    char* cp_m = cp_c + (size_t)2 * ntk * nb * d.es;
+    char* cp_r = cp_m + (size_t)ntk * nb * d.es;
+    char* cp_rm = cp_r + (size_t)mk * 2 * d.es;
+    if (rs) {
+      FT_TRY(d.copy(cp_a, mk, d.a_at(r0, r0), lda, mk, nb));
+      FT_TRY(d.copy(cp_c, 2 * ntk, d.colchk_at(2 * k, r0), d.M.ldc, 2 * ntk, nb));
+      FT_TRY(d.copy(cp_m, ntk, d.colmag_at(k, r0), d.M.ldcm, ntk, nb));
+      FT_TRY(d.copy(cp_r, mk, d.rowchk_at(r0, 2 * k), d.M.ldr, mk, 2));
+      FT_TRY(d.copy(cp_rm, mk, d.rowmag_at(r0, k), d.M.ldrm, mk, 1));
+    }
     // line 5: PD (Alg. 1: V with c(V), R_kk with r(R)) + CTF
+    auto do_pd = [&]() -> int {
+      if (d.o->pd_location == FT_PD_HOST)
+        FT_TRY(panel_geqrf_t<T>(&d.M, k, tau_all + r0, Vbuf, Tm, P0, d.info, s, &d));
+      else
+        FT_TRY(abft_panel_geqrf(&d.M, k, tau_all + r0, Vbuf, Tm, P0, d.info, as));
+      accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.info_total, r0);
+      return 0;
+    };
+    auto post_pd_checks = [&]() -> int {
+      FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_UNIT_LOWER, ABFT_COL));
+      return d.check(k, k + 1, k, k + 1, ABFT_UPPER, ABFT_ROW);
+    };
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD));
-    if (d.o->pd_location == FT_PD_HOST)
-      FT_TRY(panel_geqrf_t<T>(&d.M, k, tau_all + r0, Vbuf, Tm, P0, d.info, s, &d));
-    else
-      FT_TRY(abft_panel_geqrf(&d.M, k, tau_all + r0, Vbuf, Tm, P0, d.info, as));
-    accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.info_total, r0);
+    FT_TRY(do_pd());
     FT_TRY(d.restore_onchip());
     FT_TRY(d.inject_at(k, FT_AT_POST_PD));
-    // line 7: check V (UNIT_LOWER on the diagonal, c) and R_kk (UPPER, r)
+    // line 7: check V (UNIT_LOWER on the diagonal, c) and R_kk (UPPER, r);
+    // 2D -> restore the copy and redo the PD once
     if (ft) {
-      FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_UNIT_LOWER, ABFT_COL));
-      FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_UPPER, ABFT_ROW));
+      if (rs) FT_TRY(d.snap_uncorrectable());
+      FT_TRY(post_pd_checks());
+      int delta = 0;
+      if (rs) FT_TRY(d.uncorrectable_added(&delta));
+      if (delta > 0) {
+        FT_TRY(d.take_back_uncorrectable(delta));
+        FT_TRY(d.copy(d.a_at(r0, r0), lda, cp_a, mk, mk, nb));
+        FT_TRY(d.copy(d.colchk_at(2 * k, r0), d.M.ldc, cp_c, 2 * ntk, 2 * ntk, nb));
+        FT_TRY(d.copy(d.colmag_at(k, r0), d.M.ldcm, cp_m, ntk, ntk, nb));
+        FT_TRY(d.copy(d.rowchk_at(r0, 2 * k), d.M.ldr, cp_r, mk, mk, 2));
+        FT_TRY(d.copy(d.rowmag_at(r0, k), d.M.ldrm, cp_rm, mk, mk, 1));
+        FT_TRY(do_pd());
+        FT_TRY(post_pd_checks());
+      }
     }
     if (k == nt - 1) break;
     // QR's TMU reads all of A2 (W = T^T V^T A2): A2 is a reference part, so it

@@ -196,7 +196,7 @@ __global__ void __launch_bounds__(256) lu_perm_cols_kernel(T* A, int64_t lda, in
   const int64_t c = blockIdx.x;
   const int64_t r0 = (int64_t)k * nb, r1 = r0 + nb;
   const bool panel = c >= r0 && c < r1;
-  if (panel && !colchk) return;
+  if (panel && (!colchk || !pcopy)) return;  // no pcopy: restart undo, the panel is restored from its copy
   const int n = *nrows;
   const T* col = panel ? pcopy + (c - r0) * ldp - r0 : A + c * lda;
   for (int s = threadIdx.x; s < n; s += blockDim.x) xs[s] = col[S[s]];
@@ -327,6 +327,12 @@ __global__ void lu_fig4a_repair_kernel(LuRepairArgs r) {
     if (threadIdx.x == 0) atomicAdd(&r.rep_counts[0], 1);
     __syncthreads();
   }
+}
+
+// Inverse of the (S, src) permutation: sinv[src[s]] = s.
+__global__ void lu_invert_perm_kernel(const int32_t* src, const int32_t* nrows, int32_t* sinv) {
+  const int n = *nrows;
+  for (int s = threadIdx.x; s < n; s += blockDim.x) sinv[src[s]] = s;
 }
 
 static unsigned blocks_for(int64_t work, int per) {
@@ -468,6 +474,51 @@ static int panel_getrf_impl(const abft_mat_t* mat, int32_t k, int64_t* ipiv, con
   return 0;
 }
 
+// f1 (L430): take back the row swaps the last panel_getrf_impl(k) on this
+// stream applied outside its panel (same scratch layout: moved rows S, src,
+// tile bounds, count), with the column-checksum deltas and the row checksums
+// moving back.  The panel and its checksums are restored by the caller.
+static int panel_getrf_undo(const abft_mat_t* mat, int k, cudaStream_t s) {
+  using namespace abft;
+  const int64_t nb = mat->nb, n = mat->n, nt = n / nb, r0 = k * nb, mk = n - r0;
+  const size_t es = mat->dtype == ABFT_F64 ? 8 : 4;
+  const bool ft = mat->colchk != nullptr;
+  const size_t copy_bytes = ft ? (size_t)mk * nb * es : 0;
+  const size_t off_piv = (copy_bytes + 255) / 256 * 256;
+  const size_t off_rows = off_piv + ((size_t)nb * 4 + 255) / 256 * 256;
+  const size_t off_src = off_rows + (size_t)2 * nb * 8;
+  const size_t off_tb = off_src + (size_t)2 * nb * 4;
+  const size_t off_nrows = off_tb + ((size_t)nt + 2) * 4;
+  void* scr = nullptr;
+  FT_TRY(scratch(s, 10, off_nrows + 4, &scr));  // the buffer the PD used (only grows)
+  char* base = (char*)scr;
+  const int64_t* rows = (const int64_t*)(base + off_rows);
+  const int32_t* src = (const int32_t*)(base + off_src);
+  const int32_t* tb = (const int32_t*)(base + off_tb);
+  const int32_t* nrows = (const int32_t*)(base + off_nrows);
+  void* si = nullptr;
+  FT_TRY(scratch(s, 11, (size_t)2 * nb * 4, &si));
+  int32_t* sinv = (int32_t*)si;
+  lu_invert_perm_kernel<<<1, 1024, 0, s>>>(src, nrows, sinv);
+  if (mat->dtype == ABFT_F64) {
+    lu_perm_cols_kernel<double><<<(unsigned)n, 256, 0, s>>>((double*)mat->A, mat->lda, (int)nb, k, (int)nt, rows, sinv,
+                                                            tb, nrows, nullptr, 0, (double*)mat->colchk, mat->ldc,
+                                                            (double*)mat->colmag, mat->ldcm);
+    lu_perm_rowchk_kernel<double><<<(unsigned)(nt - k), 256, 0, s>>>((double*)mat->rowchk, mat->ldr,
+                                                                    (double*)mat->rowmag, mat->ldrm, k, rows, sinv,
+                                                                    nrows);
+  } else {
+    lu_perm_cols_kernel<float><<<(unsigned)n, 256, 0, s>>>((float*)mat->A, mat->lda, (int)nb, k, (int)nt, rows, sinv,
+                                                           tb, nrows, nullptr, 0, (float*)mat->colchk, mat->ldc,
+                                                           (float*)mat->colmag, mat->ldcm);
+    lu_perm_rowchk_kernel<float><<<(unsigned)(nt - k), 256, 0, s>>>((float*)mat->rowchk, mat->ldr,
+                                                                   (float*)mat->rowmag, mat->ldrm, k, rows, sinv,
+                                                                   nrows);
+  }
+  ABFT_CUDA_TRY(cudaGetLastError());
+  return 0;
+}
+
 // ----------------------------------------------------------------- driver --
 extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t lda, int64_t* ipiv,
                         const ft_opts_t* o, ft_stats_t* stats, int64_t* info_out) {
@@ -500,28 +551,77 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     // Alg. 2 lines 3-4: check the column panel to be decomposed (c + r)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
     if (ft) FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH));
+    // Local restart (f1, L430): the column panel with its checksums is copied
+    // after its pre-op check; layout in rsv: panel | c | m_c | r | m_r
+    const bool rs = ft && o->restart;
+    const int64_t mk = n - r0;
+    const int ntk = (int)(nt - k);
+    char* rb = (char*)c->rsv;
+    char* cp_a = rb;
+    char* cp_c = cp_a + (size_t)mk * nb * d.es;
+    char* cp_m = cp_c + (size_t)2 * ntk * nb * d.es;
+    char* cp_r = cp_m + (size_t)ntk * nb * d.es;
+    char* cp_rm = cp_r + (size_t)mk * 2 * d.es;
+    if (rs) {
+      FT_TRY(d.copy(cp_a, mk, d.a_at(r0, r0), lda, mk, nb));
+      FT_TRY(d.copy(cp_c, 2 * ntk, d.colchk_at(2 * k, r0), d.M.ldc, 2 * ntk, nb));
+      FT_TRY(d.copy(cp_m, ntk, d.colmag_at(k, r0), d.M.ldcm, ntk, nb));
+      FT_TRY(d.copy(cp_r, mk, d.rowchk_at(r0, 2 * k), d.M.ldr, mk, 2));
+      FT_TRY(d.copy(cp_rm, mk, d.rowmag_at(r0, k), d.M.ldrm, mk, 1));
+    }
     // line 5: PD with pivoting, swap rule, c(L), r(U_kk)
+    auto do_pd = [&]() -> int {
+      FT_TRY(panel_getrf_impl(&d.M, k, ipiv + r0, ft ? &d.tol : nullptr, ft ? &d.R : nullptr, c->fixlog,
+                              c->fixcap, d.nfix, c->linv, c->uinv, d.info, as,
+                              o->pd_location == FT_PD_HOST ? &d : nullptr));
+      if (ft && k < nt - 1) ++d.n_checks;  // the pre-swap row check (c-14b)
+      accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.info_total, r0);
+      return 0;
+    };
+    auto post_pd_checks = [&]() -> int {
+      FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_UNIT_LOWER, ABFT_COL));
+      return d.check(k, k + 1, k, k + 1, ABFT_UPPER, ABFT_ROW);
+    };
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD));
-    FT_TRY(panel_getrf_impl(&d.M, k, ipiv + r0, ft ? &d.tol : nullptr, ft ? &d.R : nullptr, c->fixlog, c->fixcap,
-                            d.nfix, c->linv, c->uinv, d.info, as, o->pd_location == FT_PD_HOST ? &d : nullptr));
-    if (ft && k < nt - 1) ++d.n_checks;  // the pre-swap row check (c-14b)
-    accum_info_kernel<<<1, 1, 0, s>>>(d.info, d.info_total, r0);
+    FT_TRY(do_pd());
     FT_TRY(d.restore_onchip());
     FT_TRY(d.inject_at(k, FT_AT_POST_PD));
     // line 7: check the decomposed panel: L (UNIT_LOWER on the diagonal, c) and U_kk (r)
     if (ft) {
-      FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_UNIT_LOWER, ABFT_COL));
-      FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_UPPER, ABFT_ROW));
+      if (rs) FT_TRY(d.snap_uncorrectable());
+      FT_TRY(post_pd_checks());
+      int delta = 0;
+      if (rs) FT_TRY(d.uncorrectable_added(&delta));
+      if (delta > 0) {  // 2D after the PD: undo its swaps, restore the copy, redo
+        FT_TRY(d.take_back_uncorrectable(delta));
+        FT_TRY(panel_getrf_undo(&d.M, k, s));
+        FT_TRY(d.copy(d.a_at(r0, r0), lda, cp_a, mk, mk, nb));
+        FT_TRY(d.copy(d.colchk_at(2 * k, r0), d.M.ldc, cp_c, 2 * ntk, 2 * ntk, nb));
+        FT_TRY(d.copy(d.colmag_at(k, r0), d.M.ldcm, cp_m, ntk, ntk, nb));
+        FT_TRY(d.copy(d.rowchk_at(r0, 2 * k), d.M.ldr, cp_r, mk, mk, 2));
+        FT_TRY(d.copy(d.rowmag_at(r0, k), d.M.ldrm, cp_rm, mk, mk, 1));
+        FT_TRY(do_pd());
+        FT_TRY(post_pd_checks());
+      }
     }
     if (k == nt - 1) break;
     // line 8: check the row panel to be updated (c + r)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PU_CHECK));
     if (ft) FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_BOTH));
+    // local restart copy of the row panel: A12 | r(A12) | m_r(A12)
+    char* pu_a = rb;
+    char* pu_r = pu_a + (size_t)nb * nk * d.es;
+    char* pu_rm = pu_r + (size_t)nb * m2 * d.es;
+    if (rs) {
+      FT_TRY(d.copy(pu_a, nb, d.a_at(r0, r1), lda, nb, nk));
+      FT_TRY(d.copy(pu_r, nb, d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, nb, m2));
+      FT_TRY(d.copy(pu_rm, nb, d.rowmag_at(r0, k + 1), d.M.ldrm, nb, m2 / 2));
+    }
     // line 9: PU  U12 = L_kk^-1 A12 (DGEMM with the PD's inverse) + r rule
     FT_TRY(d.inject_at(k, FT_AT_PRE_PU));
     const bool refresh = d.diag_touched_before_pu(k);
     if (refresh) FT_TRY(abft_tri_inverse(dtype, 'L', 'U', nb, d.a_at(r0, r0), lda, c->linv, nb, as));
-    {
+    auto pu_data = [&]() -> int {
       cublasHandle_t h = blas_handle(s, lk);
       cublasStatus_t st;
       if (dtype == ABFT_F64) {
@@ -535,16 +635,33 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       }
       lk.unlock();
       if (st != CUBLAS_STATUS_SUCCESS) return ABFT_E_CUBLAS;
-      FT_TRY(abft::copy2d(d.a_at(r0, r1), lda * d.es, c->putmp, nb * d.es, nb * d.es, nk, s));
-    }
+      return abft::copy2d(d.a_at(r0, r1), lda * d.es, c->putmp, nb * d.es, nb * d.es, nk, s);
+    };
+    auto pu_chk = [&]() -> int {  // r(U_kJ) = L_kk^-1 r(A_kJ), m_r <- |L_kk^-1| m_r  (c-13)
+      return abft_update_trsm_inv(dtype, 'L', 'N', nb, c->linv, nb, d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, m2,
+                                  d.rowmag_at(r0, k + 1), d.M.ldrm, m2 / 2, as);
+    };
+    FT_TRY(pu_data());
     FT_TRY(d.restore_onchip());
     if (refresh) FT_TRY(abft_tri_inverse(dtype, 'L', 'U', nb, d.a_at(r0, r0), lda, c->linv, nb, as));
-    if (ft)  // r(U_kJ) = L_kk^-1 r(A_kJ), m_r <- |L_kk^-1| m_r  (c-13)
-      FT_TRY(abft_update_trsm_inv(dtype, 'L', 'N', nb, c->linv, nb, d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, m2,
-                                  d.rowmag_at(r0, k + 1), d.M.ldrm, m2 / 2, as));
+    if (ft) FT_TRY(pu_chk());
     FT_TRY(d.inject_at(k, FT_AT_POST_PU));
-    // line 10: check the updated row panel (r)
-    if (ft) FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW));
+    // line 10: check the updated row panel (r); 2D -> local restart of the PU (L430, L434)
+    if (ft) {
+      if (rs) FT_TRY(d.snap_uncorrectable());
+      FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW));
+      int delta = 0;
+      if (rs) FT_TRY(d.uncorrectable_added(&delta));
+      if (delta > 0) {
+        FT_TRY(d.take_back_uncorrectable(delta));
+        FT_TRY(d.copy(d.a_at(r0, r1), lda, pu_a, nb, nb, nk));
+        FT_TRY(d.copy(d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, pu_r, nb, nb, m2));
+        FT_TRY(d.copy(d.rowmag_at(r0, k + 1), d.M.ldrm, pu_rm, nb, nb, m2 / 2));
+        FT_TRY(pu_data());
+        FT_TRY(pu_chk());
+        FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW));
+      }
+    }
     // line 12: TMU  A22 -= L21 U12 (DGEMM on tensor cores) + c-13 rules
     FT_TRY(d.inject_at(k, FT_AT_PRE_TMU));
     {

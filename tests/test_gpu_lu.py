@@ -154,3 +154,35 @@ def test_config3_shape_error_free(lib, ctx):
     PA = A0[torch.tensor(pm, device="cuda")[rows]]
     R = PA - L[rows] @ U
     assert R.abs().max().item() <= 1e-10 * A0.abs().max().item() * n ** 0.5
+
+
+# ---- f1 local restart (L430): parity with the oracle's restart -------------
+def _gpu_getrf_rs(lib, ctx, A_np, nb, inject, restart):
+    A = dev(A_np)
+    ipiv = torch.zeros(A.shape[0], dtype=torch.int64, device="cuda")
+    inj = [(f.iter, f.point, f.kind, f.target, f.gi, f.gj, si.mask_of(f.bits)) for f in inject]
+    rc, info, stats = lib.ft_getrf(ctx, A, nb, ipiv, inject=inj, restart=restart)
+    torch.cuda.synchronize()
+    return host(A), ipiv.cpu().numpy() - 1, rc, stats
+
+
+@pytest.mark.parametrize("k,point,kind,gi,gj,bit", [
+    (1, dr.AT_PRE_PD, dr.KIND_PERSIST, 200, 66, 62),   # consumed by getrf, other pivots
+    (1, dr.AT_PRE_PD, dr.KIND_PERSIST, 130, 70, 60),
+    (1, dr.AT_PRE_PD, dr.KIND_PERSIST, 64, 64, 55),
+    (2, dr.AT_PRE_PU, dr.KIND_ONCHIP, 140, 130, 60),   # L_kk read by the PU: U12 2D
+])
+def test_lu_restart_parity(lib, ctx, k, point, kind, gi, gj, bit):
+    nb = 64
+    A = si.general(256, seed=31)
+    inj = [dr.Inject(k, point, kind, 0, gi, gj, (bit,))]
+    ref, pref, _ = dr.ft_getrf(A, nb)
+    o_lu, o_piv, ost = dr.ft_getrf(A, nb, inject=inj)
+    LU, piv, rc, st = _gpu_getrf_rs(lib, ctx, A, nb, inj, True)
+    assert ost.restarts == 1 and ost.uncorrectable == 0
+    assert rc == 0 and st.restarts == 1 and st.uncorrectable == 0
+    assert list(st.counts) == ost.counts and st.n_checks == ost.n_checks
+    assert np.array_equal(piv, pref)
+    assert np.abs(LU - ref).max() <= 1e-12 * np.abs(ref).max()
+    _, _, rc0, st0 = _gpu_getrf_rs(lib, ctx, A, nb, inj, False)
+    assert rc0 == lib.E_UNCORRECTABLE and st0.restarts == 0
