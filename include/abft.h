@@ -350,6 +350,15 @@ typedef struct {
                             (abft_verify / abft_locate_correct; uncorrectable -> re-send), then the
                             PD checksum rule and the post-PD check run on the device as usual.
                             The host waits for the device once per iteration. */
+  int32_t fig4b;         /* 1 (default): Fig. 4b on-chip 1D detection (L359, f1) — when a pre-PD / pre-PU
+                            check of iteration k corrected a 1D pattern (class 1D_ROW / 1D_COL: several
+                            errors in one row / column of a block, the trace of an on-chip fault in the
+                            previous TMU), the whole trailing matrix is checked right away (ft_potrf,
+                            ft_getrf; ft_geqrf checks all of A2 before every TMU anyway).  Decided on the
+                            device: without such a fix the check's kernels exit at once. */
+  int32_t trailing_check_period; /* P > 0: check the whole trailing matrix after the TMU of every P-th
+                            iteration (L359: "periodically check the correctness of trailing matrix
+                            ... to avoid 2D propagation"); 0 (default): never */
 } ft_opts_t;
 
 /* Host-side statistics, filled after the driver's final synchronisation. */

@@ -136,4 +136,15 @@ int counters_get(cudaStream_t s, size_t n_ints, int** out);
 // Device-to-device 2-D copy (pitches and width in bytes) with an SM kernel:
 // cudaMemcpy2DAsync D2D of column panels runs far below HBM bandwidth.
 int copy2d(void* dst, size_t dpitch, const void* src, size_t spitch, size_t width, size_t height, cudaStream_t s);
+
+// Device-side gate of the verify / locate launches issued by this host
+// thread (drivers only, not part of the C ABI): when non-null, every CTA of
+// those kernels returns at once unless *gate != 0, so a conditional check
+// (Fig. 4b, f1) costs two empty launches and no host synchronisation.
+const int32_t*& launch_gate();
+struct GateScope {
+  const int32_t* prev;
+  explicit GateScope(const int32_t* g) : prev(launch_gate()) { launch_gate() = g; }
+  ~GateScope() { launch_gate() = prev; }
+};
 }  // namespace abft

@@ -47,6 +47,7 @@ struct LocArgs {
   int32_t max_fixes;
   int32_t* n_fixes;
   int64_t ntiles;
+  const int32_t* gate;  // nullable: run only if *gate != 0
 };
 
 template <typename T>
@@ -135,6 +136,7 @@ struct Action {
 
 template <typename T>
 __global__ void __launch_bounds__(kLThreads) locate_correct_kernel(LocArgs p) {
+  if (p.gate && *p.gate == 0) return;
   extern __shared__ __align__(16) unsigned char sm[];
   const int nb = p.nb;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -614,6 +616,7 @@ extern "C" int abft_locate_correct(const abft_mat_t* m, const abft_tiles_t* t, i
   a.max_fixes = max_fixes;
   a.n_fixes = n_fixes;
   a.ntiles = abft::tiles_count(*t);
+  a.gate = abft::launch_gate();
   if (a.ntiles == 0) return 0;
   cudaStream_t s = (cudaStream_t)stream;
   return m->dtype == ABFT_F64 ? abft::launch_locate<double>(a, s) : abft::launch_locate<float>(a, s);

@@ -106,6 +106,7 @@ struct PassArgs {
   void* symws;      // [ntiles][3][NB] SYM column sums of slabbed diagonal tiles
   int* ticket;      // [nsuper] self-resetting
   int* tflags;      // [ntiles] self-resetting
+  const int32_t* gate;  // nullable: run only if *gate != 0 (driver-side conditional checks)
 };
 
 template <typename T, int VEC>
@@ -180,6 +181,7 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
   __shared__ int s_colflags[K], s_ncols[K], s_nrows[K], s_rowflags[K];
   __shared__ int s_last;
 
+  if (p.gate && *p.gate == 0) return;  // whole grid skips (uniform): no barrier or ticket touched
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int64_t unit = blockIdx.x;
   const int64_t sup = unit / p.nslab;
@@ -700,6 +702,7 @@ static int run_pass(const abft_mat_t* m, const abft_tiles_t* t, int which, const
   a.ldrm = m->ldrm;
   a.tiles = *t;
   a.which = which;
+  a.gate = launch_gate();
   const size_t es = m->dtype == ABFT_F64 ? 8 : 4;
   a.use_bulk = ((uintptr_t)m->A % 16 == 0) && ((m->lda * es) % 16 == 0);
   if (verify) {

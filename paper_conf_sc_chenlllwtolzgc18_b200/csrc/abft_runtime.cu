@@ -100,6 +100,11 @@ int copy2d(void* dst, size_t dpitch, const void* src, size_t spitch, size_t widt
   return 0;
 }
 
+const int32_t*& launch_gate() {
+  static thread_local const int32_t* g = nullptr;
+  return g;
+}
+
 __global__ void inject_kernel64(uint64_t* p, int64_t off, uint64_t mask) { p[off] ^= mask; }
 __global__ void inject_kernel32(uint32_t* p, int64_t off, uint32_t mask) { p[off] ^= mask; }
 

@@ -72,6 +72,21 @@ inline int grow_buffer(void*& p, size_t& have, size_t need) {
 // offset by the panel origin.
 static __global__ void drv_add_i32_kernel(int32_t* p, int32_t v) { *p += v; }
 
+// Fig. 4b gate: did the fixes logged since the start of the iteration include
+// a 1D pattern (class 1D_ROW / 1D_COL)?  Counts the gated checks that run.
+static __global__ void fig4b_gate_kernel(const abft_fix_t* fixes, int cap, const int32_t* from, const int32_t* to,
+                                         int32_t* gate, int32_t* runs) {
+  const int n0 = *from, n1 = min(*to, cap);
+  int hit = 0;
+  for (int f = n0 + (int)threadIdx.x; f < n1; f += blockDim.x)
+    hit |= fixes[f].kind == ABFT_FIX_DATA && (fixes[f].cls == ABFT_CLS_1D_ROW || fixes[f].cls == ABFT_CLS_1D_COL);
+  hit = __any_sync(0xffffffffu, hit);
+  if (threadIdx.x == 0) {
+    *gate = hit;
+    if (hit) ++*runs;
+  }
+}
+
 static __global__ void accum_info_kernel(int32_t* tile_info, int32_t* total, int64_t offset) {
   if (*tile_info != 0 && *total == 0) *total = (int32_t)(*tile_info + offset);
   *tile_info = 0;
@@ -102,6 +117,9 @@ struct Driver {
   double ms_host = 0.0;
   double host_phase[4] = {};           // ABFT_HOST_TIMING=1: per-phase host ms (stderr at the end)
   int32_t* ctf_cnt = nullptr;          // device: flagged entries of one CTF check (QR, f2)
+  int32_t* gate4b = nullptr;           // device: Fig. 4b gate of this iteration
+  int32_t* gated_runs = nullptr;       // device: gated checks that ran
+  int32_t* iter_mark = nullptr;        // device: fix-log position at the start of the iteration
   int ctf_flagged = 0, ctf_recomputed = 0;
   std::vector<std::pair<int, int>> xfer_used;  // (iter, point) transfer faults already applied
 
@@ -141,6 +159,9 @@ struct Driver {
     mark2 = snap + 1;
     xcounts = counts + 16;
     ctf_cnt = counts + 24;
+    gate4b = counts + 25;
+    gated_runs = counts + 26;
+    iter_mark = counts + 27;
     if (o->abft && o->restart)
       FT_TRY(grow_buffer(c->rsv, c->rsv_bytes,
                          ((size_t)n * nb + (size_t)nb * nb + 3 * (size_t)nt * nb + 4 * nb + 3 * (size_t)n) * es));
@@ -263,6 +284,26 @@ struct Driver {
     if (rows <= 0 || cols <= 0) return 0;
     return abft::copy2d(dst, ldd * es, src, lds * es, rows * es, cols, s);
   }
+  // f1 hooks: the fix-log position at the start of iteration k; the Fig. 4b
+  // check (gated on a 1D fix since then); the periodic trailing check.
+  int begin_iteration() {
+    ABFT_CUDA_TRY(cudaMemcpyAsync(iter_mark, nfix, 4, cudaMemcpyDeviceToDevice, s));
+    return 0;
+  }
+  int fig4b_check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only) {
+    if (!o->fig4b || I0 >= I1) return 0;
+    fig4b_gate_kernel<<<1, 32, 0, s>>>(c->fixlog, c->fixcap, iter_mark, nfix, gate4b, gated_runs);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    GateScope g(gate4b);
+    FT_TRY(check(I0, I1, J0, J1, view, which, lower_only));
+    --n_checks;  // counted on the device when it runs
+    return 0;
+  }
+  int periodic_check(int k, int I0, int I1, int J0, int J1, int view, bool lower_only) {
+    const int P = o->trailing_check_period;
+    if (P <= 0 || (k + 1) % P != 0 || I0 >= I1) return 0;
+    return check(I0, I1, J0, J1, view, ABFT_BOTH, lower_only);
+  }
   void* colchk_at(int64_t r, int64_t col) { return (char*)M.colchk + (r + col * M.ldc) * es; }
   void* colmag_at(int64_t r, int64_t col) { return (char*)M.colmag + (r + col * M.ldcm) * es; }
   void* rowchk_at(int64_t r, int64_t col) { return (char*)M.rowchk + (r + col * M.ldr) * es; }
@@ -271,7 +312,7 @@ struct Driver {
 
   // The single host synchronisation: counters, info and the fix log.
   int finish(std::chrono::steady_clock::time_point t0, ft_stats_t* stats, int64_t* info_out) {
-    int32_t h[8 + 8];
+    int32_t h[32];
     ABFT_CUDA_TRY(cudaMemcpyAsync(h, counts, sizeof(h), cudaMemcpyDeviceToHost, s));
     if (o->fix_log && o->fix_log_cap > 0)
       ABFT_CUDA_TRY(cudaMemcpyAsync(o->fix_log, c->fixlog, sizeof(abft_fix_t) * std::min(o->fix_log_cap, c->fixcap),
@@ -286,7 +327,7 @@ struct Driver {
       stats->repairs_applied = h[11];
       stats->repairs_skipped = h[12];
       stats->uncorrectable = h[ABFT_CNT_UNCORRECTABLE];
-      stats->n_checks = n_checks;
+      stats->n_checks = n_checks + h[26];
       stats->restarts = restarts;
       stats->ms_total = std::chrono::duration<double, std::milli>(t1 - t0).count();
       int32_t* x = &stats->xfer_d2h_flagged;

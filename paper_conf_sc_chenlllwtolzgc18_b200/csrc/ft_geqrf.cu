@@ -540,6 +540,7 @@ static int geqrf_driver(Driver& d, ft_ctx* c, T* tau_all) {
       FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_UNIT_LOWER, ABFT_COL));
       qr_consumed_fault_kernel<<<1, 1, 0, s>>>(c->fixlog, c->fixcap, d.nfix, d.mark, r0, r1, d.rep, d.counts);
       FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW));
+      FT_TRY(d.periodic_check(k, k + 1, (int)nt, k + 1, (int)nt, ABFT_GENERAL, false));  // L359
     }
   }
   return 0;

@@ -548,6 +548,7 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
   for (int k = 0; k < nt; ++k) {
     const int64_t r0 = k * nb, r1 = r0 + nb, nk = n - r1;
     const int m2 = (int)(2 * (nt - k - 1));
+    if (ft) FT_TRY(d.begin_iteration());
     // Alg. 2 lines 3-4: check the column panel to be decomposed (c + r)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
     if (ft) FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH));
@@ -617,6 +618,8 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       FT_TRY(d.copy(pu_r, nb, d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, nb, m2));
       FT_TRY(d.copy(pu_rm, nb, d.rowmag_at(r0, k + 1), d.M.ldrm, nb, m2 / 2));
     }
+    // Fig. 4b (L359): a 1D pattern fixed in this iteration -> check the trailing matrix
+    if (ft) FT_TRY(d.fig4b_check(k + 1, (int)nt, k + 1, (int)nt, ABFT_GENERAL, ABFT_BOTH, false));
     // line 9: PU  U12 = L_kk^-1 A12 (DGEMM with the PD's inverse) + r rule
     FT_TRY(d.inject_at(k, FT_AT_PRE_PU));
     const bool refresh = d.diag_touched_before_pu(k);
@@ -723,6 +726,7 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
           lu_fig4a_repair_kernel<float><<<1, 256, 0, s>>>(ra);
         ABFT_CUDA_TRY(cudaGetLastError());
       }
+      FT_TRY(d.periodic_check(k, k + 1, (int)nt, k + 1, (int)nt, ABFT_GENERAL, false));  // L359
     }
   }
   return d.finish(t0, stats, info_out);

@@ -225,6 +225,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     const int64_t r1 = (k + 1) * nb;  // first row/col after the panel
     const int64_t nk = n - r1;        // trailing size
     const int m2 = (int)(2 * (nt - k - 1));
+    if (ft) FT_TRY(d.begin_iteration());
     // Alg. 2 lines 3-4: check the panel to be decomposed (diag tile, SYM view, both)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
     if (ft) FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_SYM_LOWER, ABFT_BOTH));
@@ -328,6 +329,10 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       FT_TRY(copy2d(pu_m, m2 / 2, d.colmag_at(k + 1, r0), d.M.ldcm, m2 / 2, nb));
     }
     if (defer_pd) FT_TRY(pd_restart());
+    // Fig. 4b (L359): a 1D pattern fixed by this iteration's pre-PD / pre-PU
+    // checks is the trace of an on-chip fault in the last TMU: check the
+    // whole trailing matrix now (gated on the device)
+    if (ft) FT_TRY(d.fig4b_check(k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, ABFT_BOTH, true));
     // line 9: PU  L_ik = A_ik L_kk^-T  (+ c(L_ik) = c(A_ik) L_kk^-T, c-12)
     auto pu_data = [&]() -> int {
       cublasHandle_t h = blas_handle(s, lk);
@@ -452,6 +457,8 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
           fig4a_repair_kernel<float><<<1, 256, 0, s>>>(ra);
         ABFT_CUDA_TRY(cudaGetLastError());
       }
+      // periodic trailing-matrix check (L359)
+      FT_TRY(d.periodic_check(k, k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, true));
     }
   }
   return d.finish(t0, stats, info_out);

@@ -159,3 +159,28 @@ def test_config2_shape_error_free_and_injected(lib, ctx):
     torch.cuda.synchronize()
     assert rc == 0 and stats.counts[5] == 1
     assert (torch.tril(A) - L).abs().max().item() <= 1e-12 * L.abs().max().item()
+
+
+# ---- f1: Fig. 4b on-chip 1D detection and the periodic trailing check ------
+_ONCHIP_PAIR = [dr.Inject(1, dr.AT_PRE_TMU, dr.KIND_ONCHIP, 0, 197, 40, (55,)),
+                dr.Inject(2, dr.AT_PRE_TMU, dr.KIND_ONCHIP, 0, 212, 67, (55,))]
+
+
+@pytest.mark.parametrize("fig4b,period", [(True, 0), (False, 0), (False, 1), (True, 2)])
+def test_fig4b_and_periodic_parity(lib, ctx, fig4b, period):
+    A_np = si.spd(256, seed=41)
+    o_L, ost = dr.ft_potrf(A_np, 32, inject=_ONCHIP_PAIR, fig4b=fig4b, restart=False,
+                           trailing_check_period=period)
+    A = dev(A_np)
+    inj = [(f.iter, f.point, f.kind, f.target, f.gi, f.gj, si.mask_of(f.bits)) for f in _ONCHIP_PAIR]
+    log = torch.zeros(8192 * lib.FIX_BYTES, dtype=torch.uint8, device="cuda")
+    rc, info, st = lib.ft_potrf(ctx, A, 32, inject=inj, fix_log=log, restart=False, fig4b=fig4b,
+                                trailing_check_period=period)
+    torch.cuda.synchronize()
+    fixes = lib.decode_fixes(log, st.n_fixes)
+    assert (rc == lib.E_UNCORRECTABLE) == (ost.uncorrectable > 0)
+    assert st.n_checks == ost.n_checks
+    if ost.uncorrectable == 0:
+        assert list(st.counts) == ost.counts
+        assert sorted((f[0], f[1], f[4]) for f in fixes) == sorted((f.gi, f.gj, f.cls) for f in ost.fixes)
+        assert np.abs(np.tril(host(A)) - o_L).max() <= 1e-12 * np.abs(o_L).max()

@@ -353,3 +353,41 @@ def test_qr_pd_consumed_fault_restart(bit, gi, gj):
     qr, tau, st = dr.ft_geqrf(A, 64, inject=inj)
     assert st.uncorrectable == 0 and st.restarts == 1
     assert np.abs(qr - ref).max() <= 1e-12 * np.abs(ref).max() and np.abs(tau - tref).max() <= 1e-12
+
+
+# ---- f1 Fig. 4b on-chip 1D detection and the periodic trailing check (L359) -
+# Two on-chip faults in consecutive TMUs hit cached panel values of rows 197
+# and 212 (both in tile row 6): each leaves a 1D row/column error across the
+# trailing matrix; left alone they meet in tiles (6, 3..6) as a 2D error.
+_ONCHIP_PAIR = [dr.Inject(1, dr.AT_PRE_TMU, dr.KIND_ONCHIP, 0, 197, 40, (55,)),
+                dr.Inject(2, dr.AT_PRE_TMU, dr.KIND_ONCHIP, 0, 212, 67, (55,))]
+
+
+def test_fig4b_stops_onchip_1d_errors_from_accumulating():
+    A = si.spd(256, seed=41)
+    Lref, _ = dr.ft_potrf(A, 32)
+    _, s0 = dr.ft_potrf(A, 32, inject=_ONCHIP_PAIR, fig4b=False, restart=False)
+    assert s0.uncorrectable >= 1
+    L, st = dr.ft_potrf(A, 32, inject=_ONCHIP_PAIR, restart=False)
+    assert st.uncorrectable == 0
+    assert [c[1] for c in st.checks].count("fig4b") == 2
+    assert any(f.cls in (ck.CLS_1D_ROW, ck.CLS_1D_COL) for f in st.fixes)
+    assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
+
+
+def test_periodic_trailing_check_also_stops_the_accumulation():
+    A = si.spd(256, seed=41)
+    Lref, _ = dr.ft_potrf(A, 32)
+    L, st = dr.ft_potrf(A, 32, inject=_ONCHIP_PAIR, fig4b=False, restart=False, trailing_check_period=1)
+    assert st.uncorrectable == 0
+    assert [c[1] for c in st.checks].count("periodic") == 256 // 32 - 1
+    assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
+
+
+def test_fig4b_silent_without_faults():
+    A = si.spd(256, seed=42)
+    _, st = dr.ft_potrf(A, 32)
+    assert "fig4b" not in [c[1] for c in st.checks]
+    G = si.general(256, seed=43)
+    _, _, st = dr.ft_getrf(G, 32, trailing_check_period=3)
+    assert [c[1] for c in st.checks].count("periodic") == 2 and st.counts == [0] * 8
