@@ -44,17 +44,23 @@ struct Handles {
   std::mutex mu;
 };
 std::mutex g_hmu;
-Handles& handles_for_device() {
-  static auto* m = new std::unordered_map<int, Handles*>();
+// One cuBLAS / cuSOLVER handle pair per (device, stream): library calls issued
+// on different streams at the same time (the drivers' side stream) must not
+// share a handle's workspace.
+Handles& handles_for(cudaStream_t s) {
+  static auto* m = new std::unordered_map<uint64_t, Handles*>();
   int dev = 0;
   cudaGetDevice(&dev);
+  const uint64_t key = (reinterpret_cast<uint64_t>(s) << 8) ^ (uint64_t)dev;
   std::lock_guard<std::mutex> g(g_hmu);
-  auto it = m->find(dev);
+  auto it = m->find(key);
   if (it != m->end()) return *it->second;
   Handles* h = new Handles();
   cublasCreate(&h->blas);
   cusolverDnCreate(&h->solver);
-  (*m)[dev] = h;
+  cublasSetStream(h->blas, s);
+  cusolverDnSetStream(h->solver, s);
+  (*m)[key] = h;
   return *h;
 }
 
@@ -90,16 +96,13 @@ int scratch_get(cudaStream_t s, int slot, size_t bytes, void** out) {
 }  // namespace
 
 cublasHandle_t blas_handle(cudaStream_t s, std::unique_lock<std::mutex>& lk) {
-  Handles& h = handles_for_device();
+  Handles& h = handles_for(s);
   lk = std::unique_lock<std::mutex>(h.mu);
-  cublasSetStream(h.blas, s);
   return h.blas;
 }
 cusolverDnHandle_t solver_handle(cudaStream_t s, std::unique_lock<std::mutex>& lk) {
-  Handles& h = handles_for_device();
+  Handles& h = handles_for(s);
   lk = std::unique_lock<std::mutex>(h.mu);
-  cusolverDnSetStream(h.solver, s);
-  cublasSetStream(h.blas, s);
   return h.solver;
 }
 int scratch(cudaStream_t s, int slot, size_t bytes, void** out) { return scratch_get(s, slot, bytes, out); }

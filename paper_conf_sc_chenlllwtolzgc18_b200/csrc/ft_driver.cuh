@@ -252,10 +252,12 @@ struct Driver {
     onchip_pending.clear();
     return 0;
   }
-  int check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only = false) {
+  int check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only = false,
+            cudaStream_t on = nullptr) {
     abft_tiles_t t{I0, I1, J0, J1, lower_only ? 1 : 0, view};
-    FT_TRY(abft_verify(&M, &t, which, &tol, &R, (abft_stream_t)s));
-    FT_TRY(abft_locate_correct(&M, &t, which, &tol, &R, c->fixlog, c->fixcap, nfix, (abft_stream_t)s));
+    const abft_stream_t st = (abft_stream_t)(on ? on : s);
+    FT_TRY(abft_verify(&M, &t, which, &tol, &R, st));
+    FT_TRY(abft_locate_correct(&M, &t, which, &tol, &R, c->fixlog, c->fixcap, nfix, st));
     ++n_checks;
     return 0;
   }

@@ -625,19 +625,27 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     const bool refresh = d.diag_touched_before_pu(k);
     if (refresh) FT_TRY(abft_tri_inverse(dtype, 'L', 'U', nb, d.a_at(r0, r0), lda, c->linv, nb, as));
     auto pu_data = [&]() -> int {
+      // not in place: from the local-restart copy of A12 straight into A12 when
+      // there is one (no fault plan: copy == A12), else via scratch + copy back
+      const bool from_copy = rs && o->n_inject == 0;
+      const void* src = from_copy ? (const void*)pu_a : d.a_at(r0, r1);
+      const int lds = from_copy ? (int)nb : (int)lda;
+      void* dst = from_copy ? d.a_at(r0, r1) : c->putmp;
+      const int ldd = from_copy ? (int)lda : (int)nb;
       cublasHandle_t h = blas_handle(s, lk);
       cublasStatus_t st;
       if (dtype == ABFT_F64) {
         const double one = 1.0, zero = 0.0;
         st = cublasDgemm(h, CUBLAS_OP_N, CUBLAS_OP_N, (int)nb, (int)nk, (int)nb, &one, (const double*)c->linv,
-                         (int)nb, (const double*)d.a_at(r0, r1), (int)lda, &zero, (double*)c->putmp, (int)nb);
+                         (int)nb, (const double*)src, lds, &zero, (double*)dst, ldd);
       } else {
         const float one = 1.0f, zero = 0.0f;
         st = cublasSgemm(h, CUBLAS_OP_N, CUBLAS_OP_N, (int)nb, (int)nk, (int)nb, &one, (const float*)c->linv, (int)nb,
-                         (const float*)d.a_at(r0, r1), (int)lda, &zero, (float*)c->putmp, (int)nb);
+                         (const float*)src, lds, &zero, (float*)dst, ldd);
       }
       lk.unlock();
       if (st != CUBLAS_STATUS_SUCCESS) return ABFT_E_CUBLAS;
+      if (from_copy) return 0;
       return abft::copy2d(d.a_at(r0, r1), lda * d.es, c->putmp, nb * d.es, nb * d.es, nk, s);
     };
     auto pu_chk = [&]() -> int {  // r(U_kJ) = L_kk^-1 r(A_kJ), m_r <- |L_kk^-1| m_r  (c-13)

@@ -337,21 +337,28 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     auto pu_data = [&]() -> int {
       cublasHandle_t h = blas_handle(s, lk);
       if (o->pu_gemm) {
-        // L21 = A21 L_kk^-T as a DGEMM with the explicit inverse (tensor cores),
-        // written to scratch and copied back
+        // L21 = A21 L_kk^-T as a DGEMM with the explicit inverse (tensor cores).
+        // The GEMM cannot run in place: it reads the local-restart copy of A21
+        // when there is one (no fault plan: the copy equals A21) and writes
+        // A21 directly, else it writes scratch that is copied back.
+        const bool from_copy = rs && o->n_inject == 0;
+        const void* src = from_copy ? (const void*)pu_a : d.a_at(r1, r0);
+        const int lds = from_copy ? (int)nk : (int)lda;
+        void* dst = from_copy ? d.a_at(r1, r0) : c->putmp;
+        const int ldd = from_copy ? (int)lda : (int)nk;
         cublasStatus_t st;
         if (dtype == ABFT_F64) {
           const double one = 1.0, zero = 0.0;
-          st = cublasDgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)nk, (int)nb, (int)nb, &one, (const double*)d.a_at(r1, r0),
-                           (int)lda, (const double*)c->linv, (int)nb, &zero, (double*)c->putmp, (int)nk);
+          st = cublasDgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)nk, (int)nb, (int)nb, &one, (const double*)src, lds,
+                           (const double*)c->linv, (int)nb, &zero, (double*)dst, ldd);
         } else {
           const float one = 1.0f, zero = 0.0f;
-          st = cublasSgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)nk, (int)nb, (int)nb, &one, (const float*)d.a_at(r1, r0),
-                           (int)lda, (const float*)c->linv, (int)nb, &zero, (float*)c->putmp, (int)nk);
+          st = cublasSgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)nk, (int)nb, (int)nb, &one, (const float*)src, lds,
+                           (const float*)c->linv, (int)nb, &zero, (float*)dst, ldd);
         }
         lk.unlock();
         if (st != CUBLAS_STATUS_SUCCESS) return ABFT_E_CUBLAS;
-        FT_TRY(abft::copy2d(d.a_at(r1, r0), lda * d.es, c->putmp, nk * d.es, nk * d.es, nb, s));
+        if (!from_copy) FT_TRY(abft::copy2d(d.a_at(r1, r0), lda * d.es, c->putmp, nk * d.es, nk * d.es, nb, s));
       } else {
         cublasStatus_t st;
         if (dtype == ABFT_F64) {
@@ -402,6 +409,10 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     }
     // line 12: TMU  A22 -= L21 L21^T (DSYRK on tensor cores) + checksum rules c-12
     FT_TRY(d.inject_at(k, FT_AT_PRE_TMU));
+    // (Running the checksum rule and the panel re-check on a second stream
+    // next to the DSYRK was measured: no gain at any stream priority — the
+    // DSYRK keeps every SM busy — so everything stays on one stream.)
+    cudaStream_t cs = s;
     {
       cublasHandle_t h = blas_handle(s, lk);
       if (dtype == ABFT_F64) {
@@ -423,13 +434,13 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       FT_TRY(abft_update_syrk(dtype, nb, nt - k - 1, d.a_at(r1, k * nb), lda, d.colchk_at(2 * (k + 1), k * nb), d.M.ldc,
                               d.colmag_at(k + 1, k * nb), d.M.ldcm, d.colchk_at(2 * (k + 1), r1),
                               d.rowchk_at(r1, 2 * (k + 1)), d.M.ldr, d.colmag_at(k + 1, r1), d.rowmag_at(r1, k + 1),
-                              d.M.ldrm, as));
+                              d.M.ldrm, (abft_stream_t)cs));
     }
     FT_TRY(d.inject_at(k, FT_AT_POST_TMU));
     // line 13: heuristic panel re-check for the TMU (Fig. 4a) + guarded repair (c-25)
     if (ft) {
-      ABFT_CUDA_TRY(cudaMemcpyAsync(d.mark, d.nfix, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
-      FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
+      ABFT_CUDA_TRY(cudaMemcpyAsync(d.mark, d.nfix, sizeof(int32_t), cudaMemcpyDeviceToDevice, cs));
+      FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL, false, cs));
       if (o->fig4a_repair) {
         RepairArgs ra{};
         ra.A = dA;
@@ -452,9 +463,9 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
         ra.rep_counts = d.rep;
         ra.counts = d.counts;
         if (dtype == ABFT_F64)
-          fig4a_repair_kernel<double><<<1, 256, 0, s>>>(ra);
+          fig4a_repair_kernel<double><<<1, 256, 0, cs>>>(ra);
         else
-          fig4a_repair_kernel<float><<<1, 256, 0, s>>>(ra);
+          fig4a_repair_kernel<float><<<1, 256, 0, cs>>>(ra);
         ABFT_CUDA_TRY(cudaGetLastError());
       }
       // periodic trailing-matrix check (L359)
