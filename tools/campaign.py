@@ -2,9 +2,13 @@
 one random single fault per run at a random Alg. 2 hook of a random
 iteration, for ft_potrf / ft_getrf / ft_geqrf on the GPU, graded as the
 paper's outcomes (L580): Y = fixed (factor equals the fault-free one within
-1e-12), R = detected but uncorrectable (restart needed), N = not detected /
+1e-12; "restarts" counts the runs that needed the local restart, f1),
+R = detected but uncorrectable (complete restart needed), N = not detected /
 silently wrong.  Faults use exponent/sign bits (52–63), i.e. the MUST band
-of reading c-10 for O(1) elements.  Writes gpurun_out/campaign.json.
+of reading c-10 for O(1) elements.  QR runs also draw faults in the CTF T
+(f2); a fourth campaign, "host", runs ft_potrf / ft_getrf with the PD on the
+host (FT_PD_HOST) and draws D2H / H2D transfer faults (Alg. 2 lines 3, 6).
+Writes gpurun_out/campaign.json.
 
   python tools/campaign.py [trials_per_driver] [n] [nb]
 """
@@ -19,7 +23,8 @@ import torch
 import synth_inputs as si
 from paper_conf_sc_chenlllwtolzgc18_b200 import abft
 
-AT = dict(PRE_PD_CHECK=0, PRE_PD=1, POST_PD=2, PRE_PU_CHECK=3, PRE_PU=4, POST_PU=5, PRE_TMU=6, POST_TMU=7)
+AT = dict(PRE_PD_CHECK=0, PRE_PD=1, POST_PD=2, PRE_PU_CHECK=3, PRE_PU=4, POST_PU=5, PRE_TMU=6, POST_TMU=7,
+          D2H=8, H2D=9)
 
 
 def plan(kind, n, nb, g):
@@ -53,7 +58,19 @@ def plan(kind, n, nb, g):
         else:
             gi, gj = int(g.integers(r1, n)), int(g.integers(r1, n))
     bit = int(g.integers(52, 64))
-    return (k, point, 1 if onchip else 0, 0, gi, gj, 1 << bit), bit
+    target = 0
+    if kind == "geqrf" and point == AT["POST_PD"] and g.random() < 0.25:  # CTF T (f2)
+        target, gi, gj = 3, int(g.integers(0, nb)), int(g.integers(0, nb))
+        gi, gj = min(gi, gj), max(gi, gj)  # upper triangle incl. the diagonal
+    if kind.startswith("host"):
+        point = AT["D2H"] if g.random() < 0.5 else AT["H2D"]
+        onchip = False
+        rows = nb if kind == "host_potrf" else n - r0
+        gi, gj = r0 + int(g.integers(0, rows)), int(g.integers(r0, r1))
+        if kind == "host_potrf":
+            a, b = gi, gj
+            gi, gj = max(a, b), min(a, b)
+    return (k, point, 1 if onchip else 0, target, gi, gj, 1 << bit), bit
 
 
 def main():
@@ -61,21 +78,23 @@ def main():
     n = int(sys.argv[2]) if len(sys.argv) > 2 else 1024
     nb = int(sys.argv[3]) if len(sys.argv) > 3 else 128
     ctx = abft.Context()
+    ctx.set_host_lapack()
     g = si.rng(2018)
     report = {"n": n, "nb": nb, "trials": trials, "bits": "52-63"}
-    for kind in ("potrf", "getrf", "geqrf"):
-        A0 = si.spd_device(n, seed=1) if kind == "potrf" else si.general_device(n, seed=1)
+    for kind in ("potrf", "getrf", "geqrf", "host_potrf", "host_getrf"):
+        pd = abft.PD_HOST if kind.startswith("host") else abft.PD_DEVICE
+        A0 = si.spd_device(n, seed=1) if kind.endswith("potrf") else si.general_device(n, seed=1)
         A = torch.empty_like(A0.t()).t()
         piv = torch.zeros(n, dtype=torch.int64, device="cuda")
         tau = torch.zeros(n, dtype=torch.float64, device="cuda")
 
         def run(inj):
             A.copy_(A0)
-            if kind == "potrf":
-                rc, info, st = abft.ft_potrf(ctx, A, nb, inject=inj)
+            if kind.endswith("potrf"):
+                rc, info, st = abft.ft_potrf(ctx, A, nb, inject=inj, pd_location=pd)
                 out = torch.tril(A).clone()
-            elif kind == "getrf":
-                rc, info, st = abft.ft_getrf(ctx, A, nb, piv, inject=inj)
+            elif kind.endswith("getrf"):
+                rc, info, st = abft.ft_getrf(ctx, A, nb, piv, inject=inj, pd_location=pd)
                 out = A.clone()
             else:
                 rc, info, st = abft.ft_geqrf(ctx, A, nb, tau, inject=inj)
@@ -85,12 +104,13 @@ def main():
 
         _, _, ref = run(())
         scale = ref.abs().max().item()
-        out = {"Y": 0, "R": 0, "N": 0, "detected": 0, "cases": []}
+        out = {"Y": 0, "R": 0, "N": 0, "detected": 0, "restarts": 0, "cases": []}
         for t in range(trials):
             inj, bit = plan(kind, n, nb, g)
             rc, st, res = run([inj])
             err = (res - ref).abs().max().item() / scale
-            det = st.counts[0] > 0 or st.uncorrectable > 0
+            det = (st.counts[0] > 0 or st.uncorrectable > 0 or st.restarts > 0 or st.ctf_flagged > 0
+                   or st.xfer_d2h_flagged > 0 or st.xfer_h2d_flagged > 0)
             if rc == abft.E_UNCORRECTABLE:
                 o = "R"
             elif err <= 1e-12:
@@ -99,8 +119,11 @@ def main():
                 o = "N"
             out[o] += 1
             out["detected"] += int(det)
+            out["restarts"] += int(st.restarts > 0)
             out["cases"].append({"inject": list(inj[:6]), "bit": bit, "outcome": o, "rel_err": err,
-                                 "fixes": st.n_fixes, "repairs": st.repairs_applied})
+                                 "fixes": st.n_fixes, "repairs": st.repairs_applied, "restarts": st.restarts,
+                                 "ctf": st.ctf_recomputed, "xfer_fixed": st.xfer_d2h_fixed + st.xfer_h2d_fixed,
+                                 "retransfers": st.xfer_retransfers + st.xfer_resends})
         report[kind] = out
         print(kind, {k: v for k, v in out.items() if k != "cases"}, flush=True)
         del A, A0
