@@ -45,7 +45,8 @@ struct ft_ctx {
   size_t aux_bytes = 0;
   void* rsv = nullptr;  // local-restart copies (f1): PD tile + PU panel with checksums
   size_t rsv_bytes = 0;
-  int32_t* hpin = nullptr;  // pinned host words for the restart read-back
+  int32_t* hpin = nullptr;  // pinned host words (read-backs), mapped into the device address space
+  int32_t* hpin_dev = nullptr;  // device alias of hpin (a kernel writes read-back words straight to the host)
   cudaEvent_t ev = nullptr;  // marks the PD-check read-back (restart decision)
   // FT_PD_HOST (ft_host.cu): host LAPACK, pinned panel staging, device guard
   void* lapack = nullptr;  // dlopen handle
@@ -71,6 +72,14 @@ inline int grow_buffer(void*& p, size_t& have, size_t need) {
 // LAPACK info of the whole factorization: first failing panel's local value
 // offset by the panel origin.
 static __global__ void drv_add_i32_kernel(int32_t* p, int32_t v) { *p += v; }
+
+// Restart read-back (f1): the uncorrectable errors a check added, written to
+// mapped host memory by one thread (replaces two device-to-host copies on
+// the stream's critical path).
+static __global__ void drv_delta_to_host_kernel(const int32_t* now, const int32_t* snap, volatile int32_t* host) {
+  *host = *now - *snap;
+}
+static __global__ void drv_word_to_host_kernel(const int32_t* src, volatile int32_t* host) { *host = *src; }
 
 // Fig. 4b gate: did the fixes logged since the start of the iteration include
 // a 1D pattern (class 1D_ROW / 1D_COL)?  Counts the gated checks that run.
@@ -268,12 +277,27 @@ struct Driver {
     ABFT_CUDA_TRY(cudaMemcpyAsync(snap, counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToDevice, s));
     return 0;
   }
-  int uncorrectable_added(int* delta) {
-    ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin, snap, 4, cudaMemcpyDeviceToHost, s));
-    ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin + 1, counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToHost, s));
-    ABFT_CUDA_TRY(cudaStreamSynchronize(s));
-    *delta = c->hpin[1] - c->hpin[0];
+  int post_delta(int slot) {  // queue the read-back of the check just issued into hpin[slot]
+    drv_delta_to_host_kernel<<<1, 1, 0, s>>>(counts + ABFT_CNT_UNCORRECTABLE, snap, c->hpin_dev + slot);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    ABFT_CUDA_TRY(cudaEventRecord(c->ev, s));
     return 0;
+  }
+  int post_word(const int32_t* src, int slot) {  // queue the read-back of one device word into hpin[slot]
+    drv_word_to_host_kernel<<<1, 1, 0, s>>>(src, c->hpin_dev + slot);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    ABFT_CUDA_TRY(cudaEventRecord(c->ev, s));
+    return 0;
+  }
+  int32_t host_word(int slot) const { return ((volatile int32_t*)c->hpin)[slot]; }
+  int wait_delta(int slot, int* delta) {
+    ABFT_CUDA_TRY(cudaEventSynchronize(c->ev));
+    *delta = ((volatile int32_t*)c->hpin)[slot];
+    return 0;
+  }
+  int uncorrectable_added(int* delta) {
+    FT_TRY(post_delta(0));
+    return wait_delta(0, delta);
   }
   int take_back_uncorrectable(int delta) {
     ++restarts;

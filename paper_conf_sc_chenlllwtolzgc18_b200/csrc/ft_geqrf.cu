@@ -385,38 +385,53 @@ static int ctf_eval(cudaStream_t s, int64_t mk, int nb, const T* Vbuf, const T* 
   return 0;
 }
 
-// f2 for iteration k: check T, recompute it from V (the CTF of
-// panel_geqrf_t: T = (striu(V^T V) + diag(1/tau))^-1) if flagged, check again;
-// a T still flagged is uncorrectable.  One host read-back per call.
+// f2 for iteration k, in two halves so that its host read-back can share one
+// wait with the PD restart decision: ctf_issue rebuilds V from memory,
+// evaluates E and queues the flag count into hpin[1]; ctf_resolve (after the
+// caller waited) recomputes T from V (the CTF of panel_geqrf_t:
+// T = (striu(V^T V) + diag(1/tau))^-1) if flagged and checks again; a T still
+// flagged is uncorrectable.
+struct CtfWork {
+  void* sv;
+  double g4;
+};
+
 template <typename T>
-static int ctf_check(Driver& d, ft_ctx* c, int64_t mk, T* Vbuf, T* Tm, const T* tau) {
+static int ctf_issue(Driver& d, int64_t mk, T* Vbuf, T* Tm, CtfWork* w) {
   cudaStream_t s = d.s;
   const int nb = (int)d.nb;
-  void* sv = nullptr;
-  FT_TRY(scratch(s, 17, ((size_t)nb * nb * 4 + nb) * sizeof(T), &sv));
-  T* S = reinterpret_cast<T*>(sv);
+  FT_TRY(scratch(s, 17, ((size_t)nb * nb * 4 + nb) * sizeof(T), &w->sv));
+  T* S = reinterpret_cast<T*>(w->sv);
+  T* W = S + (size_t)nb * nb;
+  T* TST = W + (size_t)nb * nb;
+  T* a = TST + (size_t)2 * nb * nb;
+  const double m = (double)(mk + nb), u = Prec<T>::u;
+  w->g4 = 4.0 * d.tol.scale * m * u / (1.0 - m * u);
+  qr_build_v_kernel<T><<<blocks_of(mk * nb), 256, 0, s>>>(Vbuf, mk, nb, reinterpret_cast<T*>(d.a_at(d.n - mk, d.n - mk)),
+                                                         d.lda);
+  FT_TRY(ctf_eval<T>(s, mk, nb, Vbuf, Tm, S, W, TST, a, w->g4, d.ctf_cnt));
+  return d.post_word(d.ctf_cnt, 1);
+}
+
+template <typename T>
+static int ctf_resolve(Driver& d, int64_t mk, T* Vbuf, T* Tm, const T* tau, const CtfWork& w) {
+  if (d.host_word(1) == 0) return 0;
+  cudaStream_t s = d.s;
+  const int nb = (int)d.nb;
+  T* S = reinterpret_cast<T*>(w.sv);
   T* W = S + (size_t)nb * nb;
   T* TST = W + (size_t)nb * nb;
   T* Ti = TST + (size_t)nb * nb;
   T* a = Ti + (size_t)nb * nb;
-  const double m = (double)(mk + nb), u = Prec<T>::u;
-  const double g4 = 4.0 * d.tol.scale * m * u / (1.0 - m * u);
-  int32_t* cnt = d.ctf_cnt;
-  qr_build_v_kernel<T><<<blocks_of(mk * nb), 256, 0, s>>>(Vbuf, mk, nb, reinterpret_cast<T*>(d.a_at(d.n - mk, d.n - mk)),
-                                                         d.lda);
-  FT_TRY(ctf_eval<T>(s, mk, nb, Vbuf, Tm, S, W, TST, a, g4, cnt));
-  ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin + 4, cnt, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-  ABFT_CUDA_TRY(cudaStreamSynchronize(s));
-  if (c->hpin[4] == 0) return 0;
   ++d.ctf_flagged;
   qr_tinv_kernel<T><<<blocks_of((int64_t)nb * nb), 256, 0, s>>>(Ti, S, tau, nb);
   FT_TRY(abft_tri_inverse(d.dtype, 'U', 'N', nb, Ti, nb, Tm, nb, (abft_stream_t)s));
   qr_fix_zero_tau_kernel<T><<<(unsigned)nb, 128, 0, s>>>(Tm, tau, nb);
   ++d.ctf_recomputed;
-  FT_TRY(ctf_eval<T>(s, mk, nb, Vbuf, Tm, S, W, TST, a, g4, cnt));
-  ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin + 4, cnt, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-  ABFT_CUDA_TRY(cudaStreamSynchronize(s));
-  if (c->hpin[4] != 0) add_i32_kernel_qr<<<1, 1, 0, s>>>(d.counts + ABFT_CNT_UNCORRECTABLE, 1);
+  FT_TRY(ctf_eval<T>(s, mk, nb, Vbuf, Tm, S, W, TST, a, w.g4, d.ctf_cnt));
+  FT_TRY(d.post_word(d.ctf_cnt, 1));
+  ABFT_CUDA_TRY(cudaEventSynchronize(d.c->ev));
+  if (d.host_word(1) != 0) add_i32_kernel_qr<<<1, 1, 0, s>>>(d.counts + ABFT_CNT_UNCORRECTABLE, 1);
   return 0;
 }
 }  // namespace abft
@@ -480,29 +495,49 @@ static int geqrf_driver(Driver& d, ft_ctx* c, T* tau_all) {
     FT_TRY(d.restore_onchip());
     FT_TRY(d.inject_at(k, FT_AT_POST_PD));
     // line 7: check V (UNIT_LOWER on the diagonal, c) and R_kk (UPPER, r);
-    // 2D -> restore the copy and redo the PD once
+    // 2D -> restore the copy and redo the PD once.  The decision's read-back
+    // shares one host wait with the CTF check's (the A2 check in between is
+    // independent of the panel).
+    auto restart_pd = [&]() -> int {
+      FT_TRY(d.copy(d.a_at(r0, r0), lda, cp_a, mk, mk, nb));
+      FT_TRY(d.copy(d.colchk_at(2 * k, r0), d.M.ldc, cp_c, 2 * ntk, 2 * ntk, nb));
+      FT_TRY(d.copy(d.colmag_at(k, r0), d.M.ldcm, cp_m, ntk, ntk, nb));
+      FT_TRY(d.copy(d.rowchk_at(r0, 2 * k), d.M.ldr, cp_r, mk, mk, 2));
+      FT_TRY(d.copy(d.rowmag_at(r0, k), d.M.ldrm, cp_rm, mk, mk, 1));
+      FT_TRY(do_pd());
+      return post_pd_checks();
+    };
     if (ft) {
       if (rs) FT_TRY(d.snap_uncorrectable());
       FT_TRY(post_pd_checks());
+      if (rs) FT_TRY(d.post_delta(0));
+    }
+    if (k == nt - 1) {
       int delta = 0;
-      if (rs) FT_TRY(d.uncorrectable_added(&delta));
+      if (rs) FT_TRY(d.wait_delta(0, &delta));
       if (delta > 0) {
         FT_TRY(d.take_back_uncorrectable(delta));
-        FT_TRY(d.copy(d.a_at(r0, r0), lda, cp_a, mk, mk, nb));
-        FT_TRY(d.copy(d.colchk_at(2 * k, r0), d.M.ldc, cp_c, 2 * ntk, 2 * ntk, nb));
-        FT_TRY(d.copy(d.colmag_at(k, r0), d.M.ldcm, cp_m, ntk, ntk, nb));
-        FT_TRY(d.copy(d.rowchk_at(r0, 2 * k), d.M.ldr, cp_r, mk, mk, 2));
-        FT_TRY(d.copy(d.rowmag_at(r0, k), d.M.ldrm, cp_rm, mk, mk, 1));
-        FT_TRY(do_pd());
-        FT_TRY(post_pd_checks());
+        FT_TRY(restart_pd());
       }
+      break;
     }
-    if (k == nt - 1) break;
     // QR's TMU reads all of A2 (W = T^T V^T A2): A2 is a reference part, so it
     // is checked before the TMU (Alg. 2 line 8 for QR, reading c-25q)
     if (ft) FT_TRY(d.check(k, (int)nt, k + 1, (int)nt, ABFT_GENERAL, ABFT_BOTH));
     // f2 (L263): T carries no checksum; verify the orthogonality of I - V T V^T
-    if (ft) FT_TRY(ctf_check<T>(d, c, mk, Vbuf, Tm, tau_all + r0));
+    if (ft) {
+      CtfWork cw{};
+      FT_TRY(ctf_issue<T>(d, mk, Vbuf, Tm, &cw));
+      ABFT_CUDA_TRY(cudaEventSynchronize(c->ev));  // one wait: PD decision + CTF flags
+      const int delta = rs ? d.host_word(0) : 0;
+      if (delta > 0) {
+        FT_TRY(d.take_back_uncorrectable(delta));
+        FT_TRY(restart_pd());  // new V and T: check them again
+        FT_TRY(ctf_issue<T>(d, mk, Vbuf, Tm, &cw));
+        ABFT_CUDA_TRY(cudaEventSynchronize(c->ev));
+      }
+      FT_TRY(ctf_resolve<T>(d, mk, Vbuf, Tm, tau_all + r0, cw));
+    }
     // line 12: TMU  A2 <- (I - V T V^T)^T A2 = A2 - V W,  W = T^T V^T A2
     FT_TRY(d.inject_at(k, FT_AT_PRE_TMU));
     const bool touched = d.o->n_inject > 0;  // V re-read from memory after hooks

@@ -165,7 +165,8 @@ extern "C" int ft_ctx_create(ft_ctx_t** ctx, int32_t device, abft_stream_t strea
     delete c;
     return ABFT_E_NOMEM;
   }
-  if (cudaHostAlloc((void**)&c->hpin, 16 * sizeof(int32_t), cudaHostAllocDefault) != cudaSuccess ||
+  if (cudaHostAlloc((void**)&c->hpin, 16 * sizeof(int32_t), cudaHostAllocMapped) != cudaSuccess ||
+      cudaHostGetDevicePointer((void**)&c->hpin_dev, c->hpin, 0) != cudaSuccess ||
       cudaEventCreateWithFlags(&c->ev, cudaEventDisableTiming) != cudaSuccess) {
     cudaFree(c->fixlog);
     if (c->hpin) cudaFreeHost(c->hpin);
@@ -249,19 +250,11 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     char* pu_m = pu_c + (size_t)m2 * nb * d.es;
     // restart decision: snapshot the uncorrectable count before a check, read
     // both words back into pinned memory after it (8 bytes, one event)
-    auto post_readback = [&](int32_t* snap) -> int {
-      ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin, snap, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-      ABFT_CUDA_TRY(cudaMemcpyAsync(c->hpin + 1, d.counts + ABFT_CNT_UNCORRECTABLE, sizeof(int32_t),
-                                    cudaMemcpyDeviceToHost, s));
-      ABFT_CUDA_TRY(cudaEventRecord(c->ev, s));
-      return 0;
-    };
+    auto post_readback = [&](int32_t*) -> int { return d.post_delta(0); };
     static const bool dbg_nosync = getenv("ABFT_DBG_RESTART_NOSYNC") != nullptr;
     auto readback_delta = [&](int* delta) -> int {  // uncorrectable errors the check added
       if (dbg_nosync) { *delta = 0; return 0; }
-      ABFT_CUDA_TRY(cudaEventSynchronize(c->ev));
-      *delta = c->hpin[1] - c->hpin[0];
-      return 0;
+      return d.wait_delta(0, delta);
     };
     if (rs) {
       FT_TRY(copy2d(pd_a, nb, d.a_at(r0, r0), lda, nb, nb));
