@@ -24,6 +24,11 @@ global tile's).  Iteration k of Alg. 2 (L368-L378):
      a value corrected there was already consumed by the update, which the
      distributed driver reports as uncorrectable (no distributed repair).
 
+Local restart (f1, L430): the owner of A_kk and the panel owners copy the
+input of their PD / PU with its checksums after the pre-op check; a 2D error
+left by their post-op check (read back on the host: one wait per op) restores
+the copy and redoes the op once, before anything is broadcast.
+
 Only panels, checksums and int32 error reports cross the interconnect;
 torch.distributed is plumbing (NCCL on the GPU box; gloo with CUDA tensors
 when several ranks share one GPU in the tests).  Every arithmetic step is a
@@ -182,10 +187,11 @@ class MgpuStats:
     tmu_consumed: int = 0
     info: int = 0
     uncorrectable: int = 0
+    restarts: int = 0
 
 
 def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0, inject=(), group=None,
-                  tmu_groups=32):
+                  tmu_groups=32, restart=True):
     """Fault-tolerant lower Cholesky of the distributed matrix in place.
     A_loc: this rank's local column-major matrix (from scatter_tiles).
     inject: (iter, point, gi, gj, xor_mask, rank) with global (gi, gj);
@@ -246,6 +252,22 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
             t = tiles_I.index(gi // nb)
             abft.abft_inject(buf.L, t * nb + gi % nb, gj % nb, mask)
 
+    restarts = [0]
+    rs = abft_on and restart
+
+    def snapshot(*ts):
+        return [t.clone() for t in ts] + [rep.counts[abft.NCOUNTS - 1].clone()]
+
+    def added_2d(snap):
+        """2D errors the post-op check added (host read-back, f1)."""
+        return int((rep.counts[abft.NCOUNTS - 1] - snap[-1]).item())
+
+    def restore(snap, *ts):
+        for t, c in zip(ts, snap[:-1]):
+            t.copy_(c)
+        rep.counts[abft.NCOUNTS - 1] = snap[-1]
+        restarts[0] += 1
+
     def sub(m: abft.Mat, il, jl):
         """One local tile as its own 1x1-tile Mat (views into m's arrays)."""
         r0, c0 = il * nb, jl * nb
@@ -276,10 +298,16 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
             hook(k, abft.AT_PRE_PD_CHECK)
             if abft_on:
                 check(D, abft.tiles(0, 1, 0, 1, False, abft.SYM_LOWER), abft.BOTH)
+            if rs:
+                pd_snap = snapshot(D.A, D.colchk, D.colmag)
             hook(k, abft.AT_PRE_PD)
             abft.abft_panel_potrf(D, infos[k:k + 1], Linv)
             hook(k, abft.AT_POST_PD)
             if abft_on:
+                check(D, abft.tiles(0, 1, 0, 1, False, abft.LOWER), abft.COL)
+            if rs and added_2d(pd_snap) > 0:  # local restart of the PD (L430)
+                restore(pd_snap, D.A, D.colchk, D.colmag)
+                abft.abft_panel_potrf(D, infos[k:k + 1], Linv)
                 check(D, abft.tiles(0, 1, 0, 1, False, abft.LOWER), abft.COL)
             diag_buf.L.copy_(D.A)
             if abft_on:
@@ -302,13 +330,24 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
             hook(k, abft.AT_PRE_PU_CHECK)
             if abft_on:
                 check(mat, abft.tiles(ir0, lay.mt_loc, jk, jk + 1), abft.BOTH)
+            pan = (A_loc[r0:, jk * nb:(jk + 1) * nb],) + ((mat.colchk[2 * ir0:, jk * nb:(jk + 1) * nb],
+                                                            mat.colmag[ir0:, jk * nb:(jk + 1) * nb]) if abft_on else ())
+            if rs:
+                pu_snap = snapshot(*pan)
+
+            def pu():
+                abft.abft_update_trsm_inv("R", "T", Linv, pan[0], cnt * nb)
+                if abft_on:
+                    abft.abft_update_trsm_inv("R", "T", Linv, pan[1], 2 * cnt, pan[2], cnt)
+
             hook(k, abft.AT_PRE_PU)
-            abft.abft_update_trsm_inv("R", "T", Linv, A_loc[r0:, jk * nb:(jk + 1) * nb], cnt * nb)
-            if abft_on:
-                abft.abft_update_trsm_inv("R", "T", Linv, mat.colchk[2 * ir0:, jk * nb:(jk + 1) * nb], 2 * cnt,
-                                          mat.colmag[ir0:, jk * nb:(jk + 1) * nb], cnt)
+            pu()
             hook(k, abft.AT_POST_PU)
             if abft_on:
+                check(mat, abft.tiles(ir0, lay.mt_loc, jk, jk + 1), abft.COL)
+            if rs and added_2d(pu_snap) > 0:  # local restart of the PU (L430, L434)
+                restore(pu_snap, *pan)
+                pu()
                 check(mat, abft.tiles(ir0, lay.mt_loc, jk, jk + 1), abft.COL)
         # ---- 4. broadcast the panel pieces (one per process row)
         pieces = []
@@ -386,7 +425,8 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
 
     # ---- error reports: one all-reduce of the int32 counters (L361-L363)
     rep_counts = rep.counts if rep is not None else torch.zeros(abft.NCOUNTS, dtype=torch.int32, device=dev)
-    summary = torch.cat([rep_counts, cb_total, consumed, infos, bflag.reshape(-1)])
+    nrs = torch.tensor([restarts[0]], dtype=torch.int32, device=dev)
+    summary = torch.cat([rep_counts, cb_total, consumed, infos, bflag.reshape(-1), nrs])
     if world > 1:
         dist.all_reduce(summary, op=dist.ReduceOp.SUM, group=group)
     h = summary.cpu().tolist()
@@ -395,7 +435,8 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
     st.bcast_counts = h[8:16]
     st.tmu_consumed = h[16]
     inf = h[17:17 + nt]
-    bf = h[17 + nt:]
+    bf = h[17 + nt:-1]
+    st.restarts = h[-1]
     for kk in range(nt):
         if inf[kk] and not st.info:
             st.info = kk * nb + inf[kk]

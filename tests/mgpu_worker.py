@@ -7,7 +7,7 @@ import sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
 
-def run(rank, world, port, n, nb, grid, inject, out_path, abft_on, seed):
+def run(rank, world, port, n, nb, grid, inject, out_path, abft_on, seed, restart=True):
     import torch
     import torch.distributed as dist
 
@@ -21,12 +21,12 @@ def run(rank, world, port, n, nb, grid, inject, out_path, abft_on, seed):
         lay = mgpu.Layout(n, nb, P, Q, rank)
         A = torch.from_numpy(si.spd(n, seed=seed))
         A_loc = mgpu.scatter_tiles(A, lay)
-        rc, st = mgpu.ft_potrf_mgpu(A_loc, lay, abft_on=abft_on, inject=inject)
+        rc, st = mgpu.ft_potrf_mgpu(A_loc, lay, abft_on=abft_on, inject=inject, restart=restart)
         torch.cuda.synchronize()
         L = mgpu.gather_tiles(A_loc, lay)
         if rank == 0:
             torch.save({"L": torch.tril(L), "rc": rc, "counts": st.counts, "bcast_counts": st.bcast_counts,
                         "bcast_events": st.bcast_events, "tmu_consumed": st.tmu_consumed, "info": st.info,
-                        "uncorrectable": st.uncorrectable}, out_path)
+                        "uncorrectable": st.uncorrectable, "restarts": st.restarts}, out_path)
     finally:
         dist.destroy_process_group()

@@ -28,11 +28,11 @@ def _port():
     return p
 
 
-def _run(tmp_path, n, nb, grid, inject=(), abft_on=True, seed=11):
+def _run(tmp_path, n, nb, grid, inject=(), abft_on=True, seed=11, restart=True):
     world = grid[0] * grid[1]
     out = str(tmp_path / f"mgpu_{grid[0]}x{grid[1]}.pt")
-    mp.spawn(mgpu_worker.run, args=(world, _port(), n, nb, grid, list(inject), out, abft_on, seed), nprocs=world,
-             join=True)
+    mp.spawn(mgpu_worker.run, args=(world, _port(), n, nb, grid, list(inject), out, abft_on, seed, restart),
+             nprocs=world, join=True)
     return torch.load(out)
 
 
@@ -96,4 +96,18 @@ def test_communication_fault_one_receiver(tmp_path, grid):
     assert r["bcast_counts"][5] >= 1  # an element fixed in a received copy
     kinds = [e[4] for e in r["bcast_events"]]
     assert kinds == ["communication"], r["bcast_events"]
+    assert np.abs(r["L"].numpy() - _ref(n)).max() <= 1e-12 * np.abs(_ref(n)).max()
+
+
+@pytest.mark.parametrize("grid", [(1, 1), (2, 2)])
+def test_pd_consumed_fault_local_restart(tmp_path, grid):
+    """A DRAM flip in A_kk between its pre-PD check and the PD is consumed by
+    the PD (2D in L_kk): the owner restores its pre-PD copy and redoes the PD
+    before the broadcast (f1, L430); without the restart it is uncorrectable."""
+    n, nb = 512, 64
+    inj = [(2, abft.AT_PRE_PD, 2 * nb + 40, 2 * nb + 9, BIT)]
+    r0 = _run(tmp_path, n, nb, grid, inject=inj, restart=False)
+    assert r0["rc"] == abft.E_UNCORRECTABLE
+    r = _run(tmp_path, n, nb, grid, inject=inj)
+    assert r["rc"] == 0 and r["restarts"] == 1, r
     assert np.abs(r["L"].numpy() - _ref(n)).max() <= 1e-12 * np.abs(_ref(n)).max()
