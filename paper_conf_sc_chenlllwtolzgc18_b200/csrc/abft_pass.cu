@@ -34,7 +34,7 @@ constexpr int kWarps = kThreads / 32;
 // NB = checksum tile; K = vertically adjacent tiles streamed by one CTA
 // (K > 1 for small tiles: one K*NB-row bulk copy per column and a K-times
 // longer CTA lifetime; GENERAL views only).
-template <typename T, int NB, int K>
+template <typename T, int NB, int K, bool VERIFY = false>
 struct PassCfg {
   static constexpr int RK = K * NB;              // rows per CTA
   static constexpr int GC = NB < 64 ? NB : 64;  // group columns (slab granularity)
@@ -46,8 +46,11 @@ struct PassCfg {
   static constexpr int CC = CC_RAW < GC ? (CC_RAW < 1 ? 1 : CC_RAW) : GC;  // columns per stage
   static constexpr int STAGE_ELEMS = CC * RK;
   static constexpr int STAGE_BYTES = STAGE_ELEMS * (int)sizeof(T);
-  // keep the whole CTA <= ~110 KiB (2 CTAs / SM): ring = budget - side area
-  static constexpr int SIDE_BYTES = RK * 3 * (int)sizeof(T);
+  // keep the whole CTA <= ~110 KiB (2 CTAs / SM): ring = budget - side area.
+  // Side area: SYM column sums / maintained column checksums, and for verify
+  // the recomputed column sums (compared after the stage loop, see below)
+  static constexpr int REC_ELEMS = VERIFY ? RK * 3 : 0;
+  static constexpr int SIDE_BYTES = (RK * 3 + REC_ELEMS) * (int)sizeof(T);
   static constexpr int RING_BYTES = RK >= 256 ? (96 * 1024 < 108 * 1024 - SIDE_BYTES ? 96 * 1024
                                                                                         : 108 * 1024 - SIDE_BYTES)
                                               : 48 * 1024;
@@ -70,7 +73,7 @@ struct PassCfg {
   static constexpr int CQ = CC_BIG_RAW < GC ? (CC_BIG_RAW < 1 ? 1 : CC_BIG_RAW) : GC;
   static_assert(CC % CQ == 0, "row-sum chunk must divide the stage");
   static constexpr size_t SMEM = (size_t)NSTAGE * STAGE_BYTES   // ring
-                                 + (size_t)RK * 3 * sizeof(T)   // SYM sums / maintained column checksums
+                                 + (size_t)(RK * 3 + REC_ELEMS) * sizeof(T)  // side area
                                  + 2 * NSTAGE * sizeof(uint64_t) + 64;  // full / empty barriers
   static_assert(CC >= 1 && GC % CC == 0, "stage must divide group");
   static_assert(NB % 32 == 0, "a tile column must be a multiple of 32 rows");
@@ -169,14 +172,19 @@ __device__ __forceinline__ void super_of(const abft_tiles_t& t, int K, int64_t s
   Ib = t.I0 + (int)(su % nIk) * K;
 }
 
+// Two CTAs per SM need <= 96 registers per thread: 2 x 9 warps spread over
+// the 4 SM sub-partitions put 5 warps on one of them (16K registers each).
+// The verify variant of stacked tiles otherwise takes 111 and runs one CTA
+// per SM (fp32 nb=256 verify at 2.5 TB/s, ncu r01).
 template <typename T, int NB, int K, bool VERIFY>
-__global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
-  using C = PassCfg<T, NB, K>;
+__global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched with kBlock threads
+  using C = PassCfg<T, NB, K, VERIFY>;
   constexpr int RK = C::RK;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   T* ring = reinterpret_cast<T*>(smem_raw);
   T* symacc = ring + (size_t)C::NSTAGE * C::STAGE_ELEMS;  // [K][3][NB]
-  uint64_t* full = reinterpret_cast<uint64_t*>(symacc + 3 * RK);
+  T* rec = symacc + 3 * RK;                               // verify: recomputed [K][3][NB]
+  uint64_t* full = reinterpret_cast<uint64_t*>(rec + C::REC_ELEMS);
   uint64_t* empty = full + C::NSTAGE;
   __shared__ int s_colflags[K], s_ncols[K], s_nrows[K], s_rowflags[K];
   __shared__ int s_last;
@@ -286,22 +294,41 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
       cc2[1] = pw;
       if (colmag) colmag[I + gj * p.ldcm] = pa;
     } else {
+      // verify: park the recomputed sums; the comparisons run after the stage
+      // loop, one column per thread (a per-column compare by one lane inside
+      // the loop serialised the warps: fp32 nb=256 verify 3.9 vs 5.4 TB/s)
+      T* rc = rec + (size_t)t * 3 * NB;
       const int idx = jl - c0;
+      rc[idx] = pe;
+      rc[NB + idx] = pw;
+      rc[2 * NB + idx] = pa;
+    }
+  };
+  // verify: compare the slab's columns (maintained in symacc, recomputed in rec)
+  auto compare_cols = [&]() {
+#pragma unroll
+    for (int t = 0; t < K; ++t) {
+      const int I = Ib + t;
       const T* sa = symacc + (size_t)t * 3 * NB;
-      double m = p.use_mag ? (double)sa[2 * NB + idx] : (double)pa;
-      T de, dw;
-      int f = check_pair<T>(sa[idx], sa[NB + idx], pe, pw, m, p.tau_fac, NB, &de, &dw);
-      if (dcol) {
-        dcol[(int64_t)2 * I + gj * p.ldc] = de;
-        dcol[(int64_t)2 * I + 1 + gj * p.ldc] = dw;
-      }
-      my_colflags[t] |= f;
-      my_ncols[t] += f & 1;
-      if (p.refresh && !(f & 1)) {
-        T* cc2 = colchk + (int64_t)2 * I + gj * p.ldc;
-        cc2[0] = pe;
-        cc2[1] = pw;
-        if (colmag) colmag[I + gj * p.ldcm] = pa;
+      const T* rc = rec + (size_t)t * 3 * NB;
+      for (int idx = tid; idx < cols; idx += kThreads) {
+        const int64_t gj = (int64_t)J * NB + c0 + idx;
+        const T pe = rc[idx], pw = rc[NB + idx], pa = rc[2 * NB + idx];
+        const double m = p.use_mag ? (double)sa[2 * NB + idx] : (double)pa;
+        T de, dw;
+        const int f = check_pair<T>(sa[idx], sa[NB + idx], pe, pw, m, p.tau_fac, NB, &de, &dw);
+        if (dcol) {
+          dcol[(int64_t)2 * I + gj * p.ldc] = de;
+          dcol[(int64_t)2 * I + 1 + gj * p.ldc] = dw;
+        }
+        my_colflags[t] |= f;
+        my_ncols[t] += f & 1;
+        if (p.refresh && !(f & 1)) {
+          T* cc2 = colchk + (int64_t)2 * I + gj * p.ldc;
+          cc2[0] = pe;
+          cc2[1] = pw;
+          if (colmag) colmag[I + gj * p.ldcm] = pa;
+        }
       }
     }
   };
@@ -439,6 +466,10 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
   }
 
   // ---------------- column flags of this CTA ------------------------------
+  if (VERIFY && !sym && (p.which & ABFT_COL)) {
+    consumer_sync();  // every column of the slab is parked in rec
+    compare_cols();
+  }
   if (VERIFY) {
 #pragma unroll
     for (int t = 0; t < K; ++t) {
@@ -591,7 +622,7 @@ __global__ void __launch_bounds__(kBlock) checksum_pass_kernel(PassArgs p) {
 // ------------------------------------------------------------ launcher --
 template <typename T, int NB, int K, bool VERIFY>
 static int launch_k(PassArgs& a, int64_t ntiles, cudaStream_t s) {
-  using C = PassCfg<T, NB, K>;
+  using C = PassCfg<T, NB, K, VERIFY>;
   auto kern = checksum_pass_kernel<T, NB, K, VERIFY>;
   static bool attr_done = false;  // per instantiation
   if (!attr_done) {
