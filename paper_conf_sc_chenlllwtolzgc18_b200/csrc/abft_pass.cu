@@ -23,6 +23,7 @@
 //    last-arriving CTA of a tile (atomic ticket) finishes it and resets the
 //    ticket (no memset launches, no host sync).
 #include <algorithm>
+#include <cstdlib>
 
 #include "abft_common.cuh"
 
@@ -105,6 +106,7 @@ struct PassArgs {
   void* drow;
   int32_t* counts;
   int K;            // tiles per unit (vertical stack), see PassCfg
+  int mode;         // unit decode: PASS_RECT / PASS_SEG / PASS_DIAG (see below)
   void* part;       // [nsuper][GROUPS][K*NB][3] (slabbed units only)
   void* symws;      // [ntiles][3][NB] SYM column sums of slabbed diagonal tiles
   int* ticket;      // [nsuper] self-resetting
@@ -160,9 +162,61 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 // it, so warps never wait for each other inside the stage loop.
 constexpr int kBlock = kThreads + 32;
 
-// Unit decode: K == 1 follows the tile enumeration (lower_only aware); K > 1
-// stacks K consecutive tile rows of one tile column (rectangular ranges only).
-__device__ __forceinline__ void super_of(const abft_tiles_t& t, int K, int64_t su, int& Ib, int& J) {
+// Unit decode.
+//  PASS_RECT: K == 1 follows the tile enumeration (lower_only aware, the
+//    diagonal tiles in diag_view); K > 1 stacks K consecutive tile rows of one
+//    tile column of a rectangular range whose height K divides.
+//  PASS_SEG: the tiles of each tile column that are checked in the GENERAL
+//    view form <= 2 contiguous segments (lower_only clips the top; a diagonal
+//    tile with a masked view is left out and splits the column); each segment
+//    is cut into stacks of K tiles, the last one ragged (kv < K tiles).
+//  PASS_DIAG: only the diagonal tiles of the range, one per unit (K == 1),
+//    in diag_view — the companion launch of a PASS_SEG launch.
+enum { PASS_RECT = 0, PASS_SEG = 1, PASS_DIAG = 2 };
+
+__host__ __device__ __forceinline__ int64_t seg_units(int len, int K) { return len > 0 ? (len + K - 1) / K : 0; }
+
+// returns the number of units when u is past the end (host: count with u = -1)
+__host__ __device__ inline int64_t seg_of(const abft_tiles_t& t, int K, int64_t u, int& Ib, int& J, int& kv) {
+  const bool split = t.diag_view != ABFT_GENERAL;
+  int64_t seen = 0;
+  for (int Jc = t.J0; Jc < t.J1; ++Jc) {
+    const int lo = t.lower_only ? (t.I0 > Jc ? t.I0 : Jc) : t.I0;
+    int a1 = t.I1, b0 = 0, b1 = 0;
+    if (split && Jc >= lo && Jc < t.I1) {
+      a1 = Jc;
+      b0 = Jc + 1;
+      b1 = t.I1;
+    }
+    const int64_t ua = seg_units(a1 - lo, K), ub = seg_units(b1 - b0, K);
+    if (u >= seen && u < seen + ua) {
+      J = Jc;
+      Ib = lo + (int)(u - seen) * K;
+      kv = a1 - Ib < K ? a1 - Ib : K;
+      return -1;
+    }
+    if (u >= seen + ua && u < seen + ua + ub) {
+      J = Jc;
+      Ib = b0 + (int)(u - seen - ua) * K;
+      kv = b1 - Ib < K ? b1 - Ib : K;
+      return -1;
+    }
+    seen += ua + ub;
+  }
+  return seen;
+}
+
+__device__ __forceinline__ void super_of(const abft_tiles_t& t, int mode, int K, int64_t su, int& Ib, int& J,
+                                         int& kv) {
+  kv = K;
+  if (mode == PASS_SEG) {
+    seg_of(t, K, su, Ib, J, kv);
+    return;
+  }
+  if (mode == PASS_DIAG) {
+    Ib = J = (t.I0 > t.J0 ? t.I0 : t.J0) + (int)su;
+    return;
+  }
   if (K == 1) {
     tile_of(t, su, Ib, J);
     return;
@@ -194,9 +248,10 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
   const int64_t unit = blockIdx.x;
   const int64_t sup = unit / p.nslab;
   const int slab = (int)(unit % p.nslab);
-  int Ib, J;
-  super_of(p.tiles, K, sup, Ib, J);
-  const int view = (K == 1 && Ib == J) ? p.tiles.diag_view : ABFT_GENERAL;
+  int Ib, J, kv;
+  super_of(p.tiles, p.mode, K, sup, Ib, J, kv);
+  const int RV = K == 1 ? NB : kv * NB;  // valid rows of this unit (ragged PASS_SEG stacks: kv < K)
+  const int view = (K == 1 && Ib == J && p.mode != PASS_SEG) ? p.tiles.diag_view : ABFT_GENERAL;
   const bool sym = view == ABFT_SYM_LOWER;
   const int nslab = p.nslab;
   // SYM column sums of a split tile go through the workspace (the finishing
@@ -235,11 +290,11 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
         if (g >= C::NSTAGE) mbar_wait(&empty[slot], (uint32_t)(((g / C::NSTAGE) - 1) & 1));
         T* dst = ring + (size_t)slot * C::STAGE_ELEMS;
         fence_proxy_async();
-        mbar_arrive_expect_tx(&full[slot], C::STAGE_BYTES);
+        mbar_arrive_expect_tx(&full[slot], (uint32_t)(C::CC * RV * sizeof(T)));
         const T* src = tileA + (int64_t)(c0 + g * C::CC) * p.lda;
 #pragma unroll 1
         for (int cc = 0; cc < C::CC; ++cc)
-          bulk_g2s(dst + cc * RK, src + (int64_t)cc * p.lda, RK * sizeof(T), &full[slot]);
+          bulk_g2s(dst + cc * RK, src + (int64_t)cc * p.lda, RV * sizeof(T), &full[slot]);
       }
     }
     return;
@@ -267,7 +322,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
   // strided load per column inside the stage loop.  For non-SYM tiles the
   // SYM area is free and holds them: per tile [e | w | mag] x cols.
   if (VERIFY && !sym && (p.which & ABFT_COL)) {
-    for (int idx = tid; idx < K * cols; idx += kThreads) {
+    for (int idx = tid; idx < kv * cols; idx += kThreads) {
       const int t = idx / cols, c = idx - t * cols;
       const int64_t gj = (int64_t)J * NB + c0 + c;
       T* sa = symacc + (size_t)t * 3 * NB;
@@ -308,6 +363,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
   auto compare_cols = [&]() {
 #pragma unroll
     for (int t = 0; t < K; ++t) {
+      if (t >= kv) break;
       const int I = Ib + t;
       const T* sa = symacc + (size_t)t * 3 * NB;
       const T* rc = rec + (size_t)t * 3 * NB;
@@ -343,7 +399,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
       const T* src = tileA + (int64_t)(c0 + s * C::CC) * p.lda;
       for (int idx = tid; idx < C::STAGE_ELEMS; idx += kThreads) {
         int cc = idx / RK, r = idx % RK;
-        buf[idx] = src[(int64_t)cc * p.lda + r];
+        if (r < RV) buf[idx] = src[(int64_t)cc * p.lda + r];
       }
       consumer_sync();
     }
@@ -365,7 +421,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
           (void)dummy;
           const int t = k / C::KPT;
           const int kl = k - t * C::KPT;
-          T xv[C::VEC];
+          T xv[C::VEC];  // rows of a ragged stack's missing tiles (t >= kv) are stale smem, never finished
           load_vec<T, C::VEC>(xv, col + (32 * k + lane) * C::VEC);
 #pragma unroll
           for (int v = 0; v < C::VEC; ++v) {
@@ -383,7 +439,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
             w = fadd(w, shfl_xor(w, m));
             a2 = fadd(a2, shfl_xor(a2, m));
           }
-          if (lane == t) finish_col(t, jl, e, w, a2);  // tiles finished by different lanes in parallel
+          if (lane == t && t < kv) finish_col(t, jl, e, w, a2);  // tiles finished by different lanes in parallel
         }
       } else {  // masked diagonal views (K == 1 only)
         T pe = T(0), pw = T(0), pa = T(0);
@@ -408,7 +464,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
 #pragma unroll
     for (int q = 0; q < C::RPT; ++q) {
       const int r = tid + q * kThreads;
-      if (r < RK) {
+      if (r < RV) {
         if (view == ABFT_GENERAL) {
           // per CQ-column chunk: sum (jl+1) x with jl = base + cq  =  (base + 1) * S0 + sum_cq cq*x
 #pragma unroll
@@ -448,7 +504,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
 #pragma unroll
       for (int q = 0; q < C::RPT; ++q) {
         const int r = tid + q * kThreads;
-        if (r < RK) {
+        if (r < RV) {
           if (nslab == 1) {
             tot[q].e = fadd(tot[q].e, grp[q].e);
             tot[q].w = fadd(tot[q].w, grp[q].w);
@@ -502,7 +558,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
 #pragma unroll
     for (int q = 0; q < C::RPT; ++q) {
       const int r = tid + q * kThreads;
-      if (r < RK) {
+      if (r < RV) {
         for (int g = 0; g < C::GROUPS; ++g) {
           const T* src = partT + (((size_t)sup * C::GROUPS + g) * RK + r) * 3;
           tot[q].e = fadd(tot[q].e, __ldcg(src + 0));
@@ -535,7 +591,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
 #pragma unroll
   for (int q = 0; q < C::RPT; ++q) {
     const int rr = tid + q * kThreads;
-    if (rr >= RK) continue;
+    if (rr >= RV) continue;
     const int t = rr / NB, r = rr - t * NB;
     const int I = Ib + t;
     T re = tot[q].e, rw = tot[q].w, ra = tot[q].a;
@@ -607,7 +663,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
   }
   if (!VERIFY) return;
   consumer_sync();
-  if (tid < K) {
+  if (tid < kv) {
     const int t = tid, I = Ib + t;
     const int cf = s_colflags[t], rf = s_rowflags[t];
     const int st = ((cf & 1) ? ABFT_ST_COL : 0) | ((rf & 1) ? ABFT_ST_ROW : 0) | (((cf | rf) & 2) ? ABFT_ST_NONFINITE : 0);
@@ -621,7 +677,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
 
 // ------------------------------------------------------------ launcher --
 template <typename T, int NB, int K, bool VERIFY>
-static int launch_k(PassArgs& a, int64_t ntiles, cudaStream_t s) {
+static int launch_k(PassArgs& a, int64_t nsup, cudaStream_t s) {
   using C = PassCfg<T, NB, K, VERIFY>;
   auto kern = checksum_pass_kernel<T, NB, K, VERIFY>;
   static bool attr_done = false;  // per instantiation
@@ -635,11 +691,13 @@ static int launch_k(PassArgs& a, int64_t ntiles, cudaStream_t s) {
     cudaGetDevice(&dev);
     if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms <= 0) sms = 148;
   }
-  const int64_t nsup = ntiles / K;
+  const int64_t ntiles = nsup * K;  // tile slots of the workspace (ragged stacks included)
   // slabs: aim for >= 2 CTAs per SM when the unit count is small
   int nslab = 1;
   const int max_slab = C::GROUPS;
   while (nslab < max_slab && nsup * nslab < 2LL * sms) nslab *= 2;
+  static const int force_slab = getenv("ABFT_NSLAB") ? atoi(getenv("ABFT_NSLAB")) : 0;  // tuning experiments only
+  if (force_slab > 0) nslab = std::min(force_slab, max_slab);
   a.nslab = nslab;
   a.K = K;
   if (nslab > 1) {
@@ -661,24 +719,33 @@ static int launch_k(PassArgs& a, int64_t ntiles, cudaStream_t s) {
   return 0;
 }
 
-// Small tiles are streamed K at a time (K*NB*s >= 4 KiB per column copy)
-// when the range is rectangular, GENERAL everywhere and divisible by K.
+// Small tiles are streamed K at a time (K*NB*s >= 4 KiB per column copy):
+// a rectangular GENERAL range whose height K divides in one PASS_RECT
+// launch; any other range (lower_only, ragged height, masked diagonal view)
+// as PASS_SEG stacks of its GENERAL tiles plus, when the diagonal view is
+// masked, one PASS_DIAG launch over the diagonal tiles.
 template <typename T, int NB, bool VERIFY>
 static int launch_nb(PassArgs& a, int64_t ntiles, cudaStream_t s) {
   constexpr int KR = 4096 / (NB * (int)sizeof(T));
   constexpr int KBIG = KR < 1 ? 1 : (KR > 8 ? 8 : KR);
   constexpr int VEC = NB >= 32 * (16 / (int)sizeof(T)) ? 16 / (int)sizeof(T) : 1;
   constexpr bool can = KBIG > 1 && NB % (32 * VEC) == 0;
+  a.mode = PASS_RECT;
   if constexpr (can) {
     const abft_tiles_t& t = a.tiles;
-    const bool touches_diag = t.I0 < t.J1 && t.J0 < t.I1;
-    const bool general = !t.lower_only && (t.diag_view == ABFT_GENERAL || !touches_diag);
-    if (general) {
-      int K = KBIG;
-      while (K > 1 && (t.I1 - t.I0) % K) K /= 2;
-      if (K == KBIG) return launch_k<T, NB, KBIG, VERIFY>(a, ntiles, s);
-      if (K >= 2 && KBIG >= 4 && K == KBIG / 2) return launch_k<T, NB, (KBIG >= 4 ? KBIG / 2 : 1), VERIFY>(a, ntiles, s);
+    const int D0 = std::max(t.I0, t.J0), D1 = std::min(t.I1, t.J1);
+    const bool split = t.diag_view != ABFT_GENERAL && D1 > D0;
+    if (!t.lower_only && !split && (t.I1 - t.I0) % KBIG == 0) return launch_k<T, NB, KBIG, VERIFY>(a, ntiles / KBIG, s);
+    if (split) {
+      a.mode = PASS_DIAG;
+      const int rc = launch_k<T, NB, 1, VERIFY>(a, D1 - D0, s);
+      if (rc) return rc;
     }
+    int Ib, J, kv;
+    const int64_t nseg = seg_of(t, KBIG, -1, Ib, J, kv);
+    if (nseg == 0) return 0;
+    a.mode = PASS_SEG;
+    return launch_k<T, NB, KBIG, VERIFY>(a, nseg, s);
   }
   return launch_k<T, NB, 1, VERIFY>(a, ntiles, s);
 }

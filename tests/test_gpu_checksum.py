@@ -290,3 +290,93 @@ def test_full_size_sampled_tiles(lib, prec):
         rg = host(mat.rowchk[I * nb:(I + 1) * nb, 2 * J:2 * J + 2])
         assert normwise_err(cg, c, X, 0) <= TOL[prec]
         assert normwise_err(rg, r, X, 1) <= TOL[prec]
+
+
+# Ranges the launcher cuts into ragged stacks of K tiles (PASS_SEG) plus a
+# diagonal-only launch when the diagonal view is masked (PASS_DIAG): lower-only
+# triangles, offset sub-ranges, heights K does not divide, masked diagonals
+# that split a tile column in two.  (I0, I1, J0, J1, lower_only, view) with
+# I1/J1 = None for nt.
+SEG_RANGES = [(0, None, 0, None, True, ck.SYM_LOWER), (0, None, 0, None, True, ck.GENERAL),
+              (2, None, 1, -2, True, ck.LOWER), (1, -1, 0, 3, False, ck.GENERAL),
+              (0, None, 0, None, False, ck.UNIT_LOWER), (3, None, 0, None, False, ck.UPPER)]
+
+
+def _seg_case(nb):
+    nt = 19 if nb <= 64 else (11 if nb == 128 else 7)
+    return nt, nt * nb
+
+
+def _rng(r, nt):
+    I0, I1, J0, J1, lower, view = r
+    fix = lambda v: nt if v is None else (nt + v if v < 0 else v)  # noqa: E731
+    return fix(I0), fix(I1), fix(J0), fix(J1), lower, view
+
+
+@pytest.mark.parametrize("prec,nb", [("f64", 32), ("f64", 64), ("f64", 128), ("f64", 256), ("f32", 32),
+                                     ("f32", 128), ("f32", 256), ("f32", 512)])
+@pytest.mark.parametrize("ri", range(len(SEG_RANGES)))
+def test_encode_segmented_ranges_bit_exact(lib, prec, nb, ri):
+    nt, n = _seg_case(nb)
+    I0, I1, J0, J1, lower, view = _rng(SEG_RANGES[ri], nt)
+    A = si.integers(n, seed=nb + ri, R=8 if prec == "f32" else 1000)
+    if view == ck.SYM_LOWER:
+        A = A + A.T
+    mat = lib.Mat.alloc(dev(A, TDT[prec]), nb)
+    lib.abft_encode(mat, lib.tiles(I0, I1, J0, J1, lower, view))
+    torch.cuda.synchronize()
+    st = ck.State.alloc(A.astype(np.float64), nb, prec=prec)
+    tt = ck.Tiles(I0, I1, J0, J1, lower, view)
+    ck.encode(st, tt)
+    g = gpu_state_to_oracle(mat, prec)
+    seen = set(tt)
+    assert seen
+    for I in range(nt):
+        for J in range(nt):
+            cs, rs = slice(J * nb, (J + 1) * nb), slice(I * nb, (I + 1) * nb)
+            if (I, J) in seen:  # exact sums of integers: every order gives the same bits
+                assert np.array_equal(g.colchk[2 * I:2 * I + 2, cs], st.colchk[2 * I:2 * I + 2, cs]), (I, J)
+                assert np.array_equal(g.rowchk[rs, 2 * J:2 * J + 2], st.rowchk[rs, 2 * J:2 * J + 2]), (I, J)
+                assert np.array_equal(g.colmag[I, cs], st.colmag[I, cs]), (I, J)
+                assert np.array_equal(g.rowmag[rs, J], st.rowmag[rs, J]), (I, J)
+            else:  # tiles outside the range are not written
+                assert not g.colchk[2 * I:2 * I + 2, cs].any() and not g.rowchk[rs, 2 * J:2 * J + 2].any(), (I, J)
+
+
+@pytest.mark.parametrize("prec,nb", [("f64", 32), ("f64", 256), ("f32", 64), ("f32", 512)])
+def test_verify_segmented_after_rect_encode_is_exactly_zero(lib, prec, nb):
+    """c-27 pin across launch shapes: checksums written by a full rectangular
+    encode (PASS_RECT stacks) are recomputed bit-identically by the ragged
+    PASS_SEG stacks of lower-only / offset / ragged-height verifies."""
+    nt, n = _seg_case(nb)
+    A = si.general(n, seed=nb)
+    mat, _ = _encode(lib, A, nb, prec)
+    rep = lib.Report.alloc(mat, deltas=True)
+    tol = lib.abft_tol_t(ck.TOL_MAGNITUDE, 1.0)
+    for r in SEG_RANGES[1:4]:
+        I0, I1, J0, J1, lower, _ = _rng(r, nt)
+        lib.abft_verify(mat, lib.tiles(I0, I1, J0, J1, lower, ck.GENERAL), ck.BOTH, tol, rep)
+    torch.cuda.synchronize()
+    assert torch.count_nonzero(rep.dcol) == 0 and torch.count_nonzero(rep.drow) == 0
+    assert torch.count_nonzero(rep.status) == 0 and torch.count_nonzero(rep.counts) == 0
+
+
+@pytest.mark.parametrize("prec,nb", [("f64", 64), ("f32", 256)])
+def test_verify_segmented_flags_every_tile(lib, prec, nb):
+    """One MUST-band corruption in every tile of a lower-only SYM range: the
+    ragged stacks and the diagonal launch flag exactly those tiles."""
+    nt, n = _seg_case(nb)
+    A = si.spd(n, seed=9)
+    mat, t = _encode(lib, A, nb, prec, view=ck.SYM_LOWER, lower_only=True)
+    for I in range(nt):
+        for J in range(I + 1):
+            i, j = (I * nb + 5, J * nb + 3)
+            mat.A[i, j] += 1e3
+    rep = lib.Report.alloc(mat)
+    lib.abft_verify(mat, t, ck.BOTH, lib.abft_tol_t(ck.TOL_MAGNITUDE, 1.0), rep)
+    torch.cuda.synchronize()
+    s = host(rep.status)
+    for I in range(nt):
+        for J in range(nt):
+            assert (s[I, J] != 0) == (I >= J), (I, J, s[I, J])
+    assert int(rep.counts[0].item()) == nt * (nt + 1) // 2
