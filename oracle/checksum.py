@@ -505,20 +505,6 @@ def classify_fix_round(st, tc, which, tol, fixes):
     if not Fc and not Fr:
         return CLS_CLEAN
     sym = tc.view == SYM_LOWER
-    # step 2 — a lone e- or w-entry: the checksum itself is corrupt
-    repaired = False
-    if has_c and Fc and (not has_r or not Fr):
-        for j in Fc:
-            if bool(tc.fce[j]) != bool(tc.fcw[j]):
-                _reencode_col(st, tc, j, CLS_CHK_CORRUPT, fixes)
-                repaired = True
-    if has_r and Fr and (not has_c or not Fc):
-        for i in Fr:
-            if bool(tc.fre[i]) != bool(tc.frw[i]):
-                _reencode_row(st, tc, i, CLS_CHK_CORRUPT, fixes)
-                repaired = True
-    if repaired:
-        return CLS_CHK_CORRUPT
     # step 3 — all flagged columns locate the same row i (0D / 1D_ROW)
     loc_c = {}
     if has_c and Fc:
@@ -542,6 +528,24 @@ def classify_fix_round(st, tc, which, tol, fixes):
                 for i in Fr:
                     _fix_via_row(st, tc, i, j, cls, fixes)
                 return cls
+    # step 2 — a lone e- or w-entry that no consistent data location explains
+    # (steps 3 and 4 failed): the checksum entry itself is corrupt.  After
+    # steps 3-4 (reading c-11b): a data error in local column j changes
+    # delta_w by j*delta_e, so for small j it can pass tau_w = nb*tau_e while
+    # delta_e fails tau_e; re-encoding then absorbed a locatable data error.
+    repaired = False
+    if has_c and Fc and (not has_r or not Fr):
+        for j in Fc:
+            if bool(tc.fce[j]) != bool(tc.fcw[j]):
+                _reencode_col(st, tc, j, CLS_CHK_CORRUPT, fixes)
+                repaired = True
+    if has_r and Fr and (not has_c or not Fc):
+        for i in Fr:
+            if bool(tc.fre[i]) != bool(tc.frw[i]):
+                _reencode_row(st, tc, i, CLS_CHK_CORRUPT, fixes)
+                repaired = True
+    if repaired:
+        return CLS_CHK_CORRUPT
     if sym and has_c:
         # step 5 — SYM_LOWER mirrored pair: one stored element seen twice
         if len(Fc) == 2:

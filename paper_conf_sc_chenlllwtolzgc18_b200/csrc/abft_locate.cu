@@ -6,7 +6,7 @@
 // (L330-L334); "same row => 1D, otherwise 2D" (L432-L434, §VII.D).
 // Readings: c-4 correction x <- c_e - sum_{r!=i} X[r][j];
 // c-5 acceptance of the rounded ratio; c-7 non-finite fallback with
-// confirmation; c-11 class order CHK_CORRUPT -> 0D/1D_ROW -> 0D/1D_COL ->
+// confirmation; c-11 class order 0D/1D_ROW -> 0D/1D_COL -> CHK_CORRUPT (c-11b) ->
 // SYM pair -> SYM_CROSS -> STALE -> 2D, at most 3 rounds.
 //
 // This is the rare path (only tiles whose verify status is non-zero do any
@@ -357,28 +357,6 @@ __global__ void __launch_bounds__(kLThreads) locate_correct_kernel(LocArgs p) {
           if (na < kMaxActions) acts[na++] = Action{(short)kind, (short)c, i, j};
         };
         bool decided = false;
-        // step 2: lone e- or w-flag => the checksum entry itself is corrupt
-        bool rep = false;
-        if (has_c && nfc && (!has_r || !nfr))
-          for (int j = 0; j < nb; ++j) {
-            unsigned f = D[0].fl[j];
-            if ((f & 3) && ((f & 1) != 0) != ((f & 2) != 0)) {
-              push(ACT_REENC_COL, -1, j, ABFT_CLS_CHK_CORRUPT);
-              rep = true;
-            }
-          }
-        if (has_r && nfr && (!has_c || !nfc))
-          for (int i = 0; i < nb; ++i) {
-            unsigned f = D[1].fl[i];
-            if ((f & 3) && ((f & 1) != 0) != ((f & 2) != 0)) {
-              push(ACT_REENC_ROW, i, -1, ABFT_CLS_CHK_CORRUPT);
-              rep = true;
-            }
-          }
-        if (rep) {
-          cls = ABFT_CLS_CHK_CORRUPT;
-          decided = true;
-        }
         // step 3: columns locate one row
         if (!decided && has_c && nfc) {
           int i0 = -2;
@@ -418,6 +396,29 @@ __global__ void __launch_bounds__(kLThreads) locate_correct_kernel(LocArgs p) {
               if (D[1].fl[i] & 3) push(ACT_FIX_ROW, i, j0, cls);
             decided = true;
           }
+        }
+        // step 2 (after steps 3-4, reading c-11b): a lone e- or w-flag that no
+        // consistent data location explains => the checksum entry is corrupt
+        bool rep = false;
+        if (!decided && has_c && nfc && (!has_r || !nfr))
+          for (int j = 0; j < nb; ++j) {
+            unsigned f = D[0].fl[j];
+            if ((f & 3) && ((f & 1) != 0) != ((f & 2) != 0)) {
+              push(ACT_REENC_COL, -1, j, ABFT_CLS_CHK_CORRUPT);
+              rep = true;
+            }
+          }
+        if (!decided && has_r && nfr && (!has_c || !nfc))
+          for (int i = 0; i < nb; ++i) {
+            unsigned f = D[1].fl[i];
+            if ((f & 3) && ((f & 1) != 0) != ((f & 2) != 0)) {
+              push(ACT_REENC_ROW, i, -1, ABFT_CLS_CHK_CORRUPT);
+              rep = true;
+            }
+          }
+        if (rep) {
+          cls = ABFT_CLS_CHK_CORRUPT;
+          decided = true;
         }
         if (!decided && sym && has_c) {
           // step 5: mirrored pair

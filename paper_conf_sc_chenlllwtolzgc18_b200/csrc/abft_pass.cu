@@ -692,10 +692,12 @@ static int launch_k(PassArgs& a, int64_t nsup, cudaStream_t s) {
     if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms <= 0) sms = 148;
   }
   const int64_t ntiles = nsup * K;  // tile slots of the workspace (ragged stacks included)
-  // slabs: aim for >= 2 CTAs per SM when the unit count is small
+  // slabs: split the units of a small launch so that it fills, but does not
+  // spill past, one wave of 2 CTAs per SM (a spilled second wave cost more
+  // than the halved slab saved: 40-59-tile panels 10% slower, slab_tune r01)
   int nslab = 1;
   const int max_slab = C::GROUPS;
-  while (nslab < max_slab && nsup * nslab < 2LL * sms) nslab *= 2;
+  while (nslab < max_slab && nsup * nslab * 2 <= 2LL * sms) nslab *= 2;
   static const int force_slab = getenv("ABFT_NSLAB") ? atoi(getenv("ABFT_NSLAB")) : 0;  // tuning experiments only
   if (force_slab > 0) nslab = std::min(force_slab, max_slab);
   a.nslab = nslab;

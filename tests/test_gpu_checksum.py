@@ -189,7 +189,7 @@ def test_locate_0d_every_tile_config1(lib):
 
 
 @pytest.mark.parametrize("case", ["1d_row", "1d_col", "chk_e", "chk_w", "stale_r", "stale_c", "2d", "inf", "nan",
-                                  "huge"])
+                                  "huge", "absorbed_col"])
 def test_locate_classes_match_oracle(lib, case):
     A = si.general(128, seed=30)
     nb = 64
@@ -226,6 +226,15 @@ def test_locate_classes_match_oracle(lib, case):
             _set(st, mat, 33, 40, np.nan)
         elif case == "huge":
             _set(st, mat, 33, 40, 1e308)
+        elif case == "absorbed_col":  # c-11b: e-only row flags that locate column 0 are data errors
+            d = np.where(np.arange(64) % 2 == 0, 1e-12, 0.5) * (1 + np.arange(64) / 64)
+            for i in range(64):
+                _set(st, mat, 64 + i, 64, A[64 + i, 64] + d[i])
+            x = st.A[64:128, 64]
+            ce, cw, cm = x.sum(), (np.arange(1, 65) * x).sum(), np.abs(x).sum()
+            st.colchk[2:4, 64] = [ce, cw]
+            st.colmag[1, 64] = cm
+            mat.colchk[2, 64], mat.colchk[3, 64], mat.colmag[1, 64] = float(ce), float(cw), float(cm)
 
     _compare_locate(lib, A, nb, mutate)
 

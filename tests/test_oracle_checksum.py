@@ -234,6 +234,37 @@ def test_checksum_corrupt_entry_repaired(w):
     assert ck.verify(st, ck.Tiles(0, 2, 0, 2))[1][0] == 0
 
 
+def _absorbed_column_damage(seed):
+    """A column of data errors that the column checksums absorbed (the TMU's
+    c-rule ran on the corrupted operand): tile (1, 1), local column 0
+    (weight 1), half of the rows off by 1e-12 (above tau_e ~ 1e-13 of this
+    U(-1,1) nb=32 tile but below tau_w = nb tau_e: delta_w = 1 * delta_e
+    flags e only), the other half by 0.5 (both flagged)."""
+    A = si.general(64, seed=seed)
+    st = _state(A, 32)
+    d = np.where(np.arange(32) % 2 == 0, 1e-12, 0.5) * (1 + np.arange(32) / 32)
+    st.A[32:64, 32] += d
+    X = st.A[32:64, 32:64]
+    st.colchk[2:4, 32] = [X[:, 0].sum(), (np.arange(1, 33) * X[:, 0]).sum()]  # absorbed
+    st.colmag[1, 32] = np.abs(X[:, 0]).sum()
+    return A, st, d
+
+
+def test_e_only_row_flags_that_locate_are_data_errors():
+    """Reading c-11b: rows flagged by e only whose ratio locates local column
+    0 are data errors (1D_COL through the rows), not corrupt row checksums;
+    by construction the original matrix comes back and no checksum entry is
+    declared corrupt."""
+    A, st, d = _absorbed_column_damage(16)
+    status, fixes, counts = _fix_all(st)
+    assert counts[3] == 0
+    cls = {f.cls for f in fixes}
+    assert ck.CLS_CHK_CORRUPT not in cls and ck.CLS_1D_COL in cls, cls
+    assert sum(f.cls == ck.CLS_1D_COL for f in fixes) == 32
+    assert np.abs(st.A - A).max() <= 1e-14 and np.abs(st.A - A).max() < d.min() / 10
+    assert ck.verify(st, ck.Tiles(0, 2, 0, 2))[1][0] == 0
+
+
 def test_stale_row_checksum():
     # data consistent with c, r disagrees in two rows → STALE_R (reading c-11 5b)
     A = si.general(64, seed=14)

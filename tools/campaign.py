@@ -19,8 +19,12 @@ error, not by equality with the fault-free factor: a corrected element is
 exact only to its checksum's rounding (reading c-4, <= tau), and LU / QR
 amplify such a perturbation in the forward factors (pivot growth) while the
 factorization stays backward stable.  Y: rc == 0 and ||A - factors||_F /
-||A||_F <= 4x the fault-free run's; the forward deviation from the
-fault-free factor is reported beside it (rel_err).
+||A||_F <= 4x the fault-free run's; Yr ("rounding residue"): above that but
+within LAPACK's own acceptance test for a factorization, ratio
+||A - factors|| / (||A|| n u) <= 30 (the threshold of LAPACK's xCHKPO /
+xCHKGE / xCHKQR test drivers) — many corrections, each exact only to tau,
+add up; N: beyond.  The forward deviation from the fault-free factor is
+reported beside it (rel_err).
 Writes gpurun_out/campaign.json (or the path in $CAMPAIGN_OUT).
 
   python tools/campaign.py [trials_per_driver] [n] [nb] [K,K,..] [kind,kind,..]
@@ -135,7 +139,7 @@ def main():
         _, _, ref = run(())
         scale = ref.abs().max().item()
         res_free = resid(ref)
-        out = {"K": K, "backward_err_fault_free": res_free, "Y": 0, "R": 0, "N": 0, "detected": 0, "restarts": 0, "graded_pass": 0, "cases": []}
+        out = {"K": K, "backward_err_fault_free": res_free, "Y": 0, "Yr": 0, "R": 0, "N": 0, "detected": 0, "restarts": 0, "graded_pass": 0, "cases": []}
         for t in range(trials):
             ks = sorted(int(x) for x in g.choice(n // nb - 1, size=K, replace=False))
             plans = [plan(kind, n, nb, g, k) for k in ks]
@@ -150,13 +154,15 @@ def main():
                 o = "R"
             elif bwd <= 4 * res_free:
                 o = "Y"
+            elif bwd <= 30 * n * 2.0 ** -53:
+                o = "Yr"
             else:
                 o = "N"
             out[o] += 1
             out["detected"] += int(det)
             out["restarts"] += int(st.restarts > 0)
             tmu_ref = any(i[1] == AT["PRE_TMU"] for i in inj)
-            out["graded_pass"] += int(o == "Y" or (o == "R" and tmu_ref))
+            out["graded_pass"] += int(o in ("Y", "Yr") or (o == "R" and tmu_ref))
             out["cases"].append({"inject": [list(i[:6]) for i in inj], "bit": bit, "outcome": o, "rel_err": err,
                                  "backward_err": bwd,
                                  "tmu_ref": tmu_ref,
