@@ -362,12 +362,12 @@ def potrf_overhead(abft, si, n, nb, reps, host_pd=True):
     A = torch.empty_like(A0.t()).t()
     ctx = abft.Context()
 
-    def run(ft, restart=True, pd=abft.PD_DEVICE):
+    def run(ft, restart=True, pd=abft.PD_DEVICE, scheme=abft.SCHEME_NEW):
         A.copy_(A0)
         torch.cuda.synchronize()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record()
-        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart, pd_location=pd)
+        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart, pd_location=pd, scheme=scheme)
         b.record()
         torch.cuda.synchronize()
         assert rc == 0 and info == 0
@@ -387,6 +387,16 @@ def potrf_overhead(abft, si, n, nb, reps, host_pd=True):
     t_nors.sort()
     ft_ms, plain_ms = t_ft[len(t_ft) // 2], t_plain[len(t_plain) // 2]
     nors_ms = t_nors[len(t_nors) // 2]
+    # the checking schemes the paper compares (L542, L653 Figs. 12-14; c-34),
+    # same driver, same plain baseline, no restart (so that every scheme is
+    # timed alike: SINGLE_PRE has no post-op check to restart from)
+    schemes = {}
+    for name, sc in (("new", abft.SCHEME_NEW), ("full_post", abft.SCHEME_FULL_POST),
+                     ("single_post", abft.SCHEME_SINGLE_POST), ("single_pre", abft.SCHEME_SINGLE_PRE)):
+        run(True, restart=False, scheme=sc)
+        ts = sorted(run(True, restart=False, scheme=sc)[0] for _ in range(max(1, reps - 1)))
+        tm = ts[len(ts) // 2]
+        schemes[name] = {"ms_ft": tm, "overhead_pct": 100.0 * (tm - plain_ms) / plain_ms}
     host = None
     if host_pd:  # Alg. 2 lines 3-7 with the PD on the host (FT_PD_HOST)
         import os
@@ -413,7 +423,8 @@ def potrf_overhead(abft, si, n, nb, reps, host_pd=True):
     return {"n": n, "nb": nb, "ms_ft": ft_ms, "ms_plain": plain_ms,
             "overhead_pct": 100.0 * (ft_ms - plain_ms) / plain_ms, "cusolver_potrf_ms": cus,
             "ms_ft_no_restart": nors_ms, "overhead_pct_no_restart": 100.0 * (nors_ms - plain_ms) / plain_ms,
-            "tflops_ft": n ** 3 / 3 / (ft_ms / 1e3) / 1e12, "reps": reps, "host_pd": host}
+            "tflops_ft": n ** 3 / 3 / (ft_ms / 1e3) / 1e12, "reps": reps, "host_pd": host,
+            "schemes_no_restart": schemes}
 
 
 def mgpu_overhead(si, n, nb, reps, world, rank):

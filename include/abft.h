@@ -290,7 +290,9 @@ ABFT_API int abft_update_trsm_inv(int32_t dtype, char side, char trans, int64_t 
  *   r(A_IJ) -= P[2J.., cols of I]^T        for I >= J  (Rr: rowchk block, ldr)
  * and, when mL != NULL, with Q = m_c(L21) |L21|^T: Cm += Q (lower tiles),
  * Rm += Q^T (c-6).  L21: ntk*nb x nb (ldl); cL: 2ntk x nb panel column
- * checksums (ld ldc, the colchk leading dimension); mL: ntk x nb (ldcm). */
+ * checksums (ld ldc, the colchk leading dimension); mL: ntk x nb (ldcm).
+ * Rr == NULL (with Rm == NULL): column rule only (the single-side checking
+ * schemes of ft_opts_t.scheme). */
 ABFT_API int abft_update_syrk(int32_t dtype, int64_t nb, int64_t ntk, const void *L21, int64_t ldl,
                               const void *cL, int64_t ldc, const void *mL, int64_t ldcm, void *Cc,
                               void *Rr, int64_t ldr, void *Cm, void *Rm, int64_t ldrm, abft_stream_t stream);
@@ -359,7 +361,21 @@ typedef struct {
   int32_t trailing_check_period; /* P > 0: check the whole trailing matrix after the TMU of every P-th
                             iteration (L359: "periodically check the correctness of trailing matrix
                             ... to avoid 2D propagation"); 0 (default): never */
+  int32_t scheme;        /* FT_SCHEME_* (ft_potrf only; ft_getrf / ft_geqrf return -7 for anything but
+                            FT_SCHEME_NEW): the checking scheme, for the paper's comparison of
+                            schemes (L35, L47, L542, Table VIII, Figs. 12-14; reading c-34) */
 } ft_opts_t;
+
+/* ft_opts_t.scheme (reading c-34).  NEW: the paper's scheme, Alg. 2 (full
+ * checksums, pre-op checks of PD / PU inputs, post-op checks of their outputs,
+ * the Fig. 4a heuristic TMU check).  FULL_POST: full checksums [13], every
+ * op's output checked after it (L_kk, the panel, the whole trailing matrix
+ * after each TMU).  SINGLE_POST: column checksums only [51, 52], the same
+ * post-op checks on c.  SINGLE_PRE: column checksums only [11], every op's
+ * input checked before it (A_kk, the panel, panel + trailing matrix before
+ * each TMU).  Single-side schemes neither maintain nor check row checksums.
+ * Local restart (restart=1) applies where a post-op check exists. */
+enum { FT_SCHEME_NEW = 0, FT_SCHEME_FULL_POST = 1, FT_SCHEME_SINGLE_POST = 2, FT_SCHEME_SINGLE_PRE = 3 };
 
 /* Host-side statistics, filled after the driver's final synchronisation. */
 typedef struct {

@@ -35,6 +35,7 @@ AT_PRE_PU, AT_POST_PU, AT_PRE_TMU, AT_POST_TMU = 4, 5, 6, 7
 AT_D2H, AT_H2D = 8, 9
 KIND_PERSIST, KIND_ONCHIP = 0, 1
 PD_DEVICE, PD_HOST = 0, 1
+SCHEME_NEW, SCHEME_FULL_POST, SCHEME_SINGLE_POST, SCHEME_SINGLE_PRE = 0, 1, 2, 3  # ft_opts_t.scheme (c-34)
 
 
 # ------------------------------------------------------------- structs ----
@@ -81,7 +82,7 @@ class ft_opts_t(C.Structure):
                 ("fig4a_repair", C.c_int32), ("n_inject", C.c_int32), ("inject", C.POINTER(ft_inject_t)),
                 ("fix_log", C.c_void_p), ("fix_log_cap", C.c_int32), ("pu_gemm", C.c_int32),
                 ("refresh", C.c_int32), ("restart", C.c_int32), ("pd_location", C.c_int32),
-                ("fig4b", C.c_int32), ("trailing_check_period", C.c_int32)]
+                ("fig4b", C.c_int32), ("trailing_check_period", C.c_int32), ("scheme", C.c_int32)]
 
 
 class ft_stats_t(C.Structure):
@@ -370,13 +371,13 @@ def host_lapack_path():
 
 
 def _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh=True, restart=True,
-          pd_location=PD_DEVICE, fig4b=True, period=0):
+          pd_location=PD_DEVICE, fig4b=True, period=0, scheme=0):
     inj = (ft_inject_t * max(1, len(inject)))()
     for k, f in enumerate(inject):
         inj[k] = ft_inject_t(*f)
     opts = ft_opts_t(nb, int(abft), tol_kind, tol_scale, int(fig4a_repair), len(inject), inj,
                      _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES, int(pu_gemm),
-                     int(refresh), int(restart), int(pd_location), int(fig4b), int(period))
+                     int(refresh), int(restart), int(pd_location), int(fig4b), int(period), int(scheme))
     return opts, inj
 
 
@@ -431,13 +432,14 @@ def ft_geqrf(ctx: Context, A: torch.Tensor, nb: int, tau: torch.Tensor, abft=Tru
 
 def ft_potrf(ctx: Context, A: torch.Tensor, nb: int, abft=True, tol_kind=TOL_MAGNITUDE, tol_scale=1.0,
              fig4a_repair=True, inject=(), fix_log=None, pu_gemm=True, refresh=True, restart=True,
-             pd_location=PD_DEVICE, fig4b=True, trailing_check_period=0):
+             pd_location=PD_DEVICE, fig4b=True, trailing_check_period=0, scheme=0):
     """Fault-tolerant lower Cholesky in place on a column-major A.  Returns
     (rc, info, stats) with rc 0 or E_UNCORRECTABLE (other codes raise).
-    pd_location=PD_HOST needs ctx.set_host_lapack() first."""
+    pd_location=PD_HOST needs ctx.set_host_lapack() first.  scheme: SCHEME_*
+    (the checking scheme, include/abft.h ft_opts_t.scheme)."""
     n = A.shape[0]
     opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh, restart,
-                       pd_location, fig4b, trailing_check_period)
+                       pd_location, fig4b, trailing_check_period, scheme)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_potrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), C.byref(opts), C.byref(stats), C.byref(info))

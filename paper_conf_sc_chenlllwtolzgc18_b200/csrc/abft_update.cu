@@ -401,9 +401,9 @@ int update_syrk_t(int64_t nb, int64_t ntk, const T* L21, int64_t ldl, const T* c
                          &zero, P, (int)M2));
   }
   syrk_scatter_col_kernel<T><<<grid_for(M2 * nk), 256, 0, s>>>(Cc, ldc, P, M2, nk, (int)nb, 2, T(-1));
-  syrk_scatter_row_kernel<T><<<grid_for(M2 * nk), 256, 0, s>>>(Rr, ldr, P, M2, nk, (int)nb, 2, T(-1));
+  if (Rr) syrk_scatter_row_kernel<T><<<grid_for(M2 * nk), 256, 0, s>>>(Rr, ldr, P, M2, nk, (int)nb, 2, T(-1));
   ABFT_CUDA_TRY(cudaGetLastError());
-  if (mL && Cm && Rm) {
+  if (mL && Cm) {
     void* av = nullptr;
     rc = scratch_get(s, 3, (size_t)nk * nb * sizeof(T), &av);
     if (rc) return rc;
@@ -417,7 +417,7 @@ int update_syrk_t(int64_t nb, int64_t ntk, const T* L21, int64_t ldl, const T* c
                            &zero, P, (int)ntk));
     }
     syrk_scatter_col_kernel<T><<<grid_for(ntk * nk), 256, 0, s>>>(Cm, ldcm, P, ntk, nk, (int)nb, 1, T(1));
-    syrk_scatter_row_kernel<T><<<grid_for(ntk * nk), 256, 0, s>>>(Rm, ldrm, P, ntk, nk, (int)nb, 1, T(1));
+    if (Rm) syrk_scatter_row_kernel<T><<<grid_for(ntk * nk), 256, 0, s>>>(Rm, ldrm, P, ntk, nk, (int)nb, 1, T(1));
     ABFT_CUDA_TRY(cudaGetLastError());
   }
   return 0;
@@ -554,8 +554,8 @@ extern "C" int abft_update_syrk(int32_t dtype, int64_t nb, int64_t ntk, const vo
   if (ntk == 0) return 0;
   if (!L21 || ldl < ntk * nb) return -4;
   if (!cL || !Cc || ldc < 2 * ntk) return -6;
-  if (!Rr || ldr < ntk * nb) return -11;
-  if (mL && (!Cm || !Rm || ldcm < ntk || ldrm < ntk * nb)) return -8;
+  if (Rr && ldr < ntk * nb) return -11;
+  if (mL && (!Cm || (Rr && !Rm) || ldcm < ntk || (Rm && ldrm < ntk * nb))) return -8;
   cudaStream_t s = (cudaStream_t)stream;
   if (dtype == ABFT_F64)
     return abft::update_syrk_t<double>(nb, ntk, (const double*)L21, ldl, (const double*)cL, ldc, (const double*)mL,

@@ -208,6 +208,14 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
   if (!dA) return -4;
   if (lda < std::max<int64_t>(1, n)) return -5;
   if (o->n_inject < 0 || (o->n_inject > 0 && !o->inject)) return -6;
+  if (o->scheme < FT_SCHEME_NEW || o->scheme > FT_SCHEME_SINGLE_PRE) return -6;
+  // checking scheme (reading c-34): which checks run, and on which checksums
+  const int scheme = o->scheme;
+  const bool s_new = scheme == FT_SCHEME_NEW;
+  const bool single = scheme == FT_SCHEME_SINGLE_POST || scheme == FT_SCHEME_SINGLE_PRE;
+  const bool pre_checks = s_new || scheme == FT_SCHEME_SINGLE_PRE;  // PD / PU inputs
+  const bool post_checks = scheme != FT_SCHEME_SINGLE_PRE;          // PD / PU outputs
+  const int W = single ? ABFT_COL : ABFT_BOTH;
   ABFT_CUDA_TRY(cudaSetDevice(c->device));
   Driver d;
   FT_TRY(d.setup(c, dtype, n, nb, dA, lda, o, /*lu=*/false));
@@ -220,7 +228,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
 
   if (ft) {
     abft_tiles_t all{0, (int)nt, 0, (int)nt, 1, ABFT_SYM_LOWER};
-    FT_TRY(abft_encode(&d.M, &all, ABFT_BOTH, as));
+    FT_TRY(abft_encode(&d.M, &all, W, as));
   }
   for (int k = 0; k < nt; ++k) {
     const int64_t r1 = (k + 1) * nb;  // first row/col after the panel
@@ -229,11 +237,11 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft) FT_TRY(d.begin_iteration());
     // Alg. 2 lines 3-4: check the panel to be decomposed (diag tile, SYM view, both)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
-    if (ft) FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_SYM_LOWER, ABFT_BOTH));
+    if (ft && pre_checks) FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_SYM_LOWER, W));
     // Local restart (f1, L430): the PD input tile and the PU input panel are
     // copied (with their checksums) right after their pre-op checks; a 2D
     // error left by the post-op check restores the copy and redoes the op.
-    const bool rs = ft && o->restart;
+    const bool rs = ft && o->restart && post_checks;
     const int64_t r0 = (int64_t)k * nb;
     char* rbuf = (char*)c->rsv;
     auto copy2d = [&](void* dst, int64_t ldd, const void* src, int64_t lds, int64_t rows, int64_t cols) -> int {
@@ -289,7 +297,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     FT_TRY(d.restore_onchip());
     FT_TRY(d.inject_at(k, FT_AT_POST_PD));
     // line 7: check the decomposed panel (LOWER view, c only; c-24)
-    if (ft) {
+    if (ft && post_checks) {
       if (rs) ABFT_CUDA_TRY(cudaMemcpyAsync(d.snap, d.counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToDevice, s));
       FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_LOWER, ABFT_COL));
       if (rs) FT_TRY(post_readback(d.snap));
@@ -315,7 +323,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (k == nt - 1) break;
     // line 8: check the panel to be updated (both checksums)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PU_CHECK));
-    if (ft) FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH));
+    if (ft && pre_checks) FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, W));
     if (rs) {
       FT_TRY(copy2d(pu_a, nk, d.a_at(r1, r0), lda, nk, nb));
       FT_TRY(copy2d(pu_c, m2, d.colchk_at(2 * (k + 1), r0), d.M.ldc, m2, nb));
@@ -325,7 +333,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     // Fig. 4b (L359): a 1D pattern fixed by this iteration's pre-PD / pre-PU
     // checks is the trace of an on-chip fault in the last TMU: check the
     // whole trailing matrix now (gated on the device)
-    if (ft) FT_TRY(d.fig4b_check(k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, ABFT_BOTH, true));
+    if (ft && s_new) FT_TRY(d.fig4b_check(k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, ABFT_BOTH, true));
     // line 9: PU  L_ik = A_ik L_kk^-T  (+ c(L_ik) = c(A_ik) L_kk^-T, c-12)
     auto pu_data = [&]() -> int {
       cublasHandle_t h = blas_handle(s, lk);
@@ -381,7 +389,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft) FT_TRY(pu_chk());
     FT_TRY(d.inject_at(k, FT_AT_POST_PU));
     // line 10: check the updated panel (c only; 1D_ROW fixable, 2D -> restart, L434)
-    if (ft) {
+    if (ft && post_checks) {
       if (rs) ABFT_CUDA_TRY(cudaMemcpyAsync(d.snap, d.counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToDevice, s));
       FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
       int delta = 0;
@@ -399,6 +407,11 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
         FT_TRY(pu_chk());
         FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
       }
+    }
+    // prior-operation scheme [11]: the TMU's inputs (panel, trailing matrix) before it
+    if (ft && scheme == FT_SCHEME_SINGLE_PRE) {
+      FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
+      FT_TRY(d.check(k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, ABFT_COL, true));
     }
     // line 12: TMU  A22 -= L21 L21^T (DSYRK on tensor cores) + checksum rules c-12
     FT_TRY(d.inject_at(k, FT_AT_PRE_TMU));
@@ -426,12 +439,15 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       // c(A_ij) -= c(L_ik) L_jk^T and r(A_ij) -= L_ik c(L_jk)^T from one product (c-12, L189)
       FT_TRY(abft_update_syrk(dtype, nb, nt - k - 1, d.a_at(r1, k * nb), lda, d.colchk_at(2 * (k + 1), k * nb), d.M.ldc,
                               d.colmag_at(k + 1, k * nb), d.M.ldcm, d.colchk_at(2 * (k + 1), r1),
-                              d.rowchk_at(r1, 2 * (k + 1)), d.M.ldr, d.colmag_at(k + 1, r1), d.rowmag_at(r1, k + 1),
-                              d.M.ldrm, (abft_stream_t)cs));
+                              single ? nullptr : d.rowchk_at(r1, 2 * (k + 1)), d.M.ldr, d.colmag_at(k + 1, r1),
+                              single ? nullptr : d.rowmag_at(r1, k + 1), d.M.ldrm, (abft_stream_t)cs));
     }
     FT_TRY(d.inject_at(k, FT_AT_POST_TMU));
+    // post-operation schemes [13], [51, 52]: the TMU's output, the whole trailing matrix
+    if (ft && (scheme == FT_SCHEME_FULL_POST || scheme == FT_SCHEME_SINGLE_POST))
+      FT_TRY(d.check(k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, W, true));
     // line 13: heuristic panel re-check for the TMU (Fig. 4a) + guarded repair (c-25)
-    if (ft) {
+    if (ft && s_new) {
       ABFT_CUDA_TRY(cudaMemcpyAsync(d.mark, d.nfix, sizeof(int32_t), cudaMemcpyDeviceToDevice, cs));
       FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL, false, cs));
       if (o->fig4a_repair) {

@@ -391,3 +391,78 @@ def test_fig4b_silent_without_faults():
     G = si.general(256, seed=43)
     _, _, st = dr.ft_getrf(G, 32, trailing_check_period=3)
     assert [c[1] for c in st.checks].count("periodic") == 2 and st.counts == [0] * 8
+
+
+# ---------------------------------------------- checking schemes (c-34) --
+# The four schemes the paper compares (L542, Table VIII; L343, L355): the new
+# scheme (Alg. 2), full checksums with post-operation checks [13], column
+# checksums with post-operation checks [51, 52], column checksums with
+# prior-operation checks [11].
+SCHEMES = [dr.SCHEME_NEW, dr.SCHEME_FULL_POST, dr.SCHEME_SINGLE_POST, dr.SCHEME_SINGLE_PRE]
+
+
+@pytest.mark.parametrize("scheme", SCHEMES)
+def test_scheme_error_free_matches_lapack(scheme):
+    A = si.spd(256, seed=31)
+    L, st = dr.ft_potrf(A, 32, scheme=scheme)
+    Lref = np.linalg.cholesky(A)
+    assert st.counts == [0] * 8 and not st.fixes
+    assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
+
+
+# iteration-0 checks of each scheme: (phase, tile range, view, which), n=128 nb=32
+SCHEME_CHECKS = {
+    dr.SCHEME_NEW: [("pre_pd", 0, 1, 0, 1, ck.SYM_LOWER, ck.BOTH), ("post_pd", 0, 1, 0, 1, ck.LOWER, ck.COL),
+                    ("pre_pu", 1, 4, 0, 1, ck.GENERAL, ck.BOTH), ("post_pu", 1, 4, 0, 1, ck.GENERAL, ck.COL),
+                    ("post_tmu", 1, 4, 0, 1, ck.GENERAL, ck.COL)],
+    dr.SCHEME_FULL_POST: [("post_pd", 0, 1, 0, 1, ck.LOWER, ck.COL), ("post_pu", 1, 4, 0, 1, ck.GENERAL, ck.COL),
+                          ("post_tmu_trailing", 1, 4, 1, 4, ck.SYM_LOWER, ck.BOTH)],
+    dr.SCHEME_SINGLE_POST: [("post_pd", 0, 1, 0, 1, ck.LOWER, ck.COL), ("post_pu", 1, 4, 0, 1, ck.GENERAL, ck.COL),
+                            ("post_tmu_trailing", 1, 4, 1, 4, ck.SYM_LOWER, ck.COL)],
+    dr.SCHEME_SINGLE_PRE: [("pre_pd", 0, 1, 0, 1, ck.SYM_LOWER, ck.COL), ("pre_pu", 1, 4, 0, 1, ck.GENERAL, ck.COL),
+                           ("pre_tmu_panel", 1, 4, 0, 1, ck.GENERAL, ck.COL),
+                           ("pre_tmu_trailing", 1, 4, 1, 4, ck.SYM_LOWER, ck.COL)],
+}
+
+
+@pytest.mark.parametrize("scheme", SCHEMES)
+def test_scheme_check_sequence(scheme):
+    """Each scheme checks what its definition says, in that order: inputs
+    before the op (prior-operation, [11]), outputs after it (post-operation,
+    [13], [51, 52]), or both for PD/PU plus the Fig. 4a panel re-check
+    (Alg. 2).  Single-side schemes check column checksums only."""
+    _, st = dr.ft_potrf(si.spd(128, seed=32), 32, scheme=scheme)
+    got = [c[1:] for c in st.checks if c[0] == 0]
+    assert got == SCHEME_CHECKS[scheme]
+
+
+# (fault, outcome per scheme NEW / FULL_POST / SINGLE_POST / SINGLE_PRE) at n=256 nb=32,
+# outcomes: Y = fixed (factor == LAPACK's within 1e-12), R = detected, uncorrectable
+SCHEME_OUTCOMES = [
+    # on-chip fault in a panel element during the TMU (L355): row AND column p of
+    # the trailing matrix damaged (1D).  Full checksums fix 1D, single-side cannot
+    # ("cannot tolerate errors causing 1D error propagation", L544)
+    (dr.Inject(1, dr.AT_PRE_TMU, dr.KIND_ONCHIP, 0, 140, 40, (52,)), "YYRR"),
+    # DRAM fault in A_kk between ops: a prior-operation check catches it before
+    # the PD; a post-operation check finds the PD output inconsistent with the
+    # copy taken after the fault -> 2D (L355: check before AND after PD)
+    (dr.Inject(2, dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 0, 70, 66, (61,)), "YRRY"),
+    # DRAM fault in the TMU reference part: only the Fig. 4a re-check + repair
+    # (L357-L359) recovers it; the other schemes detect it (R)
+    (dr.Inject(1, dr.AT_PRE_TMU, dr.KIND_PERSIST, 0, 140, 40, (52,)), "YRRR"),
+    # 0D computation fault in the trailing matrix: every scheme fixes it
+    (dr.Inject(1, dr.AT_POST_TMU, dr.KIND_PERSIST, 0, 200, 150, (60,)), "YYYY"),
+]
+
+
+@pytest.mark.parametrize("case", range(len(SCHEME_OUTCOMES)))
+def test_scheme_outcomes(case):
+    f, expect = SCHEME_OUTCOMES[case]
+    A = si.spd(256, seed=3)
+    Lref = np.linalg.cholesky(A)
+    got = ""
+    for scheme in SCHEMES:
+        L, st = dr.ft_potrf(A, 32, inject=[f], scheme=scheme)
+        ok = np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
+        got += "R" if st.uncorrectable else ("Y" if ok else "N")
+    assert got == expect

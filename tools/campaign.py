@@ -27,6 +27,10 @@ add up; N: beyond.  The forward deviation from the fault-free factor is
 reported beside it (rel_err).
 Writes gpurun_out/campaign.json (or the path in $CAMPAIGN_OUT).
 
+Kinds potrf:full_post, potrf:single_post, potrf:single_pre run ft_potrf
+with the other checking schemes the paper compares (L542, Table VIII;
+ft_opts_t.scheme, reading c-34) on the same fault draws.
+
   python tools/campaign.py [trials_per_driver] [n] [nb] [K,K,..] [kind,kind,..]
 """
 import json
@@ -100,7 +104,12 @@ def main():
     ctx.set_host_lapack()
     g = si.rng(2018)
     report = {"n": n, "nb": nb, "trials": trials, "bits": "52-63", "K": Ks}
-    for kind, K in [(kd, K) for kd in kinds for K in Ks]:
+    SCHEME = {"": abft.SCHEME_NEW, "full_post": abft.SCHEME_FULL_POST, "single_post": abft.SCHEME_SINGLE_POST,
+              "single_pre": abft.SCHEME_SINGLE_PRE}
+    for label, K in [(kd, K) for kd in kinds for K in Ks]:
+        kind, _, sname = label.partition(":")
+        scheme = SCHEME[sname]
+        g = si.rng(2018 + K)  # every driver / scheme sees the same draw sequence for a given K
         pd = abft.PD_HOST if kind.startswith("host") else abft.PD_DEVICE
         A0 = si.spd_device(n, seed=1) if kind.endswith("potrf") else si.general_device(n, seed=1)
         A = torch.empty_like(A0.t()).t()
@@ -125,7 +134,7 @@ def main():
         def run(inj):
             A.copy_(A0)
             if kind.endswith("potrf"):
-                rc, info, st = abft.ft_potrf(ctx, A, nb, inject=inj, pd_location=pd)
+                rc, info, st = abft.ft_potrf(ctx, A, nb, inject=inj, pd_location=pd, scheme=scheme)
                 out = torch.tril(A).clone()
             elif kind.endswith("getrf"):
                 rc, info, st = abft.ft_getrf(ctx, A, nb, piv, inject=inj, pd_location=pd)
@@ -169,8 +178,8 @@ def main():
                                  "fixes": st.n_fixes, "repairs": st.repairs_applied, "restarts": st.restarts,
                                  "ctf": st.ctf_recomputed, "xfer_fixed": st.xfer_d2h_fixed + st.xfer_h2d_fixed,
                                  "retransfers": st.xfer_retransfers + st.xfer_resends})
-        report[kind if len(Ks) == 1 else f"{kind}_K{K}"] = out
-        print(kind, {k: v for k, v in out.items() if k != "cases"}, flush=True)
+        report[label if len(Ks) == 1 else f"{label}_K{K}"] = out
+        print(label, {k: v for k, v in out.items() if k != "cases"}, flush=True)
         del A, A0
         torch.cuda.empty_cache()
     os.makedirs("gpurun_out", exist_ok=True)
