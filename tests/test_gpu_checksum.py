@@ -277,11 +277,12 @@ def test_inject_is_xor(lib):
     assert A[5, 7].item() == si.flip_bits(before, [62])
 
 
-@pytest.mark.parametrize("prec", ["f64", "f32"])
-def test_full_size_sampled_tiles(lib, prec):
-    """BASELINE config-4 sized matrix (n=16384, nb=512): sampled tiles vs the
+@pytest.mark.parametrize("prec,n", [("f64", 16384), ("f32", 16384), ("f64", 30720)])
+def test_full_size_sampled_tiles(lib, prec, n):
+    """BASELINE config-4 sized matrices (n=16384, nb=512) and the bench's own
+    launch (fp64 n=30720 nb=512, the metric's size): sampled tiles vs the
     oracle, plus the verify-after-encode invariant over the whole matrix."""
-    n, nb = 16384, 512
+    nb = 512
     A = si.general_device(n, seed=7, dtype=TDT[prec])
     mat = lib.Mat.alloc(A, nb)
     t = lib.tiles(0, n // nb, 0, n // nb)

@@ -161,6 +161,32 @@ def test_config2_shape_error_free_and_injected(lib, ctx):
     assert (torch.tril(A) - L).abs().max().item() <= 1e-12 * L.abs().max().item()
 
 
+def test_metric_size_potrf(lib, ctx):
+    """The metric's ft_potrf (n=30720 nb=512, as bench.py runs it): sampled
+    residual rows of the error-free factor, then one MUST-band DRAM fault in
+    the trailing matrix and one on-chip fault in the panel during the TMU,
+    both fixed (the factor equals the fault-free one within 1e-12)."""
+    n, nb = 30720, 512
+    A = si.spd_device(n, seed=6)
+    A0 = A.clone()
+    rc, info, stats = lib.ft_potrf(ctx, A, nb)
+    torch.cuda.synchronize()
+    assert rc == 0 and info == 0 and list(stats.counts) == [0] * 8
+    g = si.rng(10)
+    rows = torch.tensor(sorted(g.choice(n, 32, replace=False)), device="cuda")
+    Lr = torch.tril(A)[rows]
+    R = A0[rows] - Lr @ torch.tril(A).T
+    assert R.abs().max().item() <= 1e-12 * n
+    ref = torch.tril(A).clone()
+    A.copy_(A0)
+    inj = [(20, lib.AT_POST_TMU, lib.KIND_PERSIST, 0, 25000, 15000, 1 << 60),
+           (40, lib.AT_PRE_TMU, lib.KIND_ONCHIP, 0, 29000, 20600, 1 << 55)]
+    rc, info, stats = lib.ft_potrf(ctx, A, nb, inject=inj)
+    torch.cuda.synchronize()
+    assert rc == 0 and stats.uncorrectable == 0 and stats.n_fixes >= 2
+    assert (torch.tril(A) - ref).abs().max().item() <= 1e-12 * ref.abs().max().item()
+
+
 # ---- f1: Fig. 4b on-chip 1D detection and the periodic trailing check ------
 _ONCHIP_PAIR = [dr.Inject(1, dr.AT_PRE_TMU, dr.KIND_ONCHIP, 0, 197, 40, (55,)),
                 dr.Inject(2, dr.AT_PRE_TMU, dr.KIND_ONCHIP, 0, 212, 67, (55,))]
