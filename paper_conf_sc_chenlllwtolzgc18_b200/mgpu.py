@@ -22,7 +22,9 @@ global tile's).  Iteration k of Alg. 2 (L368-L378):
      c-6, c-12), grouped tile columns per call (`abft_update_gemm`);
   6. the received panel is re-checked after the trailing update (Fig. 4a);
      a value corrected there was already consumed by the update, which the
-     distributed driver reports as uncorrectable (no distributed repair).
+     distributed driver reports as uncorrectable (no distributed repair);
+     the panel owners re-check their stored pieces too (the factor itself,
+     which no update read: a fault there is a plain fix).
 
 Local restart (f1, L430): the owner of A_kk and the panel owners copy the
 input of their PD / PU with its checksums after the pre-op check; a 2D error
@@ -422,6 +424,12 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
         elif ncol == 0 or Lrow is None:
             hook(k, abft.AT_PRE_TMU)
             hook(k, abft.AT_POST_TMU)
+        # ---- 6b. the panel owners' stored pieces (the factor itself): Alg. 2
+        # line 13 re-checks the panel after the TMU; here the update read the
+        # broadcast copies (checked above), so a fault in the stored piece
+        # since its post-PU check was consumed by nobody and is a plain fix
+        if abft_on and q == kq and cnt > 0:
+            check(mat, abft.tiles(ir0, lay.mt_loc, jk, jk + 1), abft.COL)
 
     # ---- error reports: one all-reduce of the int32 counters (L361-L363)
     rep_counts = rep.counts if rep is not None else torch.zeros(abft.NCOUNTS, dtype=torch.int32, device=dev)

@@ -69,6 +69,8 @@ BIT = 1 << 61  # exponent bit: a MUST-band fault (reading c-10)
     (0, abft.AT_PRE_PU_CHECK, 300, 20),   # panel before PU
     (2, abft.AT_POST_PU, 450, 140),       # updated panel
     (0, abft.AT_POST_TMU, 400, 200),      # trailing tile after the update (caught when it becomes panel)
+    (1, abft.AT_PRE_TMU, 300, 70),        # owner's stored panel after its broadcast (Alg. 2 line 13)
+    (2, abft.AT_POST_TMU, 470, 150),      # owner's stored panel after the update
 ])
 def test_single_fault_corrected(tmp_path, case):
     n, nb = 512, 64
