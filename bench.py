@@ -362,12 +362,13 @@ def potrf_overhead(abft, si, n, nb, reps, host_pd=True):
     A = torch.empty_like(A0.t()).t()
     ctx = abft.Context()
 
-    def run(ft, restart=True, pd=abft.PD_DEVICE, scheme=abft.SCHEME_NEW):
+    def run(ft, restart=True, pd=abft.PD_DEVICE, scheme=abft.SCHEME_NEW, gemm=False):
         A.copy_(A0)
         torch.cuda.synchronize()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record()
-        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart, pd_location=pd, scheme=scheme)
+        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart, pd_location=pd, scheme=scheme,
+                                     checksum_gemm=gemm)
         b.record()
         torch.cuda.synchronize()
         assert rc == 0 and info == 0
@@ -391,10 +392,14 @@ def potrf_overhead(abft, si, n, nb, reps, host_pd=True):
     # same driver, same plain baseline, no restart (so that every scheme is
     # timed alike: SINGLE_PRE has no post-op check to restart from)
     schemes = {}
-    for name, sc in (("new", abft.SCHEME_NEW), ("full_post", abft.SCHEME_FULL_POST),
-                     ("single_post", abft.SCHEME_SINGLE_POST), ("single_pre", abft.SCHEME_SINGLE_PRE)):
-        run(True, restart=False, scheme=sc)
-        ts = sorted(run(True, restart=False, scheme=sc)[0] for _ in range(max(1, reps - 1)))
+    # ("new_gemm_checks": the new scheme with the checks' recalculation done by
+    # cuBLAS GEMMs, the paper's "without the optimized kernel", L653-L657)
+    for name, sc, gm in (("new", abft.SCHEME_NEW, False), ("new_gemm_checks", abft.SCHEME_NEW, True),
+                         ("full_post", abft.SCHEME_FULL_POST, False),
+                         ("single_post", abft.SCHEME_SINGLE_POST, False),
+                         ("single_pre", abft.SCHEME_SINGLE_PRE, False)):
+        run(True, restart=False, scheme=sc, gemm=gm)
+        ts = sorted(run(True, restart=False, scheme=sc, gemm=gm)[0] for _ in range(max(1, reps - 1)))
         tm = ts[len(ts) // 2]
         schemes[name] = {"ms_ft": tm, "overhead_pct": 100.0 * (tm - plain_ms) / plain_ms}
     host = None

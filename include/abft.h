@@ -168,6 +168,16 @@ ABFT_API int abft_encode(const abft_mat_t *mat, const abft_tiles_t *tiles, int32
 ABFT_API int abft_verify(const abft_mat_t *mat, const abft_tiles_t *tiles, int32_t which,
                 const abft_tol_t *tol, const abft_report_t *report, abft_stream_t stream);
 
+/* Prior-art baseline (row f3; L35, L442): abft_verify with the checksums
+ * recomputed as matrix products c = [v1 v2]^T X, r = X [v1 v2] by cuBLAS
+ * (strided-batched GEMMs per tile column; masked diagonal views materialized
+ * first), then the same test and report as abft_verify.  Needs the
+ * magnitude arrays of every checked direction (ABFT_E_UNSUPPORTED
+ * otherwise: a product cannot form e^T|X|); tol->refresh is ignored.  Exists
+ * to measure what the fused single-pass kernel buys (the paper's L657). */
+ABFT_API int abft_verify_gemm(const abft_mat_t *mat, const abft_tiles_t *tiles, int32_t which,
+                const abft_tol_t *tol, const abft_report_t *report, abft_stream_t stream);
+
 /* a3 — abft_locate_correct.  For every tile of the range whose
  * report->status has COL or ROW set: up to 3 rounds of recompute ->
  * classify (c-11: CHK_CORRUPT, STALE_R/C, 0D, 1D_ROW, 1D_COL, SYM_LOWER
@@ -361,6 +371,10 @@ typedef struct {
   int32_t trailing_check_period; /* P > 0: check the whole trailing matrix after the TMU of every P-th
                             iteration (L359: "periodically check the correctness of trailing matrix
                             ... to avoid 2D propagation"); 0 (default): never */
+  int32_t checksum_gemm; /* 1: every check of ft_potrf recomputes the checksums with abft_verify_gemm
+                            (the prior-art GEMM-based recalculation, L442) instead of the fused pass;
+                            no refresh, no Fig. 4b check.  For the paper's comparison "with / without
+                            the optimized checksum kernel" (L653-L657).  Default 0. */
   int32_t scheme;        /* FT_SCHEME_* (ft_potrf only; ft_getrf / ft_geqrf return -7 for anything but
                             FT_SCHEME_NEW): the checking scheme, for the paper's comparison of
                             schemes (L35, L47, L542, Table VIII, Figs. 12-14; reading c-34) */

@@ -82,7 +82,8 @@ class ft_opts_t(C.Structure):
                 ("fig4a_repair", C.c_int32), ("n_inject", C.c_int32), ("inject", C.POINTER(ft_inject_t)),
                 ("fix_log", C.c_void_p), ("fix_log_cap", C.c_int32), ("pu_gemm", C.c_int32),
                 ("refresh", C.c_int32), ("restart", C.c_int32), ("pd_location", C.c_int32),
-                ("fig4b", C.c_int32), ("trailing_check_period", C.c_int32), ("scheme", C.c_int32)]
+                ("fig4b", C.c_int32), ("trailing_check_period", C.c_int32), ("checksum_gemm", C.c_int32),
+                ("scheme", C.c_int32)]
 
 
 class ft_stats_t(C.Structure):
@@ -101,6 +102,7 @@ _P = C.POINTER
 _sig = {
     "abft_encode": [_P(abft_mat_t), _P(abft_tiles_t), _i32, _vp],
     "abft_verify": [_P(abft_mat_t), _P(abft_tiles_t), _i32, _P(abft_tol_t), _P(abft_report_t), _vp],
+    "abft_verify_gemm": [_P(abft_mat_t), _P(abft_tiles_t), _i32, _P(abft_tol_t), _P(abft_report_t), _vp],
     "abft_locate_correct": [_P(abft_mat_t), _P(abft_tiles_t), _i32, _P(abft_tol_t), _P(abft_report_t),
                             _vp, _i32, _vp, _vp],
     "abft_inject": [_vp, _i32, _i64, _u64, _vp],
@@ -265,6 +267,13 @@ def abft_verify(mat: Mat, t: abft_tiles_t, which, tol: abft_tol_t, rep: Report, 
                                                 _stream(stream)))
 
 
+def abft_verify_gemm(mat: Mat, t: abft_tiles_t, which, tol: abft_tol_t, rep: Report, stream=None):
+    """Prior-art baseline: abft_verify with the checksums recomputed by cuBLAS GEMMs."""
+    m, r = mat.c(), rep.c()
+    return _check("abft_verify_gemm", _L.abft_verify_gemm(C.byref(m), C.byref(t), which, C.byref(tol), C.byref(r),
+                                                          _stream(stream)))
+
+
 def abft_locate_correct(mat: Mat, t: abft_tiles_t, which, tol: abft_tol_t, rep: Report,
                         fixes: torch.Tensor, n_fixes: torch.Tensor, stream=None):
     """fixes: uint8 device buffer of k*FIX_BYTES bytes; n_fixes: int32[1]."""
@@ -371,13 +380,14 @@ def host_lapack_path():
 
 
 def _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh=True, restart=True,
-          pd_location=PD_DEVICE, fig4b=True, period=0, scheme=0):
+          pd_location=PD_DEVICE, fig4b=True, period=0, scheme=0, checksum_gemm=False):
     inj = (ft_inject_t * max(1, len(inject)))()
     for k, f in enumerate(inject):
         inj[k] = ft_inject_t(*f)
     opts = ft_opts_t(nb, int(abft), tol_kind, tol_scale, int(fig4a_repair), len(inject), inj,
                      _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES, int(pu_gemm),
-                     int(refresh), int(restart), int(pd_location), int(fig4b), int(period), int(scheme))
+                     int(refresh), int(restart), int(pd_location), int(fig4b), int(period), int(checksum_gemm),
+                     int(scheme))
     return opts, inj
 
 
@@ -432,14 +442,15 @@ def ft_geqrf(ctx: Context, A: torch.Tensor, nb: int, tau: torch.Tensor, abft=Tru
 
 def ft_potrf(ctx: Context, A: torch.Tensor, nb: int, abft=True, tol_kind=TOL_MAGNITUDE, tol_scale=1.0,
              fig4a_repair=True, inject=(), fix_log=None, pu_gemm=True, refresh=True, restart=True,
-             pd_location=PD_DEVICE, fig4b=True, trailing_check_period=0, scheme=0):
+             pd_location=PD_DEVICE, fig4b=True, trailing_check_period=0, scheme=0, checksum_gemm=False):
     """Fault-tolerant lower Cholesky in place on a column-major A.  Returns
     (rc, info, stats) with rc 0 or E_UNCORRECTABLE (other codes raise).
     pd_location=PD_HOST needs ctx.set_host_lapack() first.  scheme: SCHEME_*
-    (the checking scheme, include/abft.h ft_opts_t.scheme)."""
+    (the checking scheme, include/abft.h ft_opts_t.scheme); checksum_gemm: the
+    checks recompute checksums by GEMMs (prior-art baseline, abft_verify_gemm)."""
     n = A.shape[0]
     opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh, restart,
-                       pd_location, fig4b, trailing_check_period, scheme)
+                       pd_location, fig4b, trailing_check_period, scheme, checksum_gemm)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_potrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), C.byref(opts), C.byref(stats), C.byref(info))

@@ -265,7 +265,10 @@ struct Driver {
             cudaStream_t on = nullptr) {
     abft_tiles_t t{I0, I1, J0, J1, lower_only ? 1 : 0, view};
     const abft_stream_t st = (abft_stream_t)(on ? on : s);
-    FT_TRY(abft_verify(&M, &t, which, &tol, &R, st));
+    if (o->checksum_gemm)  // prior-art GEMM recalculation (f3 baseline)
+      FT_TRY(abft_verify_gemm(&M, &t, which, &tol, &R, st));
+    else
+      FT_TRY(abft_verify(&M, &t, which, &tol, &R, st));
     FT_TRY(abft_locate_correct(&M, &t, which, &tol, &R, c->fixlog, c->fixcap, nfix, st));
     ++n_checks;
     return 0;
@@ -317,7 +320,7 @@ struct Driver {
     return 0;
   }
   int fig4b_check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only) {
-    if (!o->fig4b || I0 >= I1) return 0;
+    if (!o->fig4b || o->checksum_gemm || I0 >= I1) return 0;  // GEMMs cannot honour the device gate
     fig4b_gate_kernel<<<1, 32, 0, s>>>(c->fixlog, c->fixcap, iter_mark, nfix, gate4b, gated_runs);
     ABFT_CUDA_TRY(cudaGetLastError());
     GateScope g(gate4b);

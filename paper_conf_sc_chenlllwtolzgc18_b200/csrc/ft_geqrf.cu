@@ -594,7 +594,7 @@ extern "C" int ft_geqrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
   if (lda < std::max<int64_t>(1, n)) return -5;
   if (!tau) return -6;
   if (o->n_inject < 0 || (o->n_inject > 0 && !o->inject)) return -7;
-  if (o->scheme != FT_SCHEME_NEW) return -7;  // checking-scheme comparison: ft_potrf only (c-34)
+  if (o->scheme != FT_SCHEME_NEW || o->checksum_gemm) return -7;  // scheme / GEMM-check comparisons: ft_potrf only
   ABFT_CUDA_TRY(cudaSetDevice(c->device));
   Driver d;
   FT_TRY(d.setup(c, dtype, n, nb, dA, lda, o, /*lu=*/true));

@@ -390,3 +390,56 @@ def test_verify_segmented_flags_every_tile(lib, prec, nb):
         for J in range(nt):
             assert (s[I, J] != 0) == (I >= J), (I, J, s[I, J])
     assert int(rep.counts[0].item()) == nt * (nt + 1) // 2
+
+
+# ---- f3 baseline: the GEMM-based recalculation (abft_verify_gemm) --------
+@pytest.mark.parametrize("prec", ["f64", "f32"])
+@pytest.mark.parametrize("rng_case", ["full", "sym_lower", "lower_col"])
+def test_verify_gemm_matches_fused(lib, prec, rng_case):
+    """The prior-art GEMM recalculation (L442) reaches the same verdicts as the
+    fused pass: identical tile status and counts on MUST-band corruptions, and
+    deltas equal within the normwise tolerance of c-1."""
+    nb, n = 64, 384
+    A = si.spd(n, seed=12) if rng_case != "full" else si.general(n, seed=12)
+    view = {"full": ck.GENERAL, "sym_lower": ck.SYM_LOWER, "lower_col": ck.LOWER}[rng_case]
+    lower = rng_case != "full"
+    which = ck.COL if rng_case == "lower_col" else ck.BOTH
+    mat, t = _encode(lib, A, nb, prec, view=view, lower_only=lower, which=which)
+    for gi, gj in [(70, 3), (200, 130), (383, 320), (5, 0)]:
+        if not lower or gi >= gj:
+            mat.A[gi, gj] += 7.0
+    mat.colchk[2 * 3, 200] += 50.0
+    tol = lib.abft_tol_t(ck.TOL_MAGNITUDE, 1.0, 0)
+    r1, r2 = lib.Report.alloc(mat, deltas=True), lib.Report.alloc(mat, deltas=True)
+    lib.abft_verify(mat, t, which, tol, r1)
+    lib.abft_verify_gemm(mat, t, which, tol, r2)
+    torch.cuda.synchronize()
+    assert torch.equal(r1.status, r2.status) and torch.equal(r1.counts, r2.counts), (r1.counts, r2.counts)
+    assert int(r1.counts[0]) >= 3
+    scale = {"f64": 1e-12, "f32": 1e-5}[prec] * float(mat.A.abs().sum(0).max())
+    assert float((r1.dcol - r2.dcol).abs().max()) <= scale * nb
+    if which & ck.ROW:
+        assert float((r1.drow - r2.drow).abs().max()) <= scale * nb
+
+
+def test_potrf_with_gemm_checks(lib):
+    """ft_potrf with the checks' recalculation done by GEMMs (the paper's
+    'without the optimized kernel' variant, L653): error free it equals LAPACK;
+    a MUST-band fault is fixed exactly as with the fused pass."""
+    ctx = lib.Context()
+    A_np = si.spd(1024, seed=13)
+    Lref = np.linalg.cholesky(A_np)
+    inj = [(3, lib.AT_POST_TMU, lib.KIND_PERSIST, 0, 900, 700, 1 << 60),
+           (2, lib.AT_PRE_PU_CHECK, lib.KIND_PERSIST, 0, 600, 300, 1 << 58)]
+    outs = []
+    for gemm in (False, True):
+        for plan in ((), inj):
+            A = dev(A_np)
+            log = torch.zeros(1024 * lib.FIX_BYTES, dtype=torch.uint8, device="cuda")
+            rc, info, st = lib.ft_potrf(ctx, A, 128, inject=plan, fix_log=log, checksum_gemm=gemm)
+            torch.cuda.synchronize()
+            L = np.tril(host(A))
+            assert rc == 0 and info == 0
+            assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
+            outs.append(sorted((f[0], f[1], f[4]) for f in lib.decode_fixes(log, st.n_fixes)))
+    assert outs[0] == outs[2] == [] and outs[1] == outs[3] and len(outs[1]) == 2
