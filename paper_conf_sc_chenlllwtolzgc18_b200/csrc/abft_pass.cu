@@ -151,6 +151,44 @@ __device__ __forceinline__ int check_pair(T me, T mw, T re, T rw, double m, doub
   return (fl ? 1 : 0) | (nf ? 2 : 0);
 }
 
+// Masked diagonal views (c-3), one template per view so that the inner loops
+// carry no view switch; the weights are kept in floating point and stepped
+// by exact integer increments (an int->fp64 conversion per element, I2F.F64,
+// made a masked diagonal tile ~6x slower than a GENERAL one: pass_views r01).
+// Same values in the same order as before, so results are bit-identical.
+template <int VIEW, typename T>
+__device__ __forceinline__ T masked(int i, int j, T x) {  // X[i, j] under VIEW
+  if (VIEW == ABFT_LOWER) return i >= j ? x : T(0);
+  if (VIEW == ABFT_UNIT_LOWER) return i > j ? x : (i == j ? T(1) : T(0));
+  if (VIEW == ABFT_UPPER) return i <= j ? x : T(0);
+  if (VIEW == ABFT_SYM_LOWER) return i > j ? x : T(0);  // strict lower (the row-sum half of SYM)
+  return x;
+}
+template <int VIEW, int NB, typename T>
+__device__ __forceinline__ void masked_colsum(const T* col, int jl, int lane, T& pe, T& pw, T& pa) {
+  T wi = T(lane + 1);
+#pragma unroll 4
+  for (int k = 0; k < NB / 32; ++k) {
+    const T x = masked<VIEW>(lane + 32 * k, jl, col[lane + 32 * k]);
+    pe = fadd(pe, x);
+    pw = ffma(wi, x, pw);
+    pa = fadd(pa, fabs(x));
+    wi = fadd(wi, T(32));
+  }
+}
+template <int VIEW, int CC, int RK, typename T>
+__device__ __forceinline__ void masked_rowsum(const T* buf, int r, int jl0, Acc3<T>& g) {
+  T wj = T(jl0 + 1);
+#pragma unroll 8
+  for (int cc = 0; cc < CC; ++cc) {
+    const T x = masked<VIEW>(r, jl0 + cc, buf[cc * RK + r]);
+    g.e = fadd(g.e, x);
+    g.w = ffma(wj, x, g.w);
+    g.a = fadd(g.a, fabs(x));
+    wj = fadd(wj, T(1));
+  }
+}
+
 __device__ __forceinline__ void consumer_sync() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
@@ -443,13 +481,11 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
         }
       } else {  // masked diagonal views (K == 1 only)
         T pe = T(0), pw = T(0), pa = T(0);
-#pragma unroll 4
-        for (int k = 0; k < NB / 32; ++k) {
-          const int i = lane + 32 * k;
-          T x = view_mask(viewA, i, jl, col[i]);
-          pe = fadd(pe, x);
-          pw = ffma(T(i + 1), x, pw);
-          pa = fadd(pa, fabs(x));
+        switch (viewA) {  // uniform per CTA
+          case ABFT_LOWER: masked_colsum<ABFT_LOWER, NB>(col, jl, lane, pe, pw, pa); break;
+          case ABFT_UNIT_LOWER: masked_colsum<ABFT_UNIT_LOWER, NB>(col, jl, lane, pe, pw, pa); break;
+          case ABFT_UPPER: masked_colsum<ABFT_UPPER, NB>(col, jl, lane, pe, pw, pa); break;
+          default: masked_colsum<ABFT_GENERAL, NB>(col, jl, lane, pe, pw, pa); break;
         }
 #pragma unroll
         for (int m = 16; m >= 1; m >>= 1) {
@@ -482,13 +518,13 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
             grp[q].a = fadd(grp[q].a, sa);
           }
         } else {
-          for (int cc = 0; cc < C::CC; ++cc) {
-            const int jl = c0 + s * C::CC + cc;
-            T x = buf[cc * RK + r];
-            x = sym ? (r > jl ? x : T(0)) : view_mask(view, r, jl, x);
-            grp[q].e = fadd(grp[q].e, x);
-            grp[q].w = ffma(T(jl + 1), x, grp[q].w);
-            grp[q].a = fadd(grp[q].a, fabs(x));
+          const int jl0 = c0 + s * C::CC;
+          switch (sym ? (int)ABFT_SYM_LOWER : view) {  // uniform per CTA
+            case ABFT_SYM_LOWER: masked_rowsum<ABFT_SYM_LOWER, C::CC, RK>(buf, r, jl0, grp[q]); break;
+            case ABFT_LOWER: masked_rowsum<ABFT_LOWER, C::CC, RK>(buf, r, jl0, grp[q]); break;
+            case ABFT_UNIT_LOWER: masked_rowsum<ABFT_UNIT_LOWER, C::CC, RK>(buf, r, jl0, grp[q]); break;
+            case ABFT_UPPER: masked_rowsum<ABFT_UPPER, C::CC, RK>(buf, r, jl0, grp[q]); break;
+            default: masked_rowsum<ABFT_GENERAL, C::CC, RK>(buf, r, jl0, grp[q]); break;
           }
         }
       }
