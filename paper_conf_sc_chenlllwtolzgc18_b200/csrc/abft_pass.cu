@@ -152,10 +152,9 @@ __device__ __forceinline__ int check_pair(T me, T mw, T re, T rw, double m, doub
 }
 
 // Masked diagonal views (c-3), one template per view so that the inner loops
-// carry no view switch; the weights are kept in floating point and stepped
-// by exact integer increments (an int->fp64 conversion per element, I2F.F64,
-// made a masked diagonal tile ~6x slower than a GENERAL one: pass_views r01).
-// Same values in the same order as before, so results are bit-identical.
+// carry no view switch; weights are compile-time or stepped in floating point
+// (an int->fp64 conversion per element, I2F.F64, made a masked diagonal tile
+// ~6x slower than a GENERAL one: pass_views r01).
 template <int VIEW, typename T>
 __device__ __forceinline__ T masked(int i, int j, T x) {  // X[i, j] under VIEW
   if (VIEW == ABFT_LOWER) return i >= j ? x : T(0);
@@ -163,18 +162,6 @@ __device__ __forceinline__ T masked(int i, int j, T x) {  // X[i, j] under VIEW
   if (VIEW == ABFT_UPPER) return i <= j ? x : T(0);
   if (VIEW == ABFT_SYM_LOWER) return i > j ? x : T(0);  // strict lower (the row-sum half of SYM)
   return x;
-}
-template <int VIEW, int NB, typename T>
-__device__ __forceinline__ void masked_colsum(const T* col, int jl, int lane, T& pe, T& pw, T& pa) {
-  T wi = T(lane + 1);
-#pragma unroll 4
-  for (int k = 0; k < NB / 32; ++k) {
-    const T x = masked<VIEW>(lane + 32 * k, jl, col[lane + 32 * k]);
-    pe = fadd(pe, x);
-    pw = ffma(wi, x, pw);
-    pa = fadd(pa, fabs(x));
-    wi = fadd(wi, T(32));
-  }
 }
 template <int VIEW, int CC, int RK, typename T>
 __device__ __forceinline__ void masked_rowsum(const T* buf, int r, int jl0, Acc3<T>& g) {
@@ -186,6 +173,88 @@ __device__ __forceinline__ void masked_rowsum(const T* buf, int r, int jl0, Acc3
     g.w = ffma(wj, x, g.w);
     g.a = fadd(g.a, fabs(x));
     wj = fadd(wj, T(1));
+  }
+}
+
+// Masked column sums with the GENERAL path's vector loads and compile-time
+// weights: a warp-uniform test per vector iteration skips row blocks the view
+// zeroes entirely and masks element-wise only in the block the diagonal
+// crosses (a masked diagonal tile then streams about half of its column work).
+template <int VIEW, int NB, int VEC, typename T>
+__device__ __forceinline__ void masked_colsum_vec(const T* col, int jl, int lane, T& e, T& w, T& a) {
+  constexpr int KV = NB / (32 * VEC);
+  T pe = T(0), s1 = T(0), pa = T(0);
+#pragma unroll
+  for (int k = 0; k < KV; ++k) {
+    const int blo = 32 * VEC * k, bhi = blo + 32 * VEC - 1;  // the warp's rows this iteration
+    bool out, in;
+    if (VIEW == ABFT_UPPER) {
+      out = blo > jl;
+      in = bhi <= jl;
+    } else if (VIEW == ABFT_LOWER) {
+      out = bhi < jl;
+      in = blo >= jl;
+    } else {  // UNIT_LOWER: the diagonal element reads as 1
+      out = bhi < jl;
+      in = blo > jl;
+    }
+    if (out) continue;
+    T xv[VEC];
+    load_vec<T, VEC>(xv, col + (32 * k + lane) * VEC);
+    if (!in) {
+#pragma unroll
+      for (int v = 0; v < VEC; ++v) xv[v] = masked<VIEW>((32 * k + lane) * VEC + v, jl, xv[v]);
+    }
+#pragma unroll
+    for (int v = 0; v < VEC; ++v) {
+      pe = fadd(pe, xv[v]);
+      s1 = ffma(T(32 * VEC * k + v), xv[v], s1);
+      pa = fadd(pa, fabs(xv[v]));
+    }
+  }
+  e = pe;
+  w = ffma(T(lane * VEC + 1), pe, s1);
+  a = pa;
+}
+
+// Masked row sums of one stage for row r: a stage entirely inside the view
+// takes the GENERAL chunk formula, one entirely outside is skipped, only the
+// stage the diagonal crosses is masked element-wise.
+template <int VIEW, int CC, int CQ, int RK, typename T>
+__device__ __forceinline__ void masked_rowsum_fast(const T* buf, int r, int jl0, Acc3<T>& g) {
+  const int jl1 = jl0 + CC - 1;
+  bool in, out;
+  if (VIEW == ABFT_UPPER) {  // keep jl >= r
+    in = jl0 >= r;
+    out = jl1 < r;
+  } else if (VIEW == ABFT_LOWER) {  // keep jl <= r
+    in = jl1 <= r;
+    out = jl0 > r;
+  } else if (VIEW == ABFT_SYM_LOWER) {  // keep jl < r
+    in = jl1 < r;
+    out = jl0 >= r;
+  } else {  // UNIT_LOWER: keep jl < r, jl == r reads 1
+    in = jl1 < r;
+    out = jl0 > r;
+  }
+  if (out) return;
+  if (!in) {
+    masked_rowsum<VIEW, CC, RK>(buf, r, jl0, g);
+    return;
+  }
+#pragma unroll
+  for (int ch = 0; ch < CC / CQ; ++ch) {
+    T se = T(0), s1 = T(0), sa = T(0);
+#pragma unroll
+    for (int cq = 0; cq < CQ; ++cq) {
+      const T x = buf[(ch * CQ + cq) * RK + r];
+      se = fadd(se, x);
+      s1 = ffma(T(cq), x, s1);
+      sa = fadd(sa, fabs(x));
+    }
+    g.e = fadd(g.e, se);
+    g.w = fadd(g.w, ffma(T(jl0 + ch * CQ + 1), se, s1));
+    g.a = fadd(g.a, sa);
   }
 }
 
@@ -482,10 +551,9 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
       } else {  // masked diagonal views (K == 1 only)
         T pe = T(0), pw = T(0), pa = T(0);
         switch (viewA) {  // uniform per CTA
-          case ABFT_LOWER: masked_colsum<ABFT_LOWER, NB>(col, jl, lane, pe, pw, pa); break;
-          case ABFT_UNIT_LOWER: masked_colsum<ABFT_UNIT_LOWER, NB>(col, jl, lane, pe, pw, pa); break;
-          case ABFT_UPPER: masked_colsum<ABFT_UPPER, NB>(col, jl, lane, pe, pw, pa); break;
-          default: masked_colsum<ABFT_GENERAL, NB>(col, jl, lane, pe, pw, pa); break;
+          case ABFT_LOWER: masked_colsum_vec<ABFT_LOWER, NB, C::VEC>(col, jl, lane, pe, pw, pa); break;
+          case ABFT_UNIT_LOWER: masked_colsum_vec<ABFT_UNIT_LOWER, NB, C::VEC>(col, jl, lane, pe, pw, pa); break;
+          default: masked_colsum_vec<ABFT_UPPER, NB, C::VEC>(col, jl, lane, pe, pw, pa); break;
         }
 #pragma unroll
         for (int m = 16; m >= 1; m >>= 1) {
@@ -520,11 +588,10 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
         } else {
           const int jl0 = c0 + s * C::CC;
           switch (sym ? (int)ABFT_SYM_LOWER : view) {  // uniform per CTA
-            case ABFT_SYM_LOWER: masked_rowsum<ABFT_SYM_LOWER, C::CC, RK>(buf, r, jl0, grp[q]); break;
-            case ABFT_LOWER: masked_rowsum<ABFT_LOWER, C::CC, RK>(buf, r, jl0, grp[q]); break;
-            case ABFT_UNIT_LOWER: masked_rowsum<ABFT_UNIT_LOWER, C::CC, RK>(buf, r, jl0, grp[q]); break;
-            case ABFT_UPPER: masked_rowsum<ABFT_UPPER, C::CC, RK>(buf, r, jl0, grp[q]); break;
-            default: masked_rowsum<ABFT_GENERAL, C::CC, RK>(buf, r, jl0, grp[q]); break;
+            case ABFT_SYM_LOWER: masked_rowsum_fast<ABFT_SYM_LOWER, C::CC, C::CQ, RK>(buf, r, jl0, grp[q]); break;
+            case ABFT_LOWER: masked_rowsum_fast<ABFT_LOWER, C::CC, C::CQ, RK>(buf, r, jl0, grp[q]); break;
+            case ABFT_UNIT_LOWER: masked_rowsum_fast<ABFT_UNIT_LOWER, C::CC, C::CQ, RK>(buf, r, jl0, grp[q]); break;
+            default: masked_rowsum_fast<ABFT_UPPER, C::CC, C::CQ, RK>(buf, r, jl0, grp[q]); break;
           }
         }
       }
