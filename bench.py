@@ -49,14 +49,14 @@ def peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def ncu_traffic():
+def ncu_traffic(n=None, nb=None):
     """dram read+write bytes per launch of the dominant kernel from the
-    committed `ncu --set full` summary (profiles/), or None."""
+    committed `ncu --set full` summary (profiles/) of the same (n, nb), or None."""
     p = os.path.join(ROOT, "profiles", "ncu_verify_summary.json")
     try:
         with open(p) as f:
             d = json.load(f)
-        if d.get("n") == N_MAT and d.get("nb") == NB:
+        if d.get("n") == (n or N_MAT) and d.get("nb") == (nb or NB):
             return float(d["dram_bytes_per_launch"])
     except Exception:
         pass
@@ -209,9 +209,17 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # BENCH_SHARED_GPU=1 (tests only): every rank on cuda:0 over gloo, so the
+    # N>1 code path can be exercised on a one-GPU box; numbers are not valid
+    shared = os.environ.get("BENCH_SHARED_GPU") == "1"
+    if shared:
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     n, nb = args.n, NB
     es = 8
     # ---- workload: each rank holds its own n x n block-cyclic share (weak) ----
@@ -337,10 +345,11 @@ def run_ours(args):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"encode+verify(+locate) fp64 n={n} nb={nb} per GPU, U(-1,1), full matrix "
                                    f"(BASELINE configs[3] shape at the n={N_MAT} metric size)",
-                       "n": n, "nb": nb, "tiles_per_gpu": (n // nb) ** 2, "l2": "inputs larger than L2 (7.55 GB/pass)",
+                       "n": n, "nb": nb, "tiles_per_gpu": (n // nb) ** 2, "l2": f"inputs larger than L2 ({pass_bytes / 1e9:.2f} GB/pass vs "
+                                                         f"{torch.cuda.get_device_properties(0).L2_cache_size / 1e6:.0f} MB L2)",
                        "parallelism": f"tiles block-cyclic, dp{world}", "ft_potrf_n": args.potrf_n},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": ncu_traffic(), "kernel": dom,
+                         "frac": achieved / peak, "traffic": ncu_traffic(n, nb), "kernel": dom,
                          "bytes_per_launch": pass_bytes, "ms_per_launch": dom_ms, "peak_source": peak_src,
                          "encode_GBs": pass_bytes / (enc_ms / 1e3) / 1e9,
                          "verify_GBs": pass_bytes / (ver_ms / 1e3) / 1e9,
@@ -548,7 +557,7 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=N_MAT)
+    ap.add_argument("--matrix-n", dest="n", type=int, default=N_MAT)  # not "--n": torchrun would take it
     ap.add_argument("--potrf-n", type=int, default=N_MAT)
     ap.add_argument("--potrf-reps", type=int, default=3)
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
