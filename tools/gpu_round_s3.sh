@@ -3,6 +3,7 @@
 # of the checksum pass (reduced to CSV on the box), ft_potrf kernel breakdown.
 mkdir -p gpurun_out/s3
 python __graft_entry__.py smoke > gpurun_out/s3/smoke.log 2>&1; tail -1 gpurun_out/s3/smoke.log
+python -m pytest tests -q -m gpu > gpurun_out/s3/gpu_tests.log 2>&1; tail -1 gpurun_out/s3/gpu_tests.log
 timeout 1200 python bench.py --steps 10 --warmup 3 > gpurun_out/s3/bench.log 2>&1
 tail -1 gpurun_out/s3/bench.log | cut -c1-300
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/s3/bench_launches.csv \
