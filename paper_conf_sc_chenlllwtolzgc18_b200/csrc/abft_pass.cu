@@ -511,9 +511,9 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
       consumer_sync();
     }
     // ---------------- phase A: column sums (one warp per column) ----------
+    // this warp's columns of the stage: (s*CC + cc) % kWarps == warp (no per-column skip test)
 #pragma unroll 1
-    for (int cc = 0; cc < C::CC; ++cc) {
-      if (((s * C::CC + cc) & (kWarps - 1)) != warp) continue;
+    for (int cc = (warp - s * C::CC) & (kWarps - 1); cc < C::CC; cc += kWarps) {
       const int jl = c0 + s * C::CC + cc;  // tile-local column
       const T* col = buf + cc * RK;
       if (viewA == ABFT_GENERAL) {
