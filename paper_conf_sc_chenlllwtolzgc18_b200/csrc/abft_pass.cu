@@ -50,7 +50,12 @@ struct PassCfg {
   // keep the whole CTA <= ~110 KiB (2 CTAs / SM): ring = budget - side area.
   // Side area: SYM column sums / maintained column checksums, and for verify
   // the recomputed column sums (compared after the stage loop, see below)
-  static constexpr int REC_ELEMS = VERIFY ? RK * 3 : 0;
+  // verify parks the recomputed column sums of a non-SYM tile in the SYM
+  // area (a SYM tile keeps its column sums there and parks nothing), so the
+  // side area is RK*3 for both; the maintained checksums are read from
+  // global memory at compare time (a 12 KiB smaller side area gives fp64
+  // nb=512 verify a third 32 KiB ring stage)
+  static constexpr int REC_ELEMS = 0;
   static constexpr int SIDE_BYTES = (RK * 3 + REC_ELEMS) * (int)sizeof(T);
   static constexpr int RING_BYTES = RK >= 256 ? (96 * 1024 < 108 * 1024 - SIDE_BYTES ? 96 * 1024
                                                                                         : 108 * 1024 - SIDE_BYTES)
@@ -344,8 +349,8 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
   extern __shared__ __align__(128) unsigned char smem_raw[];
   T* ring = reinterpret_cast<T*>(smem_raw);
   T* symacc = ring + (size_t)C::NSTAGE * C::STAGE_ELEMS;  // [K][3][NB]
-  T* rec = symacc + 3 * RK;                               // verify: recomputed [K][3][NB]
-  uint64_t* full = reinterpret_cast<uint64_t*>(rec + C::REC_ELEMS);
+  T* rec = symacc;                                        // verify: recomputed [K][3][NB] (non-SYM tiles)
+  uint64_t* full = reinterpret_cast<uint64_t*>(symacc + 3 * RK + C::REC_ELEMS);
   uint64_t* empty = full + C::NSTAGE;
   __shared__ int s_colflags[K], s_ncols[K], s_nrows[K], s_rowflags[K];
   __shared__ int s_last;
@@ -424,21 +429,6 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
     my_colflags[t] = 0;
     my_ncols[t] = 0;
   }
-  // verify: fetch the maintained column checksums (and magnitudes) of this
-  // slab once, while the TMA prologue is in flight, instead of one dependent
-  // strided load per column inside the stage loop.  For non-SYM tiles the
-  // SYM area is free and holds them: per tile [e | w | mag] x cols.
-  if (VERIFY && !sym && (p.which & ABFT_COL)) {
-    for (int idx = tid; idx < kv * cols; idx += kThreads) {
-      const int t = idx / cols, c = idx - t * cols;
-      const int64_t gj = (int64_t)J * NB + c0 + c;
-      T* sa = symacc + (size_t)t * 3 * NB;
-      sa[c] = colchk[(int64_t)2 * (Ib + t) + gj * p.ldc];
-      sa[NB + c] = colchk[(int64_t)2 * (Ib + t) + 1 + gj * p.ldc];
-      if (p.use_mag) sa[2 * NB + c] = colmag[(Ib + t) + gj * p.ldcm];
-    }
-    consumer_sync();
-  }
   // column finish of tile row Ib+t: encode writes c (and m_c); verify compares (c-6, c-7)
   auto finish_col = [&](int t, int jl, T pe, T pw, T pa) {
     if (sym) {
@@ -466,20 +456,20 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
       rc[2 * NB + idx] = pa;
     }
   };
-  // verify: compare the slab's columns (maintained in symacc, recomputed in rec)
+  // verify: compare the slab's columns (recomputed in rec, maintained from global)
   auto compare_cols = [&]() {
 #pragma unroll
     for (int t = 0; t < K; ++t) {
       if (t >= kv) break;
       const int I = Ib + t;
-      const T* sa = symacc + (size_t)t * 3 * NB;
       const T* rc = rec + (size_t)t * 3 * NB;
       for (int idx = tid; idx < cols; idx += kThreads) {
         const int64_t gj = (int64_t)J * NB + c0 + idx;
+        const T me = colchk[(int64_t)2 * I + gj * p.ldc], mw = colchk[(int64_t)2 * I + 1 + gj * p.ldc];
         const T pe = rc[idx], pw = rc[NB + idx], pa = rc[2 * NB + idx];
-        const double m = p.use_mag ? (double)sa[2 * NB + idx] : (double)pa;
+        const double m = p.use_mag ? (double)colmag[I + gj * p.ldcm] : (double)pa;
         T de, dw;
-        const int f = check_pair<T>(sa[idx], sa[NB + idx], pe, pw, m, p.tau_fac, NB, &de, &dw);
+        const int f = check_pair<T>(me, mw, pe, pw, m, p.tau_fac, NB, &de, &dw);
         if (dcol) {
           dcol[(int64_t)2 * I + gj * p.ldc] = de;
           dcol[(int64_t)2 * I + 1 + gj * p.ldc] = dw;
