@@ -136,6 +136,21 @@ class Clocks:
 
 
 # ------------------------------------------------------------- reference --
+def workload_config(n, nb, world, potrf_n):
+    """The `config` object of both arms' JSON lines (same workload named)."""
+    try:
+        import torch
+
+        l2 = torch.cuda.get_device_properties(0).L2_cache_size if torch.cuda.is_available() else 126 * 2 ** 20
+    except Exception:
+        l2 = 126 * 2 ** 20
+    return {"workload": f"encode+verify(+locate) fp64 n={n} nb={nb} per GPU, U(-1,1), full matrix "
+                        f"(BASELINE configs[3] shape at the n={N_MAT} metric size)",
+            "n": n, "nb": nb, "tiles_per_gpu": (n // nb) ** 2,
+            "l2": f"inputs larger than L2 ({alg_bytes(n, nb, 8) / 1e9:.2f} GB/pass vs {l2 / 1e6:.0f} MB L2)",
+            "parallelism": f"tiles block-cyclic, dp{world}", "ft_potrf_n": potrf_n}
+
+
 def run_reference(args):
     """The oracle on the host cores: encode + verify of a bounded sample of
     nb x nb tiles of the same fp64 U(-1,1) workload, same byte formula."""
@@ -167,10 +182,10 @@ def run_reference(args):
         "impl": "reference", "metric": METRIC, "value": val, "unit": "GB/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": f"encode+verify fp64 nb={nb}, oracle sample of {n_tiles_sample} tiles per step "
-                               f"(of the n={N_MAT} matrix)", "n": N_MAT, "nb": nb},
+        "config": workload_config(args.n, nb, int(os.environ.get("WORLD_SIZE", "1")), args.potrf_n),
         "cpu_baseline": {"value": val, "unit": "GB/s", "cores": cores, "kind": "oracle",
-                         "sample": f"{n_tiles_sample} tiles of {nb}x{nb} fp64 per step"},
+                         "sample": f"{n_tiles_sample} tiles of {nb}x{nb} fp64 per step (a bounded sample of the "
+                                   f"n={args.n} workload; GB/s with the same per-tile byte formula)"},
         "e2e": {"value": val, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -343,11 +358,7 @@ def run_ours(args):
             "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"encode+verify(+locate) fp64 n={n} nb={nb} per GPU, U(-1,1), full matrix "
-                                   f"(BASELINE configs[3] shape at the n={N_MAT} metric size)",
-                       "n": n, "nb": nb, "tiles_per_gpu": (n // nb) ** 2, "l2": f"inputs larger than L2 ({pass_bytes / 1e9:.2f} GB/pass vs "
-                                                         f"{torch.cuda.get_device_properties(0).L2_cache_size / 1e6:.0f} MB L2)",
-                       "parallelism": f"tiles block-cyclic, dp{world}", "ft_potrf_n": args.potrf_n},
+            "config": workload_config(n, nb, world, args.potrf_n),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": ncu_traffic(n, nb), "kernel": dom,
                          "bytes_per_launch": pass_bytes, "ms_per_launch": dom_ms, "peak_source": peak_src,
