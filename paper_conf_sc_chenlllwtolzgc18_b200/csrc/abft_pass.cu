@@ -438,17 +438,9 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
       return;
     }
     if (!(p.which & ABFT_COL)) return;
-    const int I = Ib + t;
-    const int64_t gj = (int64_t)J * NB + jl;
-    if (!VERIFY) {
-      T* cc2 = colchk + (int64_t)2 * I + gj * p.ldc;
-      cc2[0] = pe;
-      cc2[1] = pw;
-      if (colmag) colmag[I + gj * p.ldcm] = pa;
-    } else {
-      // verify: park the recomputed sums; the comparisons run after the stage
-      // loop, one column per thread (a per-column compare by one lane inside
-      // the loop serialised the warps: fp32 nb=256 verify 3.9 vs 5.4 TB/s)
+    {  // park the sums; encode's stores / verify's comparisons run after the
+      // stage loop, one column per thread (a per-column compare by one lane
+      // inside the loop serialised the warps: fp32 nb=256 verify 3.9 vs 5.4 TB/s)
       T* rc = rec + (size_t)t * 3 * NB;
       const int idx = jl - c0;
       rc[idx] = pe;
@@ -615,9 +607,25 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
   }
 
   // ---------------- column flags of this CTA ------------------------------
-  if (VERIFY && !sym && (p.which & ABFT_COL)) {
+  if (!sym && (p.which & ABFT_COL)) {
     consumer_sync();  // every column of the slab is parked in rec
-    compare_cols();
+    if (VERIFY) {
+      compare_cols();
+    } else {  // encode: one column per thread
+#pragma unroll
+      for (int t = 0; t < K; ++t) {
+        if (t >= kv) break;
+        const int I = Ib + t;
+        const T* rc = rec + (size_t)t * 3 * NB;
+        for (int idx = tid; idx < cols; idx += kThreads) {
+          const int64_t gj = (int64_t)J * NB + c0 + idx;
+          T* cc2 = colchk + (int64_t)2 * I + gj * p.ldc;
+          cc2[0] = rc[idx];
+          cc2[1] = rc[NB + idx];
+          if (colmag) colmag[I + gj * p.ldcm] = rc[2 * NB + idx];
+        }
+      }
+    }
   }
   if (VERIFY) {
 #pragma unroll
