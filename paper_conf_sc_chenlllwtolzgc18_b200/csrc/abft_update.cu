@@ -161,16 +161,6 @@ static cublasStatus_t gemm(cublasHandle_t h, cublasOperation_t ta, cublasOperati
                            float* C, int ldc) {
   return cublasSgemm(h, ta, tb, m, n, k, al, A, lda, B, ldb, be, C, ldc);
 }
-static cublasStatus_t trsm(cublasHandle_t h, cublasSideMode_t sd, cublasFillMode_t ul, cublasOperation_t tr,
-                           cublasDiagType_t dg, int m, int n, const double* al, const double* A, int lda, double* B,
-                           int ldb) {
-  return cublasDtrsm(h, sd, ul, tr, dg, m, n, al, A, lda, B, ldb);
-}
-static cublasStatus_t trsm(cublasHandle_t h, cublasSideMode_t sd, cublasFillMode_t ul, cublasOperation_t tr,
-                           cublasDiagType_t dg, int m, int n, const float* al, const float* A, int lda, float* B,
-                           int ldb) {
-  return cublasStrsm(h, sd, ul, tr, dg, m, n, al, A, lda, B, ldb);
-}
 
 static cublasOperation_t op_of(char t) { return (t == 'T' || t == 't') ? CUBLAS_OP_T : CUBLAS_OP_N; }
 

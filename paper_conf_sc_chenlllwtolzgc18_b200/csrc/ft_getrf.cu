@@ -353,11 +353,6 @@ __global__ void lu_invert_perm_kernel(const int32_t* src, const int32_t* nrows, 
   for (int s = threadIdx.x; s < n; s += blockDim.x) sinv[src[s]] = s;
 }
 
-static unsigned blocks_for(int64_t work, int per) {
-  int64_t g = (work + per - 1) / per;
-  return (unsigned)(g < 1 ? 1 : (g > 148 * 32 ? 148 * 32 : g));
-}
-
 }  // namespace abft
 
 // ------------------------------------------------------------ panel getrf --
