@@ -40,9 +40,11 @@ struct PassCfg {
   static constexpr int RK = K * NB;              // rows per CTA
   static constexpr int GC = NB < 64 ? NB : 64;  // group columns (slab granularity)
   static constexpr int COL_BYTES = RK * (int)sizeof(T);
-  // ~32 KiB stages, 16 KiB when a column is 8 KiB so that the ring still
-  // holds >= 4 stages within the 2-CTAs-per-SM budget
-  static constexpr int STAGE_TARGET = COL_BYTES >= 8192 ? 16 * 1024 : 32 * 1024;
+  // 32 KiB stages for every column size (fp64 nb=1024, 8-KiB columns, had
+  // 16 KiB stages of 2 columns: the row-sum chunk CQ fell to 2 columns, the
+  // per-chunk work per element rose ~1.5x, and the pass ran at 5.1-6.1 TB/s;
+  // with 4-column stages 6.3-7.0 TB/s, pass_views r01)
+  static constexpr int STAGE_TARGET = 32 * 1024;
   static constexpr int CC_RAW = STAGE_TARGET / COL_BYTES;
   static constexpr int CC = CC_RAW < GC ? (CC_RAW < 1 ? 1 : CC_RAW) : GC;  // columns per stage
   static constexpr int STAGE_ELEMS = CC * RK;
@@ -75,7 +77,7 @@ struct PassCfg {
   static constexpr int KBIG_RAW = 4096 / (NB * (int)sizeof(T));
   static constexpr int KBIG = KBIG_RAW < 1 ? 1 : (KBIG_RAW > 8 ? 8 : KBIG_RAW);
   static constexpr int COLB_BIG = KBIG * NB * (int)sizeof(T);
-  static constexpr int CC_BIG_RAW = (COLB_BIG >= 8192 ? 16 * 1024 : 32 * 1024) / COLB_BIG;
+  static constexpr int CC_BIG_RAW = (32 * 1024) / COLB_BIG;
   static constexpr int CQ = CC_BIG_RAW < GC ? (CC_BIG_RAW < 1 ? 1 : CC_BIG_RAW) : GC;
   static_assert(CC % CQ == 0, "row-sum chunk must divide the stage");
   static constexpr size_t SMEM = (size_t)NSTAGE * STAGE_BYTES   // ring
