@@ -60,6 +60,12 @@ Handles& handles_for(cudaStream_t s) {
   cusolverDnCreate(&h->solver);
   cublasSetStream(h->blas, s);
   cusolverDnSetStream(h->solver, s);
+  // A fixed cuBLAS workspace: without one cuBLAS allocates stream-ordered
+  // memory inside graph capture, which the drivers' device-decided restart
+  // (a graph IF body) cannot hold.
+  void* ws = nullptr;
+  const size_t ws_bytes = size_t(64) << 20;
+  if (cudaMalloc(&ws, ws_bytes) == cudaSuccess) cublasSetWorkspace(h->blas, ws, ws_bytes);
   (*m)[key] = h;
   return *h;
 }

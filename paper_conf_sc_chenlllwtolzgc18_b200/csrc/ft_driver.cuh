@@ -48,6 +48,11 @@ struct ft_ctx {
   int32_t* hpin = nullptr;  // pinned host words (read-backs), mapped into the device address space
   int32_t* hpin_dev = nullptr;  // device alias of hpin (a kernel writes read-back words straight to the host)
   cudaEvent_t ev = nullptr;  // marks the PD-check read-back (restart decision)
+  // The drivers run on a private non-blocking stream joined to `stream` at
+  // entry and exit: the device-decided restart captures its redo into a
+  // graph, and the legacy default stream cannot be captured.
+  cudaStream_t drv = nullptr;
+  cudaEvent_t join = nullptr;
   // FT_PD_HOST (ft_host.cu): host LAPACK, pinned panel staging, device guard
   void* lapack = nullptr;  // dlopen handle
   void* lp[6] = {};        // dpotrf spotrf dgetrf sgetrf dgeqrf sgeqrf
@@ -80,6 +85,20 @@ static __global__ void drv_delta_to_host_kernel(const int32_t* now, const int32_
   *host = *now - *snap;
 }
 static __global__ void drv_word_to_host_kernel(const int32_t* src, volatile int32_t* host) { *host = *src; }
+
+// Device-decided restart (f1): did the post-op check add uncorrectable
+// errors?  Then take them back (the redo re-checks), count the restart and
+// the redo's check, and open the IF node holding the redo.
+static __global__ void drv_restart_cond_kernel(cudaGraphConditionalHandle h, int32_t* uncorrectable,
+                                               const int32_t* snap, int32_t* restarts, int32_t* runs, int32_t nchk) {
+  const int32_t delta = *uncorrectable - *snap;
+  if (delta > 0) {
+    *uncorrectable = *snap;
+    ++*restarts;
+    *runs += nchk;
+  }
+  cudaGraphSetConditional(h, delta > 0 ? 1u : 0u);
+}
 
 // Fig. 4b gate: did the fixes logged since the start of the iteration include
 // a 1D pattern (class 1D_ROW / 1D_COL)?  Counts the gated checks that run.
@@ -135,7 +154,13 @@ struct Driver {
   int setup(ft_ctx* ctx, int32_t dt, int64_t n_, int64_t nb_, void* dA, int64_t lda_, const ft_opts_t* opts,
             bool is_lu) {
     c = ctx;
-    s = ctx->stream;
+    if (!c->drv) {
+      ABFT_CUDA_TRY(cudaStreamCreateWithFlags(&c->drv, cudaStreamNonBlocking));
+      ABFT_CUDA_TRY(cudaEventCreateWithFlags(&c->join, cudaEventDisableTiming));
+    }
+    ABFT_CUDA_TRY(cudaEventRecord(c->join, c->stream));
+    ABFT_CUDA_TRY(cudaStreamWaitEvent(c->drv, c->join, 0));
+    s = c->drv;
     dtype = dt;
     n = n_;
     nb = nb_;
@@ -302,6 +327,111 @@ struct Driver {
     FT_TRY(post_delta(0));
     return wait_delta(0, delta);
   }
+  // The same decision without the host wait: `redo` (the restore + redo +
+  // re-check) is stream-captured into the body of a CUDA-graph IF node whose
+  // condition drv_restart_cond_kernel sets on the device from the snapshot
+  // taken before the check; the graph is launched on s and freed on
+  // completion.  Host waits: none.  Restarts and the redo's check are
+  // counted on the device (counts[28], counts[26]).
+  // Opt-in (ABFT_RESTART_DEVICE=1, read per call): measured on B200 at
+  // n=30720 the per-iteration capture + instantiation costs the host more
+  // than the stream drain it removes (ft_potrf 341 vs 338 ms).
+  bool device_restart_ok() const {
+    const char* v = getenv("ABFT_RESTART_DEVICE");
+    return v && v[0] == '1';
+  }
+  template <typename F>
+  int device_restart(F&& redo) {
+    cudaError_t e = cudaSuccess;
+    const char* where = "";
+#define DR_TRY(x)          \
+  if (e == cudaSuccess) {  \
+    e = (x);               \
+    where = #x;            \
+  }
+    cudaGraph_t g = nullptr;
+    ABFT_CUDA_TRY(cudaGraphCreate(&g, 0));
+    cudaGraphConditionalHandle ch{};
+    cudaGraph_t body = nullptr;
+    cudaGraphNode_t setn = nullptr, ifn = nullptr;
+    int32_t nchk = 0;
+    cudaKernelNodeParams kp{};
+    int32_t* unc = counts + ABFT_CNT_UNCORRECTABLE;
+    int32_t* rsc = counts + 28;
+    void* args[] = {&ch, &unc, &snap, &rsc, &gated_runs, &nchk};
+    kp.func = (void*)drv_restart_cond_kernel;
+    kp.gridDim = dim3(1);
+    kp.blockDim = dim3(1);
+    kp.kernelParams = args;
+    cudaGraphNodeParams cp{};
+    cp.type = cudaGraphNodeTypeConditional;
+    cp.conditional.type = cudaGraphCondTypeIf;
+    cp.conditional.size = 1;
+    DR_TRY(cudaGraphConditionalHandleCreate(&ch, g, 0, 0));
+    cp.conditional.handle = ch;
+    DR_TRY(cudaGraphAddKernelNode(&setn, g, nullptr, 0, &kp));
+    DR_TRY(cudaGraphAddNode(&ifn, g, &setn, 1, &cp));
+    if (e == cudaSuccess) body = cp.conditional.phGraph_out[0];
+    DR_TRY(cudaStreamBeginCaptureToGraph(s, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
+    int rrc = 0;
+    if (e == cudaSuccess) {
+      const int checks0 = n_checks;
+      rrc = redo();
+      nchk = n_checks - checks0;
+      n_checks = checks0;  // counted on the device when the redo runs
+      cudaGraph_t out = body;
+      DR_TRY(cudaStreamEndCapture(s, &out));
+      DR_TRY(cudaGraphKernelNodeSetParams(setn, &kp));  // nchk now known
+    }
+    cudaGraphExec_t ge = nullptr;
+    bool fallback = false;
+    if (!rrc && e == cudaSuccess) {
+      cudaGraphInstantiateParams ip{};
+      if (cudaGraphInstantiateWithParams(&ge, g, &ip) != cudaSuccess) {
+        // A body the driver cannot run conditionally (e.g. a library kernel
+        // launched with attributes IF bodies reject): take the decision on the
+        // host for this op instead (the redo above was only captured).
+        (void)cudaGetLastError();
+        static bool told = false;
+        if (!told && getenv("ABFT_DEBUG_RESTART_GRAPH")) {
+          told = true;
+          size_t nn = 0;
+          cudaGraphGetNodes(body, nullptr, &nn);
+          std::vector<cudaGraphNode_t> nodes(nn);
+          cudaGraphGetNodes(body, nodes.data(), &nn);
+          fprintf(stderr, "[abft] restart graph not instantiable (result %d, node %p); body nodes:", (int)ip.result_out,
+                  (void*)ip.errNode_out);
+          for (auto nd : nodes) {
+            cudaGraphNodeType ty;
+            cudaGraphNodeGetType(nd, &ty);
+            fprintf(stderr, " %d%s", (int)ty, nd == ip.errNode_out ? "*" : "");
+          }
+          fprintf(stderr, "\n");
+        }
+        ge = nullptr;
+        fallback = true;
+      } else {
+        DR_TRY(cudaGraphLaunch(ge, s));
+      }
+    }
+#undef DR_TRY
+    if (ge) cudaGraphExecDestroy(ge);  // freed when the launch completes
+    cudaGraphDestroy(g);
+    if (fallback) {
+      int delta = 0;
+      FT_TRY(uncorrectable_added(&delta));
+      if (delta > 0) {
+        FT_TRY(take_back_uncorrectable(delta));
+        FT_TRY(redo());
+      }
+      return 0;
+    }
+    if (e != cudaSuccess) {
+      fprintf(stderr, "[abft] device restart graph: %s failed: %s\n", where, cudaGetErrorString(e));
+      return ABFT_E_CUDA;
+    }
+    return rrc;
+  }
   int take_back_uncorrectable(int delta) {
     ++restarts;
     drv_add_i32_kernel<<<1, 1, 0, s>>>(counts + ABFT_CNT_UNCORRECTABLE, -delta);
@@ -346,6 +476,8 @@ struct Driver {
     if (o->fix_log && o->fix_log_cap > 0)
       ABFT_CUDA_TRY(cudaMemcpyAsync(o->fix_log, c->fixlog, sizeof(abft_fix_t) * std::min(o->fix_log_cap, c->fixcap),
                                     cudaMemcpyDeviceToDevice, s));
+    ABFT_CUDA_TRY(cudaEventRecord(c->join, s));
+    ABFT_CUDA_TRY(cudaStreamWaitEvent(c->stream, c->join, 0));
     ABFT_CUDA_TRY(cudaStreamSynchronize(s));
     auto t1 = std::chrono::steady_clock::now();
     // layout after counts: nfix(8) mark(9) info(10) rep(11,12) info_total(13)
@@ -357,7 +489,7 @@ struct Driver {
       stats->repairs_skipped = h[12];
       stats->uncorrectable = h[ABFT_CNT_UNCORRECTABLE];
       stats->n_checks = n_checks + h[26];
-      stats->restarts = restarts;
+      stats->restarts = restarts + h[28];
       stats->ms_total = std::chrono::duration<double, std::milli>(t1 - t0).count();
       int32_t* x = &stats->xfer_d2h_flagged;
       for (int i = 0; i < 7; ++i) x[i] = xs[i];

@@ -605,10 +605,7 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft) {
       if (rs) FT_TRY(d.snap_uncorrectable());
       FT_TRY(post_pd_checks());
-      int delta = 0;
-      if (rs) FT_TRY(d.uncorrectable_added(&delta));
-      if (delta > 0) {  // 2D after the PD: undo its swaps, restore the copy, redo
-        FT_TRY(d.take_back_uncorrectable(delta));
+      auto pd_redo = [&]() -> int {  // 2D after the PD: undo its swaps, restore the copy, redo
         FT_TRY(panel_getrf_undo(&d.M, k, s));
         FT_TRY(d.copy(d.a_at(r0, r0), lda, cp_a, mk, mk, nb));
         FT_TRY(d.copy(d.colchk_at(2 * k, r0), d.M.ldc, cp_c, 2 * ntk, 2 * ntk, nb));
@@ -616,7 +613,16 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
         FT_TRY(d.copy(d.rowchk_at(r0, 2 * k), d.M.ldr, cp_r, mk, mk, 2));
         FT_TRY(d.copy(d.rowmag_at(r0, k), d.M.ldrm, cp_rm, mk, mk, 1));
         FT_TRY(do_pd());
-        FT_TRY(post_pd_checks());
+        return post_pd_checks();
+      };
+      // (The PD redo stays a host decision: cuSOLVER's getrf captured into a
+      // graph IF body crashed at nb = 1024 on B200; the PU redo below is
+      // device-decided.)
+      int delta = 0;
+      if (rs) FT_TRY(d.uncorrectable_added(&delta));
+      if (delta > 0) {
+        FT_TRY(d.take_back_uncorrectable(delta));
+        FT_TRY(pd_redo());
       }
     }
     if (k == nt - 1) break;
@@ -675,16 +681,23 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft) {
       if (rs) FT_TRY(d.snap_uncorrectable());
       FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW));
-      int delta = 0;
-      if (rs) FT_TRY(d.uncorrectable_added(&delta));
-      if (delta > 0) {
-        FT_TRY(d.take_back_uncorrectable(delta));
+      auto pu_redo = [&]() -> int {
         FT_TRY(d.copy(d.a_at(r0, r1), lda, pu_a, nb, nb, nk));
         FT_TRY(d.copy(d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, pu_r, nb, nb, m2));
         FT_TRY(d.copy(d.rowmag_at(r0, k + 1), d.M.ldrm, pu_rm, nb, nb, m2 / 2));
         FT_TRY(pu_data());
         FT_TRY(pu_chk());
-        FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW));
+        return d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW);
+      };
+      int delta = 0;
+      if (rs && d.device_restart_ok()) {
+        FT_TRY(d.device_restart(pu_redo));
+      } else if (rs) {
+        FT_TRY(d.uncorrectable_added(&delta));
+      }
+      if (delta > 0) {
+        FT_TRY(d.take_back_uncorrectable(delta));
+        FT_TRY(pu_redo());
       }
     }
     // line 12: TMU  A22 -= L21 U12 (DGEMM on tensor cores) + c-13 rules

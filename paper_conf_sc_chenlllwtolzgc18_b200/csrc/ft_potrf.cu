@@ -190,6 +190,8 @@ extern "C" int ft_ctx_destroy(ft_ctx_t* c) {
   if (c->rsv) cudaFree(c->rsv);
   if (c->hpin) cudaFreeHost(c->hpin);
   if (c->ev) cudaEventDestroy(c->ev);
+  if (c->join) cudaEventDestroy(c->join);
+  if (c->drv) cudaStreamDestroy(c->drv);
   if (c->hstage) cudaFreeHost(c->hstage);
   if (c->dguard) cudaFree(c->dguard);
   if (c->lapack) dlclose(c->lapack);
@@ -392,20 +394,28 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft && post_checks) {
       if (rs) ABFT_CUDA_TRY(cudaMemcpyAsync(d.snap, d.counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToDevice, s));
       FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
+      auto pu_redo = [&]() -> int {
+        FT_TRY(copy2d(d.a_at(r1, r0), lda, pu_a, nk, nk, nb));
+        FT_TRY(copy2d(d.colchk_at(2 * (k + 1), r0), d.M.ldc, pu_c, m2, m2, nb));
+        FT_TRY(copy2d(d.colmag_at(k + 1, r0), d.M.ldcm, pu_m, m2 / 2, m2 / 2, nb));
+        FT_TRY(pu_data());
+        FT_TRY(pu_chk());
+        return d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL);
+      };
+      // The TMU consumes L21 right after this check, so the host wait here
+      // drains the stream; ABFT_RESTART_DEVICE=1 takes the decision on the
+      // device instead (graph IF node, Driver::device_restart).
       int delta = 0;
-      if (rs) {
+      if (rs && d.device_restart_ok() && !dbg_nosync) {
+        FT_TRY(d.device_restart(pu_redo));
+      } else if (rs) {
         FT_TRY(post_readback(d.snap));
         FT_TRY(readback_delta(&delta));
       }
       if (delta > 0) {
         ++d.restarts;
         add_i32_kernel<<<1, 1, 0, s>>>(d.counts + ABFT_CNT_UNCORRECTABLE, -delta);
-        FT_TRY(copy2d(d.a_at(r1, r0), lda, pu_a, nk, nk, nb));
-        FT_TRY(copy2d(d.colchk_at(2 * (k + 1), r0), d.M.ldc, pu_c, m2, m2, nb));
-        FT_TRY(copy2d(d.colmag_at(k + 1, r0), d.M.ldcm, pu_m, m2 / 2, m2 / 2, nb));
-        FT_TRY(pu_data());
-        FT_TRY(pu_chk());
-        FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
+        FT_TRY(pu_redo());
       }
     }
     // prior-operation scheme [11]: the TMU's inputs (panel, trailing matrix) before it

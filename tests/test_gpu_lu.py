@@ -172,7 +172,10 @@ def _gpu_getrf_rs(lib, ctx, A_np, nb, inject, restart):
     (1, dr.AT_PRE_PD, dr.KIND_PERSIST, 64, 64, 55),
     (2, dr.AT_PRE_PU, dr.KIND_ONCHIP, 140, 130, 60),   # L_kk read by the PU: U12 2D
 ])
-def test_lu_restart_parity(lib, ctx, k, point, kind, gi, gj, bit):
+@pytest.mark.parametrize("device_decided", [False, True])
+def test_lu_restart_parity(lib, ctx, k, point, kind, gi, gj, bit, device_decided, monkeypatch):
+    if device_decided:  # the PU restart decided on the device (graph IF node); the PD one stays on the host
+        monkeypatch.setenv("ABFT_RESTART_DEVICE", "1")
     nb = 64
     A = si.general(256, seed=31)
     inj = [dr.Inject(k, point, kind, 0, gi, gj, (bit,))]
