@@ -415,6 +415,12 @@ typedef struct {
   int32_t ctf_recomputed;       /* T recomputed from V after a flagged check */
 } ft_stats_t;
 
+/* A driver context on `device`; the ft_* drivers are ordered on `stream`
+ * (any stream, the legacy default one included): internally they run on a
+ * private non-blocking stream of the context that waits for `stream` at entry
+ * and that `stream` waits for at exit (so the optional device-decided restart
+ * below can capture its redo into a CUDA graph).  Owned by the caller; free
+ * with ft_ctx_destroy. */
 ABFT_API int ft_ctx_create(ft_ctx_t **ctx, int32_t device, abft_stream_t stream);
 ABFT_API int ft_ctx_destroy(ft_ctx_t *ctx);
 
@@ -432,9 +438,12 @@ ABFT_API int ft_ctx_set_host_lapack(ft_ctx_t *ctx, const char *path);
  * -> check L_kk (LOWER, c) -> check panel A_ik (both) -> PU + a5 -> check
  * L_ik (c) -> TMU (DSYRK on tensor cores) + a6 -> heuristic re-check of L_ik
  * (Fig. 4a) with the guarded trailing repair (c-25).  Checksums are
- * allocated inside ctx.  Synchronises the host once at the end.  Returns
- * ABFT_E_UNCORRECTABLE if a 2D error remained (restart is out of scope,
- * DESIGN.md §8).  *info (host) follows LAPACK potrf. */
+ * allocated inside ctx.  Synchronises the host once at the end, plus one
+ * wait per post-op check when opts->restart (the local-restart decision, f1
+ * L430; with the environment variable ABFT_RESTART_DEVICE=1 the post-PU
+ * decision is taken on the device by a CUDA-graph IF node instead, DESIGN.md
+ * §2.10).  Returns ABFT_E_UNCORRECTABLE if a 2D error remained after the
+ * restart (or without it).  *info (host) follows LAPACK potrf. */
 ABFT_API int ft_potrf(ft_ctx_t *ctx, int32_t dtype, int64_t n, void *dA, int64_t lda,
              const ft_opts_t *opts, ft_stats_t *stats, int64_t *info);
 
