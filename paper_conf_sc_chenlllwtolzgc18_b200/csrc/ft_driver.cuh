@@ -151,6 +151,16 @@ struct Driver {
   int ctf_flagged = 0, ctf_recomputed = 0;
   std::vector<std::pair<int, int>> xfer_used;  // (iter, point) transfer faults already applied
 
+  Driver() = default;
+  Driver(const Driver&) = delete;
+  Driver& operator=(const Driver&) = delete;
+  // Every exit (error returns included) orders the caller's stream after the
+  // work queued on the private one.
+  ~Driver() {
+    if (c && c->drv && s == c->drv && cudaEventRecord(c->join, s) == cudaSuccess)
+      cudaStreamWaitEvent(c->stream, c->join, 0);
+  }
+
   int setup(ft_ctx* ctx, int32_t dt, int64_t n_, int64_t nb_, void* dA, int64_t lda_, const ft_opts_t* opts,
             bool is_lu) {
     c = ctx;
