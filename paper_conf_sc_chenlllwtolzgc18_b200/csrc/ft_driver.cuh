@@ -157,9 +157,14 @@ struct Driver {
   // Every exit (error returns included) orders the caller's stream after the
   // work queued on the private one.
   ~Driver() {
+    if (rs_exec) cudaGraphExecDestroy(rs_exec);  // freed when its queued launches complete
+    if (rs_instantiations && getenv("ABFT_DEBUG_RESTART_GRAPH"))
+      fprintf(stderr, "[abft] restart graphs: %d instantiated, %d updated\n", rs_instantiations, rs_updates);
     if (c && c->drv && s == c->drv && cudaEventRecord(c->join, s) == cudaSuccess)
       cudaStreamWaitEvent(c->stream, c->join, 0);
   }
+  cudaGraphExec_t rs_exec = nullptr;  // device-decided restart: the last executable graph
+  int rs_instantiations = 0, rs_updates = 0;
 
   int setup(ft_ctx* ctx, int32_t dt, int64_t n_, int64_t nb_, void* dA, int64_t lda_, const ft_opts_t* opts,
             bool is_lu) {
@@ -395,6 +400,25 @@ struct Driver {
     }
     cudaGraphExec_t ge = nullptr;
     bool fallback = false;
+    if (!rrc && e == cudaSuccess && rs_exec) {
+      // Same topology as the previous iteration's graph (the usual case):
+      // update the executable graph in place instead of instantiating anew
+      // (launches already queued keep their parameters).
+      cudaGraphExecUpdateResultInfo ui{};
+      if (cudaGraphExecUpdate(rs_exec, g, &ui) == cudaSuccess) {
+        ++rs_updates;
+        DR_TRY(cudaGraphLaunch(rs_exec, s));
+        cudaGraphDestroy(g);
+        if (e != cudaSuccess) {
+          fprintf(stderr, "[abft] device restart graph: %s failed: %s\n", where, cudaGetErrorString(e));
+          return ABFT_E_CUDA;
+        }
+        return 0;
+      }
+      (void)cudaGetLastError();
+      cudaGraphExecDestroy(rs_exec);  // freed when its queued launches complete
+      rs_exec = nullptr;
+    }
     if (!rrc && e == cudaSuccess) {
       cudaGraphInstantiateParams ip{};
       if (cudaGraphInstantiateWithParams(&ge, g, &ip) != cudaSuccess) {
@@ -421,11 +445,14 @@ struct Driver {
         ge = nullptr;
         fallback = true;
       } else {
+        ++rs_instantiations;
         DR_TRY(cudaGraphLaunch(ge, s));
+        rs_exec = ge;  // kept for the next iteration's update
+        ge = nullptr;
       }
     }
 #undef DR_TRY
-    if (ge) cudaGraphExecDestroy(ge);  // freed when the launch completes
+    if (ge) cudaGraphExecDestroy(ge);
     cudaGraphDestroy(g);
     if (fallback) {
       int delta = 0;
