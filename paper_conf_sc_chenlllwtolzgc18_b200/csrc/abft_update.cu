@@ -380,6 +380,48 @@ __global__ void syrk_scatter_row_kernel(T* __restrict__ R, int64_t ldr, const T*
   }
 }
 
+// Both scatters from one read of P (nb % 32 == 0): a block owns a 32 x 32
+// piece of P (32 columns x inside one tile column J = x / nb), stages it in
+// shared memory, adds them to C with y as the fast index and to R, through
+// the transpose, with x as the fast index — coalesced on both sides.  Same
+// element operations as the two kernels above (bit-identical results).
+template <typename T>
+__global__ void __launch_bounds__(256) syrk_scatter_kernel(T* __restrict__ C, int64_t ldc, T* __restrict__ R,
+                                                           int64_t ldr, const T* __restrict__ P, int64_t M,
+                                                           int64_t nk, int nb, int rows_per_tile, T sign) {
+  __shared__ T tile[32][33];
+  const int64_t x0 = (int64_t)blockIdx.x * 32, y0 = (int64_t)blockIdx.y * 32;
+  const int64_t J = x0 / nb;
+  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+#pragma unroll
+  for (int j = ty; j < 32; j += 8) {
+    const int64_t x = x0 + j, y = y0 + tx;
+    const bool in = x < nk && y < M;
+    const T v = in ? P[y + x * M] : T(0);
+    tile[j][tx] = v;
+    if (in && y / rows_per_tile >= J) C[y + x * ldc] += sign * v;
+  }
+  if (!R) return;
+  __syncthreads();
+#pragma unroll
+  for (int i = ty; i < 32; i += 8) {
+    const int64_t y = y0 + i, x = x0 + tx;
+    if (x < nk && y < M && J >= y / rows_per_tile) R[x + y * ldr] += sign * tile[tx][i];
+  }
+}
+
+template <typename T>
+static void scatter_both(T* C, int64_t ldc, T* R, int64_t ldr, const T* P, int64_t M, int64_t nk, int64_t nb, int rpt,
+                         T sign, cudaStream_t s) {
+  if (nb % 32 == 0) {
+    const dim3 grid((unsigned)((nk + 31) / 32), (unsigned)((M + 31) / 32));
+    syrk_scatter_kernel<T><<<grid, 256, 0, s>>>(C, ldc, R, ldr, P, M, nk, (int)nb, rpt, sign);
+    return;
+  }
+  syrk_scatter_col_kernel<T><<<grid_for(M * nk), 256, 0, s>>>(C, ldc, P, M, nk, (int)nb, rpt, sign);
+  if (R) syrk_scatter_row_kernel<T><<<grid_for(M * nk), 256, 0, s>>>(R, ldr, P, M, nk, (int)nb, rpt, sign);
+}
+
 template <typename T>
 int update_syrk_t(int64_t nb, int64_t ntk, const T* L21, int64_t ldl, const T* cL, int64_t ldc, const T* mL,
                   int64_t ldcm, T* Cc, T* Rr, int64_t ldr, T* Cm, T* Rm, int64_t ldrm, cudaStream_t s) {
@@ -396,8 +438,7 @@ int update_syrk_t(int64_t nb, int64_t ntk, const T* L21, int64_t ldl, const T* c
     ABFT_CUBLAS_TRY(gemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)M2, (int)nk, (int)nb, &one, cL, (int)ldc, L21, (int)ldl,
                          &zero, P, (int)M2));
   }
-  syrk_scatter_col_kernel<T><<<grid_for(M2 * nk), 256, 0, s>>>(Cc, ldc, P, M2, nk, (int)nb, 2, T(-1));
-  if (Rr) syrk_scatter_row_kernel<T><<<grid_for(M2 * nk), 256, 0, s>>>(Rr, ldr, P, M2, nk, (int)nb, 2, T(-1));
+  scatter_both<T>(Cc, ldc, Rr, ldr, P, M2, nk, nb, 2, T(-1), s);
   ABFT_CUDA_TRY(cudaGetLastError());
   if (mL && Cm) {
     void* av = nullptr;
@@ -412,8 +453,7 @@ int update_syrk_t(int64_t nb, int64_t ntk, const T* L21, int64_t ldl, const T* c
       ABFT_CUBLAS_TRY(gemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)ntk, (int)nk, (int)nb, &one, mL, (int)ldcm, aL, (int)nk,
                            &zero, P, (int)ntk));
     }
-    syrk_scatter_col_kernel<T><<<grid_for(ntk * nk), 256, 0, s>>>(Cm, ldcm, P, ntk, nk, (int)nb, 1, T(1));
-    if (Rm) syrk_scatter_row_kernel<T><<<grid_for(ntk * nk), 256, 0, s>>>(Rm, ldrm, P, ntk, nk, (int)nb, 1, T(1));
+    scatter_both<T>(Cm, ldcm, Rm, ldrm, P, ntk, nk, nb, 1, T(1), s);
     ABFT_CUDA_TRY(cudaGetLastError());
   }
   return 0;
