@@ -422,8 +422,14 @@ def qr_pd_alg1(st: State, k: int):
         V = np.tril(P, -1)
         V[:nb, :nb] += np.eye(nb)
         T = qr_T(V, tau)
-        st.rowmag[r0:n, k] = mr + np.abs(V) @ (np.abs(T).T @ (np.abs(V).T @ mr))
+        st.rowmag[r0:n, k] = qr_rowmag_rule(V, T, mr)
     return tau
+
+
+def qr_rowmag_rule(V, T, mr):
+    """Row magnitudes through r <- (I − V T^T V^T) r, the QR row rule of both
+    the PD (r(R) = Q^T r(P)) and the TMU (c-6): m_r + |V| (|T|^T (|V|^T m_r))."""
+    return mr + np.abs(V) @ (np.abs(T).T @ (np.abs(V).T @ mr))
 
 
 def qr_V(st: State, k: int):
@@ -492,5 +498,4 @@ def qr_tmu_chk(st: State, k: int, V, T, Wm):
     st.rowchk[r0:n, 2 * (k + 1):] = rA - V @ (T.T @ (V.T @ rA))
     if st.colmag is not None:
         st.colmag[k:, r1:n] += st.colmag[k:, r0:r1] @ np.abs(Wm)
-        mr = st.rowmag[r0:n, k + 1:]
-        st.rowmag[r0:n, k + 1:] = mr + np.abs(V) @ (np.abs(T).T @ (np.abs(V).T @ mr))
+        st.rowmag[r0:n, k + 1:] = qr_rowmag_rule(V, T, st.rowmag[r0:n, k + 1:])

@@ -38,6 +38,32 @@ def spd(n: int, seed: int = 0, dtype=np.float64) -> np.ndarray:
     return S.astype(dtype)
 
 
+def stieltjes(n: int, seed: int = 0, dtype=np.float64) -> np.ndarray:
+    """n*I - B with B symmetric, B_ij ~ U(0,1) off the diagonal, B_ii = 0:
+    a diagonally dominant SPD matrix with non-positive off-diagonal entries
+    (a Stieltjes matrix).  Used by the magnitude pins: its Cholesky factor
+    keeps one sign pattern, so the absolute-value computation has no
+    cancellation off the diagonal."""
+    M = rng(seed).uniform(0.0, 1.0, size=(n, n))
+    B = (M + M.T) * 0.5
+    B[np.diag_indices(n)] = 0.0
+    S = -B
+    S[np.diag_indices(n)] = float(n)
+    return S.astype(dtype)
+
+
+def m_matrix(n: int, seed: int = 0, dtype=np.float64) -> np.ndarray:
+    """n*I - B with B_ij ~ U(0,1) off the diagonal (B_ii = 0): a
+    column-diagonally-dominant nonsingular M-matrix (partial pivoting never
+    swaps; L and U keep non-positive off-diagonal entries).  Magnitude pins
+    for LU, like `stieltjes` for Cholesky."""
+    B = rng(seed).uniform(0.0, 1.0, size=(n, n))
+    B[np.diag_indices(n)] = 0.0
+    S = -B
+    S[np.diag_indices(n)] = float(n)
+    return S.astype(dtype)
+
+
 def integers(m: int, n: int | None = None, seed: int = 0, R: int = 64, dtype=np.float64) -> np.ndarray:
     """Integer-valued matrix in [-R, R]; every checksum of it is an exactly
     representable integer, so sums are bit-exact in any order."""
