@@ -52,9 +52,18 @@ def test_not_spd_info(lib, ctx):
     assert info == 64 + 7
 
 
-def _compare(lib, ctx, A, nb, injects, fig4a=True):
-    Lo, so = dr.ft_potrf(A, nb, inject=injects, fig4a_repair=fig4a)
-    Lg, rc, info, sg, fg = _gpu_potrf(lib, ctx, A, nb, inject=injects, fig4a=fig4a)
+def _compare(lib, ctx, A, nb, injects, fig4a=True, prec="f64"):
+    """Same fault plan on the oracle driver and the GPU driver: counters, fix
+    positions / classes / kinds, restarts and repairs identical; factors
+    within 1e-12 (fp64) / 1e-5 (fp32) of LAPACK's.  fp32: the GPU factors in
+    fp32, the oracle carries fp32 inputs, fp32 flips and fp32 thresholds
+    (u = 2^-24) in fp64 arithmetic; MUST-band faults take the same decisions."""
+    vtol = 1e-12 if prec == "f64" else 1e-5
+    if prec == "f32":
+        A = A.astype(np.float32).astype(np.float64)
+    Lo, so = dr.ft_potrf(A, nb, prec=prec, inject=injects, fig4a_repair=fig4a)
+    Lg, rc, info, sg, fg = _gpu_potrf(lib, ctx, A, nb, inject=injects, fig4a=fig4a,
+                                      dtype=torch.float64 if prec == "f64" else torch.float32)
     assert (rc == lib.E_UNCORRECTABLE) == (so.uncorrectable > 0)
     assert sg.repairs_skipped == so.repairs_skipped
     if so.repairs_skipped:
@@ -69,8 +78,8 @@ def _compare(lib, ctx, A, nb, injects, fig4a=True):
     assert (rc == lib.E_UNCORRECTABLE) == (so.uncorrectable > 0)
     if so.uncorrectable == 0:
         Lref = np.linalg.cholesky(A)
-        assert np.abs(Lg - Lref).max() <= 1e-12 * np.abs(Lref).max()
-        assert np.abs(Lo - Lref).max() <= 1e-12 * np.abs(Lref).max()
+        assert np.abs(Lg - Lref).max() <= vtol * np.abs(Lref).max()
+        assert np.abs(Lo - Lref).max() <= vtol * np.abs(Lref).max()
     return so, sg
 
 
@@ -99,6 +108,35 @@ def test_fault_campaign_parity(lib, ctx, case):
     point, kind, target, gi, gj, bits = CASES[case]
     A = si.spd(256, seed=0)
     _compare(lib, ctx, A, 32, [dr.Inject(2, point, kind, target, gi, gj, bits)])
+
+
+# fp32 (every entry point takes ABFT_F32; BASELINE's 1e-5): the same fault
+# kinds with the flips moved into the fp32 word (fp64 bit b -> b - 32: the
+# exponent/sign bits stay exponent/sign bits, 52-54 become mantissa 20-22)
+CASES_F32 = CASES
+
+
+@pytest.mark.parametrize("case", range(len(CASES_F32)))
+def test_fault_campaign_parity_f32(lib, ctx, case):
+    point, kind, target, gi, gj, bits = CASES_F32[case]
+    A = si.spd(256, seed=0)
+    _compare(lib, ctx, A, 32, [dr.Inject(2, point, kind, target, gi, gj, tuple(b - 32 for b in bits))], prec="f32")
+
+
+@pytest.mark.parametrize("case", [
+    # (iter, point, kind, gi, gj, bits): the metric's tile size nb=512 on n=2048
+    (1, dr.AT_POST_TMU, dr.KIND_PERSIST, 1900, 1300, (60,)),   # trailing computation error -> 0D
+    (1, dr.AT_PRE_TMU, dr.KIND_PERSIST, 1500, 700, (54,)),     # DRAM in the TMU reference part -> Fig. 4a repair
+    (1, dr.AT_PRE_TMU, dr.KIND_ONCHIP, 1700, 600, (56,)),      # on-chip panel value during the TMU -> 1D + Fig. 4b
+    (0, dr.AT_PRE_PU, dr.KIND_ONCHIP, 100, 50, (58,)),         # on-chip in L_kk during the PU -> 2D -> restart
+    (2, dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 1200, 1100, (62,)),  # DRAM in A_kk before its check
+])
+def test_fault_parity_nb512(lib, ctx, case):
+    """One-fault driver parity against the ORACLE at the metric's nb=512
+    (n=2048, 4 tile columns), not against the GPU's own fault-free run."""
+    k, point, kind, gi, gj, bits = case
+    A = si.spd(2048, seed=77)
+    _compare(lib, ctx, A, 512, [dr.Inject(k, point, kind, 0, gi, gj, bits)])
 
 
 def test_fig4a_off_matches_oracle(lib, ctx):
