@@ -438,10 +438,10 @@ ABFT_API int ft_ctx_set_host_lapack(ft_ctx_t *ctx, const char *path);
  * -> check L_kk (LOWER, c) -> check panel A_ik (both) -> PU + a5 -> check
  * L_ik (c) -> TMU (DSYRK on tensor cores) + a6 -> heuristic re-check of L_ik
  * (Fig. 4a) with the guarded trailing repair (c-25).  Checksums are
- * allocated inside ctx.  Synchronises the host once at the end, plus one
- * wait per post-op check when opts->restart (the local-restart decision, f1
- * L430; with the environment variable ABFT_RESTART_DEVICE=1 the post-PU
- * decision is taken on the device by a CUDA-graph IF node instead, DESIGN.md
+ * allocated inside ctx.  Synchronises the host once at the end, plus, when
+ * opts->restart, one wait per iteration for the post-PD local-restart
+ * decision (f1, L430); the post-PU restart is decided on the device (its
+ * redo is queued as gated kernels that run only after a 2D error, DESIGN.md
  * §2.10).  Returns ABFT_E_UNCORRECTABLE if a 2D error remained after the
  * restart (or without it).  *info (host) follows LAPACK potrf. */
 ABFT_API int ft_potrf(ft_ctx_t *ctx, int32_t dtype, int64_t n, void *dA, int64_t lda,

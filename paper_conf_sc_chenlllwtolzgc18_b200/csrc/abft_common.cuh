@@ -135,7 +135,17 @@ int workspace_get(cudaStream_t s, size_t bytes, void** out);
 int counters_get(cudaStream_t s, size_t n_ints, int** out);
 // Device-to-device 2-D copy (pitches and width in bytes) with an SM kernel:
 // cudaMemcpy2DAsync D2D of column panels runs far below HBM bandwidth.
+// Honours launch_gate() (below) like the verify / locate launches.
 int copy2d(void* dst, size_t dpitch, const void* src, size_t spitch, size_t width, size_t height, cudaStream_t s);
+// C (M x N, ld ldc) = op(A) op(B) with optional |.| on A or B, every CTA
+// returning at once when *gate == 0 (abft_gated.cu; the local-restart redo).
+int gemm_gated(int32_t dtype, bool ta, bool tb, bool absa, bool absb, int64_t M, int64_t N, int64_t K, const void* A,
+               int64_t lda, const void* B, int64_t ldb, void* C, int64_t ldc, const int32_t* gate, cudaStream_t s);
+// Free the per-stream pools (workspace, counters: abft_runtime.cu) and the
+// per-stream library handles and scratch (abft_update.cu) of a stream that is
+// about to be destroyed.  The stream must be idle.
+void release_stream_pools(cudaStream_t s);
+void release_stream_handles(cudaStream_t s);
 
 // Device-side gate of the verify / locate launches issued by this host
 // thread (drivers only, not part of the C ABI): when non-null, every CTA of

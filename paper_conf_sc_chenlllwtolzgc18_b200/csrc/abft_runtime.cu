@@ -69,9 +69,19 @@ int counters_get(cudaStream_t s, size_t n, int** out) {
   return 0;
 }
 
+void release_stream_pools(cudaStream_t s) {
+  std::lock_guard<std::mutex> g(g_mu);
+  auto it = pools().find(key_of(s));
+  if (it == pools().end()) return;
+  if (it->second.ws) cudaFree(it->second.ws);
+  if (it->second.ctr) cudaFree(it->second.ctr);
+  pools().erase(it);
+}
+
 template <typename V>
 __global__ void __launch_bounds__(256) copy2d_kernel(char* __restrict__ dst, size_t dpitch, const char* __restrict__ src,
-                                                     size_t spitch, size_t wv, size_t height) {
+                                                     size_t spitch, size_t wv, size_t height, const int32_t* gate) {
+  if (gate && *gate == 0) return;
   for (size_t c = blockIdx.y; c < height; c += gridDim.y) {
     const V* sc = reinterpret_cast<const V*>(src + c * spitch);
     V* dc = reinterpret_cast<V*>(dst + c * dpitch);
@@ -90,11 +100,12 @@ int copy2d(void* dst, size_t dpitch, const void* src, size_t spitch, size_t widt
   dim3 g(gx, std::min<unsigned>(gy, 65535u));
   char* d = (char*)dst;
   const char* r = (const char*)src;
+  const int32_t* gate = launch_gate();
   switch (vb) {
-    case 16: copy2d_kernel<int4><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height); break;
-    case 8: copy2d_kernel<int2><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height); break;
-    case 4: copy2d_kernel<int><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height); break;
-    default: copy2d_kernel<char><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height); break;
+    case 16: copy2d_kernel<int4><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height, gate); break;
+    case 8: copy2d_kernel<int2><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height, gate); break;
+    case 4: copy2d_kernel<int><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height, gate); break;
+    default: copy2d_kernel<char><<<g, 256, 0, s>>>(d, dpitch, r, spitch, wv, height, gate); break;
   }
   ABFT_CUDA_TRY(cudaGetLastError());
   return 0;

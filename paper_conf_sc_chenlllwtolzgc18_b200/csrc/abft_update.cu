@@ -47,26 +47,27 @@ std::mutex g_hmu;
 // One cuBLAS / cuSOLVER handle pair per (device, stream): library calls issued
 // on different streams at the same time (the drivers' side stream) must not
 // share a handle's workspace.
-Handles& handles_for(cudaStream_t s) {
+std::unordered_map<uint64_t, Handles*>& handle_map() {
   static auto* m = new std::unordered_map<uint64_t, Handles*>();
+  return *m;
+}
+uint64_t handle_key(cudaStream_t s) {
   int dev = 0;
   cudaGetDevice(&dev);
-  const uint64_t key = (reinterpret_cast<uint64_t>(s) << 8) ^ (uint64_t)dev;
+  return (reinterpret_cast<uint64_t>(s) << 8) ^ (uint64_t)dev;
+}
+Handles& handles_for(cudaStream_t s) {
+  const uint64_t key = handle_key(s);
   std::lock_guard<std::mutex> g(g_hmu);
-  auto it = m->find(key);
-  if (it != m->end()) return *it->second;
+  auto& m = handle_map();
+  auto it = m.find(key);
+  if (it != m.end()) return *it->second;
   Handles* h = new Handles();
   cublasCreate(&h->blas);
   cusolverDnCreate(&h->solver);
   cublasSetStream(h->blas, s);
   cusolverDnSetStream(h->solver, s);
-  // A fixed cuBLAS workspace: without one cuBLAS allocates stream-ordered
-  // memory inside graph capture, which the drivers' device-decided restart
-  // (a graph IF body) cannot hold.
-  void* ws = nullptr;
-  const size_t ws_bytes = size_t(64) << 20;
-  if (cudaMalloc(&ws, ws_bytes) == cudaSuccess) cublasSetWorkspace(h->blas, ws, ws_bytes);
-  (*m)[key] = h;
+  m[key] = h;
   return *h;
 }
 
@@ -76,13 +77,20 @@ struct Scratch {
   size_t bytes = 0;
 };
 std::mutex g_smu;
-int scratch_get(cudaStream_t s, int slot, size_t bytes, void** out) {
+constexpr int kScratchSlots = 32;  // slots in use: 1-23
+std::unordered_map<uint64_t, Scratch>& scratch_map() {
   static auto* m = new std::unordered_map<uint64_t, Scratch>();
+  return *m;
+}
+uint64_t scratch_key(cudaStream_t s, int slot) {
   int dev = 0;
   cudaGetDevice(&dev);
-  uint64_t key = (reinterpret_cast<uint64_t>(s) << 12) ^ ((uint64_t)dev << 4) ^ (uint64_t)slot;
+  return (reinterpret_cast<uint64_t>(s) << 12) ^ ((uint64_t)dev << 4) ^ (uint64_t)slot;
+}
+int scratch_get(cudaStream_t s, int slot, size_t bytes, void** out) {
+  const uint64_t key = scratch_key(s, slot);
   std::lock_guard<std::mutex> g(g_smu);
-  Scratch& sc = (*m)[key];
+  Scratch& sc = scratch_map()[key];
   if (sc.bytes < bytes) {
     if (sc.p) {
       ABFT_CUDA_TRY(cudaStreamSynchronize(s));
@@ -112,6 +120,28 @@ cusolverDnHandle_t solver_handle(cudaStream_t s, std::unique_lock<std::mutex>& l
   return h.solver;
 }
 int scratch(cudaStream_t s, int slot, size_t bytes, void** out) { return scratch_get(s, slot, bytes, out); }
+
+void release_stream_handles(cudaStream_t s) {
+  {
+    std::lock_guard<std::mutex> g(g_hmu);
+    auto& m = handle_map();
+    auto it = m.find(handle_key(s));
+    if (it != m.end()) {
+      cublasDestroy(it->second->blas);
+      cusolverDnDestroy(it->second->solver);
+      delete it->second;
+      m.erase(it);
+    }
+  }
+  std::lock_guard<std::mutex> g(g_smu);
+  auto& m = scratch_map();
+  for (int slot = 0; slot < kScratchSlots; ++slot) {
+    auto it = m.find(scratch_key(s, slot));
+    if (it == m.end()) continue;
+    if (it->second.p) cudaFree(it->second.p);
+    m.erase(it);
+  }
+}
 
 // ---------------------------------------------------- elementwise kernels --
 // dst (rows x cols, ld = rows) = |src (ld = lds)|

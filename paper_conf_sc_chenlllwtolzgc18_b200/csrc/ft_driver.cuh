@@ -86,18 +86,18 @@ static __global__ void drv_delta_to_host_kernel(const int32_t* now, const int32_
 }
 static __global__ void drv_word_to_host_kernel(const int32_t* src, volatile int32_t* host) { *host = *src; }
 
-// Device-decided restart (f1): did the post-op check add uncorrectable
-// errors?  Then take them back (the redo re-checks), count the restart and
-// the redo's check, and open the IF node holding the redo.
-static __global__ void drv_restart_cond_kernel(cudaGraphConditionalHandle h, int32_t* uncorrectable,
-                                               const int32_t* snap, int32_t* restarts, int32_t* runs, int32_t nchk) {
+// Device-decided local restart (f1, L430): did the post-op check add
+// uncorrectable errors?  Then take them back (the redo re-checks), count the
+// restart and the redo's checks, and open the gate of the redo's launches.
+static __global__ void drv_restart_gate_kernel(int32_t* uncorrectable, const int32_t* snap, int32_t* gate,
+                                               int32_t* restarts, int32_t* runs, int32_t nchk) {
   const int32_t delta = *uncorrectable - *snap;
+  *gate = delta > 0;
   if (delta > 0) {
     *uncorrectable = *snap;
     ++*restarts;
     *runs += nchk;
   }
-  cudaGraphSetConditional(h, delta > 0 ? 1u : 0u);
 }
 
 // Fig. 4b gate: did the fixes logged since the start of the iteration include
@@ -148,6 +148,7 @@ struct Driver {
   int32_t* gate4b = nullptr;           // device: Fig. 4b gate of this iteration
   int32_t* gated_runs = nullptr;       // device: gated checks that ran
   int32_t* iter_mark = nullptr;        // device: fix-log position at the start of the iteration
+  int32_t* gate_rs = nullptr;          // device: gate of the device-decided restart's redo
   int ctf_flagged = 0, ctf_recomputed = 0;
   std::vector<std::pair<int, int>> xfer_used;  // (iter, point) transfer faults already applied
 
@@ -157,14 +158,9 @@ struct Driver {
   // Every exit (error returns included) orders the caller's stream after the
   // work queued on the private one.
   ~Driver() {
-    if (rs_exec) cudaGraphExecDestroy(rs_exec);  // freed when its queued launches complete
-    if (rs_instantiations && getenv("ABFT_DEBUG_RESTART_GRAPH"))
-      fprintf(stderr, "[abft] restart graphs: %d instantiated, %d updated\n", rs_instantiations, rs_updates);
     if (c && c->drv && s == c->drv && cudaEventRecord(c->join, s) == cudaSuccess)
       cudaStreamWaitEvent(c->stream, c->join, 0);
   }
-  cudaGraphExec_t rs_exec = nullptr;  // device-decided restart: the last executable graph
-  int rs_instantiations = 0, rs_updates = 0;
 
   int setup(ft_ctx* ctx, int32_t dt, int64_t n_, int64_t nb_, void* dA, int64_t lda_, const ft_opts_t* opts,
             bool is_lu) {
@@ -211,6 +207,7 @@ struct Driver {
     gate4b = counts + 25;
     gated_runs = counts + 26;
     iter_mark = counts + 27;
+    gate_rs = counts + 29;  // counts + 28: restarts decided on the device
     if (o->abft && o->restart)
       FT_TRY(grow_buffer(c->rsv, c->rsv_bytes,
                          ((size_t)n * nb + (size_t)nb * nb + 3 * (size_t)nt * nb + 4 * nb + 3 * (size_t)n) * es));
@@ -342,132 +339,22 @@ struct Driver {
     FT_TRY(post_delta(0));
     return wait_delta(0, delta);
   }
-  // The same decision without the host wait: `redo` (the restore + redo +
-  // re-check) is stream-captured into the body of a CUDA-graph IF node whose
-  // condition drv_restart_cond_kernel sets on the device from the snapshot
-  // taken before the check; the graph is launched on s and freed on
-  // completion.  Host waits: none.  Restarts and the redo's check are
-  // counted on the device (counts[28], counts[26]).
-  // Opt-in (ABFT_RESTART_DEVICE=1, read per call): measured on B200 at
-  // n=30720 the per-iteration capture + instantiation costs the host more
-  // than the stream drain it removes (ft_potrf 341 vs 338 ms).
-  bool device_restart_ok() const {
-    const char* v = getenv("ABFT_RESTART_DEVICE");
-    return v && v[0] == '1';
-  }
+  // The same decision without a host wait (the PU restarts): `redo` queues
+  // the restore / redo / re-check as gated launches (copy2d, gemm_gated,
+  // verify and locate all return at once while the gate is closed) after
+  // drv_restart_gate_kernel has compared the counter with the snapshot.  The
+  // redo's `nchk` checks and the restart are counted on the device
+  // (counts[26], counts[28]) when the gate opens.
   template <typename F>
-  int device_restart(F&& redo) {
-    cudaError_t e = cudaSuccess;
-    const char* where = "";
-#define DR_TRY(x)          \
-  if (e == cudaSuccess) {  \
-    e = (x);               \
-    where = #x;            \
-  }
-    cudaGraph_t g = nullptr;
-    ABFT_CUDA_TRY(cudaGraphCreate(&g, 0));
-    cudaGraphConditionalHandle ch{};
-    cudaGraph_t body = nullptr;
-    cudaGraphNode_t setn = nullptr, ifn = nullptr;
-    int32_t nchk = 0;
-    cudaKernelNodeParams kp{};
-    int32_t* unc = counts + ABFT_CNT_UNCORRECTABLE;
-    int32_t* rsc = counts + 28;
-    void* args[] = {&ch, &unc, &snap, &rsc, &gated_runs, &nchk};
-    kp.func = (void*)drv_restart_cond_kernel;
-    kp.gridDim = dim3(1);
-    kp.blockDim = dim3(1);
-    kp.kernelParams = args;
-    cudaGraphNodeParams cp{};
-    cp.type = cudaGraphNodeTypeConditional;
-    cp.conditional.type = cudaGraphCondTypeIf;
-    cp.conditional.size = 1;
-    DR_TRY(cudaGraphConditionalHandleCreate(&ch, g, 0, 0));
-    cp.conditional.handle = ch;
-    DR_TRY(cudaGraphAddKernelNode(&setn, g, nullptr, 0, &kp));
-    DR_TRY(cudaGraphAddNode(&ifn, g, &setn, 1, &cp));
-    if (e == cudaSuccess) body = cp.conditional.phGraph_out[0];
-    DR_TRY(cudaStreamBeginCaptureToGraph(s, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
-    int rrc = 0;
-    if (e == cudaSuccess) {
-      const int checks0 = n_checks;
-      rrc = redo();
-      nchk = n_checks - checks0;
-      n_checks = checks0;  // counted on the device when the redo runs
-      cudaGraph_t out = body;
-      DR_TRY(cudaStreamEndCapture(s, &out));
-      DR_TRY(cudaGraphKernelNodeSetParams(setn, &kp));  // nchk now known
-    }
-    cudaGraphExec_t ge = nullptr;
-    bool fallback = false;
-    if (!rrc && e == cudaSuccess && rs_exec) {
-      // Same topology as the previous iteration's graph (the usual case):
-      // update the executable graph in place instead of instantiating anew
-      // (launches already queued keep their parameters).
-      cudaGraphExecUpdateResultInfo ui{};
-      if (cudaGraphExecUpdate(rs_exec, g, &ui) == cudaSuccess) {
-        ++rs_updates;
-        DR_TRY(cudaGraphLaunch(rs_exec, s));
-        cudaGraphDestroy(g);
-        if (e != cudaSuccess) {
-          fprintf(stderr, "[abft] device restart graph: %s failed: %s\n", where, cudaGetErrorString(e));
-          return ABFT_E_CUDA;
-        }
-        return 0;
-      }
-      (void)cudaGetLastError();
-      cudaGraphExecDestroy(rs_exec);  // freed when its queued launches complete
-      rs_exec = nullptr;
-    }
-    if (!rrc && e == cudaSuccess) {
-      cudaGraphInstantiateParams ip{};
-      if (cudaGraphInstantiateWithParams(&ge, g, &ip) != cudaSuccess) {
-        // A body the driver cannot run conditionally (e.g. a library kernel
-        // launched with attributes IF bodies reject): take the decision on the
-        // host for this op instead (the redo above was only captured).
-        (void)cudaGetLastError();
-        static bool told = false;
-        if (!told && getenv("ABFT_DEBUG_RESTART_GRAPH")) {
-          told = true;
-          size_t nn = 0;
-          cudaGraphGetNodes(body, nullptr, &nn);
-          std::vector<cudaGraphNode_t> nodes(nn);
-          cudaGraphGetNodes(body, nodes.data(), &nn);
-          fprintf(stderr, "[abft] restart graph not instantiable (result %d, node %p); body nodes:", (int)ip.result_out,
-                  (void*)ip.errNode_out);
-          for (auto nd : nodes) {
-            cudaGraphNodeType ty;
-            cudaGraphNodeGetType(nd, &ty);
-            fprintf(stderr, " %d%s", (int)ty, nd == ip.errNode_out ? "*" : "");
-          }
-          fprintf(stderr, "\n");
-        }
-        ge = nullptr;
-        fallback = true;
-      } else {
-        ++rs_instantiations;
-        DR_TRY(cudaGraphLaunch(ge, s));
-        rs_exec = ge;  // kept for the next iteration's update
-        ge = nullptr;
-      }
-    }
-#undef DR_TRY
-    if (ge) cudaGraphExecDestroy(ge);
-    cudaGraphDestroy(g);
-    if (fallback) {
-      int delta = 0;
-      FT_TRY(uncorrectable_added(&delta));
-      if (delta > 0) {
-        FT_TRY(take_back_uncorrectable(delta));
-        FT_TRY(redo());
-      }
-      return 0;
-    }
-    if (e != cudaSuccess) {
-      fprintf(stderr, "[abft] device restart graph: %s failed: %s\n", where, cudaGetErrorString(e));
-      return ABFT_E_CUDA;
-    }
-    return rrc;
+  int gated_restart(int nchk, F&& redo) {
+    drv_restart_gate_kernel<<<1, 1, 0, s>>>(counts + ABFT_CNT_UNCORRECTABLE, snap, gate_rs, counts + 28, gated_runs,
+                                            nchk);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    GateScope g(gate_rs);
+    const int c0 = n_checks;
+    FT_TRY(redo(gate_rs));
+    n_checks = c0;  // counted on the device when the redo runs
+    return 0;
   }
   int take_back_uncorrectable(int delta) {
     ++restarts;

@@ -681,24 +681,19 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft) {
       if (rs) FT_TRY(d.snap_uncorrectable());
       FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW));
-      auto pu_redo = [&]() -> int {
-        FT_TRY(d.copy(d.a_at(r0, r1), lda, pu_a, nb, nb, nk));
-        FT_TRY(d.copy(d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, pu_r, nb, nb, m2));
-        FT_TRY(d.copy(d.rowmag_at(r0, k + 1), d.M.ldrm, pu_rm, nb, nb, m2 / 2));
-        FT_TRY(pu_data());
-        FT_TRY(pu_chk());
+      // 2D after the PU: local restart from the pre-PU copy (L430), decided on
+      // the device (Driver::gated_restart): U12 = L_kk^-1 A12, its row
+      // checksums and magnitudes as gated GEMMs from the copy, then re-check.
+      auto pu_redo = [&](const int32_t* g) -> int {
+        FT_TRY(gemm_gated(dtype, false, false, false, false, nb, nk, nb, c->linv, nb, pu_a, nb, d.a_at(r0, r1), lda, g,
+                          s));
+        FT_TRY(gemm_gated(dtype, false, false, false, false, nb, m2, nb, c->linv, nb, pu_r, nb,
+                          d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, g, s));
+        FT_TRY(gemm_gated(dtype, false, false, true, false, nb, m2 / 2, nb, c->linv, nb, pu_rm, nb,
+                          d.rowmag_at(r0, k + 1), d.M.ldrm, g, s));
         return d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW);
       };
-      int delta = 0;
-      if (rs && d.device_restart_ok()) {
-        FT_TRY(d.device_restart(pu_redo));
-      } else if (rs) {
-        FT_TRY(d.uncorrectable_added(&delta));
-      }
-      if (delta > 0) {
-        FT_TRY(d.take_back_uncorrectable(delta));
-        FT_TRY(pu_redo());
-      }
+      if (rs) FT_TRY(d.gated_restart(1, pu_redo));
     }
     // line 12: TMU  A22 -= L21 U12 (DGEMM on tensor cores) + c-13 rules
     FT_TRY(d.inject_at(k, FT_AT_PRE_TMU));

@@ -191,7 +191,14 @@ extern "C" int ft_ctx_destroy(ft_ctx_t* c) {
   if (c->hpin) cudaFreeHost(c->hpin);
   if (c->ev) cudaEventDestroy(c->ev);
   if (c->join) cudaEventDestroy(c->join);
-  if (c->drv) cudaStreamDestroy(c->drv);
+  if (c->drv) {
+    // the library keeps cuBLAS / cuSOLVER handles, scratch and pass pools per
+    // stream: release the private stream's before the stream goes away
+    cudaStreamSynchronize(c->drv);
+    abft::release_stream_handles(c->drv);
+    abft::release_stream_pools(c->drv);
+    cudaStreamDestroy(c->drv);
+  }
   if (c->hstage) cudaFreeHost(c->hstage);
   if (c->dguard) cudaFree(c->dguard);
   if (c->lapack) dlclose(c->lapack);
@@ -258,14 +265,10 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     char* pu_a = pd_m + (size_t)nb * d.es;
     char* pu_c = pu_a + (size_t)nk * nb * d.es;
     char* pu_m = pu_c + (size_t)m2 * nb * d.es;
-    // restart decision: snapshot the uncorrectable count before a check, read
-    // both words back into pinned memory after it (8 bytes, one event)
+    // PD restart decision: snapshot the uncorrectable count before the check,
+    // read the difference back into pinned memory after it (one event)
     auto post_readback = [&](int32_t*) -> int { return d.post_delta(0); };
-    static const bool dbg_nosync = getenv("ABFT_DBG_RESTART_NOSYNC") != nullptr;
-    auto readback_delta = [&](int* delta) -> int {  // uncorrectable errors the check added
-      if (dbg_nosync) { *delta = 0; return 0; }
-      return d.wait_delta(0, delta);
-    };
+    auto readback_delta = [&](int* delta) -> int { return d.wait_delta(0, delta); };
     if (rs) {
       FT_TRY(copy2d(pd_a, nb, d.a_at(r0, r0), lda, nb, nb));
       FT_TRY(copy2d(pd_c, 2, d.colchk_at(2 * k, r0), d.M.ldc, 2, nb));
@@ -394,29 +397,19 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft && post_checks) {
       if (rs) ABFT_CUDA_TRY(cudaMemcpyAsync(d.snap, d.counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToDevice, s));
       FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
-      auto pu_redo = [&]() -> int {
-        FT_TRY(copy2d(d.a_at(r1, r0), lda, pu_a, nk, nk, nb));
-        FT_TRY(copy2d(d.colchk_at(2 * (k + 1), r0), d.M.ldc, pu_c, m2, m2, nb));
-        FT_TRY(copy2d(d.colmag_at(k + 1, r0), d.M.ldcm, pu_m, m2 / 2, m2 / 2, nb));
-        FT_TRY(pu_data());
-        FT_TRY(pu_chk());
+      // 2D after the PU: local restart from the pre-PU copy (L430), decided on
+      // the device (Driver::gated_restart): restore-and-redo as one gated
+      // GEMM per array, reading the copy and the PD's inverse, then re-check.
+      auto pu_redo = [&](const int32_t* g) -> int {
+        FT_TRY(gemm_gated(dtype, false, true, false, false, nk, nb, nb, pu_a, nk, c->linv, nb, d.a_at(r1, r0), lda, g,
+                          s));
+        FT_TRY(gemm_gated(dtype, false, true, false, false, m2, nb, nb, pu_c, m2, c->linv, nb,
+                          d.colchk_at(2 * (k + 1), r0), d.M.ldc, g, s));
+        FT_TRY(gemm_gated(dtype, false, true, false, true, m2 / 2, nb, nb, pu_m, m2 / 2, c->linv, nb,
+                          d.colmag_at(k + 1, r0), d.M.ldcm, g, s));
         return d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL);
       };
-      // The TMU consumes L21 right after this check, so the host wait here
-      // drains the stream; ABFT_RESTART_DEVICE=1 takes the decision on the
-      // device instead (graph IF node, Driver::device_restart).
-      int delta = 0;
-      if (rs && d.device_restart_ok() && !dbg_nosync) {
-        FT_TRY(d.device_restart(pu_redo));
-      } else if (rs) {
-        FT_TRY(post_readback(d.snap));
-        FT_TRY(readback_delta(&delta));
-      }
-      if (delta > 0) {
-        ++d.restarts;
-        add_i32_kernel<<<1, 1, 0, s>>>(d.counts + ABFT_CNT_UNCORRECTABLE, -delta);
-        FT_TRY(pu_redo());
-      }
+      if (rs) FT_TRY(d.gated_restart(1, pu_redo));
     }
     // prior-operation scheme [11]: the TMU's inputs (panel, trailing matrix) before it
     if (ft && scheme == FT_SCHEME_SINGLE_PRE) {

@@ -17,8 +17,8 @@ def ctx(lib):
     return lib.Context()
 
 
-def _gpu_getrf(lib, ctx, A_np, nb, inject=(), abft=True, fig4a=True):
-    A = dev(A_np)
+def _gpu_getrf(lib, ctx, A_np, nb, inject=(), abft=True, fig4a=True, dtype=torch.float64):
+    A = dev(A_np, dtype)
     n = A.shape[0]
     ipiv = torch.zeros(n, dtype=torch.int64, device="cuda")
     inj = [(f.iter, f.point, f.kind, f.target, f.gi, f.gj, si.mask_of(f.bits)) for f in inject]
@@ -57,21 +57,31 @@ def test_unprotected_same_factor(lib, ctx):
     assert np.abs(a[0] - b[0]).max() <= 1e-13 * np.abs(a[0]).max()
 
 
-def _compare(lib, ctx, A, nb, injects):
-    LUo, pivo, so = dr.ft_getrf(A, nb, inject=injects)
-    LUg, pivg, rc, info, sg, fg = _gpu_getrf(lib, ctx, A, nb, inject=injects)
+def _compare(lib, ctx, A, nb, injects, prec="f64"):
+    """fp32: the GPU factors in fp32; the oracle carries the fp32 input, fp32
+    flips and fp32 thresholds in fp64 arithmetic (pivots must still agree)."""
+    vtol = 1e-12 if prec == "f64" else 1e-5
+    if prec == "f32":
+        A = A.astype(np.float32).astype(np.float64)
+    LUo, pivo, so = dr.ft_getrf(A, nb, prec=prec, inject=injects)
+    LUg, pivg, rc, info, sg, fg = _gpu_getrf(lib, ctx, A, nb, inject=injects,
+                                             dtype=torch.float64 if prec == "f64" else torch.float32)
     assert (rc == lib.E_UNCORRECTABLE) == (so.uncorrectable > 0)
     assert sg.repairs_skipped == so.repairs_skipped
     if so.repairs_skipped:
         return so, sg
-    assert list(sg.counts) == so.counts, (list(sg.counts), so.counts)
+    # fp32: counts[3] (tiles with a non-finite delta) records fp32 overflow of
+    # the recomputed sums, which the oracle (fp32 data summed in fp64) cannot see
+    nf = [3] if prec == "f32" else []
+    assert [c for i, c in enumerate(sg.counts) if i not in nf] == [c for i, c in enumerate(so.counts) if i not in nf], \
+        (list(sg.counts), so.counts)
     assert sorted((f[0], f[1], f[4], f[5]) for f in fg) == sorted((f.gi, f.gj, f.cls, f.kind) for f in so.fixes)
     assert sg.repairs_applied == so.repairs_applied
     assert sg.n_checks == so.n_checks
     if so.uncorrectable == 0:
         lu, p = sla.lu_factor(A)
         assert np.array_equal(pivg, p) and np.array_equal(pivo, p)
-        assert np.abs(LUg - lu).max() <= 1e-12 * np.abs(lu).max()
+        assert np.abs(LUg - lu).max() <= vtol * np.abs(lu).max()
     return so, sg
 
 
@@ -99,6 +109,14 @@ def test_lu_fault_campaign_parity(lib, ctx, case):
     k, point, kind, target, gi, gj, bits = LU_CASES[case]
     A = si.general(256, seed=0)
     _compare(lib, ctx, A, 32, [dr.Inject(k, point, kind, target, gi, gj, bits)])
+
+
+@pytest.mark.parametrize("case", range(len(LU_CASES)))
+def test_lu_fault_campaign_parity_f32(lib, ctx, case):
+    """The same fault kinds in fp32 (fp64 bit b -> fp32 bit b - 32)."""
+    k, point, kind, target, gi, gj, bits = LU_CASES[case]
+    A = si.general(256, seed=0)
+    _compare(lib, ctx, A, 32, [dr.Inject(k, point, kind, target, gi, gj, tuple(b - 32 for b in bits))], prec="f32")
 
 
 def _random_lu_plan(n, nb, seed):
@@ -172,10 +190,7 @@ def _gpu_getrf_rs(lib, ctx, A_np, nb, inject, restart):
     (1, dr.AT_PRE_PD, dr.KIND_PERSIST, 64, 64, 55),
     (2, dr.AT_PRE_PU, dr.KIND_ONCHIP, 140, 130, 60),   # L_kk read by the PU: U12 2D
 ])
-@pytest.mark.parametrize("device_decided", [False, True])
-def test_lu_restart_parity(lib, ctx, k, point, kind, gi, gj, bit, device_decided, monkeypatch):
-    if device_decided:  # the PU restart decided on the device (graph IF node); the PD one stays on the host
-        monkeypatch.setenv("ABFT_RESTART_DEVICE", "1")
+def test_lu_restart_parity(lib, ctx, k, point, kind, gi, gj, bit):
     nb = 64
     A = si.general(256, seed=31)
     inj = [dr.Inject(k, point, kind, 0, gi, gj, (bit,))]

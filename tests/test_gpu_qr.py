@@ -16,10 +16,10 @@ def ctx(lib):
     return lib.Context()
 
 
-def _gpu_geqrf(lib, ctx, A_np, nb, inject=(), abft=True):
-    A = dev(A_np)
+def _gpu_geqrf(lib, ctx, A_np, nb, inject=(), abft=True, dtype=torch.float64):
+    A = dev(A_np, dtype)
     n = A.shape[0]
-    tau = torch.zeros(n, dtype=torch.float64, device="cuda")
+    tau = torch.zeros(n, dtype=dtype, device="cuda")
     inj = [(f.iter, f.point, f.kind, f.target, f.gi, f.gj, si.mask_of(f.bits)) for f in inject]
     log = torch.zeros(8192 * lib.FIX_BYTES, dtype=torch.uint8, device="cuda")
     rc, info, stats = lib.ft_geqrf(ctx, A, nb, tau, abft=abft, inject=inj, fix_log=log)
@@ -45,19 +45,27 @@ def test_unprotected_same_factor(lib, ctx):
     assert np.abs(a[0] - b[0]).max() <= 1e-13 * np.abs(a[0]).max()
 
 
-def _compare(lib, ctx, A, nb, injects):
-    Ho, tauo, so = dr.ft_geqrf(A, nb, inject=injects)
-    Hg, taug, rc, info, sg, fg = _gpu_geqrf(lib, ctx, A, nb, inject=injects)
+def _compare(lib, ctx, A, nb, injects, prec="f64"):
+    vtol = 1e-12 if prec == "f64" else 1e-5
+    if prec == "f32":
+        A = A.astype(np.float32).astype(np.float64)
+    Ho, tauo, so = dr.ft_geqrf(A, nb, prec=prec, inject=injects)
+    Hg, taug, rc, info, sg, fg = _gpu_geqrf(lib, ctx, A, nb, inject=injects,
+                                            dtype=torch.float64 if prec == "f64" else torch.float32)
     assert (rc == lib.E_UNCORRECTABLE) == (so.uncorrectable > 0)
     assert sg.repairs_skipped == so.repairs_skipped
     if so.uncorrectable:
         return so, sg
-    assert list(sg.counts) == so.counts, (list(sg.counts), so.counts)
+    # fp32: counts[3] (tiles with a non-finite delta) records fp32 overflow of
+    # the recomputed sums, which the oracle (fp32 data summed in fp64) cannot see
+    nf = [3] if prec == "f32" else []
+    assert [c for i, c in enumerate(sg.counts) if i not in nf] == [c for i, c in enumerate(so.counts) if i not in nf], \
+        (list(sg.counts), so.counts)
     assert sorted((f[0], f[1], f[4], f[5]) for f in fg) == sorted((f.gi, f.gj, f.cls, f.kind) for f in so.fixes)
     assert sg.n_checks == so.n_checks
     assert (sg.ctf_flagged, sg.ctf_recomputed) == (so.ctf_flagged, so.ctf_recomputed)
     h, t = np.linalg.qr(A, mode="raw")
-    assert np.abs(Hg - h.T).max() <= 1e-12 * np.abs(h).max()
+    assert np.abs(Hg - h.T).max() <= vtol * np.abs(h).max()
     return so, sg
 
 
@@ -81,6 +89,14 @@ def test_qr_fault_campaign_parity(lib, ctx, case):
     k, point, kind, target, gi, gj, bits = QR_CASES[case]
     A = si.general(256, seed=0)
     _compare(lib, ctx, A, 32, [dr.Inject(k, point, kind, target, gi, gj, bits)])
+
+
+@pytest.mark.parametrize("case", range(len(QR_CASES)))
+def test_qr_fault_campaign_parity_f32(lib, ctx, case):
+    """The same fault kinds in fp32 (fp64 bit b -> fp32 bit b - 32)."""
+    k, point, kind, target, gi, gj, bits = QR_CASES[case]
+    A = si.general(256, seed=0)
+    _compare(lib, ctx, A, 32, [dr.Inject(k, point, kind, target, gi, gj, tuple(b - 32 for b in bits))], prec="f32")
 
 
 @pytest.mark.parametrize("seed", range(8))
