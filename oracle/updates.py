@@ -75,36 +75,50 @@ def chol_pu_chk(st: State, k: int):
         st.colmag[k + 1:, s] = st.colmag[k + 1:, s] @ np.abs(tri_inv(L).T)
 
 
-def chol_tmu_data(st: State, k: int):
+def chol_tmu_data(st: State, k: int, c0: int = None, c1: int = None):
     """c-12 TMU data step, every trailing tile (i ≥ j > k):
-    A_ij −= L_ik L_jk^T on the lower triangle only (as DSYRK)."""
+    A_ij −= L_ik L_jk^T on the lower triangle only (as DSYRK).  With a
+    column range [c0, c1) (look-ahead, reading c-35) only those columns of
+    the trailing matrix are updated."""
     nb, n = st.nb, st.A.shape[0]
     s = slice(k * nb, (k + 1) * nb)
     r1 = (k + 1) * nb
+    c0 = r1 if c0 is None else c0
+    c1 = n if c1 is None else c1
     L21 = st.A[r1:n, s].copy()
-    upd = L21 @ L21.T
-    tri = np.tril(np.ones((n - r1, n - r1), dtype=bool))
-    st.A[r1:n, r1:n][tri] -= upd[tri]
+    upd = L21 @ L21[c0 - r1:c1 - r1].T  # rows r1:n, columns c0:c1
+    rows = np.arange(r1, n)[:, None]
+    cols = np.arange(c0, c1)[None, :]
+    tri = rows >= cols
+    st.A[r1:n, c0:c1][tri] -= upd[tri]
 
 
-def chol_tmu_chk(st: State, k: int):
+def chol_tmu_chk(st: State, k: int, c0: int = None, c1: int = None):
     """c-12 TMU checksum step: c(A_ij) −= c(L_ik)·L_jk^T,
     r(A_ij) −= L_ik·c(L_jk)^T (L189), m_c(A_ij) += m_c(L_ik)·|L_jk|^T,
-    m_r(A_ij) += |L_ik|·m_c(L_jk)^T (c-6)."""
+    m_r(A_ij) += |L_ik|·m_c(L_jk)^T (c-6).  With a column range [c0, c1)
+    (tile-aligned; look-ahead, reading c-35) only the tile columns j in it."""
     nb, n = st.nb, st.A.shape[0]
     s = slice(k * nb, (k + 1) * nb)
     r1 = (k + 1) * nb
+    c0 = r1 if c0 is None else c0
+    c1 = n if c1 is None else c1
+    J0, J1 = c0 // nb, c1 // nb
     L21 = st.A[r1:n, s].copy()
+    Lj = L21[c0 - r1:c1 - r1]
     cL = st.colchk[2 * (k + 1):, s].copy()
-    st.colchk[2 * (k + 1):, r1:n] -= cL @ L21.T
-    st.rowchk[r1:n, 2 * (k + 1):] -= L21 @ cL.T
+    cLj = cL[2 * (J0 - k - 1):2 * (J1 - k - 1)]
+    st.colchk[2 * (k + 1):, c0:c1] -= cL @ Lj.T
+    st.rowchk[r1:n, 2 * J0:2 * J1] -= L21 @ cLj.T
     if st.colmag is not None:
         mL = st.colmag[k + 1:, s].copy()
-        st.colmag[k + 1:, r1:n] += mL @ np.abs(L21).T
-        st.rowmag[r1:n, k + 1:] += np.abs(L21) @ mL.T
+        mLj = mL[J0 - k - 1:J1 - k - 1]
+        st.colmag[k + 1:, c0:c1] += mL @ np.abs(Lj).T
+        st.rowmag[r1:n, J0:J1] += np.abs(L21) @ mLj.T
 
 
-def chol_fig4a_repair(st: State, k: int, gi: int, gj: int, before: float, after: float):
+def chol_fig4a_repair(st: State, k: int, gi: int, gj: int, before: float, after: float, c0: int = 0,
+                      c1: int = None):
     """Reading c-25 of Fig. 4a / L359 ('we can just fix the corresponding
     rows/columns in trailing matrix'): the panel re-check after the TMU fixed
     L[p, q] by E = after − before, but the TMU had used the bad value.  With
@@ -113,8 +127,12 @@ def chol_fig4a_repair(st: State, k: int, gi: int, gj: int, before: float, after:
     r(A_i,J)[p', :] −= E·c(L_J)[:, q']^T for k < J ≤ i; magnitudes grow by
     |E| times the panel magnitude.  Guard: skipped when E is non-finite or
     |E| > 2^10·max|L_panel[:, q]|.  Returns 'applied', 'skipped' or None (not
-    a panel element of iteration k)."""
+    a panel element of iteration k).  A column range [c0, c1) (look-ahead,
+    reading c-35) restricts the repair to the trailing columns that consumed
+    the bad value: the tile column k+1 for the re-check after its update, the
+    rest for the re-check after the rest of the TMU."""
     nb, n = st.nb, st.A.shape[0]
+    c1 = n if c1 is None else c1
     r1 = (k + 1) * nb
     p, q = gi, gj
     if not (k * nb <= q < (k + 1) * nb and p >= r1):
@@ -125,15 +143,21 @@ def chol_fig4a_repair(st: State, k: int, gi: int, gj: int, before: float, after:
         return "skipped"
     i, pl, ql = p // nb, p % nb, q - k * nb
     ell = st.A[:, q]
-    st.A[p, r1:p] -= E * ell[r1:p]
-    st.A[p + 1:n, p] -= E * ell[p + 1:n]
-    st.A[p, p] -= 2.0 * E * ell[p] - E * E
+    b0, b1 = max(r1, c0), min(p, c1)
+    if b1 > b0:
+        st.A[p, b0:b1] -= E * ell[b0:b1]
+    if c0 <= p < c1:
+        st.A[p + 1:n, p] -= E * ell[p + 1:n]
+        st.A[p, p] -= 2.0 * E * ell[p] - E * E
     nt = n // nb
-    for I in range(i, nt):
-        st.colchk[2 * I:2 * I + 2, i * nb + pl] -= E * st.colchk[2 * I:2 * I + 2, k * nb + ql]
-        if st.colmag is not None:
-            st.colmag[I, i * nb + pl] += abs(E) * st.colmag[I, k * nb + ql]
+    if c0 <= p < c1:
+        for I in range(i, nt):
+            st.colchk[2 * I:2 * I + 2, i * nb + pl] -= E * st.colchk[2 * I:2 * I + 2, k * nb + ql]
+            if st.colmag is not None:
+                st.colmag[I, i * nb + pl] += abs(E) * st.colmag[I, k * nb + ql]
     for J in range(k + 1, i + 1):
+        if not c0 <= J * nb < c1:
+            continue
         st.rowchk[p, 2 * J:2 * J + 2] -= E * st.colchk[2 * J:2 * J + 2, k * nb + ql]
         if st.rowmag is not None:
             st.rowmag[p, J] += abs(E) * st.colmag[J, k * nb + ql]

@@ -466,3 +466,73 @@ def test_scheme_outcomes(case):
         ok = np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
         got += "R" if st.uncorrectable else ("Y" if ok else "N")
     assert got == expect
+
+
+# ---------------------------------------------- look-ahead (reading c-35) --
+def test_lookahead_tmu_split_equals_full_tmu():
+    """The TMU split by tile columns (column k+1, then the rest) is the same
+    update as the whole TMU: data and every checksum / magnitude array."""
+    n, nb, k = 256, 32, 1
+    st = ck.State.alloc(si.spd(n, seed=51), nb)
+    nt = n // nb
+    ck.encode(st, ck.Tiles(0, nt, 0, nt, True, ck.SYM_LOWER))
+    for kk in range(k + 1):  # factor panels 0..k so that panel k is an L panel
+        up.chol_pd_rule(st, kk)
+        up.chol_pu_data(st, kk)
+        up.chol_pu_chk(st, kk)
+        if kk < k:
+            up.chol_tmu_data(st, kk)
+            up.chol_tmu_chk(st, kk)
+    a, b = st.copy(), st.copy()
+    up.chol_tmu_data(a, k)
+    up.chol_tmu_chk(a, k)
+    r1, c2 = (k + 1) * nb, (k + 2) * nb
+    for c0, c1 in ((r1, c2), (c2, n)):
+        up.chol_tmu_data(b, k, c0, c1)
+        up.chol_tmu_chk(b, k, c0, c1)
+    for x, y in ((a.A, b.A), (a.colchk, b.colchk), (a.rowchk, b.rowchk), (a.colmag, b.colmag), (a.rowmag, b.rowmag)):
+        assert np.abs(x - y).max() <= 1e-13 * max(1.0, np.abs(x).max())
+
+
+@pytest.mark.parametrize("p", [70, 100, 200])
+def test_lookahead_restricted_repairs_add_up_to_the_full_repair(p):
+    """Reading c-35: the Fig. 4a repair restricted to tile column k+1 plus the
+    one restricted to the columns after it is the unrestricted repair."""
+    n, nb, k = 256, 32, 1
+    st = ck.State.alloc(si.spd(n, seed=52), nb)
+    nt = n // nb
+    ck.encode(st, ck.Tiles(0, nt, 0, nt, True, ck.SYM_LOWER))
+    q = k * nb + 5
+    before, after = 0.25, 0.75
+    a, b = st.copy(), st.copy()
+    assert up.chol_fig4a_repair(a, k, p, q, before, after) == "applied"
+    r1, c2 = (k + 1) * nb, (k + 2) * nb
+    up.chol_fig4a_repair(b, k, p, q, before, after, r1, c2)
+    up.chol_fig4a_repair(b, k, p, q, before, after, c2, n)
+    for x, y in ((a.A, b.A), (a.colchk, b.colchk), (a.rowchk, b.rowchk), (a.colmag, b.colmag), (a.rowmag, b.rowmag)):
+        assert np.array_equal(x, y)
+
+
+@pytest.mark.parametrize("n,nb", [(256, 32), (384, 128)])
+def test_lookahead_error_free(n, nb):
+    A = si.spd(n, seed=n + 7)
+    L, stats = dr.ft_potrf(A, nb, lookahead=True, invariant_hook=_invariant)
+    Lref = np.linalg.cholesky(A)
+    assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
+    nt = n // nb
+    assert stats.counts == [0] * 8 and stats.n_checks == 6 * (nt - 1) + 2  # one extra re-check per iteration
+
+
+@pytest.mark.parametrize("case", range(len(FIXABLE)))
+def test_lookahead_fault_outcomes_equal_alg2(case):
+    """Same faults with and without look-ahead: the same factor, fixes
+    (positions, classes) and counters (the predicate keeps Alg. 2's order
+    around every fault hook)."""
+    point, kind, gi, gj, bits = FIXABLE[case]
+    inj = [dr.Inject(2, point, kind, 0, gi, gj, bits)]
+    A = si.spd(256, seed=0)
+    L0, s0 = dr.ft_potrf(A, 32, inject=inj)
+    L1, s1 = dr.ft_potrf(A, 32, inject=inj, lookahead=True)
+    assert s1.counts == s0.counts and s1.restarts == s0.restarts and s1.repairs_applied == s0.repairs_applied
+    assert sorted((f.gi, f.gj, f.cls, f.kind) for f in s1.fixes) == sorted((f.gi, f.gj, f.cls, f.kind) for f in s0.fixes)
+    assert np.abs(L1 - L0).max() <= 1e-13 * np.abs(L0).max()
