@@ -378,6 +378,11 @@ typedef struct {
   int32_t scheme;        /* FT_SCHEME_* (ft_potrf only; ft_getrf / ft_geqrf return -7 for anything but
                             FT_SCHEME_NEW): the checking scheme, for the paper's comparison of
                             schemes (L35, L47, L542, Table VIII, Figs. 12-14; reading c-34) */
+  int32_t lookahead;     /* ft_potrf (FT_SCHEME_NEW or abft = 0): 1 = the TMU of iteration k updates tile
+                            column k+1 first (and re-checks the panel, Fig. 4a), then the PD / PU of
+                            iteration k+1 with their checks run on a second stream next to the rest of
+                            the TMU (reading c-35).  Off for an iteration whose fault hooks it would
+                            move.  Ignored by ft_getrf / ft_geqrf.  Default 0 (bindings: 1). */
 } ft_opts_t;
 
 /* ft_opts_t.scheme (reading c-34).  NEW: the paper's scheme, Alg. 2 (full

@@ -83,7 +83,7 @@ class ft_opts_t(C.Structure):
                 ("fix_log", C.c_void_p), ("fix_log_cap", C.c_int32), ("pu_gemm", C.c_int32),
                 ("refresh", C.c_int32), ("restart", C.c_int32), ("pd_location", C.c_int32),
                 ("fig4b", C.c_int32), ("trailing_check_period", C.c_int32), ("checksum_gemm", C.c_int32),
-                ("scheme", C.c_int32)]
+                ("scheme", C.c_int32), ("lookahead", C.c_int32)]
 
 
 class ft_stats_t(C.Structure):
@@ -380,14 +380,14 @@ def host_lapack_path():
 
 
 def _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh=True, restart=True,
-          pd_location=PD_DEVICE, fig4b=True, period=0, scheme=0, checksum_gemm=False):
+          pd_location=PD_DEVICE, fig4b=True, period=0, scheme=0, checksum_gemm=False, lookahead=False):
     inj = (ft_inject_t * max(1, len(inject)))()
     for k, f in enumerate(inject):
         inj[k] = ft_inject_t(*f)
     opts = ft_opts_t(nb, int(abft), tol_kind, tol_scale, int(fig4a_repair), len(inject), inj,
                      _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES, int(pu_gemm),
                      int(refresh), int(restart), int(pd_location), int(fig4b), int(period), int(checksum_gemm),
-                     int(scheme))
+                     int(scheme), int(lookahead))
     return opts, inj
 
 
@@ -442,15 +442,17 @@ def ft_geqrf(ctx: Context, A: torch.Tensor, nb: int, tau: torch.Tensor, abft=Tru
 
 def ft_potrf(ctx: Context, A: torch.Tensor, nb: int, abft=True, tol_kind=TOL_MAGNITUDE, tol_scale=1.0,
              fig4a_repair=True, inject=(), fix_log=None, pu_gemm=True, refresh=True, restart=True,
-             pd_location=PD_DEVICE, fig4b=True, trailing_check_period=0, scheme=0, checksum_gemm=False):
+             pd_location=PD_DEVICE, fig4b=True, trailing_check_period=0, scheme=0, checksum_gemm=False,
+             lookahead=True):
     """Fault-tolerant lower Cholesky in place on a column-major A.  Returns
     (rc, info, stats) with rc 0 or E_UNCORRECTABLE (other codes raise).
     pd_location=PD_HOST needs ctx.set_host_lapack() first.  scheme: SCHEME_*
     (the checking scheme, include/abft.h ft_opts_t.scheme); checksum_gemm: the
-    checks recompute checksums by GEMMs (prior-art baseline, abft_verify_gemm)."""
+    checks recompute checksums by GEMMs (prior-art baseline, abft_verify_gemm);
+    lookahead: the next panel's PD / PU next to the TMU (reading c-35)."""
     n = A.shape[0]
     opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh, restart,
-                       pd_location, fig4b, trailing_check_period, scheme, checksum_gemm)
+                       pd_location, fig4b, trailing_check_period, scheme, checksum_gemm, lookahead)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_potrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), C.byref(opts), C.byref(stats), C.byref(info))

@@ -141,6 +141,11 @@ int copy2d(void* dst, size_t dpitch, const void* src, size_t spitch, size_t widt
 // returning at once when *gate == 0 (abft_gated.cu; the local-restart redo).
 int gemm_gated(int32_t dtype, bool ta, bool tb, bool absa, bool absb, int64_t M, int64_t N, int64_t K, const void* A,
                int64_t lda, const void* B, int64_t ldb, void* C, int64_t ldc, const int32_t* gate, cudaStream_t s);
+// Cholesky TMU row-checksum rule of one trailing tile column (look-ahead):
+// re/rw (rows) -= L (rows x nb) [ce cw] and rm += |L| mc, ce/cw/mc strided
+// (abft_update.cu).
+int panel_row_rule(int32_t dtype, int64_t rows, int64_t nb, const void* L, int64_t ldl, const void* ce, const void* cw,
+                   int64_t ldc, const void* mc, int64_t ldcm, void* re, void* rw, void* rm, cudaStream_t s);
 // Free the per-stream pools (workspace, counters: abft_runtime.cu) and the
 // per-stream library handles and scratch (abft_update.cu) of a stream that is
 // about to be destroyed.  The stream must be idle.

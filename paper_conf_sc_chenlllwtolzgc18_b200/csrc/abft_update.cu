@@ -535,6 +535,69 @@ int update_gemm_t(int which, char transX, char transY, double alpha, const void*
   return 0;
 }
 
+// Row checksums of one trailing tile column J0 after the Cholesky TMU
+// (c-12, L189; the look-ahead's first part, reading c-35), every row x of the
+// panel L (rows x nb):
+//   r_e(x) -= sum_q L[x,q] c_e(L_J0)[q],  r_w(x) -= sum_q L[x,q] c_w(L_J0)[q],
+//   m_r(x) += sum_q |L[x,q]| m_c(L_J0)[q]            (c-6)
+// in ONE pass over L (the GEMM route needs |L| materialised first).  A block
+// owns 32 rows; its 8 warps split the nb columns and their partials are
+// added in warp order (deterministic).
+template <typename T>
+__global__ void __launch_bounds__(256) panel_row_rule_kernel(int64_t rows, int nb, const T* __restrict__ L, int64_t ldl,
+                                                             const T* __restrict__ ce, const T* __restrict__ cw,
+                                                             int64_t ldc, const T* __restrict__ mc, int64_t ldcm,
+                                                             T* __restrict__ re, T* __restrict__ rw,
+                                                             T* __restrict__ rm) {
+  __shared__ T part[8][3][32];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t x = (int64_t)blockIdx.x * 32 + lane;
+  const int qn = nb / 8, q0 = warp * qn;
+  T se = T(0), sw = T(0), sm = T(0);
+  if (x < rows) {
+#pragma unroll 8
+    for (int q = q0; q < q0 + qn; ++q) {
+      const T l = L[x + (int64_t)q * ldl];
+      se = fma(l, ce[(int64_t)q * ldc], se);
+      sw = fma(l, cw[(int64_t)q * ldc], sw);
+      sm = fma(fabs(l), mc ? mc[(int64_t)q * ldcm] : T(0), sm);
+    }
+  }
+  part[warp][0][lane] = se;
+  part[warp][1][lane] = sw;
+  part[warp][2][lane] = sm;
+  __syncthreads();
+  if (warp == 0 && x < rows) {
+    T e = T(0), w = T(0), m = T(0);
+#pragma unroll
+    for (int g = 0; g < 8; ++g) {
+      e += part[g][0][lane];
+      w += part[g][1][lane];
+      m += part[g][2][lane];
+    }
+    re[x] -= e;
+    rw[x] -= w;
+    if (rm) rm[x] += m;
+  }
+}
+
+int panel_row_rule(int32_t dtype, int64_t rows, int64_t nb, const void* L, int64_t ldl, const void* ce, const void* cw,
+                   int64_t ldc, const void* mc, int64_t ldcm, void* re, void* rw, void* rm, cudaStream_t s) {
+  if (rows <= 0) return 0;
+  if (nb % 8) return ABFT_E_UNSUPPORTED;
+  const unsigned grid = (unsigned)((rows + 31) / 32);
+  if (dtype == ABFT_F64)
+    panel_row_rule_kernel<double><<<grid, 256, 0, s>>>(rows, (int)nb, (const double*)L, ldl, (const double*)ce,
+                                                       (const double*)cw, ldc, (const double*)mc, ldcm, (double*)re,
+                                                       (double*)rw, (double*)rm);
+  else
+    panel_row_rule_kernel<float><<<grid, 256, 0, s>>>(rows, (int)nb, (const float*)L, ldl, (const float*)ce,
+                                                      (const float*)cw, ldc, (const float*)mc, ldcm, (float*)re,
+                                                      (float*)rw, (float*)rm);
+  ABFT_CUDA_TRY(cudaGetLastError());
+  return 0;
+}
+
 }  // namespace abft
 
 extern "C" int abft_update_trsm(int32_t dtype, char side, char uplo, char trans, char diag, int64_t nb, const void* T,

@@ -53,6 +53,12 @@ struct ft_ctx {
   // graph, and the legacy default stream cannot be captured.
   cudaStream_t drv = nullptr;
   cudaEvent_t join = nullptr;
+  // look-ahead (the next panel's PD / PU next to the current TMU): a second
+  // private stream (high priority) and its events
+  cudaStream_t side = nullptr;
+  cudaEvent_t ev_col = nullptr, ev_side = nullptr;
+  void* putmp2 = nullptr;  // PU scratch of the side stream
+  size_t putmp2_bytes = 0;
   // FT_PD_HOST (ft_host.cu): host LAPACK, pinned panel staging, device guard
   void* lapack = nullptr;  // dlopen handle
   void* lp[6] = {};        // dpotrf spotrf dgetrf sgetrf dgeqrf sgeqrf
@@ -95,8 +101,8 @@ static __global__ void drv_restart_gate_kernel(int32_t* uncorrectable, const int
   *gate = delta > 0;
   if (delta > 0) {
     *uncorrectable = *snap;
-    ++*restarts;
-    *runs += nchk;
+    atomicAdd(restarts, 1);  // shared with the other stream's gate kernels (look-ahead)
+    atomicAdd(runs, nchk);
   }
 }
 
@@ -111,7 +117,7 @@ static __global__ void fig4b_gate_kernel(const abft_fix_t* fixes, int cap, const
   hit = __any_sync(0xffffffffu, hit);
   if (threadIdx.x == 0) {
     *gate = hit;
-    if (hit) ++*runs;
+    if (hit) atomicAdd(runs, 1);
   }
 }
 
@@ -149,6 +155,27 @@ struct Driver {
   int32_t* gated_runs = nullptr;       // device: gated checks that ran
   int32_t* iter_mark = nullptr;        // device: fix-log position at the start of the iteration
   int32_t* gate_rs = nullptr;          // device: gate of the device-decided restart's redo
+  int32_t* restarts_dev = nullptr;     // device: restarts decided on the device
+  int32_t* f4b_end = nullptr;          // device: fix-log position where a deferred Fig. 4b gate stops
+  // Look-ahead (reading c-35): the next panel's PD / PU run on the context's
+  // side stream with their own report counters (so that a restart decision
+  // there never sees the main stream's checks); on_side() switches both.
+  cudaStream_t s_main = nullptr;
+  int32_t *counts_main = nullptr, *counts_side = nullptr;
+  void on_side(bool side) {
+    s = side ? c->side : s_main;
+    counts = side ? counts_side : counts_main;
+    R.counts = counts;
+  }
+  int side_setup() {
+    if (c->side) return 0;
+    int lo = 0, hi = 0;
+    ABFT_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    ABFT_CUDA_TRY(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, hi));
+    ABFT_CUDA_TRY(cudaEventCreateWithFlags(&c->ev_col, cudaEventDisableTiming));
+    ABFT_CUDA_TRY(cudaEventCreateWithFlags(&c->ev_side, cudaEventDisableTiming));
+    return 0;
+  }
   int ctf_flagged = 0, ctf_recomputed = 0;
   std::vector<std::pair<int, int>> xfer_used;  // (iter, point) transfer faults already applied
 
@@ -186,7 +213,7 @@ struct Driver {
     FT_TRY(grow_buffer(c->state, c->state_bytes, need));
     if (o->pd_location == FT_PD_HOST && !c->lapack) return ABFT_E_UNSUPPORTED;
     if (o->pd_location != FT_PD_DEVICE && o->pd_location != FT_PD_HOST) return ABFT_E_UNSUPPORTED;
-    size_t ints_need = (size_t)nt * nt + 8 + 8 + 8 + 8;
+    size_t ints_need = (size_t)nt * nt + 48;  // status | counts[32] | side counts[8] | spare
     void* ip = c->ints;
     FT_TRY(grow_buffer(ip, c->ints_n, ints_need * sizeof(int32_t)));
     c->ints = reinterpret_cast<int32_t*>(ip);
@@ -207,7 +234,12 @@ struct Driver {
     gate4b = counts + 25;
     gated_runs = counts + 26;
     iter_mark = counts + 27;
-    gate_rs = counts + 29;  // counts + 28: restarts decided on the device
+    gate_rs = counts + 29;
+    restarts_dev = counts + 28;
+    f4b_end = counts + 30;
+    counts_main = counts;
+    counts_side = counts + 32;
+    s_main = s;
     if (o->abft && o->restart)
       FT_TRY(grow_buffer(c->rsv, c->rsv_bytes,
                          ((size_t)n * nb + (size_t)nb * nb + 3 * (size_t)nt * nb + 4 * nb + 3 * (size_t)n) * es));
@@ -347,7 +379,7 @@ struct Driver {
   // (counts[26], counts[28]) when the gate opens.
   template <typename F>
   int gated_restart(int nchk, F&& redo) {
-    drv_restart_gate_kernel<<<1, 1, 0, s>>>(counts + ABFT_CNT_UNCORRECTABLE, snap, gate_rs, counts + 28, gated_runs,
+    drv_restart_gate_kernel<<<1, 1, 0, s>>>(counts + ABFT_CNT_UNCORRECTABLE, snap, gate_rs, restarts_dev, gated_runs,
                                             nchk);
     ABFT_CUDA_TRY(cudaGetLastError());
     GateScope g(gate_rs);
@@ -373,9 +405,17 @@ struct Driver {
     ABFT_CUDA_TRY(cudaMemcpyAsync(iter_mark, nfix, 4, cudaMemcpyDeviceToDevice, s));
     return 0;
   }
-  int fig4b_check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only) {
+  // mark_fig4b_end: under look-ahead the Fig. 4b check of an iteration runs
+  // after its PU (on the main stream); the gate must then see only the fixes
+  // up to where Alg. 2 puts the check (before the PU), recorded here.
+  int mark_fig4b_end() {
+    ABFT_CUDA_TRY(cudaMemcpyAsync(f4b_end, nfix, 4, cudaMemcpyDeviceToDevice, s));
+    return 0;
+  }
+  int fig4b_check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only, bool deferred = false) {
     if (!o->fig4b || o->checksum_gemm || I0 >= I1) return 0;  // GEMMs cannot honour the device gate
-    fig4b_gate_kernel<<<1, 32, 0, s>>>(c->fixlog, c->fixcap, iter_mark, nfix, gate4b, gated_runs);
+    fig4b_gate_kernel<<<1, 32, 0, s>>>(c->fixlog, c->fixcap, iter_mark, deferred ? f4b_end : nfix, gate4b,
+                                       gated_runs);
     ABFT_CUDA_TRY(cudaGetLastError());
     GateScope g(gate4b);
     FT_TRY(check(I0, I1, J0, J1, view, which, lower_only));
@@ -395,8 +435,8 @@ struct Driver {
 
   // The single host synchronisation: counters, info and the fix log.
   int finish(std::chrono::steady_clock::time_point t0, ft_stats_t* stats, int64_t* info_out) {
-    int32_t h[32];
-    ABFT_CUDA_TRY(cudaMemcpyAsync(h, counts, sizeof(h), cudaMemcpyDeviceToHost, s));
+    int32_t h[40];
+    ABFT_CUDA_TRY(cudaMemcpyAsync(h, counts_main, sizeof(h), cudaMemcpyDeviceToHost, s));
     if (o->fix_log && o->fix_log_cap > 0)
       ABFT_CUDA_TRY(cudaMemcpyAsync(o->fix_log, c->fixlog, sizeof(abft_fix_t) * std::min(o->fix_log_cap, c->fixcap),
                                     cudaMemcpyDeviceToDevice, s));
@@ -404,7 +444,8 @@ struct Driver {
     ABFT_CUDA_TRY(cudaStreamWaitEvent(c->stream, c->join, 0));
     ABFT_CUDA_TRY(cudaStreamSynchronize(s));
     auto t1 = std::chrono::steady_clock::now();
-    // layout after counts: nfix(8) mark(9) info(10) rep(11,12) info_total(13)
+    // layout after counts: nfix(8) mark(9) info(10) rep(11,12) info_total(13); side counts at 32
+    for (int i = 0; i < 8; ++i) h[i] += h[32 + i];
     if (info_out) *info_out = h[13];
     if (stats) {
       for (int i = 0; i < 8; ++i) stats->counts[i] = h[i];

@@ -82,6 +82,7 @@ struct RepairArgs {
   const int32_t* mark;
   int32_t* rep_counts;  // [0] applied, [1] skipped
   int32_t* counts;      // report counts: a skipped repair is uncorrectable (R)
+  int64_t c0, c1;       // trailing columns to repair (look-ahead, reading c-35); [0, n) = all
 };
 
 template <typename T>
@@ -122,12 +123,17 @@ __global__ void fig4a_repair_kernel(RepairArgs r) {
     const T e = (T)eps;
     const T ae = fabs(e);
     const int64_t i = p / nb, pl = p % nb, ql = q - k * nb;
-    // data: row p left of the diagonal, column p below it, and (p, p)
-    for (int64_t b = row0 + threadIdx.x; b < p; b += blockDim.x) A[p + b * r.lda] -= e * A[b + q * r.lda];
-    for (int64_t a = p + 1 + threadIdx.x; a < r.n; a += blockDim.x) A[a + p * r.lda] -= e * A[a + q * r.lda];
-    if (threadIdx.x == 0) A[p + p * r.lda] -= 2 * e * A[p + q * r.lda] - e * e;
+    // data: row p left of the diagonal, column p below it, and (p, p) —
+    // restricted to the columns [c0, c1) whose update consumed the bad value
+    const bool pin = p >= r.c0 && p < r.c1;
+    const int64_t b0 = row0 > r.c0 ? row0 : r.c0, b1 = p < r.c1 ? p : r.c1;
+    for (int64_t b = b0 + threadIdx.x; b < b1; b += blockDim.x) A[p + b * r.lda] -= e * A[b + q * r.lda];
+    if (pin) {
+      for (int64_t a = p + 1 + threadIdx.x; a < r.n; a += blockDim.x) A[a + p * r.lda] -= e * A[a + q * r.lda];
+      if (threadIdx.x == 0) A[p + p * r.lda] -= 2 * e * A[p + q * r.lda] - e * e;
+    }
     // column checksums of tile column i: c(A_Ii)[:, pl] -= E * c(L_I)[:, ql], I >= i
-    for (int64_t I = i + threadIdx.x; I < nt; I += blockDim.x) {
+    for (int64_t I = i + threadIdx.x; pin && I < nt; I += blockDim.x) {
       T* dst = colchk + 2 * I + (i * nb + pl) * r.ldc;
       const T* src = colchk + 2 * I + (k * nb + ql) * r.ldc;
       dst[0] -= e * src[0];
@@ -136,6 +142,7 @@ __global__ void fig4a_repair_kernel(RepairArgs r) {
     }
     // row checksums of tile row i: r(A_iJ)[pl, :] -= E * c(L_J)[:, ql]^T, k < J <= i
     for (int64_t J = k + 1 + threadIdx.x; J <= i; J += blockDim.x) {
+      if (J * nb < r.c0 || J * nb >= r.c1) continue;
       T* dst = rowchk + p + (2 * J) * r.ldr;
       const T* src = colchk + 2 * J + (k * nb + ql) * r.ldc;
       dst[0] -= e * src[0];
@@ -191,6 +198,15 @@ extern "C" int ft_ctx_destroy(ft_ctx_t* c) {
   if (c->hpin) cudaFreeHost(c->hpin);
   if (c->ev) cudaEventDestroy(c->ev);
   if (c->join) cudaEventDestroy(c->join);
+  if (c->ev_col) cudaEventDestroy(c->ev_col);
+  if (c->ev_side) cudaEventDestroy(c->ev_side);
+  if (c->putmp2) cudaFree(c->putmp2);
+  if (c->side) {
+    cudaStreamSynchronize(c->side);
+    abft::release_stream_handles(c->side);
+    abft::release_stream_pools(c->side);
+    cudaStreamDestroy(c->side);
+  }
   if (c->drv) {
     // the library keeps cuBLAS / cuSOLVER handles, scratch and pass pools per
     // stream: release the private stream's before the stream goes away
@@ -230,28 +246,60 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
   FT_TRY(d.setup(c, dtype, n, nb, dA, lda, o, /*lu=*/false));
   const int64_t nt = d.nt;
   const bool ft = o->abft != 0;
-  cudaStream_t s = d.s;
   std::unique_lock<std::mutex> lk;
   auto t0 = std::chrono::steady_clock::now();
-  const abft_stream_t as = (abft_stream_t)s;
+  // Look-ahead (reading c-35): the next panel's PD / PU on the side stream
+  // next to the rest of the TMU; the new scheme (or the unprotected driver).
+  const bool la_on = o->lookahead && (!ft || s_new);
+  if (la_on) FT_TRY(d.side_setup());
+  // the same predicate as oracle/drivers.py::lookahead_ok: the split must not
+  // move a fault hook relative to Alg. 2 (c-8)
+  auto la_at = [&](int k) -> bool {
+    if (k + 1 >= nt) return false;
+    // the periodic trailing check of iteration k covers tile column k+1 too
+    if (ft && o->trailing_check_period > 0 && (k + 1) % o->trailing_check_period == 0) return false;
+    const int64_t c0 = (int64_t)(k + 1) * nb, c1 = c0 + nb;
+    for (int t = 0; t < o->n_inject; ++t) {
+      const ft_inject_t& f = o->inject[t];
+      if (f.iter == k && (f.point == FT_AT_PRE_TMU || f.point == FT_AT_POST_TMU)) return false;
+      if (f.iter == k + 1 && (f.point <= FT_AT_POST_PU || f.point == FT_AT_D2H || f.point == FT_AT_H2D)) {
+        bool inside;
+        if (f.target == 0 || f.target == 1)
+          inside = f.gj >= c0 && f.gj < c1;
+        else if (f.target == 2)
+          inside = f.gj == 2 * (k + 1) || f.gj == 2 * (k + 1) + 1;
+        else
+          inside = false;
+        if (!inside) return false;
+      }
+    }
+    return true;
+  };
 
   if (ft) {
     abft_tiles_t all{0, (int)nt, 0, (int)nt, 1, ABFT_SYM_LOWER};
-    FT_TRY(abft_encode(&d.M, &all, W, as));
+    FT_TRY(abft_encode(&d.M, &all, W, (abft_stream_t)d.s));
   }
-  for (int k = 0; k < nt; ++k) {
-    const int64_t r1 = (k + 1) * nb;  // first row/col after the panel
-    const int64_t nk = n - r1;        // trailing size
+  // Local restart (f1, L430): the PD input tile and the PU input panel are
+  // copied (with their checksums) right after their pre-op checks; a 2D
+  // error left by the post-op check restores the copy and redoes the op.
+  const bool rs = ft && o->restart && post_checks;
+
+  // ---- Alg. 2 lines 3-10 of iteration k: PD and PU with their checks, on d.s
+  // (the main stream, or the side stream under look-ahead).  fig4b_here: the
+  // Fig. 4b trailing check before the PU (under look-ahead the main stream
+  // runs it after the side stream joins: it reads only the trailing matrix).
+  auto chain = [&](int k, bool fig4b_here) -> int {
+    cudaStream_t s = d.s;
+    const abft_stream_t as = (abft_stream_t)s;
+    const int64_t r0 = (int64_t)k * nb;
+    const int64_t r1 = r0 + nb;   // first row/col after the panel
+    const int64_t nk = n - r1;    // trailing size
     const int m2 = (int)(2 * (nt - k - 1));
     if (ft) FT_TRY(d.begin_iteration());
     // Alg. 2 lines 3-4: check the panel to be decomposed (diag tile, SYM view, both)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
     if (ft && pre_checks) FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_SYM_LOWER, W));
-    // Local restart (f1, L430): the PD input tile and the PU input panel are
-    // copied (with their checksums) right after their pre-op checks; a 2D
-    // error left by the post-op check restores the copy and redoes the op.
-    const bool rs = ft && o->restart && post_checks;
-    const int64_t r0 = (int64_t)k * nb;
     char* rbuf = (char*)c->rsv;
     auto copy2d = [&](void* dst, int64_t ldd, const void* src, int64_t lds, int64_t rows, int64_t cols) -> int {
       if (rows <= 0 || cols <= 0) return 0;
@@ -267,7 +315,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     char* pu_m = pu_c + (size_t)m2 * nb * d.es;
     // PD restart decision: snapshot the uncorrectable count before the check,
     // read the difference back into pinned memory after it (one event)
-    auto post_readback = [&](int32_t*) -> int { return d.post_delta(0); };
+    auto post_readback = [&]() -> int { return d.post_delta(0); };
     auto readback_delta = [&](int* delta) -> int { return d.wait_delta(0, delta); };
     if (rs) {
       FT_TRY(copy2d(pd_a, nb, d.a_at(r0, r0), lda, nb, nb));
@@ -305,12 +353,12 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft && post_checks) {
       if (rs) ABFT_CUDA_TRY(cudaMemcpyAsync(d.snap, d.counts + ABFT_CNT_UNCORRECTABLE, 4, cudaMemcpyDeviceToDevice, s));
       FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_LOWER, ABFT_COL));
-      if (rs) FT_TRY(post_readback(d.snap));
+      if (rs) FT_TRY(post_readback());
     }
     // The PD restart decision is taken after the pre-PU check has been queued
-    // (that check reads only the panel below A_kk), so the host waits on the
-    // read-back while the device is busy.  Not when the fault plan injects at
-    // the pre-PU-check point: then the paper's order is kept exactly.
+    // (that check reads only the panel below A_kk), so the host waits while the
+    // device works.  Not when the fault plan injects at the pre-PU-check point:
+    // then the paper's order is kept exactly.
     const bool defer_pd = rs && k < nt - 1 && !d.has_inject(k, FT_AT_PRE_PU_CHECK);
     auto pd_restart = [&]() -> int {
       int delta = 0;
@@ -325,7 +373,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       return d.check(k, k + 1, k, k + 1, ABFT_LOWER, ABFT_COL);
     };
     if (rs && !defer_pd) FT_TRY(pd_restart());
-    if (k == nt - 1) break;
+    if (k == nt - 1) return 0;
     // line 8: check the panel to be updated (both checksums)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PU_CHECK));
     if (ft && pre_checks) FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, W));
@@ -338,7 +386,9 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     // Fig. 4b (L359): a 1D pattern fixed by this iteration's pre-PD / pre-PU
     // checks is the trace of an on-chip fault in the last TMU: check the
     // whole trailing matrix now (gated on the device)
-    if (ft && s_new) FT_TRY(d.fig4b_check(k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, ABFT_BOTH, true));
+    if (ft && s_new && fig4b_here)
+      FT_TRY(d.fig4b_check(k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, ABFT_BOTH, true));
+    if (ft && s_new && !fig4b_here) FT_TRY(d.mark_fig4b_end());  // the deferred check's window ends here
     // line 9: PU  L_ik = A_ik L_kk^-T  (+ c(L_ik) = c(A_ik) L_kk^-T, c-12)
     auto pu_data = [&]() -> int {
       cublasHandle_t h = blas_handle(s, lk);
@@ -411,6 +461,101 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       };
       if (rs) FT_TRY(d.gated_restart(1, pu_redo));
     }
+    return 0;
+  };
+
+  // ---- TMU data step on trailing columns [c0, c1) (tile aligned, c1 = n or
+  // c0 + nb): the lower part of A[c0:n, c0:c1] -= L21 L21[c0-r1 .. c1-r1]^T
+  auto tmu_data = [&](int k, int64_t c0, int64_t c1) -> int {
+    const int64_t r0 = (int64_t)k * nb, w = c1 - c0, below = n - c1;
+    if (w <= 0) return 0;
+    cublasHandle_t h = blas_handle(d.s, lk);
+    cublasStatus_t st = CUBLAS_STATUS_SUCCESS;
+    if (dtype == ABFT_F64) {
+      const double m1 = -1.0, one = 1.0;
+      st = cublasDsyrk(h, CUBLAS_FILL_MODE_LOWER, CUBLAS_OP_N, (int)w, (int)nb, &m1, (const double*)d.a_at(c0, r0),
+                       (int)lda, &one, (double*)d.a_at(c0, c0), (int)lda);
+      if (st == CUBLAS_STATUS_SUCCESS && below > 0)
+        st = cublasDgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)below, (int)w, (int)nb, &m1, (const double*)d.a_at(c1, r0),
+                         (int)lda, (const double*)d.a_at(c0, r0), (int)lda, &one, (double*)d.a_at(c1, c0), (int)lda);
+    } else {
+      const float m1 = -1.0f, one = 1.0f;
+      st = cublasSsyrk(h, CUBLAS_FILL_MODE_LOWER, CUBLAS_OP_N, (int)w, (int)nb, &m1, (const float*)d.a_at(c0, r0),
+                       (int)lda, &one, (float*)d.a_at(c0, c0), (int)lda);
+      if (st == CUBLAS_STATUS_SUCCESS && below > 0)
+        st = cublasSgemm(h, CUBLAS_OP_N, CUBLAS_OP_T, (int)below, (int)w, (int)nb, &m1, (const float*)d.a_at(c1, r0),
+                         (int)lda, (const float*)d.a_at(c0, r0), (int)lda, &one, (float*)d.a_at(c1, c0), (int)lda);
+    }
+    lk.unlock();
+    return st == CUBLAS_STATUS_SUCCESS ? 0 : ABFT_E_CUBLAS;
+  };
+  // ---- TMU checksum rules (c-12, L189) for trailing tile columns [c0, c1)
+  auto tmu_chk = [&](int k, int64_t c0, int64_t c1) -> int {
+    const int64_t r0 = (int64_t)k * nb;
+    const abft_stream_t as = (abft_stream_t)d.s;
+    const int J0 = (int)(c0 / nb), J1 = (int)(c1 / nb);
+    if (J1 <= J0) return 0;
+    if (c1 == n) {  // tile columns J0.. (to the end): the one-product rule of the sub-problem
+      const int64_t ntk = nt - J0;
+      return abft_update_syrk(dtype, nb, ntk, d.a_at(c0, r0), lda, d.colchk_at(2 * J0, r0), d.M.ldc,
+                              d.colmag_at(J0, r0), d.M.ldcm, d.colchk_at(2 * J0, c0),
+                              single ? nullptr : d.rowchk_at(c0, 2 * J0), d.M.ldr, d.colmag_at(J0, c0),
+                              single ? nullptr : d.rowmag_at(c0, J0), d.M.ldrm, as);
+    }
+    // one tile column J0 (look-ahead's first part): every tile I >= J0 of it
+    //   c(A_I,J0) -= c(L_Ik) L_J0,k^T,  m_c += m_c(L_Ik) |L_J0,k|^T
+    //   r(A_I,J0) -= L_Ik c(L_J0,k)^T,  m_r += |L_Ik| m_c(L_J0,k)^T
+    const int64_t m2 = 2 * (nt - J0);
+    FT_TRY(abft_update_gemm(dtype, ABFT_COL, 'N', 'T', -1.0, d.colchk_at(2 * J0, r0), d.M.ldc, d.a_at(c0, r0), lda,
+                            d.colchk_at(2 * J0, c0), d.M.ldc, m2, nb, nb, d.colmag_at(J0, r0), d.M.ldcm,
+                            d.colmag_at(J0, c0), d.M.ldcm, as));
+    if (single) return 0;
+    return panel_row_rule(dtype, n - c0, nb, d.a_at(c0, r0), lda, d.colchk_at(2 * J0, r0), d.colchk_at(2 * J0 + 1, r0),
+                          d.M.ldc, d.colmag_at(J0, r0), d.M.ldcm, d.rowchk_at(c0, 2 * J0),
+                          d.rowchk_at(c0, 2 * J0 + 1), d.rowmag_at(c0, J0), d.s);
+  };
+  // ---- line 13: heuristic panel re-check for the TMU (Fig. 4a) + guarded
+  // repair (c-25) restricted to the trailing columns [c0, c1) that consumed it
+  auto recheck = [&](int k, int64_t c0, int64_t c1) -> int {
+    ABFT_CUDA_TRY(cudaMemcpyAsync(d.mark, d.nfix, sizeof(int32_t), cudaMemcpyDeviceToDevice, d.s));
+    FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
+    if (!o->fig4a_repair) return 0;
+    RepairArgs ra{};
+    ra.A = dA;
+    ra.lda = lda;
+    ra.n = n;
+    ra.nb = nb;
+    ra.k = k;
+    ra.colchk = d.M.colchk;
+    ra.rowchk = d.M.rowchk;
+    ra.colmag = d.M.colmag;
+    ra.rowmag = d.M.rowmag;
+    ra.ldc = d.M.ldc;
+    ra.ldr = d.M.ldr;
+    ra.ldcm = d.M.ldcm;
+    ra.ldrm = d.M.ldrm;
+    ra.fixes = c->fixlog;
+    ra.cap = c->fixcap;
+    ra.n_fixes = d.nfix;
+    ra.mark = d.mark;
+    ra.rep_counts = d.rep;
+    ra.counts = d.counts;
+    ra.c0 = c0;
+    ra.c1 = c1;
+    if (dtype == ABFT_F64)
+      fig4a_repair_kernel<double><<<1, 256, 0, d.s>>>(ra);
+    else
+      fig4a_repair_kernel<float><<<1, 256, 0, d.s>>>(ra);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    return 0;
+  };
+
+  bool chained = false;  // iteration k's PD / PU already ran as look-ahead
+  for (int k = 0; k < nt; ++k) {
+    if (!chained) FT_TRY(chain(k, true));
+    chained = false;
+    if (k == nt - 1) break;
+    const int64_t r1 = (int64_t)(k + 1) * nb, r2 = r1 + nb;
     // prior-operation scheme [11]: the TMU's inputs (panel, trailing matrix) before it
     if (ft && scheme == FT_SCHEME_SINGLE_PRE) {
       FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
@@ -418,68 +563,49 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     }
     // line 12: TMU  A22 -= L21 L21^T (DSYRK on tensor cores) + checksum rules c-12
     FT_TRY(d.inject_at(k, FT_AT_PRE_TMU));
+    if (la_on && la_at(k)) {
+      // look-ahead (c-35): tile column k+1 first, its re-check, then the rest
+      // of the TMU on the main stream while the side stream runs PD / PU of
+      // iteration k+1 (enqueued after the rest: the side chain's host waits
+      // then overlap the DSYRK)
+      FT_TRY(tmu_data(k, r1, r2));
+      FT_TRY(d.restore_onchip());
+      if (ft) {
+        FT_TRY(tmu_chk(k, r1, r2));
+        FT_TRY(recheck(k, r1, r2));
+      }
+      ABFT_CUDA_TRY(cudaEventRecord(c->ev_col, d.s));
+      FT_TRY(tmu_data(k, r2, n));
+      if (ft) {
+        FT_TRY(tmu_chk(k, r2, n));
+        FT_TRY(d.inject_at(k, FT_AT_POST_TMU));
+        FT_TRY(recheck(k, r2, n));
+        FT_TRY(d.periodic_check(k, k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, true));
+      }
+      ABFT_CUDA_TRY(cudaStreamWaitEvent(c->side, c->ev_col, 0));
+      d.on_side(true);
+      const int rc = chain(k + 1, false);
+      if (rc == 0) ABFT_CUDA_TRY(cudaEventRecord(c->ev_side, d.s));
+      d.on_side(false);
+      if (rc) return rc;
+      ABFT_CUDA_TRY(cudaStreamWaitEvent(d.s, c->ev_side, 0));
+      if (ft && k + 1 < nt - 1)  // Fig. 4b of iteration k+1 (reads the trailing matrix only)
+        FT_TRY(d.fig4b_check(k + 2, (int)nt, k + 2, (int)nt, ABFT_SYM_LOWER, ABFT_BOTH, true, /*deferred=*/true));
+      chained = true;
+      continue;
+    }
     // (Running the checksum rule and the panel re-check on a second stream
     // next to the DSYRK was measured: no gain at any stream priority — the
     // DSYRK keeps every SM busy — so everything stays on one stream.)
-    cudaStream_t cs = s;
-    {
-      cublasHandle_t h = blas_handle(s, lk);
-      if (dtype == ABFT_F64) {
-        const double m1 = -1.0, one = 1.0;
-        if (cublasDsyrk(h, CUBLAS_FILL_MODE_LOWER, CUBLAS_OP_N, (int)nk, (int)nb, &m1, (const double*)d.a_at(r1, k * nb),
-                        (int)lda, &one, (double*)d.a_at(r1, r1), (int)lda) != CUBLAS_STATUS_SUCCESS)
-          return ABFT_E_CUBLAS;
-      } else {
-        const float m1 = -1.0f, one = 1.0f;
-        if (cublasSsyrk(h, CUBLAS_FILL_MODE_LOWER, CUBLAS_OP_N, (int)nk, (int)nb, &m1, (const float*)d.a_at(r1, k * nb),
-                        (int)lda, &one, (float*)d.a_at(r1, r1), (int)lda) != CUBLAS_STATUS_SUCCESS)
-          return ABFT_E_CUBLAS;
-      }
-      lk.unlock();
-    }
+    FT_TRY(tmu_data(k, r1, n));
     FT_TRY(d.restore_onchip());  // on-chip flips hit the data step only (c-8)
-    if (ft) {
-      // c(A_ij) -= c(L_ik) L_jk^T and r(A_ij) -= L_ik c(L_jk)^T from one product (c-12, L189)
-      FT_TRY(abft_update_syrk(dtype, nb, nt - k - 1, d.a_at(r1, k * nb), lda, d.colchk_at(2 * (k + 1), k * nb), d.M.ldc,
-                              d.colmag_at(k + 1, k * nb), d.M.ldcm, d.colchk_at(2 * (k + 1), r1),
-                              single ? nullptr : d.rowchk_at(r1, 2 * (k + 1)), d.M.ldr, d.colmag_at(k + 1, r1),
-                              single ? nullptr : d.rowmag_at(r1, k + 1), d.M.ldrm, (abft_stream_t)cs));
-    }
+    if (ft) FT_TRY(tmu_chk(k, r1, n));  // c(A_ij) -= c(L_ik) L_jk^T, r(A_ij) -= L_ik c(L_jk)^T from one product
     FT_TRY(d.inject_at(k, FT_AT_POST_TMU));
     // post-operation schemes [13], [51, 52]: the TMU's output, the whole trailing matrix
     if (ft && (scheme == FT_SCHEME_FULL_POST || scheme == FT_SCHEME_SINGLE_POST))
       FT_TRY(d.check(k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, W, true));
-    // line 13: heuristic panel re-check for the TMU (Fig. 4a) + guarded repair (c-25)
     if (ft && s_new) {
-      ABFT_CUDA_TRY(cudaMemcpyAsync(d.mark, d.nfix, sizeof(int32_t), cudaMemcpyDeviceToDevice, cs));
-      FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL, false, cs));
-      if (o->fig4a_repair) {
-        RepairArgs ra{};
-        ra.A = dA;
-        ra.lda = lda;
-        ra.n = n;
-        ra.nb = nb;
-        ra.k = k;
-        ra.colchk = d.M.colchk;
-        ra.rowchk = d.M.rowchk;
-        ra.colmag = d.M.colmag;
-        ra.rowmag = d.M.rowmag;
-        ra.ldc = d.M.ldc;
-        ra.ldr = d.M.ldr;
-        ra.ldcm = d.M.ldcm;
-        ra.ldrm = d.M.ldrm;
-        ra.fixes = c->fixlog;
-        ra.cap = c->fixcap;
-        ra.n_fixes = d.nfix;
-        ra.mark = d.mark;
-        ra.rep_counts = d.rep;
-        ra.counts = d.counts;
-        if (dtype == ABFT_F64)
-          fig4a_repair_kernel<double><<<1, 256, 0, cs>>>(ra);
-        else
-          fig4a_repair_kernel<float><<<1, 256, 0, cs>>>(ra);
-        ABFT_CUDA_TRY(cudaGetLastError());
-      }
+      FT_TRY(recheck(k, 0, n));
       // periodic trailing-matrix check (L359)
       FT_TRY(d.periodic_check(k, k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, true));
     }

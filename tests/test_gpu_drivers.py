@@ -18,30 +18,35 @@ def ctx(lib):
     return lib.Context()
 
 
-def _gpu_potrf(lib, ctx, A_np, nb, inject=(), abft=True, fig4a=True, dtype=torch.float64):
+def _gpu_potrf(lib, ctx, A_np, nb, inject=(), abft=True, fig4a=True, dtype=torch.float64, lookahead=True):
     A = dev(A_np, dtype)
     inj = [(f.iter, f.point, f.kind, f.target, f.gi, f.gj, si.mask_of(f.bits)) for f in inject]
     log = torch.zeros(8192 * lib.FIX_BYTES, dtype=torch.uint8, device="cuda")
-    rc, info, stats = lib.ft_potrf(ctx, A, nb, abft=abft, fig4a_repair=fig4a, inject=inj, fix_log=log)
+    rc, info, stats = lib.ft_potrf(ctx, A, nb, abft=abft, fig4a_repair=fig4a, inject=inj, fix_log=log,
+                                   lookahead=lookahead)
     torch.cuda.synchronize()
     fixes = lib.decode_fixes(log, stats.n_fixes)
     return np.tril(host(A)), rc, info, stats, fixes
 
 
+@pytest.mark.parametrize("lookahead", [True, False])
 @pytest.mark.parametrize("n,nb", [(256, 32), (1024, 128), (2048, 256), (2048, 512), (4096, 1024)])
-def test_error_free_matches_lapack(lib, ctx, n, nb):
+def test_error_free_matches_lapack(lib, ctx, n, nb, lookahead):
     A = si.spd(n, seed=n)
-    L, rc, info, stats, fixes = _gpu_potrf(lib, ctx, A, nb)
+    L, rc, info, stats, fixes = _gpu_potrf(lib, ctx, A, nb, lookahead=lookahead)
     Lref = np.linalg.cholesky(A)
     assert rc == 0 and info == 0 and stats.counts[:] == [0] * 8 and not fixes
     assert np.abs(L - Lref).max() <= 1e-12 * np.abs(Lref).max()
-    assert stats.n_checks == 5 * (n // nb - 1) + 2
+    # Alg. 2: 5 checks per iteration, 2 in the last; look-ahead adds the
+    # panel re-check after the tile-column update (reading c-35)
+    assert stats.n_checks == (6 if lookahead else 5) * (n // nb - 1) + 2
 
 
-def test_unprotected_same_factor(lib, ctx):
+@pytest.mark.parametrize("lookahead", [True, False])
+def test_unprotected_same_factor(lib, ctx, lookahead):
     A = si.spd(1024, seed=1)
-    L0, *_ = _gpu_potrf(lib, ctx, A, 128, abft=False)
-    L1, *_ = _gpu_potrf(lib, ctx, A, 128, abft=True)
+    L0, *_ = _gpu_potrf(lib, ctx, A, 128, abft=False, lookahead=lookahead)
+    L1, *_ = _gpu_potrf(lib, ctx, A, 128, abft=True, lookahead=lookahead)
     assert np.abs(L0 - L1).max() <= 1e-13 * np.abs(L0).max()
 
 
@@ -52,7 +57,7 @@ def test_not_spd_info(lib, ctx):
     assert info == 64 + 7
 
 
-def _compare(lib, ctx, A, nb, injects, fig4a=True, prec="f64"):
+def _compare(lib, ctx, A, nb, injects, fig4a=True, prec="f64", lookahead=True):
     """Same fault plan on the oracle driver and the GPU driver: counters, fix
     positions / classes / kinds, restarts and repairs identical; factors
     within 1e-12 (fp64) / 1e-5 (fp32) of LAPACK's.  fp32: the GPU factors in
@@ -61,9 +66,9 @@ def _compare(lib, ctx, A, nb, injects, fig4a=True, prec="f64"):
     vtol = 1e-12 if prec == "f64" else 1e-5
     if prec == "f32":
         A = A.astype(np.float32).astype(np.float64)
-    Lo, so = dr.ft_potrf(A, nb, prec=prec, inject=injects, fig4a_repair=fig4a)
+    Lo, so = dr.ft_potrf(A, nb, prec=prec, inject=injects, fig4a_repair=fig4a, lookahead=lookahead)
     Lg, rc, info, sg, fg = _gpu_potrf(lib, ctx, A, nb, inject=injects, fig4a=fig4a,
-                                      dtype=torch.float64 if prec == "f64" else torch.float32)
+                                      dtype=torch.float64 if prec == "f64" else torch.float32, lookahead=lookahead)
     assert (rc == lib.E_UNCORRECTABLE) == (so.uncorrectable > 0)
     assert sg.repairs_skipped == so.repairs_skipped
     if so.repairs_skipped:
@@ -71,6 +76,7 @@ def _compare(lib, ctx, A, nb, injects, fig4a=True, prec="f64"):
         # matrix: the outcome is R (detected, restart); what the checks see
         # afterwards is Inf/NaN arithmetic and not compared
         return so, sg
+    assert sg.n_checks == so.n_checks
     # fp32: counts[3] (tiles with a non-finite delta) records fp32 overflow of
     # the recomputed sums, which the oracle (fp32 data summed in fp64) cannot see
     nf = [3] if prec == "f32" else []
@@ -107,11 +113,12 @@ CASES = [
 ]
 
 
+@pytest.mark.parametrize("lookahead", [True, False])
 @pytest.mark.parametrize("case", range(len(CASES)))
-def test_fault_campaign_parity(lib, ctx, case):
+def test_fault_campaign_parity(lib, ctx, case, lookahead):
     point, kind, target, gi, gj, bits = CASES[case]
     A = si.spd(256, seed=0)
-    _compare(lib, ctx, A, 32, [dr.Inject(2, point, kind, target, gi, gj, bits)])
+    _compare(lib, ctx, A, 32, [dr.Inject(2, point, kind, target, gi, gj, bits)], lookahead=lookahead)
 
 
 # fp32 (every entry point takes ABFT_F32; BASELINE's 1e-5): the same fault
@@ -238,7 +245,7 @@ _ONCHIP_PAIR = [dr.Inject(1, dr.AT_PRE_TMU, dr.KIND_ONCHIP, 0, 197, 40, (55,)),
 def test_fig4b_and_periodic_parity(lib, ctx, fig4b, period):
     A_np = si.spd(256, seed=41)
     o_L, ost = dr.ft_potrf(A_np, 32, inject=_ONCHIP_PAIR, fig4b=fig4b, restart=False,
-                           trailing_check_period=period)
+                           trailing_check_period=period, lookahead=True)
     A = dev(A_np)
     inj = [(f.iter, f.point, f.kind, f.target, f.gi, f.gj, si.mask_of(f.bits)) for f in _ONCHIP_PAIR]
     log = torch.zeros(8192 * lib.FIX_BYTES, dtype=torch.uint8, device="cuda")

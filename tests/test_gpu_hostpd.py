@@ -96,7 +96,7 @@ def test_host_pd_fault_free_matches_lapack(lib, ctx, which, abft):
 def _parity(lib, ctx, which, A, nb, inject):
     g_out, g_ex, rc, info, stats, gfix = _run(lib, ctx, which, A, nb, inject)
     if which == "potrf":
-        o_out, ost = dr.ft_potrf(A, nb, inject=inject, pd_location="host")
+        o_out, ost = dr.ft_potrf(A, nb, inject=inject, pd_location="host", lookahead=True)
         ref, _ = dr.ft_potrf(A, nb)
     elif which == "getrf":
         o_out, o_piv, ost = dr.ft_getrf(A, nb, inject=inject, pd_location="host")

@@ -33,7 +33,7 @@ def _gpu(lib, ctx, A_np, nb, scheme, inject=()):
 def test_scheme_error_free(lib, ctx, scheme, n, nb):
     A = si.spd(n, seed=n + scheme)
     L, rc, st, fixes = _gpu(lib, ctx, A, nb, scheme)
-    _, so = dr.ft_potrf(A, nb, scheme=scheme)
+    _, so = dr.ft_potrf(A, nb, scheme=scheme, lookahead=True)
     Lref = np.linalg.cholesky(A)
     assert rc == 0 and list(st.counts) == [0] * 8 and not fixes
     assert st.n_checks == so.n_checks
@@ -45,7 +45,7 @@ def test_scheme_error_free(lib, ctx, scheme, n, nb):
 def test_scheme_fault_parity(lib, ctx, scheme, case):
     f, expect = SCHEME_OUTCOMES[case]
     A = si.spd(256, seed=3)
-    Lo, so = dr.ft_potrf(A, 32, inject=[f], scheme=scheme)
+    Lo, so = dr.ft_potrf(A, 32, inject=[f], scheme=scheme, lookahead=True)
     Lg, rc, sg, fg = _gpu(lib, ctx, A, 32, scheme, inject=[f])
     assert (rc == lib.E_UNCORRECTABLE) == (so.uncorrectable > 0) == (expect[scheme] == "R")
     assert sg.restarts == so.restarts

@@ -20,13 +20,13 @@ ipiv = torch.zeros(n, dtype=torch.int64, device="cuda")
 tau = torch.zeros(n, dtype=torch.float64, device="cuda")
 
 
-def run(ft, restart=True):
+def run(ft, restart=True, la=True):
     A.copy_(A0)
     torch.cuda.synchronize()
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     a.record()
     if which == "potrf":
-        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart)
+        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart, lookahead=la)
     elif which == "getrf":
         rc, info, st = abft.ft_getrf(ctx, A, nb, ipiv, abft=ft, restart=restart)
     else:
@@ -46,6 +46,9 @@ def med(f):
 plain = med(lambda: run(False))
 ft = med(lambda: run(True))
 nors = med(lambda: run(True, restart=False))
+if which == "potrf":
+    p0, f0 = med(lambda: run(False, la=False)), med(lambda: run(True, la=False))
+    print(f"potrf without look-ahead: plain {p0:.2f} ms, ft {f0:.2f} ms ({100 * (f0 - p0) / p0:.2f}%)")
 S = A0.t().contiguous()
 torch.backends.cuda.preferred_linalg_library("cusolver")
 lib = {"potrf": lambda: torch.linalg.cholesky(S), "getrf": lambda: torch.linalg.lu_factor(S),
