@@ -152,10 +152,9 @@ def workload_config(n, nb, world, potrf_n):
 
 
 def run_reference(args):
-    """The oracle on the host cores: encode + verify of a bounded sample of
-    nb x nb tiles of the same fp64 U(-1,1) workload, same byte formula."""
-    import numpy as np
-
+    """The oracle on the host cores: each step = encode + verify of a bounded
+    sample (8 tiles) of nb x nb tiles drawn across an 8192^2 fp64 U(-1,1)
+    matrix (not cache resident), same byte formula; host BLAS on all cores."""
     import synth_inputs as si
     from oracle import checksum as ck
 
@@ -163,15 +162,19 @@ def run_reference(args):
     if rank != 0:
         return
     cores = len(os.sched_getaffinity(0))
-    nb = NB
+    nb, m = NB, 8192
     n_tiles_sample = 8  # tiles per step sample
-    st = ck.State.alloc(si.general(nb * 2, nb * 4, seed=0), nb)
-    tiles = ck.Tiles(0, 2, 0, 4)
+    st = ck.State.alloc(si.general(m, seed=0), nb)
+    mt = m // nb
+    g = si.rng(6)
     step_t = []
     for s in range(args.warmup + args.steps):
+        picks = [(int(g.integers(0, mt)), int(g.integers(0, mt))) for _ in range(n_tiles_sample)]
         t0 = time.perf_counter()
-        ck.encode(st, tiles)
-        ck.verify(st, tiles)
+        for I, J in picks:
+            t = ck.Tiles(I, I + 1, J, J + 1)
+            ck.encode(st, t)
+            ck.verify(st, t)
         dt = time.perf_counter() - t0
         if s >= args.warmup:
             step_t.append(dt)
@@ -183,33 +186,85 @@ def run_reference(args):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": workload_config(args.n, nb, int(os.environ.get("WORLD_SIZE", "1")), args.potrf_n),
-        "cpu_baseline": {"value": val, "unit": "GB/s", "cores": cores, "kind": "oracle",
-                         "sample": f"{n_tiles_sample} tiles of {nb}x{nb} fp64 per step (a bounded sample of the "
-                                   f"n={args.n} workload; GB/s with the same per-tile byte formula)"},
+        "cpu_baseline": {"value": val, "unit": "GB/s", "cores": cores, "kind": "oracle", "cpu": _cpu_model(),
+                         "sample": f"{n_tiles_sample} tiles of {nb}x{nb} fp64 per step drawn across an 8192^2 "
+                                   f"matrix (not cache resident; a bounded sample of the n={args.n} workload, "
+                                   f"GB/s with the same per-tile byte formula); host BLAS threads = {cores}"},
         "e2e": {"value": val, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
 
 
-def cpu_baseline_sample(seconds=10.0):
-    """Oracle encode+verify on host cores over a bounded sample (~10 s)."""
-    import numpy as np
+def _oracle_ev_rate(seconds, threads):
+    """Oracle encode+verify GB/s (the same per-tile byte formula as the GPU)
+    over tiles spread across an 8192 x 8192 fp64 matrix (512 MB, larger than
+    the host caches, so every tile comes from DRAM), with the host BLAS
+    limited to `threads` threads; returns (GB/s, tiles, seconds)."""
+    import threadpoolctl
 
     import synth_inputs as si
     from oracle import checksum as ck
 
-    nb = NB
-    st = ck.State.alloc(si.general(nb * 4, nb * 4, seed=1), nb)
-    tiles = ck.Tiles(0, 4, 0, 4)
-    done, t0 = 0, time.perf_counter()
-    while time.perf_counter() - t0 < seconds:
-        ck.encode(st, tiles)
-        ck.verify(st, tiles)
-        done += 16
-    dt = time.perf_counter() - t0
-    val = 2 * done * alg_bytes(nb, nb, 8) / dt / 1e9
-    return {"value": val, "unit": "GB/s", "cores": len(os.sched_getaffinity(0)), "kind": "oracle",
-            "sample": f"{done} tiles of {nb}x{nb} fp64 (encode+verify), {dt:.1f} s"}
+    nb, m = NB, 8192
+    st = ck.State.alloc(si.general(m, seed=1), nb)
+    mt = m // nb
+    order = [(I, J) for J in range(mt) for I in range(mt)]
+    g = si.rng(5)
+    g.shuffle(order)
+    done, k = 0, 0
+    with threadpoolctl.threadpool_limits(limits=threads, user_api="blas"):
+        t0 = time.perf_counter()
+        while time.perf_counter() - t0 < seconds:
+            I, J = order[k % len(order)]
+            t = ck.Tiles(I, I + 1, J, J + 1)
+            ck.encode(st, t)
+            ck.verify(st, t)
+            done += 1
+            k += 1
+        dt = time.perf_counter() - t0
+    return 2 * done * alg_bytes(nb, nb, 8) / dt / 1e9, done, dt
+
+
+def cpu_baseline_sample(seconds=10.0, potrf_n=10240):
+    """The oracle (oracle/, numpy + the host BLAS, untuned) on this box's host
+    cores: encode+verify GB/s with the host BLAS on all
+    affinity cores and on 1 core (non-cache-resident tiles), and the oracle's
+    ft_potrf wall time at n=10240 nb=512 (Alg. 2, all cores).  `cores` is the
+    BLAS thread count of the all-cores run; numpy's elementwise steps are
+    single-threaded, so that is an upper bound on the threads used."""
+    import threadpoolctl
+
+    import synth_inputs as si
+    from oracle import drivers as dr
+
+    all_cores = len(os.sched_getaffinity(0))
+    v_all, n_all, t_all = _oracle_ev_rate(seconds / 2, all_cores)
+    v_one, n_one, t_one = _oracle_ev_rate(seconds / 2, 1)
+    potrf_s = None
+    if potrf_n:
+        A = si.spd(potrf_n, seed=7)
+        with threadpoolctl.threadpool_limits(limits=all_cores, user_api="blas"):
+            t0 = time.perf_counter()
+            dr.ft_potrf(A, NB)
+            potrf_s = time.perf_counter() - t0
+    return {"value": v_all, "unit": "GB/s", "cores": all_cores, "kind": "oracle",
+            "value_1core": v_one, "cores_1core": 1,
+            "ft_potrf_s": potrf_s, "ft_potrf_n": potrf_n, "ft_potrf_cores": all_cores,
+            "cpu": _cpu_model(),
+            "sample": f"encode+verify of {n_all} (all cores, {t_all:.1f} s) / {n_one} (1 core, {t_one:.1f} s) "
+                      f"{NB}x{NB} fp64 tiles drawn across an 8192^2 matrix (512 MB, not cache resident); "
+                      f"oracle ft_potrf n={potrf_n} nb={NB} once (Alg. 2, error free)"}
+
+
+def _cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
 
 
 # ------------------------------------------------------------------ ours --

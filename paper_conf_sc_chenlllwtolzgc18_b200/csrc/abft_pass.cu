@@ -378,6 +378,12 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
   const T* tileA = A + (int64_t)J * NB * p.lda + (int64_t)Ib * NB;
   // phase-A and phase-B masks: SYM uses LOWER for columns, strict lower for rows
   const int viewA = sym ? ABFT_LOWER : view;
+  // a single-side check skips the other direction's sums (a SYM tile needs
+  // both: its column checksums are colsum(lower) + rowsum(strict lower));
+  // uniform per CTA.  COL-only verifies (post-PD / post-PU / Fig. 4a re-checks)
+  // then do half the consumer work per element.
+  const bool do_cols = sym || (p.which & ABFT_COL);
+  const bool do_rows = sym || (p.which & ABFT_ROW);
 
   if (tid == 0) {
     for (int t = 0; t < K; ++t) {
@@ -497,7 +503,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
     // ---------------- phase A: column sums (one warp per column) ----------
     // this warp's columns of the stage: (s*CC + cc) % kWarps == warp (no per-column skip test)
 #pragma unroll 1
-    for (int cc = (warp - s * C::CC) & (kWarps - 1); cc < C::CC; cc += kWarps) {
+    for (int cc = (warp - s * C::CC) & (kWarps - 1); do_cols && cc < C::CC; cc += kWarps) {
       const int jl = c0 + s * C::CC + cc;  // tile-local column
       const T* col = buf + cc * RK;
       if (viewA == ABFT_GENERAL) {
@@ -552,7 +558,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
 #pragma unroll
     for (int q = 0; q < C::RPT; ++q) {
       const int r = tid + q * kThreads;
-      if (r < RV) {
+      if (do_rows && r < RV) {
         if (view == ABFT_GENERAL) {
           // per CQ-column chunk: sum (jl+1) x with jl = base + cq  =  (base + 1) * S0 + sum_cq cq*x
 #pragma unroll
@@ -586,7 +592,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
       if (lane == 0) mbar_arrive(&empty[slot]);
     }
     const bool group_end = (((s + 1) * C::CC) % C::GC) == 0;
-    if (group_end) {
+    if (group_end && do_rows) {
       const int g = (c0 + (s + 1) * C::CC) / C::GC - 1;
 #pragma unroll
       for (int q = 0; q < C::RPT; ++q) {
@@ -661,7 +667,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
 #pragma unroll
     for (int q = 0; q < C::RPT; ++q) {
       const int r = tid + q * kThreads;
-      if (r < RV) {
+      if (do_rows && r < RV) {
         for (int g = 0; g < C::GROUPS; ++g) {
           const T* src = partT + (((size_t)sup * C::GROUPS + g) * RK + r) * 3;
           tot[q].e = fadd(tot[q].e, __ldcg(src + 0));
