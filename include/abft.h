@@ -378,6 +378,8 @@ typedef struct {
   int32_t scheme;        /* FT_SCHEME_* (ft_potrf only; ft_getrf / ft_geqrf return -7 for anything but
                             FT_SCHEME_NEW): the checking scheme, for the paper's comparison of
                             schemes (L35, L47, L542, Table VIII, Figs. 12-14; reading c-34) */
+  int32_t timing;        /* 1: per-phase device time (CUDA events on the stream each phase runs on) into
+                            ft_stats_t.ms_phase; costs two event records per timed span.  Default 0. */
   int32_t lookahead;     /* ft_potrf (FT_SCHEME_NEW or abft = 0): 1 = the TMU of iteration k updates tile
                             column k+1 first (and re-checks the panel, Fig. 4a), then the PD / PU of
                             iteration k+1 with their checks run on a second stream next to the rest of
@@ -418,7 +420,19 @@ typedef struct {
   /* ft_geqrf CTF check (row f2, L263; reading c-29) */
   int32_t ctf_flagged;          /* checks whose E = T^T V^T V T - T - T^T exceeded the bound */
   int32_t ctf_recomputed;       /* T recomputed from V after a flagged check */
+  /* outcomes by class, from the fix log of the run */
+  int32_t detected;             /* tiles a check flagged (= counts[ABFT_CNT_TILES_FLAGGED]) */
+  int32_t corrected_0d;         /* data elements fixed as 0D errors (L330) */
+  int32_t corrected_1d;         /* data elements fixed as part of a 1D pattern (1D_ROW, 1D_COL, SYM_CROSS) */
+  int32_t checksum_repaired;    /* checksum entries re-encoded (CHK_CORRUPT, STALE_R, STALE_C) */
+  int32_t comm_errors;          /* transfer-guard corrections and repeats (FT_PD_HOST, Alg. 2 lines 3-7) */
+  /* opts->timing: device ms per phase (FT_PH_*), summed over the run; the
+     phases of the look-ahead side stream overlap the main stream's */
+  double ms_phase[8];
 } ft_stats_t;
+/* ft_stats_t.ms_phase indices */
+enum { FT_PH_PD = 0, FT_PH_PU = 1, FT_PH_TMU = 2, FT_PH_RULES = 3, FT_PH_CHECKS = 4, FT_PH_RESTART = 5,
+       FT_PH_ENCODE = 6, FT_PH_OTHER = 7, FT_NPHASE = 8 };
 
 /* A driver context on `device`; the ft_* drivers are ordered on `stream`
  * (any stream, the legacy default one included): internally they run on a

@@ -83,7 +83,7 @@ class ft_opts_t(C.Structure):
                 ("fix_log", C.c_void_p), ("fix_log_cap", C.c_int32), ("pu_gemm", C.c_int32),
                 ("refresh", C.c_int32), ("restart", C.c_int32), ("pd_location", C.c_int32),
                 ("fig4b", C.c_int32), ("trailing_check_period", C.c_int32), ("checksum_gemm", C.c_int32),
-                ("scheme", C.c_int32), ("lookahead", C.c_int32)]
+                ("scheme", C.c_int32), ("timing", C.c_int32), ("lookahead", C.c_int32)]
 
 
 class ft_stats_t(C.Structure):
@@ -93,7 +93,12 @@ class ft_stats_t(C.Structure):
                 ("xfer_d2h_flagged", C.c_int32), ("xfer_d2h_fixed", C.c_int32), ("xfer_retransfers", C.c_int32),
                 ("xfer_h2d_flagged", C.c_int32), ("xfer_h2d_fixed", C.c_int32), ("xfer_resends", C.c_int32),
                 ("xfer_uncorrectable", C.c_int32), ("ms_host_pd", C.c_double),
-                ("ctf_flagged", C.c_int32), ("ctf_recomputed", C.c_int32)]
+                ("ctf_flagged", C.c_int32), ("ctf_recomputed", C.c_int32),
+                ("detected", C.c_int32), ("corrected_0d", C.c_int32), ("corrected_1d", C.c_int32),
+                ("checksum_repaired", C.c_int32), ("comm_errors", C.c_int32), ("ms_phase", C.c_double * 8)]
+
+
+PHASES = ("pd", "pu", "tmu", "rules", "checks", "restart", "encode", "other")  # ft_stats_t.ms_phase
 
 
 _L = _lib.load()
@@ -380,14 +385,15 @@ def host_lapack_path():
 
 
 def _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh=True, restart=True,
-          pd_location=PD_DEVICE, fig4b=True, period=0, scheme=0, checksum_gemm=False, lookahead=False):
+          pd_location=PD_DEVICE, fig4b=True, period=0, scheme=0, checksum_gemm=False, lookahead=False,
+          timing=False):
     inj = (ft_inject_t * max(1, len(inject)))()
     for k, f in enumerate(inject):
         inj[k] = ft_inject_t(*f)
     opts = ft_opts_t(nb, int(abft), tol_kind, tol_scale, int(fig4a_repair), len(inject), inj,
                      _ptr(fix_log), 0 if fix_log is None else fix_log.numel() // FIX_BYTES, int(pu_gemm),
                      int(refresh), int(restart), int(pd_location), int(fig4b), int(period), int(checksum_gemm),
-                     int(scheme), int(lookahead))
+                     int(scheme), int(timing), int(lookahead))
     return opts, inj
 
 
@@ -404,12 +410,12 @@ def abft_panel_getrf(mat: Mat, k: int, ipiv: torch.Tensor, Linv: torch.Tensor, U
 
 def ft_getrf(ctx: Context, A: torch.Tensor, nb: int, ipiv: torch.Tensor, abft=True, tol_kind=TOL_MAGNITUDE,
              tol_scale=1.0, fig4a_repair=True, inject=(), fix_log=None, pd_location=PD_DEVICE, restart=True,
-             fig4b=True, trailing_check_period=0):
+             fig4b=True, trailing_check_period=0, timing=False):
     """Fault-tolerant LU with partial pivoting in place on a column-major A;
     ipiv: int64 device tensor (n), receives 1-based global pivots."""
     n = A.shape[0]
     opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, True, restart=restart,
-                       pd_location=pd_location, fig4b=fig4b, period=trailing_check_period)
+                       pd_location=pd_location, fig4b=fig4b, period=trailing_check_period, timing=timing)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_getrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), _ptr(ipiv), C.byref(opts), C.byref(stats),
@@ -426,12 +432,13 @@ def abft_panel_geqrf(mat: Mat, k: int, tau: torch.Tensor, V: torch.Tensor, T: to
 
 
 def ft_geqrf(ctx: Context, A: torch.Tensor, nb: int, tau: torch.Tensor, abft=True, tol_kind=TOL_MAGNITUDE,
-             tol_scale=1.0, inject=(), fix_log=None, pd_location=PD_DEVICE, restart=True, trailing_check_period=0):
+             tol_scale=1.0, inject=(), fix_log=None, pd_location=PD_DEVICE, restart=True, trailing_check_period=0,
+             timing=False):
     """Fault-tolerant Householder QR in place on a column-major A (LAPACK
     dgeqrf storage); tau: device tensor (n) of A's dtype."""
     n = A.shape[0]
     opts, _inj = _opts(nb, abft, tol_kind, tol_scale, True, inject, fix_log, True, restart=restart,
-                       pd_location=pd_location, period=trailing_check_period)
+                       pd_location=pd_location, period=trailing_check_period, timing=timing)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_geqrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), _ptr(tau), C.byref(opts), C.byref(stats),
@@ -443,7 +450,7 @@ def ft_geqrf(ctx: Context, A: torch.Tensor, nb: int, tau: torch.Tensor, abft=Tru
 def ft_potrf(ctx: Context, A: torch.Tensor, nb: int, abft=True, tol_kind=TOL_MAGNITUDE, tol_scale=1.0,
              fig4a_repair=True, inject=(), fix_log=None, pu_gemm=True, refresh=True, restart=True,
              pd_location=PD_DEVICE, fig4b=True, trailing_check_period=0, scheme=0, checksum_gemm=False,
-             lookahead=True):
+             lookahead=True, timing=False):
     """Fault-tolerant lower Cholesky in place on a column-major A.  Returns
     (rc, info, stats) with rc 0 or E_UNCORRECTABLE (other codes raise).
     pd_location=PD_HOST needs ctx.set_host_lapack() first.  scheme: SCHEME_*
@@ -452,7 +459,7 @@ def ft_potrf(ctx: Context, A: torch.Tensor, nb: int, abft=True, tol_kind=TOL_MAG
     lookahead: the next panel's PD / PU next to the TMU (reading c-35)."""
     n = A.shape[0]
     opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, pu_gemm, refresh, restart,
-                       pd_location, fig4b, trailing_check_period, scheme, checksum_gemm, lookahead)
+                       pd_location, fig4b, trailing_check_period, scheme, checksum_gemm, lookahead, timing)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_potrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), C.byref(opts), C.byref(stats), C.byref(info))

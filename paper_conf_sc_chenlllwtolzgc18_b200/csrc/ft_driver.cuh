@@ -59,6 +59,7 @@ struct ft_ctx {
   cudaEvent_t ev_col = nullptr, ev_side = nullptr;
   void* putmp2 = nullptr;  // PU scratch of the side stream
   size_t putmp2_bytes = 0;
+  std::vector<cudaEvent_t> evpool;  // opts->timing: per-phase span events (reused across calls)
   // FT_PD_HOST (ft_host.cu): host LAPACK, pinned panel staging, device guard
   void* lapack = nullptr;  // dlopen handle
   void* lp[6] = {};        // dpotrf spotrf dgetrf sgetrf dgeqrf sgeqrf
@@ -178,6 +179,22 @@ struct Driver {
   }
   int ctf_flagged = 0, ctf_recomputed = 0;
   std::vector<std::pair<int, int>> xfer_used;  // (iter, point) transfer faults already applied
+
+  // opts->timing: spans (phase, start, end) recorded on the stream each phase runs on
+  struct Span {
+    int ph;
+    cudaEvent_t a, b;
+  };
+  std::vector<Span> spans;
+  size_t ev_used = 0;
+  cudaEvent_t ev_take() {
+    if (ev_used == c->evpool.size()) {
+      cudaEvent_t e = nullptr;
+      if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+      c->evpool.push_back(e);
+    }
+    return c->evpool[ev_used++];
+  }
 
   Driver() = default;
   Driver(const Driver&) = delete;
@@ -331,7 +348,8 @@ struct Driver {
     return 0;
   }
   int check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only = false,
-            cudaStream_t on = nullptr) {
+            cudaStream_t on = nullptr);
+  int check_impl(int I0, int I1, int J0, int J1, int view, int which, bool lower_only, cudaStream_t on) {
     abft_tiles_t t{I0, I1, J0, J1, lower_only ? 1 : 0, view};
     const abft_stream_t st = (abft_stream_t)(on ? on : s);
     if (o->checksum_gemm)  // prior-art GEMM recalculation (f3 baseline)
@@ -464,10 +482,59 @@ struct Driver {
                 host_phase[1], host_phase[2], host_phase[3]);
       stats->ctf_flagged = ctf_flagged;
       stats->ctf_recomputed = ctf_recomputed;
+      // outcomes by class from the fix log
+      stats->detected = h[ABFT_CNT_TILES_FLAGGED];
+      stats->corrected_0d = stats->corrected_1d = stats->checksum_repaired = 0;
+      const int nf = std::min(h[8], c->fixcap);
+      if (nf > 0) {
+        std::vector<abft_fix_t> fx(nf);
+        ABFT_CUDA_TRY(cudaMemcpy(fx.data(), c->fixlog, sizeof(abft_fix_t) * nf, cudaMemcpyDeviceToHost));
+        for (const abft_fix_t& f : fx) {
+          if (f.kind != ABFT_FIX_DATA)
+            ++stats->checksum_repaired;
+          else if (f.cls == ABFT_CLS_0D)
+            ++stats->corrected_0d;
+          else
+            ++stats->corrected_1d;
+        }
+      }
+      stats->comm_errors = xs[1] + xs[2] + xs[4] + xs[5];  // d2h fixed, retransfers, h2d fixed, resends
+      for (int i = 0; i < FT_NPHASE; ++i) stats->ms_phase[i] = 0.0;
+      for (const Span& sp : spans) {
+        float ms = 0.f;
+        if (cudaEventElapsedTime(&ms, sp.a, sp.b) == cudaSuccess) stats->ms_phase[sp.ph] += ms;
+      }
     }
     return h[ABFT_CNT_UNCORRECTABLE] ? ABFT_E_UNCORRECTABLE : 0;
   }
 };
+
+// opts->timing: one span of phase `ph` on the driver's current stream
+// (start recorded now, end when the scope closes).  Scopes do not nest.
+struct PhaseScope {
+  Driver& d;
+  cudaEvent_t b = nullptr;
+  cudaStream_t st = nullptr;
+  PhaseScope(Driver& dd, int ph) : d(dd) {
+    if (!dd.o->timing) return;
+    st = dd.s;
+    cudaEvent_t a = dd.ev_take();
+    b = dd.ev_take();
+    if (!a || !b || cudaEventRecord(a, st) != cudaSuccess) {
+      b = nullptr;
+      return;
+    }
+    dd.spans.push_back({ph, a, b});
+  }
+  ~PhaseScope() {
+    if (b) cudaEventRecord(b, st);
+  }
+};
+
+inline int Driver::check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only, cudaStream_t on) {
+  PhaseScope ps(*this, FT_PH_CHECKS);
+  return check_impl(I0, I1, J0, J1, view, which, lower_only, on);
+}
 
 // FT_PD_HOST (ft_host.cu): Alg. 2 lines 3-7 for the panel of iteration k,
 // rows x nb at (row0, col0) of A: guarded D2H, host check, host LAPACK

@@ -198,6 +198,7 @@ extern "C" int ft_ctx_destroy(ft_ctx_t* c) {
   if (c->hpin) cudaFreeHost(c->hpin);
   if (c->ev) cudaEventDestroy(c->ev);
   if (c->join) cudaEventDestroy(c->join);
+  for (cudaEvent_t e : c->evpool) cudaEventDestroy(e);
   if (c->ev_col) cudaEventDestroy(c->ev_col);
   if (c->ev_side) cudaEventDestroy(c->ev_side);
   if (c->putmp2) cudaFree(c->putmp2);
@@ -277,6 +278,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
   };
 
   if (ft) {
+    PhaseScope ps(d, FT_PH_ENCODE);
     abft_tiles_t all{0, (int)nt, 0, (int)nt, 1, ABFT_SYM_LOWER};
     FT_TRY(abft_encode(&d.M, &all, W, (abft_stream_t)d.s));
   }
@@ -318,11 +320,13 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     auto post_readback = [&]() -> int { return d.post_delta(0); };
     auto readback_delta = [&](int* delta) -> int { return d.wait_delta(0, delta); };
     if (rs) {
+      PhaseScope ps(d, FT_PH_RESTART);
       FT_TRY(copy2d(pd_a, nb, d.a_at(r0, r0), lda, nb, nb));
       FT_TRY(copy2d(pd_c, 2, d.colchk_at(2 * k, r0), d.M.ldc, 2, nb));
       FT_TRY(copy2d(pd_m, 1, d.colmag_at(k, r0), d.M.ldcm, 1, nb));
     }
     auto do_pd = [&]() -> int {
+      PhaseScope ps(d, FT_PH_PD);
       abft_mat_t D{};
       D.dtype = dtype;
       D.m = D.n = D.nb = nb;
@@ -378,6 +382,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     FT_TRY(d.inject_at(k, FT_AT_PRE_PU_CHECK));
     if (ft && pre_checks) FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, W));
     if (rs) {
+      PhaseScope ps(d, FT_PH_RESTART);
       FT_TRY(copy2d(pu_a, nk, d.a_at(r1, r0), lda, nk, nb));
       FT_TRY(copy2d(pu_c, m2, d.colchk_at(2 * (k + 1), r0), d.M.ldc, m2, nb));
       FT_TRY(copy2d(pu_m, m2 / 2, d.colmag_at(k + 1, r0), d.M.ldcm, m2 / 2, nb));
@@ -391,6 +396,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (ft && s_new && !fig4b_here) FT_TRY(d.mark_fig4b_end());  // the deferred check's window ends here
     // line 9: PU  L_ik = A_ik L_kk^-T  (+ c(L_ik) = c(A_ik) L_kk^-T, c-12)
     auto pu_data = [&]() -> int {
+      PhaseScope ps(d, FT_PH_PU);
       cublasHandle_t h = blas_handle(s, lk);
       if (o->pu_gemm) {
         // L21 = A21 L_kk^-T as a DGEMM with the explicit inverse (tensor cores).
@@ -432,6 +438,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       return 0;
     };
     auto pu_chk = [&]() -> int {  // c(L_ik) = c(A_ik) L_kk^-T, m_c <- m_c |L_kk^-T| with the PD's inverse (c-12, c-6)
+      PhaseScope ps(d, FT_PH_RULES);
       return abft_update_trsm_inv(dtype, 'R', 'T', nb, c->linv, nb, d.colchk_at(2 * (k + 1), r0), d.M.ldc, m2,
                                   d.colmag_at(k + 1, r0), d.M.ldcm, m2 / 2, as);
     };
@@ -451,12 +458,15 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       // the device (Driver::gated_restart): restore-and-redo as one gated
       // GEMM per array, reading the copy and the PD's inverse, then re-check.
       auto pu_redo = [&](const int32_t* g) -> int {
-        FT_TRY(gemm_gated(dtype, false, true, false, false, nk, nb, nb, pu_a, nk, c->linv, nb, d.a_at(r1, r0), lda, g,
-                          s));
-        FT_TRY(gemm_gated(dtype, false, true, false, false, m2, nb, nb, pu_c, m2, c->linv, nb,
-                          d.colchk_at(2 * (k + 1), r0), d.M.ldc, g, s));
-        FT_TRY(gemm_gated(dtype, false, true, false, true, m2 / 2, nb, nb, pu_m, m2 / 2, c->linv, nb,
-                          d.colmag_at(k + 1, r0), d.M.ldcm, g, s));
+        {
+          PhaseScope ps(d, FT_PH_RESTART);
+          FT_TRY(gemm_gated(dtype, false, true, false, false, nk, nb, nb, pu_a, nk, c->linv, nb, d.a_at(r1, r0), lda,
+                            g, s));
+          FT_TRY(gemm_gated(dtype, false, true, false, false, m2, nb, nb, pu_c, m2, c->linv, nb,
+                            d.colchk_at(2 * (k + 1), r0), d.M.ldc, g, s));
+          FT_TRY(gemm_gated(dtype, false, true, false, true, m2 / 2, nb, nb, pu_m, m2 / 2, c->linv, nb,
+                            d.colmag_at(k + 1, r0), d.M.ldcm, g, s));
+        }
         return d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL);
       };
       if (rs) FT_TRY(d.gated_restart(1, pu_redo));
@@ -469,6 +479,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
   auto tmu_data = [&](int k, int64_t c0, int64_t c1) -> int {
     const int64_t r0 = (int64_t)k * nb, w = c1 - c0, below = n - c1;
     if (w <= 0) return 0;
+    PhaseScope ps(d, FT_PH_TMU);
     cublasHandle_t h = blas_handle(d.s, lk);
     cublasStatus_t st = CUBLAS_STATUS_SUCCESS;
     if (dtype == ABFT_F64) {
@@ -495,6 +506,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     const abft_stream_t as = (abft_stream_t)d.s;
     const int J0 = (int)(c0 / nb), J1 = (int)(c1 / nb);
     if (J1 <= J0) return 0;
+    PhaseScope ps(d, FT_PH_RULES);
     if (c1 == n) {  // tile columns J0.. (to the end): the one-product rule of the sub-problem
       const int64_t ntk = nt - J0;
       return abft_update_syrk(dtype, nb, ntk, d.a_at(c0, r0), lda, d.colchk_at(2 * J0, r0), d.M.ldc,
@@ -542,6 +554,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     ra.counts = d.counts;
     ra.c0 = c0;
     ra.c1 = c1;
+    PhaseScope ps(d, FT_PH_OTHER);
     if (dtype == ABFT_F64)
       fig4a_repair_kernel<double><<<1, 256, 0, d.s>>>(ra);
     else

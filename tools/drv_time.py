@@ -68,3 +68,9 @@ cus = med(tl)
 print(f"{which} n={n} nb={nb}: plain {plain:.2f} ms, ft {ft:.2f} ms ({100 * (ft - plain) / plain:.2f}%), "
       f"ft no-restart {nors:.2f} ms ({100 * (nors - plain) / plain:.2f}%), cusolver {cus:.2f} ms "
       f"(ft vs cusolver {100 * (ft - cus) / cus:.2f}%)", flush=True)
+if which == "potrf":
+    A.copy_(A0)
+    rc, info, st = abft.ft_potrf(ctx, A, nb, timing=True)
+    torch.cuda.synchronize()
+    print("phase ms (timing run; side-stream phases overlap the main stream):",
+          {k: round(v, 2) for k, v in zip(abft.PHASES, st.ms_phase)})
