@@ -519,6 +519,7 @@ def mgpu_overhead(si, n, nb, reps, world, rank):
 
     P, Q = D.grid_shape(world)
     lay = mgpu.Layout(n, nb, P, Q, rank)
+    groups = D.Groups(P, Q)  # the broadcast communicators, created once (collective)
     A0 = si.spd_block_cyclic_device(n, nb, P, Q, rank, seed=61440)
     A = torch.empty_like(A0.t()).t()
 
@@ -529,7 +530,7 @@ def mgpu_overhead(si, n, nb, reps, world, rank):
             dist.barrier()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record()
-        rc, st = mgpu.ft_potrf_mgpu(A, lay, abft_on=ft)
+        rc, st = mgpu.ft_potrf_mgpu(A, lay, abft_on=ft, groups=groups)
         b.record()
         torch.cuda.synchronize()
         ms = a.elapsed_time(b)
@@ -551,7 +552,8 @@ def mgpu_overhead(si, n, nb, reps, world, rank):
     return {"n": n, "nb": nb, "grid": [P, Q], "ms_ft": ft_ms, "ms_plain": plain_ms,
             "overhead_pct": 100.0 * (ft_ms - plain_ms) / plain_ms,
             "tflops_ft": n ** 3 / 3 / (ft_ms / 1e3) / 1e12, "reps": reps, "timing": "min over reps, max over ranks",
-            "comm": "NCCL broadcast of L_kk and of each process row's panel piece; int32 report all-reduce"}
+            "comm": "NCCL broadcast of L_kk inside its process column and of each panel piece to the ranks "
+                    "that need it (dist.Groups); int32 decision all-reduce per round and report all-reduce"}
 
 
 def lu_qr_overhead(abft, si, n, nb, reps, host_pd=True):

@@ -9,32 +9,36 @@ global tile's).  Iteration k of Alg. 2 (L368-L378):
 
   1. owner of A_kk: pre-PD check (SYM_LOWER, c and r), PD + c(L_kk) rule
      (`abft_panel_potrf`), post-PD check (LOWER, c);
-  2. broadcast L_kk | c(L_kk) | m_c(L_kk); receivers in process column k
-     verify the received tile (communication errors, L355) and invert it;
+  2. diagonal round: L_kk | c(L_kk) | m_c(L_kk) is broadcast inside process
+     column k mod Q (the panel owners, `dist.Groups.col`); every receiver
+     verifies and corrects its copy (communication errors, L355), then the
+     owner's post-PD verdict and the receivers' flags are all-reduced in the
+     group and decided by L361-L363 (`dist.classify_bcast`): all receivers
+     flagged, or the owner's check left a 2D error -> the owner restores its
+     pre-PD copy, redoes the PD (L430) and broadcasts again; some -> the
+     receivers' local corrections stand (communication error);
   3. panel owners: pre-PU check (c and r), PU L_ik = A_ik L_kk^-T and
      c(L_ik) = c(A_ik) L_kk^-T (`abft_update_trsm_inv`), post-PU check (c);
-  4. every panel piece (the tiles of one process row) is broadcast to all
-     ranks, and every receiver verifies it against its column checksums and
-     corrects it in place (L361-L363: all receivers flagged -> the sender's
-     PD/PU was wrong; some -> communication error);
+  4. piece rounds: each process row's panel piece goes (async, all pieces at
+     once) to the ranks that need it (`dist.Groups.piece`: its process row
+     and the process columns holding its tile columns), is checked by every
+     receiver and decided as in 2 (restart -> the sender redoes its PU and
+     broadcasts the piece again);
   5. every rank updates its local trailing tiles A_IJ -= L_ik L_jk^T with
      c(A_IJ) -= c(L_ik) L_jk^T and r(A_IJ) -= L_ik c(L_jk)^T (+ magnitudes,
      c-6, c-12), grouped tile columns per call (`abft_update_gemm`);
   6. the received panel is re-checked after the trailing update (Fig. 4a);
      a value corrected there was already consumed by the update, which the
-     distributed driver reports as uncorrectable (no distributed repair);
-     the panel owners re-check their stored pieces too (the factor itself,
-     which no update read: a fault there is a plain fix).
+     distributed driver reports as uncorrectable (no distributed repair,
+     DESIGN §7 e-2); the panel owners re-check their stored pieces too.
 
-Local restart (f1, L430): the owner of A_kk and the panel owners copy the
-input of their PD / PU with its checksums after the pre-op check; a 2D error
-left by their post-op check (read back on the host: one wait per op) restores
-the copy and redoes the op once, before anything is broadcast.
-
-Only panels, checksums and int32 error reports cross the interconnect;
-torch.distributed is plumbing (NCCL on the GPU box; gloo with CUDA tensors
-when several ranks share one GPU in the tests).  Every arithmetic step is a
-C-ABI call into libabft_b200.so; the buffer packing below only moves bytes.
+Host synchronisation: one read of the all-reduced decision words per round
+(2 per iteration; the decision is control flow), none for data movement (the
+column-role index tensors are built once before the loop).  Only panels,
+checksums and int32 error reports cross the interconnect; torch.distributed
+is plumbing (NCCL on the GPU box; gloo with CUDA tensors when several ranks
+share one GPU in the tests).  Every arithmetic step is a C-ABI call into
+libabft_b200.so; the buffer packing below only moves bytes.
 """
 from __future__ import annotations
 
@@ -45,73 +49,11 @@ import torch
 import torch.distributed as dist
 
 from . import abft
-from .dist import grid_shape
+from .dist import Groups, Layout, classify_bcast, grid_shape  # noqa: F401  (re-exported)
+from .dist import decide as decide_round
 
-AT_BCAST = 8  # fault hook: a receiver's copy of the broadcast panel (communication error)
-
-
-@dataclass
-class Layout:
-    """2D block-cyclic placement of nt x nt tiles on a P x Q grid."""
-
-    n: int
-    nb: int
-    P: int
-    Q: int
-    rank: int
-
-    @property
-    def nt(self):
-        return self.n // self.nb
-
-    @property
-    def p(self):
-        return self.rank // self.Q
-
-    @property
-    def q(self):
-        return self.rank % self.Q
-
-    @property
-    def mt_loc(self):
-        return len(range(self.p, self.nt, self.P))
-
-    @property
-    def nt_loc(self):
-        return len(range(self.q, self.nt, self.Q))
-
-    def owner(self, I, J):
-        return (I % self.P) * self.Q + (J % self.Q)
-
-    @staticmethod
-    def first_at_least(x, r, S):
-        """Smallest local index i with i * S + r >= x."""
-        return max(0, -(-(x - r) // S))
-
-    def row_first(self, x, p=None):
-        return self.first_at_least(x, self.p if p is None else p, self.P)
-
-    def col_first(self, x, q=None):
-        return self.first_at_least(x, self.q if q is None else q, self.Q)
-
-    def piece_count(self, k, p):
-        """Panel tiles I > k owned by process row p (piece p of iteration k)."""
-        return max(0, len(range(p, self.nt, self.P)) - self.row_first(k + 1, p))
-
-    def to_local(self, gi, gj):
-        """Global element -> local element of its owner."""
-        I, J = gi // self.nb, gj // self.nb
-        return (I // self.P) * self.nb + gi % self.nb, (J // self.Q) * self.nb + gj % self.nb
-
-    def lcol_sources(self, k):
-        """For this rank's local trailing tile columns J > k (in order): the
-        (piece, index in piece) of L_Jk."""
-        out = []
-        for jl in range(self.col_first(k + 1), self.nt_loc):
-            J = jl * self.Q + self.q
-            pp = J % self.P
-            out.append((pp, J // self.P - self.row_first(k + 1, pp)))
-        return out
+AT_BCAST = 8   # fault hook: a receiver's copy of a broadcast panel (communication error)
+AT_SEND = 11   # fault hook: the sender's packed buffer right before its first broadcast
 
 
 def scatter_tiles(A: torch.Tensor, lay: Layout, device="cuda") -> torch.Tensor:
@@ -142,14 +84,6 @@ def gather_tiles(A_loc: torch.Tensor, lay: Layout, group=None) -> torch.Tensor:
             for jl, J in enumerate(range(L.q, L.nt, L.Q)):
                 out[I * nb:(I + 1) * nb, J * nb:(J + 1) * nb] = blk[il * nb:(il + 1) * nb, jl * nb:(jl + 1) * nb]
     return out
-
-
-def classify_bcast(nflag: int, nrecv: int) -> str:
-    """L361-L363: of the nrecv receivers of one broadcast, nflag found (and
-    corrected) corruption in their copy."""
-    if nflag == 0:
-        return "clean"
-    return "restart" if nflag >= nrecv else "communication"
 
 
 class _Piece:
@@ -193,64 +127,87 @@ class MgpuStats:
 
 
 def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0, inject=(), group=None,
-                  tmu_groups=32, restart=True):
+                  tmu_groups=32, restart=True, groups: Groups = None):
     """Fault-tolerant lower Cholesky of the distributed matrix in place.
     A_loc: this rank's local column-major matrix (from scatter_tiles).
-    inject: (iter, point, gi, gj, xor_mask, rank) with global (gi, gj);
-    point in abft.AT_* (applied by the tile's owner) or AT_BCAST (applied to
-    `rank`'s received copy of panel element (gi, gj) of iteration iter).
+    inject: (iter, point, gi, gj, xor_mask[, rank]) with global (gi, gj);
+    point in abft.AT_* (applied by the tile's owner), AT_BCAST (applied to
+    `rank`'s received copy of panel element (gi, gj) of iteration iter) or
+    AT_SEND (applied by the sender to its packed buffer before the first
+    broadcast: every receiver sees it).  groups: the broadcast communicators
+    (dist.Groups; built here when None — a collective call on every rank).
     Returns (rc, MgpuStats); rc is 0 or abft.E_UNCORRECTABLE."""
     nb, nt, P, Q = lay.nb, lay.nt, lay.P, lay.Q
     p, q = lay.p, lay.q
     dev, dt = A_loc.device, A_loc.dtype
     world = P * Q
     me = lay.rank
+    G = groups if groups is not None else Groups(P, Q, group)
+    UNC = abft.NCOUNTS - 1
     tol = abft.abft_tol_t(abft.TOL_MAGNITUDE, tol_scale, 1)
     mat = abft.Mat.alloc(A_loc, nb) if abft_on else abft.Mat(A_loc, nb)
     rep = abft.Report.alloc(mat) if abft_on else None
     rep_b = abft.Report(abft.colmajor_zeros(max(nt, 1), 1, dtype=torch.int32, device=dev),
                         torch.zeros(abft.NCOUNTS, dtype=torch.int32, device=dev))
     cb_total = torch.zeros(abft.NCOUNTS, dtype=torch.int32, device=dev)
-    bflag = torch.zeros(nt, P + 1, dtype=torch.int32, device=dev)  # [k][piece | diag]
+    bflag = torch.zeros(nt, P + 1, dtype=torch.int32, device=dev)     # [k][piece | diag]: receivers that flagged
+    brestart = torch.zeros(nt, P + 1, dtype=torch.int32, device=dev)  # [k][piece | diag]: restart + re-broadcast
     consumed = torch.zeros(1, dtype=torch.int32, device=dev)
     fixes = torch.zeros(4096 * abft.FIX_BYTES, dtype=torch.uint8, device=dev)
     nfix = torch.zeros(1, dtype=torch.int32, device=dev)
     infos = torch.zeros(max(nt, 1), dtype=torch.int32, device=dev)
     Linv = abft.colmajor_zeros(nb, nb, dtype=dt, device=dev)
     diag_buf = _Piece(1, nb, dt, dev)
+    zero1 = torch.zeros(1, dtype=torch.int32, device=dev)
+    sent = set()  # AT_SEND faults already applied (first send only)
 
-    def bcast(t, src):
-        if world > 1:
-            dist.broadcast(t, src=src, group=group)
+    # the column-role sources of every iteration, as device index tensors,
+    # built once (no host-to-device copies inside the loop)
+    lcol_idx = []
+    for k in range(nt):
+        srcs = lay.lcol_sources(k)
+        per = []
+        for pp in range(P):
+            sel = [t for t, (s_, _) in enumerate(srcs) if s_ == pp]
+            if sel:
+                per.append((pp, torch.tensor(sel, device=dev), torch.tensor([srcs[t][1] for t in sel], device=dev)))
+        lcol_idx.append((len(srcs), per))
 
     def check(m, tl, which):
         abft.abft_verify(m, tl, which, tol, rep)
         abft.abft_locate_correct(m, tl, which, tol, rep, fixes, nfix)
 
-    def check_recv(m, tl, slot_k, slot):
-        """Post-broadcast check of a received copy (L355); flags per source."""
+    def check_recv(m, tl, acc):
+        """Post-broadcast check of a received copy (L355) into the round's
+        counters `acc` (added to the run's totals once the round is decided)."""
         abft.abft_verify(m, tl, abft.COL, tol, rep_b)
         abft.abft_locate_correct(m, tl, abft.COL, tol, rep_b, fixes, nfix)
-        bflag[slot_k, slot] += (rep_b.counts[0] > 0).to(torch.int32)
-        cb_total.add_(rep_b.counts)
+        acc.add_(rep_b.counts)
         rep_b.counts.zero_()
 
     def hook(k, point):
         for f in inject:
             it, pt, gi, gj, mask = f[:5]
-            if it != k or pt != point or pt == AT_BCAST:
+            if it != k or pt != point or pt in (AT_BCAST, AT_SEND):
                 continue
             if lay.owner(gi // nb, gj // nb) == me:
                 li, lj = lay.to_local(gi, gj)
                 abft.abft_inject(A_loc, li, lj, mask)
 
-    def hook_bcast(k, buf: _Piece, tiles_I):
-        """Communication fault: flip this rank's received copy."""
-        for f in inject:
+    def hook_buf(k, point, buf: _Piece, tiles_I):
+        """A flip in a broadcast buffer: AT_BCAST in `rank`'s received copy,
+        AT_SEND in the sender's packed buffer (first send only)."""
+        for idx, f in enumerate(inject):
             it, pt, gi, gj, mask = f[:5]
             rk = f[5] if len(f) > 5 else -1
-            if it != k or pt != AT_BCAST or rk != me or gj // nb != k or gi // nb not in tiles_I:
+            if it != k or pt != point or gj // nb != k or gi // nb not in tiles_I:
                 continue
+            if point == AT_BCAST and rk != me:
+                continue
+            if point == AT_SEND:
+                if idx in sent:
+                    continue
+                sent.add(idx)
             t = tiles_I.index(gi // nb)
             abft.abft_inject(buf.L, t * nb + gi % nb, gj % nb, mask)
 
@@ -258,16 +215,12 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
     rs = abft_on and restart
 
     def snapshot(*ts):
-        return [t.clone() for t in ts] + [rep.counts[abft.NCOUNTS - 1].clone()]
-
-    def added_2d(snap):
-        """2D errors the post-op check added (host read-back, f1)."""
-        return int((rep.counts[abft.NCOUNTS - 1] - snap[-1]).item())
+        return [t.clone() for t in ts] + [rep.counts[UNC].clone()]
 
     def restore(snap, *ts):
         for t, c in zip(ts, snap[:-1]):
             t.copy_(c)
-        rep.counts[abft.NCOUNTS - 1] = snap[-1]
+        rep.counts[UNC] = snap[-1]
         restarts[0] += 1
 
     def sub(m: abft.Mat, il, jl):
@@ -278,6 +231,15 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
                         m.rowchk[r0:r0 + nb, 2 * jl:2 * jl + 2] if m.rowchk is not None else None,
                         m.colmag[il:il + 1, c0:c0 + nb] if m.colmag is not None else None,
                         m.rowmag[r0:r0 + nb, jl:jl + 1] if m.rowmag is not None else None)
+
+    def pack(buf: _Piece, A_view, c_view, m_view):
+        buf.L.copy_(A_view)
+        if abft_on:
+            buf.c.copy_(c_view)
+            buf.m.copy_(m_view)
+
+    def decide(pairs):
+        return decide_round(pairs, world)
 
     # ---- encode: the lower tiles of every local tile column (diag in SYM view)
     if abft_on:
@@ -294,6 +256,7 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
         kp, kq = k % P, k % Q
         owner_kk = kp * Q + kq
         ik, jk = k // P, k // Q
+        in_col = q == kq
         # ---- 1. PD on the owner of A_kk
         if me == owner_kk:
             D = sub(mat, ik, jk)
@@ -302,32 +265,61 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
                 check(D, abft.tiles(0, 1, 0, 1, False, abft.SYM_LOWER), abft.BOTH)
             if rs:
                 pd_snap = snapshot(D.A, D.colchk, D.colmag)
+
+            def pd():
+                abft.abft_panel_potrf(D, infos[k:k + 1], Linv)
+                if abft_on:
+                    check(D, abft.tiles(0, 1, 0, 1, False, abft.LOWER), abft.COL)
+
             hook(k, abft.AT_PRE_PD)
+            if abft_on:
+                unc0 = rep.counts[UNC].clone()
             abft.abft_panel_potrf(D, infos[k:k + 1], Linv)
             hook(k, abft.AT_POST_PD)
             if abft_on:
                 check(D, abft.tiles(0, 1, 0, 1, False, abft.LOWER), abft.COL)
-            if rs and added_2d(pd_snap) > 0:  # local restart of the PD (L430)
-                restore(pd_snap, D.A, D.colchk, D.colmag)
-                abft.abft_panel_potrf(D, infos[k:k + 1], Linv)
-                check(D, abft.tiles(0, 1, 0, 1, False, abft.LOWER), abft.COL)
-            diag_buf.L.copy_(D.A)
-            if abft_on:
-                diag_buf.c.copy_(D.colchk)
-                diag_buf.m.copy_(D.colmag)
-        # ---- 2. broadcast L_kk to the panel's process column (sent to all)
-        bcast(diag_buf.flat, owner_kk)
-        if q == kq and me != owner_kk:
-            hook_bcast(k, diag_buf, [k])
-            if abft_on:
-                check_recv(diag_buf.mat(), abft.tiles(0, 1, 0, 1, False, abft.LOWER), k, P)
-            abft.abft_tri_inverse("L", "N", diag_buf.L, Linv)
+            pack(diag_buf, D.A, D.colchk, D.colmag)
+            hook_buf(k, AT_SEND, diag_buf, [k])
+        # ---- 2. diagonal round inside process column k mod Q
+        if in_col:
+            for attempt in range(2):
+                if P > 1:
+                    dist.broadcast(diag_buf.flat, src=owner_kk, group=G.col[kq])
+                acc = torch.zeros(abft.NCOUNTS, dtype=torch.int32, device=dev)
+                if me != owner_kk:
+                    if attempt == 0:
+                        hook_buf(k, AT_BCAST, diag_buf, [k])
+                    if abft_on:
+                        check_recv(diag_buf.mat(), abft.tiles(0, 1, 0, 1, False, abft.LOWER), acc)
+                if not abft_on:
+                    break
+                word = torch.zeros(2, dtype=torch.int32, device=dev)
+                if me == owner_kk:
+                    word[0:1] = rep.counts[UNC:UNC + 1] - unc0
+                else:
+                    word[1:2] = (acc[0:1] > 0).to(torch.int32)
+                if attempt == 0 and me != owner_kk:
+                    bflag[k, P] += word[1]
+                s2d, nflag = decide([(G.col[kq], word)])[0]
+                if attempt == 1 or classify_bcast(nflag, P - 1, s2d) != "restart" or not rs:
+                    cb_total.add_(acc)
+                    break
+                # L363 / L430: restart of the PD on the owner, broadcast again
+                if me == owner_kk:
+                    restore(pd_snap, D.A, D.colchk, D.colmag)
+                    brestart[k, P] += 1
+                    unc0 = rep.counts[UNC].clone()
+                    pd()
+                    pack(diag_buf, D.A, D.colchk, D.colmag)
+            if me != owner_kk:
+                abft.abft_tri_inverse("L", "N", diag_buf.L, Linv)
         if k == nt - 1:
             break
         # ---- 3. PU on the panel owners
         ir0 = lay.row_first(k + 1)
         cnt = lay.mt_loc - ir0
-        if q == kq and cnt > 0:
+        pan = None
+        if in_col and cnt > 0:
             r0 = ir0 * nb
             hook(k, abft.AT_PRE_PU_CHECK)
             if abft_on:
@@ -343,47 +335,76 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
                     abft.abft_update_trsm_inv("R", "T", Linv, pan[1], 2 * cnt, pan[2], cnt)
 
             hook(k, abft.AT_PRE_PU)
+            if abft_on:
+                unc_pu = rep.counts[UNC].clone()
             pu()
             hook(k, abft.AT_POST_PU)
             if abft_on:
                 check(mat, abft.tiles(ir0, lay.mt_loc, jk, jk + 1), abft.COL)
-            if rs and added_2d(pu_snap) > 0:  # local restart of the PU (L430, L434)
-                restore(pu_snap, *pan)
-                pu()
-                check(mat, abft.tiles(ir0, lay.mt_loc, jk, jk + 1), abft.COL)
-        # ---- 4. broadcast the panel pieces (one per process row)
-        pieces = []
+        # ---- 4. piece rounds: each piece to the ranks that need it
+        pieces, tiles_of = [None] * P, [None] * P
         for pp in range(P):
             c_pp = lay.piece_count(k, pp)
-            buf = _Piece(c_pp, nb, dt, dev) if c_pp else None
-            pieces.append(buf)
-            if not c_pp:
-                continue
-            src = pp * Q + kq
-            if me == src:
-                buf.L.copy_(A_loc[ir0 * nb:, jk * nb:(jk + 1) * nb])
-                if abft_on:
-                    buf.c.copy_(mat.colchk[2 * ir0:, jk * nb:(jk + 1) * nb])
-                    buf.m.copy_(mat.colmag[ir0:, jk * nb:(jk + 1) * nb])
-            bcast(buf.flat, src)
-            if me != src:
+            if c_pp and me in G.piece_ranks[pp]:
+                pieces[pp] = _Piece(c_pp, nb, dt, dev)
                 first = lay.row_first(k + 1, pp)
-                tiles_I = [(first + t) * P + pp for t in range(c_pp)]
-                hook_bcast(k, buf, tiles_I)
-                if abft_on:
-                    check_recv(buf.mat(), abft.tiles(0, c_pp, 0, 1), k, pp)
+                tiles_of[pp] = [(first + t) * P + pp for t in range(c_pp)]
+        sender = [pp * Q + kq for pp in range(P)]
+        if pan is not None:
+            pack(pieces[p], pan[0], pan[1] if abft_on else None, pan[2] if abft_on else None)
+            hook_buf(k, AT_SEND, pieces[p], tiles_of[p])
+
+        def piece_round(pps, first):
+            if world > 1:
+                works = [dist.broadcast(pieces[pp].flat, src=sender[pp], group=G.piece[pp], async_op=True)
+                         for pp in pps]
+                for w in works:
+                    w.wait()
+            accs = {}
+            for pp in pps:
+                accs[pp] = torch.zeros(abft.NCOUNTS, dtype=torch.int32, device=dev)
+                if me != sender[pp]:
+                    if first:
+                        hook_buf(k, AT_BCAST, pieces[pp], tiles_of[pp])
+                    if abft_on:
+                        check_recv(pieces[pp].mat(), abft.tiles(0, pieces[pp].cnt, 0, 1), accs[pp])
+            return accs
+
+        live = [pp for pp in range(P) if pieces[pp] is not None]
+        accs = piece_round(live, True)
+        if abft_on and live:
+            words = []
+            for pp in live:
+                w = torch.zeros(2, dtype=torch.int32, device=dev)
+                if me == sender[pp]:
+                    w[0:1] = rep.counts[UNC:UNC + 1] - unc_pu
+                else:
+                    w[1:2] = (accs[pp][0:1] > 0).to(torch.int32)
+                    bflag[k, pp] += w[1]
+                words.append((G.piece[pp], w))
+            res = decide(words)
+            redo = [pp for pp, (s2d, nflag) in zip(live, res)
+                    if rs and classify_bcast(nflag, len(G.piece_ranks[pp]) - 1, s2d) == "restart"]
+            for pp in live:
+                if pp not in redo:
+                    cb_total.add_(accs[pp])
+            if redo:
+                # L363 / L430: the sender restores its pre-PU copy, redoes the
+                # PU (and its check) and the piece is broadcast again
+                if p in redo and pan is not None:
+                    restore(pu_snap, *pan)
+                    brestart[k, p] += 1
+                    pu()
+                    check(mat, abft.tiles(ir0, lay.mt_loc, jk, jk + 1), abft.COL)
+                    pack(pieces[p], pan[0], pan[1], pan[2])
+                for pp, acc in piece_round(redo, False).items():
+                    cb_total.add_(acc)
         # ---- 5. trailing update of the local tiles I >= J > k
-        srcs = lay.lcol_sources(k)
-        ncol = len(srcs)
+        ncol, per = lcol_idx[k]
         Lrow = pieces[p]
         if ncol and Lrow is not None:
             Lcol = _Piece(ncol, nb, dt, dev)
-            for pp in range(P):
-                sel = [t for t, (s, _) in enumerate(srcs) if s == pp]
-                if not sel:
-                    continue
-                dst_idx = torch.tensor(sel, device=dev)
-                src_idx = torch.tensor([srcs[t][1] for t in sel], device=dev)
+            for pp, dst_idx, src_idx in per:
                 Lcol.Lu.index_copy_(1, dst_idx, pieces[pp].Lu.index_select(1, src_idx))
                 Lcol.cu.index_copy_(1, dst_idx, pieces[pp].cu.index_select(1, src_idx))
                 Lcol.mu.index_copy_(1, dst_idx, pieces[pp].mu.index_select(1, src_idx))
@@ -421,20 +442,20 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
                 consumed.add_(nfix - before)
                 cb_total.add_(rep_b.counts)
                 rep_b.counts.zero_()
-        elif ncol == 0 or Lrow is None:
+        else:
             hook(k, abft.AT_PRE_TMU)
             hook(k, abft.AT_POST_TMU)
         # ---- 6b. the panel owners' stored pieces (the factor itself): Alg. 2
         # line 13 re-checks the panel after the TMU; here the update read the
         # broadcast copies (checked above), so a fault in the stored piece
         # since its post-PU check was consumed by nobody and is a plain fix
-        if abft_on and q == kq and cnt > 0:
+        if abft_on and in_col and cnt > 0:
             check(mat, abft.tiles(ir0, lay.mt_loc, jk, jk + 1), abft.COL)
 
     # ---- error reports: one all-reduce of the int32 counters (L361-L363)
     rep_counts = rep.counts if rep is not None else torch.zeros(abft.NCOUNTS, dtype=torch.int32, device=dev)
     nrs = torch.tensor([restarts[0]], dtype=torch.int32, device=dev)
-    summary = torch.cat([rep_counts, cb_total, consumed, infos, bflag.reshape(-1), nrs])
+    summary = torch.cat([rep_counts, cb_total, consumed, infos, bflag.reshape(-1), brestart.reshape(-1), nrs])
     if world > 1:
         dist.all_reduce(summary, op=dist.ReduceOp.SUM, group=group)
     h = summary.cpu().tolist()
@@ -443,16 +464,18 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
     st.bcast_counts = h[8:16]
     st.tmu_consumed = h[16]
     inf = h[17:17 + nt]
-    bf = h[17 + nt:-1]
+    nb_slots = nt * (P + 1)
+    bf = h[17 + nt:17 + nt + nb_slots]
+    br = h[17 + nt + nb_slots:17 + nt + 2 * nb_slots]
     st.restarts = h[-1]
     for kk in range(nt):
         if inf[kk] and not st.info:
             st.info = kk * nb + inf[kk]
         for slot in range(P + 1):
-            nflag = bf[kk * (P + 1) + slot]
-            if nflag:
-                nrecv = (P - 1) if slot == P else world - 1  # diag: the rest of process column k
-                st.bcast_events.append((kk, slot, nflag, nrecv, classify_bcast(nflag, nrecv)))
+            nflag, nre = bf[kk * (P + 1) + slot], br[kk * (P + 1) + slot]
+            if nflag or nre:
+                nrecv = (P - 1) if slot == P else len(G.piece_ranks[slot]) - 1  # diag: the rest of process column k
+                st.bcast_events.append((kk, slot, nflag, nrecv, classify_bcast(nflag, nrecv, nre)))
     st.uncorrectable = st.counts[abft.NCOUNTS - 1] + st.bcast_counts[abft.NCOUNTS - 1] + st.tmu_consumed
     rc = abft.E_UNCORRECTABLE if st.uncorrectable else 0
     return rc, st

@@ -14,6 +14,7 @@ import torch.multiprocessing as mp
 import synth_inputs as si
 from oracle import updates as ou
 from paper_conf_sc_chenlllwtolzgc18_b200 import abft, mgpu
+from paper_conf_sc_chenlllwtolzgc18_b200 import dist as D
 
 from . import mgpu_worker
 
@@ -90,9 +91,11 @@ def test_communication_fault_one_receiver(tmp_path, grid):
     world = grid[0] * grid[1]
     # iteration 1 panel element (row tile 5, column tile 1); pick a receiver that is not the sender
     k, gi, gj = 1, 5 * nb + 7, 1 * nb + 3
-    lay = mgpu.Layout(n, nb, grid[0], grid[1], 0)
-    sender = ((gi // nb) % grid[0]) * grid[1] + (k % grid[1])
-    recv = (sender + 1) % world
+    pp = (gi // nb) % grid[0]
+    sender = pp * grid[1] + (k % grid[1])
+    members = D.piece_ranks(grid[0], grid[1], pp)  # the ranks that receive this piece
+    recv = [r for r in members if r != sender][0]
+    assert world >= len(members)
     r = _run(tmp_path, n, nb, grid, inject=[(k, mgpu.AT_BCAST, gi, gj, BIT, recv)])
     assert r["rc"] == 0, r
     assert r["bcast_counts"][5] >= 1  # an element fixed in a received copy
@@ -112,4 +115,26 @@ def test_pd_consumed_fault_local_restart(tmp_path, grid):
     assert r0["rc"] == abft.E_UNCORRECTABLE
     r = _run(tmp_path, n, nb, grid, inject=inj)
     assert r["rc"] == 0 and r["restarts"] == 1, r
+    assert np.abs(r["L"].numpy() - _ref(n)).max() <= 1e-12 * np.abs(_ref(n)).max()
+
+
+@pytest.mark.parametrize("grid,what", [((1, 3), "piece"), ((2, 2), "diag"), ((2, 2), "piece")])
+def test_all_receivers_flag_restart_and_rebroadcast(tmp_path, grid, what):
+    """L361-L363 / L430: a flip in the SENDER's packed buffer reaches every
+    receiver; all of them flag their copy, so the round decides 'restart':
+    the sender redoes its PD / PU from its copy and broadcasts again; the
+    receivers' first corrections are discarded and the factor is exact."""
+    n, nb = 512, 64
+    k = 1
+    if what == "diag":
+        gi, gj = k * nb + 20, k * nb + 5
+    else:
+        gi, gj = 6 * nb + 11, k * nb + 3
+    r = _run(tmp_path, n, nb, grid, inject=[(k, mgpu.AT_SEND, gi, gj, BIT)])
+    assert r["rc"] == 0, r
+    assert r["restarts"] == 1, r
+    kinds = [e[4] for e in r["bcast_events"]]
+    assert kinds == ["restart"], r["bcast_events"]
+    ev = r["bcast_events"][0]
+    assert ev[2] == ev[3]  # every receiver flagged
     assert np.abs(r["L"].numpy() - _ref(n)).max() <= 1e-12 * np.abs(_ref(n)).max()

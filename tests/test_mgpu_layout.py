@@ -17,10 +17,10 @@ def test_layout_partitions_tiles(P, Q):
     for r in range(P * Q):
         L = mgpu.Layout(n, nb, P, Q, r)
         assert (L.p, L.q) == divmod(r, Q)
-        for I, J in D.local_tiles(r, P, Q, nt, nt):
-            assert L.owner(I, J) == r == D.owner(I, J, P, Q)
+        for I, J in L.tiles():
+            assert L.owner(I, J) == r == (I % P) * Q + J % Q
             seen[(I, J)] = r
-        assert L.mt_loc * L.nt_loc == len(D.local_tiles(r, P, Q, nt, nt))
+        assert L.mt_loc * L.nt_loc == len(L.tiles())
     assert len(seen) == nt * nt
 
 
@@ -83,6 +83,7 @@ def test_to_local():
 
 
 def test_classify_bcast():
+    assert mgpu.classify_bcast is D.classify_bcast
     assert mgpu.classify_bcast(0, 3) == "clean"
     assert mgpu.classify_bcast(1, 3) == "communication"
     assert mgpu.classify_bcast(3, 3) == "restart"

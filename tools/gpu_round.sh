@@ -1,14 +1,24 @@
 #!/bin/bash
-# One GPU session: all GPU tests, smoke, bench, ncu launch list + full capture.
-set -x
-mkdir -p gpurun_out
-python __graft_entry__.py smoke > gpurun_out/smoke.log 2>&1
-python -m pytest tests -x -q -m gpu > gpurun_out/gpu_tests.log 2>&1
-tail -5 gpurun_out/gpu_tests.log
-timeout 900 python bench.py --steps 10 --warmup 3 > gpurun_out/bench.log 2>&1
-tail -3 gpurun_out/bench.log
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv \
-   python bench.py --steps 2 --warmup 1 --no-e2e --no-potrf --no-cpu > gpurun_out/ncu_launch.log 2>&1
+# Round evidence (run under gpurun from the repo root): smoke, every GPU
+# test, the N=1 bench line, the ncu launch list of the bench step and of one
+# ft_potrf, one ncu --set full capture of the checksum pass, and
+# compute-sanitizer (racecheck, synccheck, memcheck) on tiny shapes.
+#   gpurun --timeout 3600 -- 'bash tools/gpu_round.sh r02'
+tag=${1:-round}
+out=gpurun_out/$tag
+mkdir -p $out
+python __graft_entry__.py smoke > $out/smoke.log 2>&1; tail -1 $out/smoke.log
+timeout 2400 python -m pytest tests -q -m gpu > $out/gpu_tests.log 2>&1; tail -1 $out/gpu_tests.log
+timeout 1500 python bench.py --steps 10 --warmup 3 > $out/bench.log 2>&1
+tail -1 $out/bench.log | cut -c1-300
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $out/bench_launches.csv \
+   python bench.py --steps 2 --warmup 1 --no-e2e --no-potrf --no-cpu --no-lu-qr --no-mgpu > $out/ncu_launch.log 2>&1
+timeout 900 ncu --metrics gpu__time_duration.sum,launch__grid_size --clock-control none -c 6000 --csv \
+   --log-file $out/potrf30720_launches.csv python tools/potrf_profile.py 30720 512 1 > $out/potrf_prof.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:checksum_pass -s 2 -c 2 \
-   -o gpurun_out/prof_pass -f python bench.py --steps 1 --warmup 1 --no-e2e --no-potrf --no-cpu > gpurun_out/ncu_full.log 2>&1
-tail -3 gpurun_out/ncu_full.log
+   -o $out/prof_pass -f python bench.py --steps 1 --warmup 1 --no-e2e --no-potrf --no-cpu --no-lu-qr --no-mgpu \
+   > $out/ncu_full.log 2>&1
+for tool in racecheck synccheck memcheck; do
+  timeout 900 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize_small.py > $out/sanitizer_$tool.log 2>&1
+  tail -2 $out/sanitizer_$tool.log
+done
