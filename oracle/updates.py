@@ -305,36 +305,47 @@ def lu_pu_chk(st: State, k: int):
         st.rowmag[r0:r1, k + 1:] = np.abs(tri_inv(Lkk, lower=True, unit=True)) @ st.rowmag[r0:r1, k + 1:]
 
 
-def lu_tmu_data(st: State, k: int):
-    """c-13 TMU data step: A_IJ −= L_Ik·U_kJ for every trailing tile."""
+def lu_tmu_data(st: State, k: int, c0: int = None, c1: int = None):
+    """c-13 TMU data step: A_IJ −= L_Ik·U_kJ for every trailing tile (tile
+    columns in [c0, c1) only, for the look-ahead split, reading c-35)."""
     nb, n = st.nb, st.A.shape[0]
     r0, r1 = k * nb, (k + 1) * nb
-    st.A[r1:n, r1:n] -= st.A[r1:n, r0:r1] @ st.A[r0:r1, r1:n]
+    c0 = r1 if c0 is None else c0
+    c1 = n if c1 is None else c1
+    st.A[r1:n, c0:c1] -= st.A[r1:n, r0:r1] @ st.A[r0:r1, c0:c1]
 
 
-def lu_tmu_chk(st: State, k: int):
+def lu_tmu_chk(st: State, k: int, c0: int = None, c1: int = None):
     """c-13 TMU checksum step: c(A_IJ) −= c(L_Ik)·U_kJ, r(A_IJ) −= L_Ik·r(U_kJ);
-    m_c += m_c(L)·|U|, m_r += |L|·m_r(U) (c-6)."""
+    m_c += m_c(L)·|U|, m_r += |L|·m_r(U) (c-6).  Tile-aligned column range
+    [c0, c1) as in lu_tmu_data."""
     nb, n = st.nb, st.A.shape[0]
     r0, r1 = k * nb, (k + 1) * nb
-    L21, U12 = st.A[r1:n, r0:r1], st.A[r0:r1, r1:n]
-    st.colchk[2 * (k + 1):, r1:n] -= st.colchk[2 * (k + 1):, r0:r1] @ U12
-    st.rowchk[r1:n, 2 * (k + 1):] -= L21 @ st.rowchk[r0:r1, 2 * (k + 1):]
+    c0 = r1 if c0 is None else c0
+    c1 = n if c1 is None else c1
+    J0, J1 = c0 // nb, c1 // nb
+    L21, U1j = st.A[r1:n, r0:r1], st.A[r0:r1, c0:c1]
+    st.colchk[2 * (k + 1):, c0:c1] -= st.colchk[2 * (k + 1):, r0:r1] @ U1j
+    st.rowchk[r1:n, 2 * J0:2 * J1] -= L21 @ st.rowchk[r0:r1, 2 * J0:2 * J1]
     if st.colmag is not None:
-        st.colmag[k + 1:, r1:n] += st.colmag[k + 1:, r0:r1] @ np.abs(U12)
-        st.rowmag[r1:n, k + 1:] += np.abs(L21) @ st.rowmag[r0:r1, k + 1:]
+        st.colmag[k + 1:, c0:c1] += st.colmag[k + 1:, r0:r1] @ np.abs(U1j)
+        st.rowmag[r1:n, J0:J1] += np.abs(L21) @ st.rowmag[r0:r1, J0:J1]
 
 
-def lu_fig4a_repair(st: State, k: int, gi: int, gj: int, before: float, after: float):
+def lu_fig4a_repair(st: State, k: int, gi: int, gj: int, before: float, after: float, c0: int = 0,
+                    c1: int = None):
     """Reading c-25 for LU: the post-TMU re-check corrected a panel element by
     E = after − before; the TMU had consumed the bad value.
     L21[p, q] (column panel): A[p, r1:] −= E·U[q, r1:], r(A_i,J)[p', :] −= E·r(U_J)[q, :]
       (c(A) was built from the good c(L), so only data and r change); m_r += |E|·m_r(U).
     U12[q, c] (row panel): A[r1:, c] −= L21[:, q]·E, c(A_I,j)[:, c'] −= c(L_I)[:, q]·E
       (r(A) was built from the good r(U)); m_c += |E|·m_c(L).
-    Guard as in Cholesky (2^10 × max |panel line|, finite)."""
+    Guard as in Cholesky (2^10 × max |panel line|, finite).  A column range
+    [c0, c1) (look-ahead, reading c-35) restricts the repair to the trailing
+    columns whose update consumed the bad value."""
     nb, n = st.nb, st.A.shape[0]
     nt = n // nb
+    c1 = n if c1 is None else c1
     r0, r1 = k * nb, (k + 1) * nb
     E = after - before
     if r0 <= gj < r1 and gi >= r1:  # element of L21
@@ -342,8 +353,11 @@ def lu_fig4a_repair(st: State, k: int, gi: int, gj: int, before: float, after: f
         mx = float(np.max(np.abs(st.A[r1:n, gj])))
         if not (np.isfinite(E) and abs(E) <= 1024.0 * mx):
             return "skipped"
-        st.A[p, r1:n] -= E * st.A[r0 + q, r1:n]
+        b0, b1 = max(r1, c0), min(n, c1)
+        st.A[p, b0:b1] -= E * st.A[r0 + q, b0:b1]
         for J in range(k + 1, nt):
+            if not c0 <= J * nb < c1:
+                continue
             st.rowchk[p, 2 * J:2 * J + 2] -= E * st.rowchk[r0 + q, 2 * J:2 * J + 2]
             if st.rowmag is not None:
                 st.rowmag[p, J] += abs(E) * st.rowmag[r0 + q, J]
@@ -353,6 +367,8 @@ def lu_fig4a_repair(st: State, k: int, gi: int, gj: int, before: float, after: f
         mx = float(np.max(np.abs(st.A[gi, r1:n])))
         if not (np.isfinite(E) and abs(E) <= 1024.0 * mx):
             return "skipped"
+        if not c0 <= c < c1:
+            return "applied"
         st.A[r1:n, c] -= st.A[r1:n, r0 + q] * E
         for I in range(k + 1, nt):
             st.colchk[2 * I:2 * I + 2, c] -= E * st.colchk[2 * I:2 * I + 2, r0 + q]

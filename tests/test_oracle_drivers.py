@@ -536,3 +536,59 @@ def test_lookahead_fault_outcomes_equal_alg2(case):
     assert s1.counts == s0.counts and s1.restarts == s0.restarts and s1.repairs_applied == s0.repairs_applied
     assert sorted((f.gi, f.gj, f.cls, f.kind) for f in s1.fixes) == sorted((f.gi, f.gj, f.cls, f.kind) for f in s0.fixes)
     assert np.abs(L1 - L0).max() <= 1e-13 * np.abs(L0).max()
+
+
+def test_lu_lookahead_tmu_split_and_restricted_repairs():
+    """LU (c-35): the TMU split by tile columns equals the whole TMU, and the
+    two restricted Fig. 4a repairs add up to the unrestricted one (an L21 and
+    a U12 element)."""
+    n, nb, k = 256, 32, 1
+    st = ck.State.alloc(si.general(n, seed=61), nb)
+    nt = n // nb
+    ck.encode(st, ck.Tiles(0, nt, 0, nt), ck.BOTH)
+    for kk in range(k + 1):
+        up.lu_pd(st, kk)
+        up.lu_pu_data(st, kk)
+        up.lu_pu_chk(st, kk)
+        if kk < k:
+            up.lu_tmu_data(st, kk)
+            up.lu_tmu_chk(st, kk)
+    r1, c2 = (k + 1) * nb, (k + 2) * nb
+    a, b = st.copy(), st.copy()
+    up.lu_tmu_data(a, k)
+    up.lu_tmu_chk(a, k)
+    for c0, c1 in ((r1, c2), (c2, n)):
+        up.lu_tmu_data(b, k, c0, c1)
+        up.lu_tmu_chk(b, k, c0, c1)
+    for x, y in ((a.A, b.A), (a.colchk, b.colchk), (a.rowchk, b.rowchk), (a.colmag, b.colmag), (a.rowmag, b.rowmag)):
+        assert np.abs(x - y).max() <= 1e-13 * max(1.0, np.abs(x).max())
+    for gi, gj in ((150, k * nb + 4), (k * nb + 6, 150), (k * nb + 6, r1 + 3)):
+        a, b = st.copy(), st.copy()
+        assert up.lu_fig4a_repair(a, k, gi, gj, 0.25, 0.75) == "applied"
+        up.lu_fig4a_repair(b, k, gi, gj, 0.25, 0.75, r1, c2)
+        up.lu_fig4a_repair(b, k, gi, gj, 0.25, 0.75, c2, n)
+        for x, y in ((a.A, b.A), (a.colchk, b.colchk), (a.rowchk, b.rowchk), (a.colmag, b.colmag),
+                     (a.rowmag, b.rowmag)):
+            assert np.array_equal(x, y), (gi, gj)
+
+
+@pytest.mark.parametrize("n,nb", [(256, 32), (384, 128)])
+def test_lu_lookahead_error_free(n, nb):
+    A = si.general(n, seed=n + 9)
+    LU, piv, st = dr.ft_getrf(A, nb, lookahead=True, invariant_hook=_lu_invariant)
+    lu, p = sla.lu_factor(A)
+    assert np.array_equal(piv, p) and np.abs(LU - lu).max() <= 1e-12 * np.abs(lu).max()
+    _, _, s0 = dr.ft_getrf(A, nb)
+    assert st.counts == [0] * 8 and st.n_checks == s0.n_checks + 2 * (n // nb - 1)  # both panels re-checked twice
+
+
+@pytest.mark.parametrize("case", range(len(LU_FIXABLE)))
+def test_lu_lookahead_fault_outcomes_equal_alg2(case):
+    point, kind, gi, gj, bits = LU_FIXABLE[case]
+    inj = [dr.Inject(2, point, kind, 0, gi, gj, bits)]
+    A = si.general(256, seed=0)
+    L0, p0, s0 = dr.ft_getrf(A, 32, inject=inj)
+    L1, p1, s1 = dr.ft_getrf(A, 32, inject=inj, lookahead=True)
+    assert s1.counts == s0.counts and s1.restarts == s0.restarts and s1.repairs_applied == s0.repairs_applied
+    assert sorted((f.gi, f.gj, f.cls, f.kind) for f in s1.fixes) == sorted((f.gi, f.gj, f.cls, f.kind) for f in s0.fixes)
+    assert np.array_equal(p0, p1) and np.abs(L1 - L0).max() <= 1e-13 * np.abs(L0).max()
