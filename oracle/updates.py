@@ -215,31 +215,45 @@ def lu_swap_rows(ipiv, k, nb):
     return sorted(set(rows))
 
 
-def lu_pd_apply(st: State, k: int, lu, ipiv, P0):
+def lu_pd_apply(st: State, k: int, lu, ipiv, P0, part: str = "all"):
     """c-13/c-14 PD, apply step: the row swaps on the left (factored L
     panels, c only) and right (trailing, c and r) columns with the swap rule,
     the panel's own column checksums swapped with the PRE-PD copy (L430),
     then c(L_I) = c(P~_I)·U_kk^{-1} (L_kk in UNIT_LOWER view) and
-    r(U_kk) = L_kk^{-1}·r(P~_kk), magnitudes by |U_kk^{-1}|, |L_kk^{-1}| (c-6)."""
+    r(U_kk) = L_kk^{-1}·r(P~_kk), magnitudes by |U_kk^{-1}|, |L_kk^{-1}| (c-6).
+    part (look-ahead, reading c-35): "panel" = everything inside the column
+    panel (its columns' deltas, the row checksums of tile column k, the
+    factor, the rules); "outside" = the swaps of every other column with
+    their deltas and the row checksums of tile columns > k.  The two touch
+    disjoint entries, so "panel" then "outside" equals "all"."""
     nb, n = st.nb, st.A.shape[0]
     nt = n // nb
     r0, r1 = k * nb, (k + 1) * nb
-    copy = P0.copy()
+    copy = P0.copy() if P0 is not None else None
     panel_cols = np.arange(r0, r1)
     left_cols = np.arange(0, r0)
     right_cols = np.arange(r1, n)
+    inside, outside = part in ("all", "panel"), part in ("all", "outside")
     for j in range(nb):
         p, q = r0 + j, int(ipiv[j])
         if p == q:
             continue
-        lu_swap_rule(st, p, q, panel_cols, copy[p - r0].copy(), copy[q - r0].copy(), row_chk_cols=range(k, nt))
-        copy[[p - r0, q - r0]] = copy[[q - r0, p - r0]]
+        if inside:
+            lu_swap_rule(st, p, q, panel_cols, copy[p - r0].copy(), copy[q - r0].copy(),
+                         row_chk_cols=range(k, nt) if part == "all" else range(k, k + 1))
+            copy[[p - r0, q - r0]] = copy[[q - r0, p - r0]]
+        if not outside:
+            continue
+        if part == "outside":
+            lu_swap_rule(st, p, q, [], (), (), row_chk_cols=range(k + 1, nt))
         if r0 > 0:
             lu_swap_rule(st, p, q, left_cols, st.A[p, :r0].copy(), st.A[q, :r0].copy())
         if r1 < n:
             lu_swap_rule(st, p, q, right_cols, st.A[p, r1:].copy(), st.A[q, r1:].copy())
         st.A[[p, q], :r0] = st.A[[q, p], :r0]
         st.A[[p, q], r1:] = st.A[[q, p], r1:]
+    if not inside:
+        return
     st.A[r0:n, r0:r1] = lu
     U = np.triu(lu[:nb, :nb])
     Lkk = np.tril(lu[:nb, :nb], -1) + np.eye(nb)

@@ -592,3 +592,17 @@ def test_lu_lookahead_fault_outcomes_equal_alg2(case):
     assert s1.counts == s0.counts and s1.restarts == s0.restarts and s1.repairs_applied == s0.repairs_applied
     assert sorted((f.gi, f.gj, f.cls, f.kind) for f in s1.fixes) == sorted((f.gi, f.gj, f.cls, f.kind) for f in s0.fixes)
     assert np.array_equal(p0, p1) and np.abs(L1 - L0).max() <= 1e-13 * np.abs(L0).max()
+
+
+@pytest.mark.parametrize("bit,gi,gj", [(62, 200, 66), (60, 130, 70), (55, 64, 64)])
+def test_lu_lookahead_split_pd_restart_equals_alg2(bit, gi, gj):
+    """A PD-consumed fault in a panel the look-ahead factored (split PD, c-35):
+    the restart redoes only the part inside the panel (nothing outside moved
+    yet) and ends at Alg. 2's result: same pivots, factor, counters, fixes."""
+    A = si.general(256, seed=31)
+    inj = [dr.Inject(1, dr.AT_PRE_PD, dr.KIND_PERSIST, 0, gi, gj, (bit,))]
+    l0, p0, s0 = dr.ft_getrf(A, 64, inject=inj)
+    l1, p1, s1 = dr.ft_getrf(A, 64, inject=inj, lookahead=True)
+    assert s1.restarts == s0.restarts == 1 and s1.uncorrectable == s0.uncorrectable == 0
+    assert s1.counts == s0.counts
+    assert np.array_equal(p1, p0) and np.abs(l1 - l0).max() <= 1e-13 * np.abs(l0).max()
