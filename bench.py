@@ -49,15 +49,16 @@ def peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def ncu_traffic(n=None, nb=None):
-    """dram read+write bytes per launch of the dominant kernel from the
-    committed `ncu --set full` summary (profiles/) of the same (n, nb), or None."""
+def ncu_traffic(n=None, nb=None, kernel=None):
+    """dram read+write bytes per launch of the dominant kernel (`kernel`, the
+    name bench.py reports) from the committed `ncu --set full` summary
+    (profiles/) of the same (n, nb), or None."""
     p = os.path.join(ROOT, "profiles", "ncu_verify_summary.json")
     try:
         with open(p) as f:
             d = json.load(f)
         if d.get("n") == (n or N_MAT) and d.get("nb") == (nb or NB):
-            return float(d["dram_bytes_per_launch"])
+            return float(d["kernels"][kernel]["dram_bytes_per_launch"])
     except Exception:
         pass
     return None
@@ -415,7 +416,7 @@ def run_ours(args):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": workload_config(n, nb, world, args.potrf_n),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": ncu_traffic(n, nb), "kernel": dom,
+                         "frac": achieved / peak, "traffic": ncu_traffic(n, nb, dom), "kernel": dom,
                          "bytes_per_launch": pass_bytes, "ms_per_launch": dom_ms, "peak_source": peak_src,
                          "encode_GBs": pass_bytes / (enc_ms / 1e3) / 1e9,
                          "verify_GBs": pass_bytes / (ver_ms / 1e3) / 1e9,
@@ -437,13 +438,13 @@ def potrf_overhead(abft, si, n, nb, reps, host_pd=True):
     A = torch.empty_like(A0.t()).t()
     ctx = abft.Context()
 
-    def run(ft, restart=True, pd=abft.PD_DEVICE, scheme=abft.SCHEME_NEW, gemm=False):
+    def run(ft, restart=True, pd=abft.PD_DEVICE, scheme=abft.SCHEME_NEW, gemm=False, la=True, timing=False):
         A.copy_(A0)
         torch.cuda.synchronize()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record()
         rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart, pd_location=pd, scheme=scheme,
-                                     checksum_gemm=gemm)
+                                     checksum_gemm=gemm, lookahead=la, timing=timing)
         b.record()
         torch.cuda.synchronize()
         assert rc == 0 and info == 0
@@ -452,6 +453,9 @@ def potrf_overhead(abft, si, n, nb, reps, host_pd=True):
     run(True)
     run(False)
     t_ft, t_plain, t_nors = [], [], []
+    # one run of each without look-ahead (the Alg. 2 order of round 1) for context
+    run(True, la=False)
+    nola_ft, nola_plain = run(True, la=False)[0], run(False, la=False)[0]
     for _ in range(reps):
         t_plain.append(run(False)[0])
         t, st = run(True)
@@ -473,10 +477,12 @@ def potrf_overhead(abft, si, n, nb, reps, host_pd=True):
                          ("full_post", abft.SCHEME_FULL_POST, False),
                          ("single_post", abft.SCHEME_SINGLE_POST, False),
                          ("single_pre", abft.SCHEME_SINGLE_PRE, False)):
-        run(True, restart=False, scheme=sc, gemm=gm)
-        ts = sorted(run(True, restart=False, scheme=sc, gemm=gm)[0] for _ in range(max(1, reps - 1)))
+        # all schemes in Alg. 2's sequential order (look-ahead applies to the
+        # new scheme only), against the sequential unprotected driver
+        run(True, restart=False, scheme=sc, gemm=gm, la=False)
+        ts = sorted(run(True, restart=False, scheme=sc, gemm=gm, la=False)[0] for _ in range(max(1, reps - 1)))
         tm = ts[len(ts) // 2]
-        schemes[name] = {"ms_ft": tm, "overhead_pct": 100.0 * (tm - plain_ms) / plain_ms}
+        schemes[name] = {"ms_ft": tm, "overhead_pct": 100.0 * (tm - nola_plain) / nola_plain}
     host = None
     if host_pd:  # Alg. 2 lines 3-7 with the PD on the host (FT_PD_HOST)
         import os
@@ -498,10 +504,15 @@ def potrf_overhead(abft, si, n, nb, reps, host_pd=True):
     b.record()
     torch.cuda.synchronize()
     cus = a.elapsed_time(b)
+    phases = dict(zip(abft.PHASES, run(True, timing=True)[1].ms_phase))
     del S, A, A0
     torch.cuda.empty_cache()
     return {"n": n, "nb": nb, "ms_ft": ft_ms, "ms_plain": plain_ms,
             "overhead_pct": 100.0 * (ft_ms - plain_ms) / plain_ms, "cusolver_potrf_ms": cus,
+            "overhead_vs_cusolver_pct": 100.0 * (ft_ms - cus) / cus,
+            "lookahead": True, "phases_ms": phases,
+            "no_lookahead": {"ms_ft": nola_ft, "ms_plain": nola_plain,
+                             "overhead_pct": 100.0 * (nola_ft - nola_plain) / nola_plain},
             "ms_ft_no_restart": nors_ms, "overhead_pct_no_restart": 100.0 * (nors_ms - plain_ms) / plain_ms,
             "tflops_ft": n ** 3 / 3 / (ft_ms / 1e3) / 1e12, "reps": reps, "host_pd": host,
             "schemes_no_restart": schemes}

@@ -380,11 +380,13 @@ typedef struct {
                             schemes (L35, L47, L542, Table VIII, Figs. 12-14; reading c-34) */
   int32_t timing;        /* 1: per-phase device time (CUDA events on the stream each phase runs on) into
                             ft_stats_t.ms_phase; costs two event records per timed span.  Default 0. */
-  int32_t lookahead;     /* ft_potrf (FT_SCHEME_NEW or abft = 0): 1 = the TMU of iteration k updates tile
-                            column k+1 first (and re-checks the panel, Fig. 4a), then the PD / PU of
-                            iteration k+1 with their checks run on a second stream next to the rest of
-                            the TMU (reading c-35).  Off for an iteration whose fault hooks it would
-                            move.  Ignored by ft_getrf / ft_geqrf.  Default 0 (bindings: 1). */
+  int32_t lookahead;     /* 1 = the TMU of iteration k updates tile column k+1 first (and re-checks the
+                            panel(s), Fig. 4a), then iteration k+1's panel work runs on a second stream
+                            next to the rest of the TMU (reading c-35): ft_potrf (FT_SCHEME_NEW or
+                            abft = 0) its checks, PD and PU; ft_getrf its checks and the factorization
+                            of the column panel (the swaps outside it and the PU follow the TMU).  Off
+                            for an iteration whose fault hooks it would move.  Ignored by ft_geqrf.
+                            Default 0 (bindings: 1). */
 } ft_opts_t;
 
 /* ft_opts_t.scheme (reading c-34).  NEW: the paper's scheme, Alg. 2 (full

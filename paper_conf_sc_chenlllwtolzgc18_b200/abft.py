@@ -410,12 +410,13 @@ def abft_panel_getrf(mat: Mat, k: int, ipiv: torch.Tensor, Linv: torch.Tensor, U
 
 def ft_getrf(ctx: Context, A: torch.Tensor, nb: int, ipiv: torch.Tensor, abft=True, tol_kind=TOL_MAGNITUDE,
              tol_scale=1.0, fig4a_repair=True, inject=(), fix_log=None, pd_location=PD_DEVICE, restart=True,
-             fig4b=True, trailing_check_period=0, timing=False):
+             fig4b=True, trailing_check_period=0, timing=False, lookahead=True):
     """Fault-tolerant LU with partial pivoting in place on a column-major A;
     ipiv: int64 device tensor (n), receives 1-based global pivots."""
     n = A.shape[0]
     opts, _inj = _opts(nb, abft, tol_kind, tol_scale, fig4a_repair, inject, fix_log, True, restart=restart,
-                       pd_location=pd_location, fig4b=fig4b, period=trailing_check_period, timing=timing)
+                       pd_location=pd_location, fig4b=fig4b, period=trailing_check_period, timing=timing,
+                       lookahead=lookahead)
     stats = ft_stats_t()
     info = C.c_int64()
     rc = _L.ft_getrf(ctx._h, _dt(A), n, _ptr(A), ld_of(A), _ptr(ipiv), C.byref(opts), C.byref(stats),

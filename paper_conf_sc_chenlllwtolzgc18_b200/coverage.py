@@ -61,9 +61,11 @@ OUTCOME = {
     # are seen, input (reference) errors consumed before the check are 2D for
     # PD / PU (Table V), PU output still unprotected, TMU 1D not tolerable,
     # communication after the check unseen (L346: checked before broadcast).
+    # (PD "mem_during_upd": a fault the factorization consumes spreads over
+    # L_kk — 2D for every scheme (c-17, [32]); the post-op check restarts)
     "single_post": {
         "PD": {"comp": Y, "mem_between_ref": R, "mem_between_upd": R, "mem_during_ref": R,
-               "mem_during_upd": Y, "pcie": N},
+               "mem_during_upd": R, "pcie": N},
         "PU": {"comp": N, "mem_between_ref": N, "mem_between_upd": N, "mem_during_ref": N,
                "mem_during_upd": N, "pcie": N},
         "TMU": {"comp": Y, "mem_between_ref": R, "mem_between_upd": Y, "mem_during_ref": R,
@@ -74,7 +76,7 @@ OUTCOME = {
     # (restart), communication after the check is unseen (L346).
     "full_post": {
         "PD": {"comp": Y, "mem_between_ref": R, "mem_between_upd": R, "mem_during_ref": R,
-               "mem_during_upd": Y, "pcie": N},
+               "mem_during_upd": R, "pcie": N},
         "PU": {"comp": Y, "mem_between_ref": R, "mem_between_upd": Y, "mem_during_ref": R,
                "mem_during_upd": Y, "pcie": N},
         "TMU": {"comp": Y, "mem_between_ref": Y, "mem_between_upd": Y, "mem_during_ref": Y,
@@ -87,7 +89,7 @@ OUTCOME = {
     # for faults consumed inside PD / PU, Y after the local restart).
     "ours": {
         "PD": {"comp": Y, "mem_between_ref": Y, "mem_between_upd": Y, "mem_during_ref": R,
-               "mem_during_upd": Y, "pcie": Y},
+               "mem_during_upd": R, "pcie": Y},
         "PU": {"comp": Y, "mem_between_ref": Y, "mem_between_upd": Y, "mem_during_ref": R,
                "mem_during_upd": Y, "pcie": Y},
         "TMU": {"comp": Y, "mem_between_ref": Y, "mem_between_upd": Y, "mem_during_ref": Y,
@@ -164,25 +166,80 @@ def event_probabilities(op: OpSize, rates: Rates) -> dict:
     return {"events": ev, "fault_free": clean, "single": single}
 
 
-def outcomes(op_name: str, op: OpSize, rates: Rates, scheme: str) -> dict:
+def outcomes(op_name: str, op: OpSize, rates: Rates, scheme: str, measured: dict = None) -> dict:
     """Probabilities of the four outcomes of one operation under a scheme
     (at most one fault per operation, L633: the remainder — two or more
-    faults — is reported separately as 'multi')."""
+    faults — is reported separately as 'multi').  measured (scheme "ours"
+    only): outcome fractions per (op, fault) observed by the fault campaigns
+    (`campaign_fractions`); cells the campaigns did not sample use OUTCOME."""
     e = event_probabilities(op, rates)
     out = {"fault_free": e["fault_free"], Y: 0.0, R: 0.0, N: 0.0}
     for f, p in e["single"].items():
-        out[OUTCOME[scheme][op_name][f]] += p
+        cell = (measured or {}).get(op_name, {}).get(f) if scheme == "ours" else None
+        if cell:
+            for o, frac in cell.items():
+                out[o] += p * frac
+        else:
+            out[OUTCOME[scheme][op_name][f]] += p
     out["multi"] = max(0.0, 1.0 - sum(out.values()))
     return out
 
 
+# campaign hook (tools/campaign.py `inject` entries: iter, point, kind, target,
+# gi, gj) -> the model's (op, single fault) of reading c-33.  The campaigns
+# draw PD / PU faults in the op's update part and TMU faults in its
+# reference part (the panel) or output; D2H / H2D are the PD's transfers.
+_HOOK_CELL = {(0, 0): ("PD", "mem_between_upd"), (1, 0): ("PD", "mem_during_upd"), (2, 0): ("PD", "comp"),
+              (3, 0): ("PU", "mem_between_upd"), (4, 0): ("PU", "mem_during_upd"),
+              (4, 1): ("PU", "mem_during_upd"), (5, 0): ("PU", "comp"), (6, 0): ("TMU", "mem_between_ref"),
+              (6, 1): ("TMU", "mem_during_ref"), (7, 0): ("TMU", "comp"), (8, 0): ("PD", "pcie"),
+              (9, 0): ("PD", "pcie")}
+
+
+def campaign_outcome(case: dict) -> str:
+    """A campaign run's outcome in the model's terms: fixed without a restart
+    -> fixable; fixed by the local restart -> local restart; returned
+    uncorrectable (R) or silently wrong (N) -> complete restart."""
+    if case["outcome"] in ("Y", "Yr"):
+        return R if case.get("restarts", 0) > 0 else Y
+    return N
+
+
+def campaign_fractions(campaigns) -> dict:
+    """Outcome fractions per (op, fault) from single-fault campaign runs
+    (the K = 1 sections of tools/campaign.py's JSON, any driver)."""
+    tally = {}
+    for camp in campaigns:
+        for key, sec in camp.items():
+            if not isinstance(sec, dict) or "cases" not in sec:
+                continue
+            for case in sec["cases"]:
+                if len(case["inject"]) != 1:
+                    continue
+                it, point, kind, target = case["inject"][0][:4]
+                cell = _HOOK_CELL.get((point, kind)) if target == 0 else None
+                if cell is None:
+                    continue
+                d = tally.setdefault(cell[0], {}).setdefault(cell[1], {})
+                o = campaign_outcome(case)
+                d[o] = d.get(o, 0) + 1
+    out = {}
+    for op, faults in tally.items():
+        for f, cnt in faults.items():
+            tot = sum(cnt.values())
+            out.setdefault(op, {})[f] = {o: c / tot for o, c in cnt.items()}
+            out[op][f]["runs"] = tot
+    return {op: {f: {k: v for k, v in c.items() if k != "runs"} for f, c in fs.items()} for op, fs in out.items()}, \
+        {op: {f: c["runs"] for f, c in fs.items()} for op, fs in out.items()}
+
+
 def expected_recovery_time(op_name: str, op: OpSize, rates: Rates, scheme: str, t_fix: float,
-                           t_total: float) -> float:
+                           t_total: float, measured: dict = None) -> float:
     """Expected extra time of one operation (L646: "expected time cost for
     fault recovery"): fixable -> t_fix (measured ABFT correction cost),
     local restart -> the op again (A_OP) plus t_fix, complete restart -> the
     whole factorization t_total."""
-    o = outcomes(op_name, op, rates, scheme)
+    o = outcomes(op_name, op, rates, scheme, measured)
     return o[Y] * t_fix + o[R] * (op.a_op + t_fix) + o[N] * t_total
 
 

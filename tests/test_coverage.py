@@ -64,3 +64,35 @@ def test_expected_recovery_ours_lowest():
     cost = {s: sum(cv.expected_recovery_time(n, op, rates, s, t_fix=1e-5, t_total=1.0) for n, op in ops.items())
             for s in cv.SCHEMES}
     assert cost["ours"] == min(cost.values()) and cost["ours"] < cost["single_prior"]
+
+
+def _campaigns():
+    import json
+    import os
+
+    root = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles")
+    out = []
+    for f in sorted(os.listdir(root)):
+        if "campaign_n" in f and f.endswith(".json") and "schemes" not in f:
+            with open(os.path.join(root, f)) as fh:
+                out.append(json.load(fh))
+    return out
+
+
+def test_ours_row_agrees_with_the_measured_campaigns():
+    """The 'ours' row is generated from the committed campaigns wherever they
+    sampled a cell: the reading's entry is the most frequent measured
+    outcome, and no campaign run ended silently wrong."""
+    frac, runs = cv.campaign_fractions(_campaigns())
+    assert frac, "no campaign JSON under profiles/"
+    seen = 0
+    for op, cells in frac.items():
+        for f, d in cells.items():
+            assert abs(sum(d.values()) - 1.0) < 1e-12
+            top = max(d, key=d.get)
+            assert cv.OUTCOME["ours"][op][f] == top, (op, f, d, runs[op][f])
+            seen += 1
+    assert seen >= 9  # PD / PU / TMU cells the campaigns draw (+ the PD transfers)
+    o = cv.outcomes("TMU", cv.lu_iteration(10240, 256, 2e-4, 1e-3, 3e-2)["TMU"], cv.Rates(1e-13, 1e-6, 1e-6, 1e-9),
+                    "ours", frac)
+    assert math.isclose(sum(o.values()), 1.0, rel_tol=1e-12)

@@ -99,7 +99,7 @@ def _parity(lib, ctx, which, A, nb, inject):
         o_out, ost = dr.ft_potrf(A, nb, inject=inject, pd_location="host", lookahead=True)
         ref, _ = dr.ft_potrf(A, nb)
     elif which == "getrf":
-        o_out, o_piv, ost = dr.ft_getrf(A, nb, inject=inject, pd_location="host")
+        o_out, o_piv, ost = dr.ft_getrf(A, nb, inject=inject, pd_location="host", lookahead=True)
         ref, _, _ = dr.ft_getrf(A, nb)
         assert np.array_equal(g_ex - 1, o_piv)
     else:

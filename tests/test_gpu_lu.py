@@ -17,21 +17,25 @@ def ctx(lib):
     return lib.Context()
 
 
-def _gpu_getrf(lib, ctx, A_np, nb, inject=(), abft=True, fig4a=True, dtype=torch.float64):
+def _gpu_getrf(lib, ctx, A_np, nb, inject=(), abft=True, fig4a=True, dtype=torch.float64, lookahead=True):
     A = dev(A_np, dtype)
     n = A.shape[0]
     ipiv = torch.zeros(n, dtype=torch.int64, device="cuda")
     inj = [(f.iter, f.point, f.kind, f.target, f.gi, f.gj, si.mask_of(f.bits)) for f in inject]
     log = torch.zeros(8192 * lib.FIX_BYTES, dtype=torch.uint8, device="cuda")
-    rc, info, stats = lib.ft_getrf(ctx, A, nb, ipiv, abft=abft, fig4a_repair=fig4a, inject=inj, fix_log=log)
+    rc, info, stats = lib.ft_getrf(ctx, A, nb, ipiv, abft=abft, fig4a_repair=fig4a, inject=inj, fix_log=log,
+                                   lookahead=lookahead)
     torch.cuda.synchronize()
     return host(A), ipiv.cpu().numpy() - 1, rc, info, stats, lib.decode_fixes(log, stats.n_fixes)
 
 
+@pytest.mark.parametrize("lookahead", [True, False])
 @pytest.mark.parametrize("n,nb", [(256, 32), (1024, 128), (2048, 256), (2048, 512), (4096, 1024)])
-def test_error_free_matches_lapack(lib, ctx, n, nb):
+def test_error_free_matches_lapack(lib, ctx, n, nb, lookahead):
     A = si.general(n, seed=n)
-    LU, piv, rc, info, stats, fixes = _gpu_getrf(lib, ctx, A, nb)
+    LU, piv, rc, info, stats, fixes = _gpu_getrf(lib, ctx, A, nb, lookahead=lookahead)
+    if n <= 1024:  # the check sequence of Alg. 2 (with the look-ahead's extra re-checks, c-35)
+        assert stats.n_checks == dr.ft_getrf(A, nb, lookahead=lookahead)[2].n_checks
     lu, p = sla.lu_factor(A)
     assert rc == 0 and info == 0 and list(stats.counts) == [0] * 8 and not fixes
     assert np.array_equal(piv, p)
@@ -57,15 +61,16 @@ def test_unprotected_same_factor(lib, ctx):
     assert np.abs(a[0] - b[0]).max() <= 1e-13 * np.abs(a[0]).max()
 
 
-def _compare(lib, ctx, A, nb, injects, prec="f64"):
+def _compare(lib, ctx, A, nb, injects, prec="f64", lookahead=True):
     """fp32: the GPU factors in fp32; the oracle carries the fp32 input, fp32
     flips and fp32 thresholds in fp64 arithmetic (pivots must still agree)."""
     vtol = 1e-12 if prec == "f64" else 1e-5
     if prec == "f32":
         A = A.astype(np.float32).astype(np.float64)
-    LUo, pivo, so = dr.ft_getrf(A, nb, prec=prec, inject=injects)
+    LUo, pivo, so = dr.ft_getrf(A, nb, prec=prec, inject=injects, lookahead=lookahead)
     LUg, pivg, rc, info, sg, fg = _gpu_getrf(lib, ctx, A, nb, inject=injects,
-                                             dtype=torch.float64 if prec == "f64" else torch.float32)
+                                             dtype=torch.float64 if prec == "f64" else torch.float32,
+                                             lookahead=lookahead)
     assert (rc == lib.E_UNCORRECTABLE) == (so.uncorrectable > 0)
     assert sg.repairs_skipped == so.repairs_skipped
     if so.repairs_skipped:
@@ -104,11 +109,12 @@ LU_CASES = [
 ]
 
 
+@pytest.mark.parametrize("lookahead", [True, False])
 @pytest.mark.parametrize("case", range(len(LU_CASES)))
-def test_lu_fault_campaign_parity(lib, ctx, case):
+def test_lu_fault_campaign_parity(lib, ctx, case, lookahead):
     k, point, kind, target, gi, gj, bits = LU_CASES[case]
     A = si.general(256, seed=0)
-    _compare(lib, ctx, A, 32, [dr.Inject(k, point, kind, target, gi, gj, bits)])
+    _compare(lib, ctx, A, 32, [dr.Inject(k, point, kind, target, gi, gj, bits)], lookahead=lookahead)
 
 
 @pytest.mark.parametrize("case", range(len(LU_CASES)))
@@ -195,7 +201,7 @@ def test_lu_restart_parity(lib, ctx, k, point, kind, gi, gj, bit):
     A = si.general(256, seed=31)
     inj = [dr.Inject(k, point, kind, 0, gi, gj, (bit,))]
     ref, pref, _ = dr.ft_getrf(A, nb)
-    o_lu, o_piv, ost = dr.ft_getrf(A, nb, inject=inj)
+    o_lu, o_piv, ost = dr.ft_getrf(A, nb, inject=inj, lookahead=True)
     LU, piv, rc, st = _gpu_getrf_rs(lib, ctx, A, nb, inj, True)
     assert ost.restarts == 1 and ost.uncorrectable == 0
     assert rc == 0 and st.restarts == 1 and st.uncorrectable == 0

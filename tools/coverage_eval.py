@@ -52,17 +52,28 @@ def main():
                "TMU": timed(lambda: torch.addmm(A22, A21, A12, beta=1.0, alpha=-1.0))},
     }
     rates = cv.Rates()
+    # "ours" generated from the committed single-fault campaigns (outcome
+    # fractions per op / fault, tools/campaign.py); unsampled cells: the table
+    prof = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles")
+    camps = []
+    for f in sorted(os.listdir(prof)):
+        if "campaign_n" in f and f.endswith(".json") and "schemes" not in f:
+            with open(os.path.join(prof, f)) as fh:
+                camps.append(json.load(fh))
+    measured, runs = cv.campaign_fractions(camps)
     out = {"n": n, "nb": nb, "rates": vars(rates), "a_op_s": times, "device": torch.cuda.get_device_name(),
-           "note": "one iteration at n_k = n; t_fix = 1e-5 s; complete restart = sum of the iteration's ops x n/nb"}
+           "ours_measured_fractions": measured, "ours_measured_runs": runs,
+           "note": "one iteration at n_k = n; t_fix = 1e-5 s; complete restart = sum of the iteration's ops x n/nb; "
+                   "'ours' uses the campaigns' outcome fractions where they sampled the cell"}
     for name, it in (("chol", cv.cholesky_iteration), ("lu", cv.lu_iteration)):
         t = times[name]
         ops = it(n, nb, t["PD"], t["PU"], t["TMU"])
         t_total = (t["PD"] + t["PU"] + t["TMU"]) * (n // nb) / 3.0  # ~ n/nb iterations shrinking cubically
         res = {}
         for s in cv.SCHEMES:
-            res[s] = {op: {k: v for k, v in cv.outcomes(op, ops[op], rates, s).items()} for op in cv.OPS}
+            res[s] = {op: {k: v for k, v in cv.outcomes(op, ops[op], rates, s, measured).items()} for op in cv.OPS}
             res[s]["expected_recovery_s"] = sum(
-                cv.expected_recovery_time(op, ops[op], rates, s, 1e-5, t_total) for op in cv.OPS)
+                cv.expected_recovery_time(op, ops[op], rates, s, 1e-5, t_total, measured) for op in cv.OPS)
         out[name] = res
         print(name, {s: res[s]["expected_recovery_s"] for s in cv.SCHEMES}, flush=True)
     os.makedirs("gpurun_out", exist_ok=True)

@@ -33,7 +33,7 @@ for dt in (torch.float64, torch.float32):
         print(dt, nb, n, "fixes", int(nfix.item()), "counts", rep.counts.tolist(), flush=True)
 ctx = abft.Context()
 A = abft.to_colmajor(torch.from_numpy(si.spd(1024, seed=3)).cuda())
-inj = [(2, abft.AT_PRE_PU, abft.KIND_ONCHIP, 0, 260, 130, 1 << 60),     # PU restart (gated redo)
+inj = [(2, abft.AT_PRE_PU, abft.KIND_ONCHIP, 0, 300, 270, 1 << 60),     # L_kk read by the PU: 2D, gated restart
        (4, abft.AT_POST_TMU, abft.KIND_PERSIST, 0, 900, 700, 1 << 59)]  # trailing 0D fix
 rc, info, st = abft.ft_potrf(ctx, A, 128, inject=inj)
 torch.cuda.synchronize()
