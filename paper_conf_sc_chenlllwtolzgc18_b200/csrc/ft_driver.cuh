@@ -67,6 +67,7 @@ struct ft_ctx {
   size_t hstage_bytes = 0;
   void* dguard = nullptr;  // device transfer guard
   size_t dguard_bytes = 0;
+  cudaEvent_t hchunk[4] = {};  // D2H chunk arrivals (the host checks a chunk while the next is in flight)
 };
 
 namespace abft {

@@ -145,20 +145,22 @@ int locate_ratio(double de, double dw, double te, double tw, int64_t nb) {
   return (int)j - 1;
 }
 
-// Line 4 (host check of the received panel, in place).  Returns 1 if every
-// flagged column was located and corrected, 0 if the panel must be fetched
-// again; accumulates flagged columns / fixed elements.
+// Line 4 (host check of the received panel, in place) over the nb-row tiles
+// [I0, I1).  Returns 1 if every flagged column was located and corrected, 0
+// if the panel must be fetched again; accumulates flagged columns / fixed
+// elements.
 template <typename T>
-int host_check(T* P, int64_t rows, int64_t nb, int64_t w, const T* G, int* flagged, int* fixed) {
+int host_check(T* P, int64_t rows, int64_t nb, int64_t w, const T* G, int64_t I0, int64_t I1, int* flagged,
+               int* fixed) {
   const int64_t mt = rows / nb;
   const double gam = (double)nb * Prec<T>::u / (1.0 - (double)nb * Prec<T>::u);
   std::vector<int> fl_c(w, 0), fx_c(w, 0), ok_c(w, 1);
-  parallel_cols(w, rows, [&](int64_t j0, int64_t j1) {
+  parallel_cols(w, (I1 - I0) * nb, [&](int64_t j0, int64_t j1) {
   for (int64_t j = j0; j < j1; ++j) {
     int& fl = fl_c[j];
     int& fx = fx_c[j];
     int& ok = ok_c[j];
-    for (int64_t I = 0; I < mt; ++I) {
+    for (int64_t I = I0; I < I1; ++I) {
       T* x = P + I * nb + j * rows;
       const double ge = (double)G[2 * I + j * 2 * mt], gw = (double)G[2 * I + 1 + j * 2 * mt];
       ColResid r = col_resid(x, nb, ge, gw, gam);
@@ -282,30 +284,53 @@ static int host_pd_t(Driver& d, int k, int kind, int64_t row0, int64_t col0, int
     return v;
   };
 
-  // lines 3-4: guarded D2H + host check
+  // lines 3-4: guarded D2H + host check.  The panel comes over in up to
+  // four tile-row chunks; the host checks each chunk as soon as it has
+  // arrived, so the check overlaps the rest of the copy.
   if (ft) FT_TRY(abft_encode(&P, &all, ABFT_COL, as));
   const auto d2h_faults = faults(FT_AT_D2H);
-  for (int attempt = 0; attempt < 3; ++attempt) {
-    ABFT_CUDA_TRY(cudaMemcpy2DAsync(hp, rows * es, panel, d.lda * es, rows * es, nb, cudaMemcpyDeviceToHost, s));
-    if (ft) ABFT_CUDA_TRY(cudaMemcpyAsync(hg, c->dguard, (size_t)2 * mt * nb * es, cudaMemcpyDeviceToHost, s));
-    ABFT_CUDA_TRY(cudaStreamSynchronize(s));
-    if (attempt == 0)
-      for (auto& f : d2h_faults) {
-        T* e = hp + (f.gi - row0) + (f.gj - col0) * rows;
-        if (sizeof(T) == 8) {
-          uint64_t b;
-          memcpy(&b, e, 8);
-          b ^= f.xor_mask;
-          memcpy(e, &b, 8);
-        } else {
-          uint32_t b;
-          memcpy(&b, e, 4);
-          b ^= (uint32_t)f.xor_mask;
-          memcpy(e, &b, 4);
-        }
+  const int nch = ft ? (int)std::min<int64_t>(4, mt) : 1;
+  for (int ch = 0; ch < nch; ++ch)
+    if (!c->hchunk[ch]) ABFT_CUDA_TRY(cudaEventCreateWithFlags(&c->hchunk[ch], cudaEventDisableTiming));
+  auto inject_d2h = [&](int64_t r0, int64_t r1) {  // faults in panel rows [r0, r1)
+    for (auto& f : d2h_faults) {
+      if (f.gi - row0 < r0 || f.gi - row0 >= r1) continue;
+      T* e = hp + (f.gi - row0) + (f.gj - col0) * rows;
+      if (sizeof(T) == 8) {
+        uint64_t b;
+        memcpy(&b, e, 8);
+        b ^= f.xor_mask;
+        memcpy(e, &b, 8);
+      } else {
+        uint32_t b;
+        memcpy(&b, e, 4);
+        b ^= (uint32_t)f.xor_mask;
+        memcpy(e, &b, 4);
       }
-    if (!ft) break;
-    if (host_check<T>(hp, rows, nb, nb, hg, &d.xs[0], &d.xs[1])) break;
+    }
+  };
+  for (int attempt = 0; attempt < 3; ++attempt) {
+    if (!ft) {
+      ABFT_CUDA_TRY(cudaMemcpy2DAsync(hp, rows * es, panel, d.lda * es, rows * es, nb, cudaMemcpyDeviceToHost, s));
+      ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+      if (attempt == 0) inject_d2h(0, rows);
+      break;
+    }
+    ABFT_CUDA_TRY(cudaMemcpyAsync(hg, c->dguard, (size_t)2 * mt * nb * es, cudaMemcpyDeviceToHost, s));
+    for (int ch = 0; ch < nch; ++ch) {
+      const int64_t I0 = mt * ch / nch, I1 = mt * (ch + 1) / nch;
+      ABFT_CUDA_TRY(cudaMemcpy2DAsync(hp + I0 * nb, rows * es, panel + I0 * nb, d.lda * es, (I1 - I0) * nb * es, nb,
+                                      cudaMemcpyDeviceToHost, s));
+      ABFT_CUDA_TRY(cudaEventRecord(c->hchunk[ch], s));
+    }
+    int ok = 1;
+    for (int ch = 0; ch < nch; ++ch) {
+      const int64_t I0 = mt * ch / nch, I1 = mt * (ch + 1) / nch;
+      ABFT_CUDA_TRY(cudaEventSynchronize(c->hchunk[ch]));
+      if (attempt == 0) inject_d2h(I0 * nb, I1 * nb);
+      ok &= host_check<T>(hp, rows, nb, nb, hg, I0, I1, &d.xs[0], &d.xs[1]);
+    }
+    if (ok) break;
     if (attempt < 2) {
       ++d.xs[2];
     } else {
@@ -334,11 +359,10 @@ static int host_pd_t(Driver& d, int k, int kind, int64_t row0, int64_t col0, int
     }
   }
   hcnt[8] = info > 0 ? info : 0;
-  const auto t2 = std::chrono::steady_clock::now();
-  if (ft) host_guard<T>(hp, rows, nb, nb, hg);
-  const auto t3 = std::chrono::steady_clock::now();
+  auto t2 = std::chrono::steady_clock::now(), t3 = t2;
 
-  // lines 6-7: guarded H2D + device check
+  // lines 6-7: guarded H2D + device check.  The panel goes out first and the
+  // host encodes its guard while the DMA reads the same pinned buffer.
   const auto h2d_faults = faults(FT_AT_H2D);
   for (int attempt = 0; attempt < 3; ++attempt) {
     ABFT_CUDA_TRY(cudaMemcpy2DAsync(panel, d.lda * es, hp, rows * es, rows * es, nb, cudaMemcpyHostToDevice, s));
@@ -349,6 +373,11 @@ static int host_pd_t(Driver& d, int k, int kind, int64_t row0, int64_t col0, int
       for (auto& f : h2d_faults) FT_TRY(d.inject_at_elem(f));
     }
     if (!ft) break;
+    if (attempt == 0) {
+      t2 = std::chrono::steady_clock::now();
+      host_guard<T>(hp, rows, nb, nb, hg);
+      t3 = std::chrono::steady_clock::now();
+    }
     ABFT_CUDA_TRY(cudaMemcpyAsync(c->dguard, hg, (size_t)2 * mt * nb * es, cudaMemcpyHostToDevice, s));
     ABFT_CUDA_TRY(cudaMemsetAsync(d.xcounts, 0, 8 * sizeof(int32_t), s));
     ABFT_CUDA_TRY(cudaMemcpyAsync(d.mark2, d.nfix, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));

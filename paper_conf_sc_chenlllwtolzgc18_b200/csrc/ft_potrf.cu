@@ -218,6 +218,8 @@ extern "C" int ft_ctx_destroy(ft_ctx_t* c) {
   }
   if (c->hstage) cudaFreeHost(c->hstage);
   if (c->dguard) cudaFree(c->dguard);
+  for (cudaEvent_t e : c->hchunk)
+    if (e) cudaEventDestroy(e);
   if (c->lapack) dlclose(c->lapack);
   delete c;
   return 0;

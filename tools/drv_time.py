@@ -1,7 +1,8 @@
 """Quick driver timing (CUDA events, median of reps): ft_* with ABFT (with and
 without local restart) vs the same driver unprotected, plus the cuSOLVER
 factorization as context.  Usage:
-  python tools/drv_time.py potrf|getrf|geqrf N NB [REPS]"""
+  python tools/drv_time.py potrf|getrf|geqrf N NB [REPS] [host]
+("host": the panel decomposition on the host LAPACK, FT_PD_HOST)"""
 import os
 import sys
 
@@ -13,9 +14,14 @@ from paper_conf_sc_chenlllwtolzgc18_b200 import abft
 
 which, n, nb = sys.argv[1], int(sys.argv[2]), int(sys.argv[3])
 reps = int(sys.argv[4]) if len(sys.argv) > 4 else 3
+host = len(sys.argv) > 5 and sys.argv[5] == "host"
 A0 = si.spd_device(n, seed=7) if which == "potrf" else si.general_device(n, seed=11)
 A = torch.empty_like(A0.t()).t()
 ctx = abft.Context()
+kw = {}
+if host:
+    ctx.set_host_lapack()
+    kw = {"pd_location": abft.PD_HOST}
 ipiv = torch.zeros(n, dtype=torch.int64, device="cuda")
 tau = torch.zeros(n, dtype=torch.float64, device="cuda")
 
@@ -26,11 +32,11 @@ def run(ft, restart=True, la=True):
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     a.record()
     if which == "potrf":
-        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart, lookahead=la)
+        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=ft, restart=restart, lookahead=la, **kw)
     elif which == "getrf":
-        rc, info, st = abft.ft_getrf(ctx, A, nb, ipiv, abft=ft, restart=restart)
+        rc, info, st = abft.ft_getrf(ctx, A, nb, ipiv, abft=ft, restart=restart, **kw)
     else:
-        rc, info, st = abft.ft_geqrf(ctx, A, nb, tau, abft=ft, restart=restart)
+        rc, info, st = abft.ft_geqrf(ctx, A, nb, tau, abft=ft, restart=restart, **kw)
     b.record()
     torch.cuda.synchronize()
     assert rc == 0 and info == 0 and sum(st.counts) == 0, (rc, info, list(st.counts))
@@ -65,10 +71,10 @@ def tl():
 
 
 cus = med(tl)
-print(f"{which} n={n} nb={nb}: plain {plain:.2f} ms, ft {ft:.2f} ms ({100 * (ft - plain) / plain:.2f}%), "
+print(f"{which}{' host-PD' if host else ''} n={n} nb={nb}: plain {plain:.2f} ms, ft {ft:.2f} ms ({100 * (ft - plain) / plain:.2f}%), "
       f"ft no-restart {nors:.2f} ms ({100 * (nors - plain) / plain:.2f}%), cusolver {cus:.2f} ms "
       f"(ft vs cusolver {100 * (ft - cus) / cus:.2f}%)", flush=True)
-if which == "potrf":
+if which == "potrf" and not host:
     A.copy_(A0)
     rc, info, st = abft.ft_potrf(ctx, A, nb, timing=True)
     torch.cuda.synchronize()
