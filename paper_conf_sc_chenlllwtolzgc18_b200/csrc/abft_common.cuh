@@ -146,6 +146,11 @@ int gemm_gated(int32_t dtype, bool ta, bool tb, bool absa, bool absb, int64_t M,
 // (abft_update.cu).
 int panel_row_rule(int32_t dtype, int64_t rows, int64_t nb, const void* L, int64_t ldl, const void* ce, const void* cw,
                    int64_t ldc, const void* mc, int64_t ldcm, void* re, void* rw, void* rm, cudaStream_t s);
+// fp64 Cholesky TMU checksum rule in one DMMA kernel (abft_rule_dmma.cu);
+// ABFT_E_UNSUPPORTED when nb % 32 != 0
+int update_syrk_dmma(int64_t nb, int64_t ntk, const double* L21, int64_t ldl, const double* cL, int64_t ldc,
+                     const double* mL, int64_t ldcm, double* Cc, double* Rr, int64_t ldr, double* Cm, double* Rm,
+                     int64_t ldrm, cudaStream_t s);
 // Free the per-stream pools (workspace, counters: abft_runtime.cu) and the
 // per-stream library handles and scratch (abft_update.cu) of a stream that is
 // about to be destroyed.  The stream must be idle.

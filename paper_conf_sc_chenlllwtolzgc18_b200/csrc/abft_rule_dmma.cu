@@ -1,0 +1,239 @@
+// abft_rule_dmma.cu — the Cholesky TMU checksum rule (c-12, L189; c-6) for
+// fp64 as ONE kernel on the FP64 tensor cores (DMMA, mma.sync m8n8k4).
+//
+// The rule of abft_update_syrk (abft_update.cu) for the trailing sub-problem
+// of ntk tile rows, nk = ntk * nb rows of L21:
+//   P = c(L21) L21^T   (M2 = 2 ntk rows:  c_e, c_w of every panel tile)
+//   Q = m_c(L21) |L21|^T (ntk rows: the magnitude row of every panel tile)
+//   c(A_IJ) -= P[2I.., cols of J],  r(A_IJ) -= P[2J.., cols of I]^T  (I >= J)
+//   m_c(A_IJ) += Q[I, cols of J],   m_r(A_IJ) += Q[J, cols of I]^T
+// The cuBLAS route materialises |L21| (abs_copy), runs two DGEMMs into a
+// scratch P / Q and scatters both (4 extra passes over L21-sized or P-sized
+// data, 5 launches).  Here A = [c(L21); m_c(L21)] (Mt = 3 ntk rows, padded)
+// times L21^T is ONE tiled product: the B fragment serves the checksum rows
+// as b and the magnitude rows as |b|, and the accumulators are scattered
+// straight into the four arrays (one writer per element: a fire-and-forget
+// reduction, no P / Q scratch).
+//
+// Tiling (the shape cuBLAS picks for these skinny products): CTA tile 64
+// rows of A x 32 columns, 4 warps of 32 x 16 (4 x 2 DMMA tiles), K = nb in
+// 16-deep stages through a 4-stage cp.async ring (53 KB: 4 CTAs per SM);
+// grid (Mt / 64, nk / 32), row tiles fastest so the CTAs that share an L21
+// slice run together.  Summation order: one fixed DMMA chain per output
+// element over k ascending (deterministic; not the cuBLAS order, so P and Q
+// agree with the GEMM route to rounding, well inside the checks' tau).
+#include <algorithm>
+
+#include "abft_common.cuh"
+
+namespace abft {
+namespace {
+
+constexpr int kTM = 64;       // rows of A per CTA
+constexpr int kTN = 32;       // columns per CTA
+constexpr int kBK = 16;       // k per stage
+constexpr int kStages = 4;
+constexpr int kThr = 128;     // 4 warps: 2 (m, 32 rows) x 2 (n, 16 columns)
+constexpr int kWM = 4;        // m-tiles per warp
+constexpr int kWN = 2;        // n-tiles per warp
+constexpr int kLdA = kTM + 4;  // row stride = 4 (mod 16 doubles): conflict-free fragments
+constexpr int kLdB = kTN + 4;
+constexpr size_t kRuleSmem = (size_t)kStages * kBK * (kLdA + kLdB) * sizeof(double);
+
+struct RuleArgs {
+  const double* L;  // L21, nk x nb, ld ldl
+  int64_t ldl;
+  const double* cL;  // c(L21): M2 x nb, ld ldc
+  int64_t ldc;
+  const double* mL;  // m_c(L21): ntk x nb, ld ldcm (nullable: no Q)
+  int64_t ldcm;
+  double* Cc;  // c of the trailing tiles, ld ldc
+  double* Rr;  // r, ld ldr (nullable)
+  int64_t ldr;
+  double* Cm;  // m_c, ld ldcm (nullable)
+  double* Rm;  // m_r, ld ldrm (nullable)
+  int64_t ldrm;
+  int ntk;
+  int nb;
+  int M2p;  // checksum rows padded to 8 (magnitude rows start here)
+};
+
+__device__ __forceinline__ void cp_async8(void* smem, const void* gmem, bool valid) {
+  // src-size 0: the 8 bytes are zero-filled (padding rows of A)
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(smem_u32(smem)), "l"(gmem),
+               "r"(valid ? 8 : 0)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+
+__device__ __forceinline__ void dmma(double (&d)[2], double a, double b) {
+  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+               : "+d"(d[0]), "+d"(d[1])
+               : "d"(a), "d"(b));
+}
+
+// One stage of the warp's kWM x kWN DMMA tiles: m-tiles a < AQ take b
+// (checksum rows), a >= AQ take |b| (magnitude rows).
+template <int AQ>
+__device__ __forceinline__ void stage_mma(double (&acc)[kWM][kWN][2], const double* as, const double* bs, int t) {
+#pragma unroll
+  for (int k4 = 0; k4 < kBK; k4 += 4) {
+    double bf[kWN], ba[kWN];
+#pragma unroll
+    for (int n = 0; n < kWN; ++n) {
+      bf[n] = bs[(k4 + t) * kLdB + n * 8];
+      if constexpr (AQ < kWM) ba[n] = fabs(bf[n]);
+    }
+#pragma unroll
+    for (int a = 0; a < kWM; ++a) {
+      const double af = as[(k4 + t) * kLdA + a * 8];
+#pragma unroll
+      for (int n = 0; n < kWN; ++n) {
+        if constexpr (AQ < kWM) {
+          if (a >= AQ) {
+            dmma(acc[a][n], af, ba[n]);
+            continue;
+          }
+        }
+        dmma(acc[a][n], af, bf[n]);
+      }
+    }
+  }
+}
+
+__global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
+  extern __shared__ __align__(16) double sm[];
+  double* As = sm;                                 // [kStages][kBK][kLdA]
+  double* Bs = sm + (size_t)kStages * kBK * kLdA;  // [kStages][kBK][kLdB]
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int wm = warp & 1, wn = warp >> 1;
+  const int g = lane >> 2, t = lane & 3;
+  const int r0 = blockIdx.x * kTM;                // first row of A
+  const int x0 = blockIdx.y * kTN;                // first column (row of L21)
+  const int ksteps = p.nb / kBK;
+  const int M2 = 2 * p.ntk;
+  // fill roles (fixed for the CTA): A row ra (k parity by half), L21 column cb
+  const int ra = tid % kTM, ka = tid / kTM;       // 2 threads per row: k = ka, ka + 2, ...
+  const int ya = r0 + ra, yqa = ya - p.M2p;
+  const bool isp = ya < M2, isq = p.mL && yqa >= 0 && yqa < p.ntk;
+  const double* srcA = isp ? p.cL + ya : (isq ? p.mL + yqa : p.cL);
+  const int64_t ldA = isp ? p.ldc : (isq ? p.ldcm : 0);
+  const int cb = tid % kTN, kbq = tid / kTN;      // 4 threads per column: k = kbq, kbq + 4, ...
+  const double* srcB = p.L + x0 + cb;
+  auto fill = [&](int kt, int st) {
+    const int64_t kb = (int64_t)kt * kBK;
+    double* as = As + (size_t)st * kBK * kLdA + ra;
+#pragma unroll
+    for (int kk = ka; kk < kBK; kk += kThr / kTM) cp_async8(as + kk * kLdA, srcA + (kb + kk) * ldA, isp || isq);
+    double* bs = Bs + (size_t)st * kBK * kLdB + cb;
+#pragma unroll
+    for (int kk = kbq; kk < kBK; kk += kThr / kTN) cp_async8(bs + kk * kLdB, srcB + (kb + kk) * p.ldl, true);
+  };
+#pragma unroll
+  for (int s = 0; s < kStages - 1; ++s) {
+    if (s < ksteps) fill(s, s);
+    cp_async_commit();
+  }
+  double acc[kWM][kWN][2];
+#pragma unroll
+  for (int a = 0; a < kWM; ++a)
+#pragma unroll
+    for (int n = 0; n < kWN; ++n) acc[a][n][0] = acc[a][n][1] = 0.0;
+  // this warp's m-tiles (rows r0 + 32 wm + 8a): checksum rows below aq,
+  // magnitude rows from aq on
+  const int wr0 = r0 + wm * 32;
+  const int aq = min(kWM, max(0, (p.M2p - wr0) / 8));
+  for (int kt = 0; kt < ksteps; ++kt) {
+    cp_async_wait<kStages - 2>();
+    __syncthreads();
+    const int nx = kt + kStages - 1;
+    if (nx < ksteps) fill(nx, nx % kStages);
+    cp_async_commit();
+    const double* as = As + (size_t)(kt % kStages) * kBK * kLdA + wm * 32 + g;
+    const double* bs = Bs + (size_t)(kt % kStages) * kBK * kLdB + wn * 16 + g;
+    switch (aq) {  // warp-uniform
+      case 0: stage_mma<0>(acc, as, bs, t); break;
+      case 1: stage_mma<1>(acc, as, bs, t); break;
+      case 2: stage_mma<2>(acc, as, bs, t); break;
+      case 3: stage_mma<3>(acc, as, bs, t); break;
+      default: stage_mma<4>(acc, as, bs, t); break;
+    }
+  }
+  cp_async_wait<0>();
+  // scatter: lane holds P/Q[y][x], [y][x+1] with y = wr0 + 8a + g,
+  // x = x0 + 16 wn + 8n + 2t.  The 32 columns meet at most one tile-column
+  // boundary (nb >= 32): J = J0 + (x - x0 >= bnd).  One writer per element:
+  // a reduction adds exactly what load + add + store would.
+  const int J0 = x0 / p.nb, bnd = (J0 + 1) * p.nb - x0;
+#pragma unroll
+  for (int a = 0; a < kWM; ++a) {
+    const int y = wr0 + a * 8 + g;
+    const bool q = a >= aq;
+    const int yq = y - p.M2p;
+    if (!q && y >= M2) continue;
+    if (q && (!p.Cm || yq >= p.ntk)) continue;
+    const int I = q ? yq : y / 2;
+    double* Cp = q ? p.Cm + yq : p.Cc + y;  // + x * ldC
+    double* Rp = q ? p.Rm : p.Rr;           // + x + row * ldR
+    const int64_t ldC = q ? p.ldcm : p.ldc;
+    const int64_t rowR = (int64_t)(q ? yq : y) * (q ? p.ldrm : p.ldr);
+    const double sgn = q ? 1.0 : -1.0;
+#pragma unroll
+    for (int n = 0; n < kWN; ++n)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int xx = wn * 16 + n * 8 + 2 * t + h;
+        const int J = J0 + (xx >= bnd);
+        const double v = sgn * acc[a][n][h];
+        if (I >= J) atomicAdd(Cp + (int64_t)(x0 + xx) * ldC, v);
+        if (Rp && J >= I) atomicAdd(Rp + (x0 + xx) + rowR, v);
+      }
+  }
+}
+
+}  // namespace
+
+// Returns ABFT_E_UNSUPPORTED when the shape is not covered (the caller takes
+// the cuBLAS route): nb must be a multiple of 32.
+int update_syrk_dmma(int64_t nb, int64_t ntk, const double* L21, int64_t ldl, const double* cL, int64_t ldc,
+                     const double* mL, int64_t ldcm, double* Cc, double* Rr, int64_t ldr, double* Cm, double* Rm,
+                     int64_t ldrm, cudaStream_t s) {
+  if (nb % kTN || nb <= 0) return ABFT_E_UNSUPPORTED;
+  const int64_t nk = ntk * nb;
+  if (nk == 0) return 0;
+  if (nk > (1LL << 30)) return ABFT_E_UNSUPPORTED;  // 32-bit column indices inside the kernel
+  static bool attr = false;
+  if (!attr) {
+    ABFT_CUDA_TRY(cudaFuncSetAttribute(syrk_rule_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)kRuleSmem));
+    attr = true;
+  }
+  RuleArgs a{};
+  a.L = L21;
+  a.ldl = ldl;
+  a.cL = cL;
+  a.ldc = ldc;
+  const bool mags = mL && Cm;
+  a.mL = mags ? mL : nullptr;
+  a.ldcm = ldcm;
+  a.Cc = Cc;
+  a.Rr = Rr;
+  a.ldr = ldr;
+  a.Cm = mags ? Cm : nullptr;
+  a.Rm = mags ? Rm : nullptr;
+  a.ldrm = ldrm;
+  a.ntk = (int)ntk;
+  a.nb = (int)nb;
+  a.M2p = (int)((2 * ntk + 7) / 8 * 8);
+  const int64_t Mt = a.M2p + (mags ? (ntk + 7) / 8 * 8 : 0);
+  const dim3 grid((unsigned)((Mt + kTM - 1) / kTM), (unsigned)(nk / kTN));
+  syrk_rule_dmma_kernel<<<grid, kThr, kRuleSmem, s>>>(a);
+  ABFT_CUDA_TRY(cudaGetLastError());
+  return 0;
+}
+
+}  // namespace abft

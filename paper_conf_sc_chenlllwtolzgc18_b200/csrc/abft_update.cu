@@ -457,6 +457,15 @@ int update_syrk_t(int64_t nb, int64_t ntk, const T* L21, int64_t ldl, const T* c
                   int64_t ldcm, T* Cc, T* Rr, int64_t ldr, T* Cm, T* Rm, int64_t ldrm, cudaStream_t s) {
   const int64_t nk = ntk * nb, M2 = 2 * ntk;
   if (nk == 0) return 0;
+  if constexpr (sizeof(T) == 8) {
+    // fp64: one fused DMMA kernel (abft_rule_dmma.cu); ABFT_RULE_CUBLAS=1 keeps
+    // the GEMM route below (A/B measurements)
+    static const bool gemm_route = getenv("ABFT_RULE_CUBLAS") != nullptr;
+    if (!gemm_route) {
+      const int r = update_syrk_dmma(nb, ntk, L21, ldl, cL, ldc, mL, ldcm, Cc, Rr, ldr, Cm, Rm, ldrm, s);
+      if (r != ABFT_E_UNSUPPORTED) return r;
+    }
+  }
   void* pv = nullptr;
   int rc = scratch_get(s, 7, (size_t)M2 * nk * sizeof(T), &pv);
   if (rc) return rc;
@@ -542,25 +551,44 @@ int update_gemm_t(int which, char transX, char transY, double alpha, const void*
 //   m_r(x) += sum_q |L[x,q]| m_c(L_J0)[q]            (c-6)
 // in ONE pass over L (the GEMM route needs |L| materialised first).  A block
 // owns 32 rows; its 8 warps split the nb columns and their partials are
-// added in warp order (deterministic).
+// added in warp order (deterministic).  Memory-latency bound at the panel
+// sizes of late iterations: each lane keeps 16 column loads in flight (one
+// load at a time ran 36 us per launch whatever the panel height, ncu r02a).
 template <typename T>
 __global__ void __launch_bounds__(256) panel_row_rule_kernel(int64_t rows, int nb, const T* __restrict__ L, int64_t ldl,
                                                              const T* __restrict__ ce, const T* __restrict__ cw,
                                                              int64_t ldc, const T* __restrict__ mc, int64_t ldcm,
                                                              T* __restrict__ re, T* __restrict__ rw,
                                                              T* __restrict__ rm) {
+  // the tile column's checksum vectors, staged once per block
+  __shared__ T sv[3][1024];
   __shared__ T part[8][3][32];
+  for (int q = threadIdx.x; q < nb; q += blockDim.x) {
+    sv[0][q] = ce[(int64_t)q * ldc];
+    sv[1][q] = cw[(int64_t)q * ldc];
+    sv[2][q] = mc ? mc[(int64_t)q * ldcm] : T(0);
+  }
+  __syncthreads();
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int64_t x = (int64_t)blockIdx.x * 32 + lane;
   const int qn = nb / 8, q0 = warp * qn;
   T se = T(0), sw = T(0), sm = T(0);
   if (x < rows) {
-#pragma unroll 8
-    for (int q = q0; q < q0 + qn; ++q) {
-      const T l = L[x + (int64_t)q * ldl];
-      se = fma(l, ce[(int64_t)q * ldc], se);
-      sw = fma(l, cw[(int64_t)q * ldc], sw);
-      sm = fma(fabs(l), mc ? mc[(int64_t)q * ldcm] : T(0), sm);
+    // 16 independent column loads in flight per lane, then the same
+    // sequential fma chain as one column at a time
+    const T* Lx = L + x + (int64_t)q0 * ldl;
+    for (int q = 0; q < qn; q += 16) {
+      T l[16];
+#pragma unroll
+      for (int u = 0; u < 16; ++u) l[u] = q + u < qn ? __ldg(Lx + (int64_t)(q + u) * ldl) : T(0);
+#pragma unroll
+      for (int u = 0; u < 16; ++u) {
+        if (q + u < qn) {
+          se = fma(l[u], sv[0][q0 + q + u], se);
+          sw = fma(l[u], sv[1][q0 + q + u], sw);
+          sm = fma(fabs(l[u]), sv[2][q0 + q + u], sm);
+        }
+      }
     }
   }
   part[warp][0][lane] = se;
@@ -584,7 +612,7 @@ __global__ void __launch_bounds__(256) panel_row_rule_kernel(int64_t rows, int n
 int panel_row_rule(int32_t dtype, int64_t rows, int64_t nb, const void* L, int64_t ldl, const void* ce, const void* cw,
                    int64_t ldc, const void* mc, int64_t ldcm, void* re, void* rw, void* rm, cudaStream_t s) {
   if (rows <= 0) return 0;
-  if (nb % 8) return ABFT_E_UNSUPPORTED;
+  if (nb % 8 || nb > 1024) return ABFT_E_UNSUPPORTED;
   const unsigned grid = (unsigned)((rows + 31) / 32);
   if (dtype == ABFT_F64)
     panel_row_rule_kernel<double><<<grid, 256, 0, s>>>(rows, (int)nb, (const double*)L, ldl, (const double*)ce,

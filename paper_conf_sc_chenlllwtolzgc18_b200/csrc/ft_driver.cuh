@@ -187,6 +187,15 @@ struct Driver {
     cudaEvent_t a, b;
   };
   std::vector<Span> spans;
+  // ABFT_ITER_EVENTS=1 (diagnostics): an event on the main stream at each
+  // iteration start; per-iteration ms printed to stderr by finish()
+  std::vector<cudaEvent_t> iter_ev;
+  void iter_event() {
+    static const bool on = getenv("ABFT_ITER_EVENTS") != nullptr;
+    if (!on) return;
+    cudaEvent_t e = ev_take();
+    if (e && cudaEventRecord(e, s_main) == cudaSuccess) iter_ev.push_back(e);
+  }
   size_t ev_used = 0;
   cudaEvent_t ev_take() {
     if (ev_used == c->evpool.size()) {
@@ -463,6 +472,15 @@ struct Driver {
     ABFT_CUDA_TRY(cudaStreamWaitEvent(c->stream, c->join, 0));
     ABFT_CUDA_TRY(cudaStreamSynchronize(s));
     auto t1 = std::chrono::steady_clock::now();
+    if (iter_ev.size() > 1) {
+      fprintf(stderr, "[abft] iteration ms:");
+      for (size_t i = 1; i < iter_ev.size(); ++i) {
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, iter_ev[i - 1], iter_ev[i]);
+        fprintf(stderr, " %.3f", ms);
+      }
+      fprintf(stderr, "\n");
+    }
     // layout after counts: nfix(8) mark(9) info(10) rep(11,12) info_total(13); side counts at 32
     for (int i = 0; i < 8; ++i) h[i] += h[32 + i];
     if (info_out) *info_out = h[13];

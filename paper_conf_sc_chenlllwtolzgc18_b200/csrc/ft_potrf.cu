@@ -567,6 +567,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
 
   bool chained = false;  // iteration k's PD / PU already ran as look-ahead
   for (int k = 0; k < nt; ++k) {
+    d.iter_event();
     if (!chained) FT_TRY(chain(k, true));
     chained = false;
     if (k == nt - 1) break;
@@ -625,5 +626,6 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       FT_TRY(d.periodic_check(k, k + 1, (int)nt, k + 1, (int)nt, ABFT_SYM_LOWER, true));
     }
   }
+  d.iter_event();
   return d.finish(t0, stats, info_out);
 }

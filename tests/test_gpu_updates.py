@@ -86,25 +86,36 @@ def test_panel_potrf_matches_oracle_rule(lib):
     assert np.abs(host(Linv) - np.linalg.inv(L)).max() <= 1e-12 * np.abs(np.linalg.inv(L)).max()
 
 
-def test_update_syrk_matches_oracle_rule(lib):
-    n, nb, k = 768, 128, 0
+# fp64 runs the fused DMMA kernel (abft_rule_dmma.cu): one 192-row chunk of
+# checksum rows (768/128), two chunks (2240/32: 69 tile rows -> 216 rows),
+# the metric's nb (2048/512), a later iteration, and nb=16 (cuBLAS route)
+@pytest.mark.parametrize("n,nb,k", [(768, 128, 0), (2240, 32, 0), (2048, 512, 0), (1536, 256, 2), (512, 16, 1)])
+@pytest.mark.parametrize("rows", [True, False])
+def test_update_syrk_matches_oracle_rule(lib, n, nb, k, rows):
     st = _chol_state(n, nb)
     up.chol_pd_rule(st, k)
     up.chol_pu_data(st, k)
     up.chol_pu_chk(st, k)
     mat = lib.Mat(dev(st.A), nb, dev(st.colchk), dev(st.rowchk), dev(st.colmag), dev(st.rowmag))
+    row_before = host(mat.rowchk).copy(), host(mat.rowmag).copy()
     up.chol_tmu_chk(st, k)  # the oracle's checksum step of the TMU
     r1, ntk = (k + 1) * nb, n // nb - k - 1
-    lib.abft_update_syrk(nb, ntk, mat.A[r1:, k * nb:r1], mat.colchk[2:, k * nb:r1], mat.colchk[2:, r1:],
-                         mat.rowchk[r1:, 2:], mat.colmag[1:, k * nb:r1], mat.colmag[1:, r1:], mat.rowmag[r1:, 1:])
+    k2, k1 = 2 * (k + 1), k + 1
+    lib.abft_update_syrk(nb, ntk, mat.A[r1:, k * nb:r1], mat.colchk[k2:, k * nb:r1], mat.colchk[k2:, r1:],
+                         mat.rowchk[r1:, k2:] if rows else None, mat.colmag[k1:, k * nb:r1], mat.colmag[k1:, r1:],
+                         mat.rowmag[r1:, k1:] if rows else None)
     torch.cuda.synchronize()
     g = gpu_state_to_oracle(mat)
     for I, J in ck.Tiles(k + 1, n // nb, k + 1, n // nb, True):
         cs, rs = slice(J * nb, (J + 1) * nb), slice(I * nb, (I + 1) * nb)
-        for a, b in [(g.colchk[2 * I:2 * I + 2, cs], st.colchk[2 * I:2 * I + 2, cs]),
-                     (g.rowchk[rs, 2 * J:2 * J + 2], st.rowchk[rs, 2 * J:2 * J + 2]),
-                     (g.colmag[I, cs], st.colmag[I, cs]), (g.rowmag[rs, J], st.rowmag[rs, J])]:
+        pairs = [(g.colchk[2 * I:2 * I + 2, cs], st.colchk[2 * I:2 * I + 2, cs]), (g.colmag[I, cs], st.colmag[I, cs])]
+        if rows:
+            pairs += [(g.rowchk[rs, 2 * J:2 * J + 2], st.rowchk[rs, 2 * J:2 * J + 2]),
+                      (g.rowmag[rs, J], st.rowmag[rs, J])]
+        for a, b in pairs:
             assert np.abs(a - b).max() <= 1e-12 * max(np.abs(b).max(), 1.0), (I, J)
+    if not rows:  # the single-checksum call leaves the row side alone
+        assert np.array_equal(host(mat.rowchk), row_before[0]) and np.array_equal(host(mat.rowmag), row_before[1])
 
 
 @pytest.mark.parametrize("nb", [32, 64, 128, 512, 1024])
