@@ -21,10 +21,12 @@ def _tri(nb, seed, lower=True, unit=False):
     return T
 
 
+# tile sizes from 32 to 1024, checksum-vector counts from 6 to the 118 of a
+# 60-tile panel
+@pytest.mark.parametrize("nb,nvec", [(64, 10), (512, 118), (1024, 6), (32, 10)])
 @pytest.mark.parametrize("side,uplo,trans,diag", [("R", "L", "T", "N"), ("L", "L", "N", "U"), ("L", "U", "N", "N"),
-                                                  ("R", "U", "N", "N")])
-def test_update_trsm_matches_solve(lib, side, uplo, trans, diag):
-    nb, nvec = 64, 10
+                                                  ("R", "U", "N", "N"), ("R", "L", "N", "N"), ("L", "U", "T", "N")])
+def test_update_trsm_matches_solve(lib, side, uplo, trans, diag, nb, nvec):
     T = _tri(nb, 1, uplo == "L", diag == "U")
     shape = (nvec, nb) if side == "R" else (nb, nvec)
     X = si.general(*shape, seed=2)
@@ -38,6 +40,21 @@ def test_update_trsm_matches_solve(lib, side, uplo, trans, diag):
     mref = M @ np.abs(Tinv) if side == "R" else np.abs(Tinv) @ M
     assert np.abs(host(Xd) - ref).max() <= 1e-12 * np.abs(ref).max()
     assert np.abs(host(Md) - mref).max() <= 1e-12 * np.abs(mref).max()
+
+
+@pytest.mark.parametrize("side,trans", [("R", "T"), ("L", "N")])
+def test_update_trsm_f32(lib, side, trans):
+    nb, nvec = 512, 40
+    T = _tri(nb, 4, True, False).astype(np.float32)
+    shape = (nvec, nb) if side == "R" else (nb, nvec)
+    X = si.general(*shape, seed=5).astype(np.float32)
+    Td, Xd = dev(T, torch.float32), dev(X, torch.float32)
+    lib.abft_update_trsm(side, "L", trans, "N", nb, Td, Xd, nvec)
+    torch.cuda.synchronize()
+    opT = T.astype(np.float64).T if trans == "T" else T.astype(np.float64)
+    Tinv = np.linalg.inv(opT)
+    ref = X @ Tinv if side == "R" else Tinv @ X
+    assert np.abs(host(Xd) - ref).max() <= 1e-4 * np.abs(ref).max()
 
 
 @pytest.mark.parametrize("which,tX,tY", [(1, "N", "T"), (2, "T", "N"), (1, "N", "N"), (2, "N", "N")])

@@ -37,3 +37,4 @@ for ntk in ntks:
     us = a.elapsed_time(b) / reps * 1e3
     flops = 2.0 * 3 * ntk * nk * nb
     print(f"{route} nb={nb} ntk={ntk}: {us:.1f} us  {flops / us / 1e6:.1f} TF/s", flush=True)
+
