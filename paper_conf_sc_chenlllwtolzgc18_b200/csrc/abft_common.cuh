@@ -150,7 +150,7 @@ int panel_row_rule(int32_t dtype, int64_t rows, int64_t nb, const void* L, int64
 // ABFT_E_UNSUPPORTED when nb % 32 != 0
 int update_syrk_dmma(int64_t nb, int64_t ntk, const double* L21, int64_t ldl, const double* cL, int64_t ldc,
                      const double* mL, int64_t ldcm, double* Cc, double* Rr, int64_t ldr, double* Cm, double* Rm,
-                     int64_t ldrm, cudaStream_t s);
+                     int64_t ldrm, cudaStream_t s, int64_t ntc = -1);
 // Free the per-stream pools (workspace, counters: abft_runtime.cu) and the
 // per-stream library handles and scratch (abft_update.cu) of a stream that is
 // about to be destroyed.  The stream must be idle.

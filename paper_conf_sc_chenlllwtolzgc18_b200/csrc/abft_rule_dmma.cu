@@ -198,12 +198,15 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
 }  // namespace
 
 // Returns ABFT_E_UNSUPPORTED when the shape is not covered (the caller takes
-// the cuBLAS route): nb must be a multiple of 32.
+// the cuBLAS route): nb must be a multiple of 32.  ntc < ntk restricts the
+// product to the first ntc tile columns (x < ntc nb; the look-ahead's single
+// tile column: ntc = 1 with Rr = Rm = null, c and m_c of every tile I >= J0).
 int update_syrk_dmma(int64_t nb, int64_t ntk, const double* L21, int64_t ldl, const double* cL, int64_t ldc,
                      const double* mL, int64_t ldcm, double* Cc, double* Rr, int64_t ldr, double* Cm, double* Rm,
-                     int64_t ldrm, cudaStream_t s) {
+                     int64_t ldrm, cudaStream_t s, int64_t ntc) {
   if (nb % kTN || nb <= 0) return ABFT_E_UNSUPPORTED;
-  const int64_t nk = ntk * nb;
+  if (ntc < 0) ntc = ntk;
+  const int64_t nk = ntc * nb;  // columns: the first ntc tiles of L21's rows
   if (nk == 0) return 0;
   if (nk > (1LL << 30)) return ABFT_E_UNSUPPORTED;  // 32-bit column indices inside the kernel
   static bool attr = false;

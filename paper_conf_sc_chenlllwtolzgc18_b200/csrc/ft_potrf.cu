@@ -520,9 +520,16 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     //   c(A_I,J0) -= c(L_Ik) L_J0,k^T,  m_c += m_c(L_Ik) |L_J0,k|^T
     //   r(A_I,J0) -= L_Ik c(L_J0,k)^T,  m_r += |L_Ik| m_c(L_J0,k)^T
     const int64_t m2 = 2 * (nt - J0);
-    FT_TRY(abft_update_gemm(dtype, ABFT_COL, 'N', 'T', -1.0, d.colchk_at(2 * J0, r0), d.M.ldc, d.a_at(c0, r0), lda,
+    int rc = ABFT_E_UNSUPPORTED;
+    if (dtype == ABFT_F64)  // the DMMA rule kernel restricted to this tile column (abft_rule_dmma.cu)
+      rc = update_syrk_dmma(nb, nt - J0, (const double*)d.a_at(c0, r0), lda, (const double*)d.colchk_at(2 * J0, r0),
+                            d.M.ldc, (const double*)d.colmag_at(J0, r0), d.M.ldcm, (double*)d.colchk_at(2 * J0, c0),
+                            nullptr, d.M.ldr, (double*)d.colmag_at(J0, c0), nullptr, d.M.ldrm, d.s, 1);
+    if (rc == ABFT_E_UNSUPPORTED)
+      rc = abft_update_gemm(dtype, ABFT_COL, 'N', 'T', -1.0, d.colchk_at(2 * J0, r0), d.M.ldc, d.a_at(c0, r0), lda,
                             d.colchk_at(2 * J0, c0), d.M.ldc, m2, nb, nb, d.colmag_at(J0, r0), d.M.ldcm,
-                            d.colmag_at(J0, c0), d.M.ldcm, as));
+                            d.colmag_at(J0, c0), d.M.ldcm, as);
+    FT_TRY(rc);
     if (single) return 0;
     return panel_row_rule(dtype, n - c0, nb, d.a_at(c0, r0), lda, d.colchk_at(2 * J0, r0), d.colchk_at(2 * J0 + 1, r0),
                           d.M.ldc, d.colmag_at(J0, r0), d.M.ldcm, d.rowchk_at(c0, 2 * J0),
