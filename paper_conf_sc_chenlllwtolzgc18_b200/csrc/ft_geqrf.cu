@@ -457,6 +457,7 @@ static int geqrf_driver(Driver& d, ft_ctx* c, T* tau_all) {
     FT_TRY(abft_encode(&d.M, &all, ABFT_BOTH, as));
   }
   for (int k = 0; k < nt; ++k) {
+    d.iter_event();
     const int64_t r0 = k * nb, r1 = r0 + nb, mk = n - r0, nk = n - r1;
     // Alg. 2 lines 3-4: check the column panel to be decomposed (c + r)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
@@ -603,5 +604,6 @@ extern "C" int ft_geqrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
   auto t0 = std::chrono::steady_clock::now();
   const int rc = dtype == ABFT_F64 ? geqrf_driver<double>(d, c, (double*)tau) : geqrf_driver<float>(d, c, (float*)tau);
   if (rc) return rc;
+  d.iter_event();
   return d.finish(t0, stats, info_out);
 }

@@ -881,6 +881,7 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
 
   bool chained = false;  // PD k already factored by the look-ahead (part 1)
   for (int k = 0; k < nt; ++k) {
+    d.iter_event();
     const int64_t r1 = (int64_t)(k + 1) * nb, r2 = r1 + nb;
     if (!chained)
       FT_TRY(chain_pd(k, false));
@@ -927,5 +928,6 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       FT_TRY(d.periodic_check(k, k + 1, (int)nt, k + 1, (int)nt, ABFT_GENERAL, false));  // L359
     }
   }
+  d.iter_event();
   return d.finish(t0, stats, info_out);
 }

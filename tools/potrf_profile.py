@@ -1,5 +1,6 @@
-"""Run ft_potrf once (ABFT on or off) for an ncu launch list; also prints host
-enqueue time vs device time.  Usage: python tools/potrf_profile.py N NB ABFT"""
+"""Run ft_potrf (or ft_getrf / ft_geqrf) once (ABFT on or off) for an ncu
+launch list; also prints host enqueue time vs device time.  Usage:
+  python tools/potrf_profile.py N NB ABFT [REPS [potrf|getrf|geqrf]]"""
 import os
 import sys
 import time
@@ -12,7 +13,10 @@ from paper_conf_sc_chenlllwtolzgc18_b200 import abft
 
 n, nb, ft = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3])
 reps = int(sys.argv[4]) if len(sys.argv) > 4 else 1
-A0 = si.spd_device(n, seed=7)
+which = sys.argv[5] if len(sys.argv) > 5 else "potrf"
+A0 = si.spd_device(n, seed=7) if which == "potrf" else si.general_device(n, seed=11)
+ipiv = torch.zeros(n, dtype=torch.int64, device="cuda")
+tau = torch.zeros(n, dtype=torch.float64, device="cuda")
 A = torch.empty_like(A0.t()).t()
 ctx = abft.Context()
 for r in range(reps):
@@ -21,7 +25,12 @@ for r in range(reps):
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     t0 = time.perf_counter()
     a.record()
-    rc, info, st = abft.ft_potrf(ctx, A, nb, abft=bool(ft))
+    if which == "potrf":
+        rc, info, st = abft.ft_potrf(ctx, A, nb, abft=bool(ft))
+    elif which == "getrf":
+        rc, info, st = abft.ft_getrf(ctx, A, nb, ipiv, abft=bool(ft))
+    else:
+        rc, info, st = abft.ft_geqrf(ctx, A, nb, tau, abft=bool(ft))
     b.record()
     torch.cuda.synchronize()
     t1 = time.perf_counter()
