@@ -15,6 +15,19 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
    python bench.py --steps 2 --warmup 1 --no-e2e --no-potrf --no-cpu --no-lu-qr --no-mgpu > $out/ncu_launch.log 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum,launch__grid_size --clock-control none -c 6000 --csv \
    --log-file $out/potrf30720_launches.csv python tools/potrf_profile.py 30720 512 1 > $out/potrf_prof.log 2>&1
+timeout 900 ncu --metrics gpu__time_duration.sum,launch__grid_size --clock-control none -c 6000 --csv \
+   --log-file $out/potrf30720_plain_launches.csv python tools/potrf_profile.py 30720 512 0 > $out/potrf_prof0.log 2>&1
+for ft in 0 1; do
+  timeout 900 ncu --metrics gpu__time_duration.sum,launch__grid_size --clock-control none -c 8000 --csv \
+     --log-file $out/getrf20480_ft${ft}_launches.csv python tools/potrf_profile.py 20480 512 $ft 1 getrf > /dev/null 2>&1
+done
+python tools/drv_time.py potrf 30720 512 3 > $out/drv_potrf.log 2>&1
+python tools/drv_time.py getrf 20480 512 3 > $out/drv_getrf.log 2>&1
+python tools/drv_time.py geqrf 20480 512 3 > $out/drv_geqrf.log 2>&1
+python tools/drv_time.py getrf 20480 512 3 host > $out/drv_getrf_host.log 2>&1
+python tools/rule_time.py > $out/rule_time.log 2>&1
+ABFT_RULE_CUBLAS=1 python tools/rule_time.py >> $out/rule_time.log 2>&1
+ABFT_ITER_EVENTS=1 python tools/iter_time.py 30720 512 potrf 2> $out/iter_potrf.log
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:checksum_pass -s 2 -c 2 \
    -o $out/prof_pass -f python bench.py --steps 1 --warmup 1 --no-e2e --no-potrf --no-cpu --no-lu-qr --no-mgpu \
    > $out/ncu_full.log 2>&1

@@ -1,7 +1,8 @@
 """Tiny workloads for compute-sanitizer (racecheck / synccheck / memcheck)
 of the pass (encode / verify, every launch shape: RECT, SEG, DIAG, slabbed
 tiles) and locate kernels, plus one small ft_potrf with faults (gated
-restart, Fig. 4a repair, look-ahead side stream).
+restart, Fig. 4a repair, look-ahead side stream, the DMMA TMU rule kernel,
+the panel row rule).
   compute-sanitizer --tool racecheck python tools/sanitize_small.py"""
 import os
 import sys
