@@ -1,8 +1,8 @@
 #!/bin/bash
 # Round evidence (run under gpurun from the repo root): smoke, every GPU
 # test, the N=1 bench line, the ncu launch list of the bench step and of one
-# ft_potrf, one ncu --set full capture of the checksum pass, and
-# compute-sanitizer (racecheck, synccheck, memcheck) on tiny shapes.
+# ft_potrf, one ncu --set full capture of the checksum pass (compute-sanitizer
+# is closed on the GPU pool).
 #   gpurun --timeout 3600 -- 'bash tools/gpu_round.sh r02'
 tag=${1:-round}
 out=gpurun_out/$tag
@@ -31,7 +31,3 @@ ABFT_ITER_EVENTS=1 python tools/iter_time.py 30720 512 potrf 2> $out/iter_potrf.
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:checksum_pass -s 2 -c 2 \
    -o $out/prof_pass -f python bench.py --steps 1 --warmup 1 --no-e2e --no-potrf --no-cpu --no-lu-qr --no-mgpu \
    > $out/ncu_full.log 2>&1
-for tool in racecheck synccheck memcheck; do
-  timeout 900 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize_small.py > $out/sanitizer_$tool.log 2>&1
-  tail -2 $out/sanitizer_$tool.log
-done
