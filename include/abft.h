@@ -195,6 +195,18 @@ ABFT_API int abft_locate_correct(const abft_mat_t *mat, const abft_tiles_t *tile
                         abft_fix_t *fixes, int32_t max_fixes, int32_t *n_fixes,
                         abft_stream_t stream);
 
+/* a2 + a3 fused — abft_check.  abft_verify followed by abft_locate_correct
+ * on the same range, arguments and outcomes as the two calls in sequence
+ * (status, counts, corrections and fix records equal), in ONE launch: the
+ * CTA that finishes a tile's verify and finds it flagged runs the locate /
+ * classify / correct rounds of that tile itself (a check of Alg. 2,
+ * without a separate locate launch).  Where the locate tables do not fit the
+ * pass kernel's shared memory (fp64 nb=1024) the library issues the two
+ * launches instead.  Errors as abft_verify / abft_locate_correct. */
+ABFT_API int abft_check(const abft_mat_t *mat, const abft_tiles_t *tiles, int32_t which,
+                const abft_tol_t *tol, const abft_report_t *report,
+                abft_fix_t *fixes, int32_t max_fixes, int32_t *n_fixes, abft_stream_t stream);
+
 /* Fault injection (paper §X.A): element[offset] ^= xor_mask on the
  * device (fp32 uses the low 32 bits of the mask). */
 ABFT_API int abft_inject(void *ptr, int32_t dtype, int64_t offset, uint64_t xor_mask, abft_stream_t stream);

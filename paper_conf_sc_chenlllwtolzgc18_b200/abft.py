@@ -110,6 +110,8 @@ _sig = {
     "abft_verify_gemm": [_P(abft_mat_t), _P(abft_tiles_t), _i32, _P(abft_tol_t), _P(abft_report_t), _vp],
     "abft_locate_correct": [_P(abft_mat_t), _P(abft_tiles_t), _i32, _P(abft_tol_t), _P(abft_report_t),
                             _vp, _i32, _vp, _vp],
+    "abft_check": [_P(abft_mat_t), _P(abft_tiles_t), _i32, _P(abft_tol_t), _P(abft_report_t),
+                   _vp, _i32, _vp, _vp],
     "abft_inject": [_vp, _i32, _i64, _u64, _vp],
     "abft_sizes": [_i64, _i64, _i64, _P(_i64), _P(_i64), _P(_i64), _P(_i64)],
     "abft_update_trsm": [_i32, _ch, _ch, _ch, _ch, _i64, _vp, _i64, _vp, _i64, _i64, _vp, _i64, _i64, _vp],
@@ -287,6 +289,16 @@ def abft_locate_correct(mat: Mat, t: abft_tiles_t, which, tol: abft_tol_t, rep: 
     return _check("abft_locate_correct",
                   _L.abft_locate_correct(C.byref(m), C.byref(t), which, C.byref(tol), C.byref(r), _ptr(fixes),
                                          cap, _ptr(n_fixes), _stream(stream)))
+
+
+def abft_check(mat: Mat, t: abft_tiles_t, which, tol: abft_tol_t, rep: Report,
+               fixes: torch.Tensor, n_fixes: torch.Tensor, stream=None):
+    """abft_verify + abft_locate_correct in one launch (same arguments)."""
+    m, r = mat.c(), rep.c()
+    cap = 0 if fixes is None else fixes.numel() // FIX_BYTES
+    return _check("abft_check",
+                  _L.abft_check(C.byref(m), C.byref(t), which, C.byref(tol), C.byref(r), _ptr(fixes),
+                                cap, _ptr(n_fixes), _stream(stream)))
 
 
 def abft_inject(t: torch.Tensor, i: int, j: int, mask: int, stream=None):

@@ -13,7 +13,7 @@ CSRC = os.path.join(HERE, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(HERE, "libabft_b200.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-SOURCES = ["abft_runtime.cu", "abft_pass.cu", "abft_locate.cu", "abft_update.cu", "ft_potrf.cu", "ft_getrf.cu", "ft_geqrf.cu", "ft_host.cu", "abft_verify_gemm.cu", "abft_gated.cu", "abft_rule_dmma.cu"]
+SOURCES = ["abft_runtime.cu", "abft_pass.cu", "abft_locate.cu", "abft_update.cu", "ft_potrf.cu", "ft_getrf.cu", "ft_geqrf.cu", "ft_host.cu", "abft_verify_gemm.cu", "abft_gated.cu", "abft_rule_dmma.cu", "abft_rule_small.cu"]
 FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
     "-O3", "-lineinfo", "-std=c++17",

@@ -25,7 +25,7 @@
 #include <algorithm>
 #include <cstdlib>
 
-#include "abft_common.cuh"
+#include "abft_locate.cuh"
 
 namespace abft {
 
@@ -87,6 +87,9 @@ struct PassCfg {
   static_assert(NB % 32 == 0, "a tile column must be a multiple of 32 rows");
   static_assert(K == 1 || NB % (32 * VEC) == 0, "stacked tiles need whole vectors per tile");
   static_assert(K <= 8, "at most 8 stacked tiles");
+  // the fused check's locate_tile fits in the ring + side area
+  static constexpr bool FUSE_OK =
+      VERIFY && locate_smem_bytes(NB, (int)sizeof(T)) <= (size_t)NSTAGE * STAGE_BYTES + (RK * 3 + REC_ELEMS) * sizeof(T);
 };
 
 struct PassArgs {
@@ -119,6 +122,10 @@ struct PassArgs {
   int* ticket;      // [nsuper] self-resetting
   int* tflags;      // [ntiles] self-resetting
   const int32_t* gate;  // nullable: run only if *gate != 0 (driver-side conditional checks)
+  // fused check (abft_check): the finishing CTA of a flagged tile runs
+  // locate_tile on it before exiting (no separate locate launch)
+  int fuse;
+  LocArgs loc;
 };
 
 template <typename T, int VEC>
@@ -345,7 +352,7 @@ __device__ __forceinline__ void super_of(const abft_tiles_t& t, int mode, int K,
 // The verify variant of stacked tiles otherwise takes 111 and runs one CTA
 // per SM (fp32 nb=256 verify at 2.5 TB/s, ncu r01).
 template <typename T, int NB, int K, bool VERIFY>
-__global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched with kBlock threads
+__global__ void __maxnreg__(96) checksum_pass_kernel(const __grid_constant__ PassArgs p) {  // kBlock threads
   using C = PassCfg<T, NB, K, VERIFY>;
   constexpr int RK = C::RK;
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -354,7 +361,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
   T* rec = symacc;                                        // verify: recomputed [K][3][NB] (non-SYM tiles)
   uint64_t* full = reinterpret_cast<uint64_t*>(symacc + 3 * RK + C::REC_ELEMS);
   uint64_t* empty = full + C::NSTAGE;
-  __shared__ int s_colflags[K], s_ncols[K], s_nrows[K], s_rowflags[K];
+  __shared__ int s_colflags[K], s_ncols[K], s_nrows[K], s_rowflags[K], s_st[K];
   __shared__ int s_last;
 
   if (p.gate && *p.gate == 0) return;  // whole grid skips (uniform): no barrier or ticket touched
@@ -777,14 +784,32 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(PassArgs p) {  // launched 
     const int cf = s_colflags[t], rf = s_rowflags[t];
     const int st = ((cf & 1) ? ABFT_ST_COL : 0) | ((rf & 1) ? ABFT_ST_ROW : 0) | (((cf | rf) & 2) ? ABFT_ST_NONFINITE : 0);
     p.status[I + (int64_t)J * p.ld_status] = st;
+    s_st[t] = st;
     if (st & (ABFT_ST_COL | ABFT_ST_ROW)) atomicAdd(&p.counts[ABFT_CNT_TILES_FLAGGED], 1);
     if (st & ABFT_ST_NONFINITE) atomicAdd(&p.counts[ABFT_CNT_NONFINITE], 1);
     if (s_nrows[t]) atomicAdd(&p.counts[ABFT_CNT_ROWS_FLAGGED], s_nrows[t]);
     if (s_ncols[t]) atomicAdd(&p.counts[ABFT_CNT_COLS_FLAGGED], s_ncols[t]);
   }
+  if constexpr (C::FUSE_OK) {
+    if (!p.fuse) return;
+    // fused locate (a3): the tile's sums are final; its flagged tiles are
+    // classified and corrected by this CTA, the ring and side area reused
+    // as locate_tile's shared memory (every stage is consumed, the producer
+    // warp has exited)
+    consumer_sync();
+    for (int t = 0; t < kv; ++t) {
+      if (!(s_st[t] & (ABFT_ST_COL | ABFT_ST_ROW))) continue;  // uniform
+      __threadfence();
+      locate_tile<T>(p.loc, Ib + t, J, p.status + (Ib + t) + (int64_t)J * p.ld_status, smem_raw);
+    }
+  }
 }
 
 // ------------------------------------------------------------ launcher --
+// set by launch_k when a fused check fell on an instantiation whose locate
+// tables do not fit (fp64 nb=1024): run_pass then launches locate itself
+static thread_local bool g_fuse_missed = false;
+
 template <typename T, int NB, int K, bool VERIFY>
 static int launch_k(PassArgs& a, int64_t nsup, cudaStream_t s) {
   using C = PassCfg<T, NB, K, VERIFY>;
@@ -811,6 +836,9 @@ static int launch_k(PassArgs& a, int64_t nsup, cudaStream_t s) {
   if (force_slab > 0) nslab = std::min(force_slab, max_slab);
   a.nslab = nslab;
   a.K = K;
+  const int want_fuse = a.fuse;
+  a.fuse = want_fuse && C::FUSE_OK;
+  if (want_fuse && !C::FUSE_OK) g_fuse_missed = true;  // the caller launches locate separately
   if (nslab > 1) {
     void* ws = nullptr;
     size_t bytes = (size_t)ntiles * (C::GROUPS + 1) * NB * 3 * sizeof(T);
@@ -826,6 +854,7 @@ static int launch_k(PassArgs& a, int64_t nsup, cudaStream_t s) {
   }
   dim3 grid((unsigned)(nsup * nslab));
   kern<<<grid, kBlock, C::SMEM, s>>>(a);
+  a.fuse = want_fuse;
   ABFT_CUDA_TRY(cudaGetLastError());
   return 0;
 }
@@ -893,7 +922,7 @@ int validate_mat(const abft_mat_t* m, const abft_tiles_t* t, int which) {
 }
 
 static int run_pass(const abft_mat_t* m, const abft_tiles_t* t, int which, const abft_tol_t* tol,
-                    const abft_report_t* rep, cudaStream_t s, bool verify) {
+                    const abft_report_t* rep, cudaStream_t s, bool verify, const LocArgs* loc = nullptr) {
   int rc = validate_mat(m, t, which);
   if (rc) return rc;
   const int64_t ntiles = tiles_count(*t);
@@ -929,9 +958,18 @@ static int run_pass(const abft_mat_t* m, const abft_tiles_t* t, int which, const
     a.drow = rep->drow;
     a.counts = rep->counts;
   }
+  if (loc) {
+    a.fuse = 1;
+    a.loc = *loc;
+  }
+  g_fuse_missed = false;
   if (m->dtype == ABFT_F64)
-    return verify ? launch_t<double, true>(a, m->nb, ntiles, s) : launch_t<double, false>(a, m->nb, ntiles, s);
-  return verify ? launch_t<float, true>(a, m->nb, ntiles, s) : launch_t<float, false>(a, m->nb, ntiles, s);
+    rc = verify ? launch_t<double, true>(a, m->nb, ntiles, s) : launch_t<double, false>(a, m->nb, ntiles, s);
+  else
+    rc = verify ? launch_t<float, true>(a, m->nb, ntiles, s) : launch_t<float, false>(a, m->nb, ntiles, s);
+  if (rc || !loc || !g_fuse_missed) return rc;
+  LocArgs la = *loc;
+  return launch_locate_args(la, m->dtype, s);
 }
 
 }  // namespace abft
@@ -943,6 +981,15 @@ extern "C" int abft_encode(const abft_mat_t* mat, const abft_tiles_t* tiles, int
 extern "C" int abft_verify(const abft_mat_t* mat, const abft_tiles_t* tiles, int32_t which, const abft_tol_t* tol,
                            const abft_report_t* report, abft_stream_t stream) {
   return abft::run_pass(mat, tiles, which, tol, report, (cudaStream_t)stream, true);
+}
+
+extern "C" int abft_check(const abft_mat_t* mat, const abft_tiles_t* tiles, int32_t which, const abft_tol_t* tol,
+                          const abft_report_t* report, abft_fix_t* fixes, int32_t max_fixes, int32_t* n_fixes,
+                          abft_stream_t stream) {
+  abft::LocArgs la;
+  const int rc = abft::fill_loc_args(la, mat, tiles, which, tol, report, fixes, max_fixes, n_fixes);
+  if (rc) return rc;
+  return abft::run_pass(mat, tiles, which, tol, report, (cudaStream_t)stream, true, &la);
 }
 
 extern "C" int abft_sizes(int64_t m, int64_t n, int64_t nb, int64_t* colchk_elems, int64_t* rowchk_elems,

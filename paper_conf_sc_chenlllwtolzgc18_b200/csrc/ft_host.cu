@@ -383,8 +383,7 @@ static int host_pd_t(Driver& d, int k, int kind, int64_t row0, int64_t col0, int
     ABFT_CUDA_TRY(cudaMemcpyAsync(d.mark2, d.nfix, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
     abft_tol_t tol{ABFT_TOL_POSTERIORI, 1.0, 0};
     abft_report_t R{d.status, d.nt, nullptr, nullptr, d.xcounts};
-    FT_TRY(abft_verify(&P, &all, ABFT_COL, &tol, &R, as));
-    FT_TRY(abft_locate_correct(&P, &all, ABFT_COL, &tol, &R, c->fixlog, c->fixcap, d.nfix, as));
+    FT_TRY(abft_check(&P, &all, ABFT_COL, &tol, &R, c->fixlog, c->fixcap, d.nfix, as));
     offset_fixes_kernel<<<1, 128, 0, s>>>(c->fixlog, c->fixcap, d.mark2, d.nfix, row0, col0, nb);
     ABFT_CUDA_TRY(cudaMemcpyAsync(hcnt, d.xcounts, 8 * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
     ABFT_CUDA_TRY(cudaStreamSynchronize(s));

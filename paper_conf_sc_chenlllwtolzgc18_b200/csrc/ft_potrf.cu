@@ -334,7 +334,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       D.m = D.n = D.nb = nb;
       D.A = d.a_at(r0, r0);
       D.lda = lda;
-      if (ft) {
+      if (ft && !(Driver::diag_skip() & 8)) {
         D.colchk = d.colchk_at(2 * k, r0);
         D.ldc = d.M.ldc;
         D.colmag = d.colmag_at(k, r0);
@@ -441,6 +441,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     };
     auto pu_chk = [&]() -> int {  // c(L_ik) = c(A_ik) L_kk^-T, m_c <- m_c |L_kk^-T| with the PD's inverse (c-12, c-6)
       PhaseScope ps(d, FT_PH_RULES);
+      if (Driver::diag_skip() & 8) return 0;
       return abft_update_trsm_inv(dtype, 'R', 'T', nb, c->linv, nb, d.colchk_at(2 * (k + 1), r0), d.M.ldc, m2,
                                   d.colmag_at(k + 1, r0), d.M.ldcm, m2 / 2, as);
     };
@@ -507,7 +508,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     const int64_t r0 = (int64_t)k * nb;
     const abft_stream_t as = (abft_stream_t)d.s;
     const int J0 = (int)(c0 / nb), J1 = (int)(c1 / nb);
-    if (J1 <= J0) return 0;
+    if (J1 <= J0 || (Driver::diag_skip() & 4)) return 0;
     PhaseScope ps(d, FT_PH_RULES);
     if (c1 == n) {  // tile columns J0.. (to the end): the one-product rule of the sub-problem
       const int64_t ntk = nt - J0;
@@ -540,7 +541,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
   auto recheck = [&](int k, int64_t c0, int64_t c1) -> int {
     ABFT_CUDA_TRY(cudaMemcpyAsync(d.mark, d.nfix, sizeof(int32_t), cudaMemcpyDeviceToDevice, d.s));
     FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL));
-    if (!o->fig4a_repair) return 0;
+    if (!o->fig4a_repair || (Driver::diag_skip() & 1)) return 0;
     RepairArgs ra{};
     ra.A = dA;
     ra.lda = lda;

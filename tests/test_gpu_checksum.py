@@ -121,17 +121,40 @@ def _fix_tuple_list(fixes):
     return sorted((f[0], f[1], f[4], f[5]) for f in fixes)
 
 
+def _clone_mat(lib, mat):
+    cl = lambda x: None if x is None else x.t().clone().t()  # keep the column-major strides
+    return lib.Mat(cl(mat.A), mat.nb, cl(mat.colchk), cl(mat.rowchk), cl(mat.colmag), cl(mat.rowmag))
+
+
 def _run_locate(lib, mat, t, which, view=ck.GENERAL, tol=None):
+    """abft_verify then abft_locate_correct on `mat`; and, on a copy of the
+    same corrupted state, the fused abft_check, whose status, counts, fix
+    records and corrected arrays must equal the two-launch path's bit for bit."""
     tol = tol or lib.abft_tol_t(ck.TOL_MAGNITUDE, 1.0)
+    twin = _clone_mat(lib, mat)
     rep = lib.Report.alloc(mat)
     lib.abft_verify(mat, t, which, tol, rep)
     status_v = host(rep.status.clone()).astype(int)
     fixbuf = torch.zeros(4096 * lib.FIX_BYTES, dtype=torch.uint8, device="cuda")
     nfix = torch.zeros(1, dtype=torch.int32, device="cuda")
     lib.abft_locate_correct(mat, t, which, tol, rep, fixbuf, nfix)
+    rep2 = lib.Report.alloc(twin)
+    fixbuf2 = torch.zeros_like(fixbuf)
+    nfix2 = torch.zeros_like(nfix)
+    lib.abft_check(twin, t, which, tol, rep2, fixbuf2, nfix2)
     torch.cuda.synchronize()
     n = int(nfix.item())
-    return status_v, host(rep.status).astype(int), rep.counts.cpu().numpy(), lib.decode_fixes(fixbuf, n)
+    fixes = lib.decode_fixes(fixbuf, n)
+    assert int(nfix2.item()) == n
+    assert torch.equal(rep.status, rep2.status) and torch.equal(rep.counts, rep2.counts)
+    key = lambda f: (f[0], f[1], f[4], f[5], repr(f[2]), repr(f[3]))  # NaN-safe
+    assert sorted(map(key, fixes)) == sorted(map(key, lib.decode_fixes(fixbuf2, n)))
+    for x, y in [(mat.A, twin.A), (mat.colchk, twin.colchk), (mat.rowchk, twin.rowchk), (mat.colmag, twin.colmag),
+                 (mat.rowmag, twin.rowmag)]:
+        if x is not None:
+            assert torch.equal(x.view(torch.int64 if x.dtype == torch.float64 else torch.int32),
+                               y.view(torch.int64 if y.dtype == torch.float64 else torch.int32))
+    return status_v, host(rep.status).astype(int), rep.counts.cpu().numpy(), fixes
 
 
 def _oracle_locate(st, t_or, which):

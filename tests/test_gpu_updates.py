@@ -57,6 +57,35 @@ def test_update_trsm_f32(lib, side, trans):
     assert np.abs(host(Xd) - ref).max() <= 1e-4 * np.abs(ref).max()
 
 
+# padded leading dimensions (the drivers' checksum arrays: ld = 2 nt > nvec)
+# and every vector-block tail (nvec not a multiple of the kernel's 16)
+@pytest.mark.parametrize("prec", ["f64", "f32"])
+@pytest.mark.parametrize("side,trans,nb,nvec", [("R", "T", 512, 37), ("L", "N", 256, 3), ("R", "N", 128, 17),
+                                                ("L", "T", 64, 33)])
+def test_update_trsm_inv_padded(lib, prec, side, trans, nb, nvec):
+    dt = torch.float64 if prec == "f64" else torch.float32
+    T = _tri(nb, 6, True, False)
+    if prec == "f32":
+        T = T.astype(np.float32).astype(np.float64)
+    W = np.linalg.inv(T)
+    shape = (nvec, nb) if side == "R" else (nb, nvec)
+    X = si.general(*shape, seed=7)
+    M = np.abs(si.general(*((nvec // 2 + 1, nb) if side == "R" else (nb, nvec // 2 + 1)), seed=8))
+    if prec == "f32":
+        W, X, M = (a.astype(np.float32).astype(np.float64) for a in (W, X, M))
+    Wd = dev(W, dt, ld=nb + 3)
+    Xd = dev(X, dt, ld=shape[0] + 5)
+    Md = dev(M, dt, ld=M.shape[0] + 2)
+    lib.abft_update_trsm_inv(side, trans, Wd, Xd, nvec, Md, M.shape[1] if side == "L" else M.shape[0])
+    torch.cuda.synchronize()
+    opW = W.T if trans == "T" else W
+    ref = X @ opW if side == "R" else opW @ X
+    mref = M @ np.abs(opW) if side == "R" else np.abs(opW) @ M
+    tol = 1e-12 if prec == "f64" else 1e-5
+    assert np.abs(host(Xd) - ref).max() <= tol * np.abs(ref).max()
+    assert np.abs(host(Md) - mref).max() <= tol * np.abs(mref).max()
+
+
 @pytest.mark.parametrize("which,tX,tY", [(1, "N", "T"), (2, "T", "N"), (1, "N", "N"), (2, "N", "N")])
 def test_update_gemm_matches_matmul(lib, which, tX, tY):
     M2, N, K = 12, 96, 32
