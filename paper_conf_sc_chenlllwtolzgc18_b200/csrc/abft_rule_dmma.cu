@@ -22,9 +22,13 @@
 // slice run together.  Summation order: one fixed DMMA chain per output
 // element over k ascending (deterministic; not the cuBLAS order, so P and Q
 // agree with the GEMM route to rounding, well inside the checks' tau).
+#include <cooperative_groups.h>
+
 #include <algorithm>
 
 #include "abft_common.cuh"
+
+namespace cg = cooperative_groups;
 
 namespace abft {
 namespace {
@@ -55,7 +59,8 @@ struct RuleArgs {
   int64_t ldrm;
   int ntk;
   int nb;
-  int M2p;  // checksum rows padded to 8 (magnitude rows start here)
+  int M2p;    // checksum rows padded to 8 (magnitude rows start here)
+  int split;  // K split over a (1, 1, split) cluster (small grids), partials reduced in rank order
 };
 
 __device__ __forceinline__ void cp_async8(void* smem, const void* gmem, bool valid) {
@@ -114,7 +119,9 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
   const int g = lane >> 2, t = lane & 3;
   const int r0 = blockIdx.x * kTM;                // first row of A
   const int x0 = blockIdx.y * kTN;                // first column (row of L21)
-  const int ksteps = p.nb / kBK;
+  // this CTA's k-steps: all of them, or its rank's share of a K-split cluster
+  const int kall = p.nb / kBK, z = blockIdx.z;
+  const int kbeg = z * kall / p.split, ksteps = (z + 1) * kall / p.split - kbeg;
   const int M2 = 2 * p.ntk;
   // fill roles (fixed for the CTA): A row ra (k parity by half), L21 column cb
   const int ra = tid % kTM, ka = tid / kTM;       // 2 threads per row: k = ka, ka + 2, ...
@@ -125,7 +132,7 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
   const int cb = tid % kTN, kbq = tid / kTN;      // 4 threads per column: k = kbq, kbq + 4, ...
   const double* srcB = p.L + x0 + cb;
   auto fill = [&](int kt, int st) {
-    const int64_t kb = (int64_t)kt * kBK;
+    const int64_t kb = (int64_t)(kbeg + kt) * kBK;
     double* as = As + (size_t)st * kBK * kLdA + ra;
 #pragma unroll
     for (int kk = ka; kk < kBK; kk += kThr / kTM) cp_async8(as + kk * kLdA, srcA + (kb + kk) * ldA, isp || isq);
@@ -164,6 +171,35 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
     }
   }
   cp_async_wait<0>();
+  if (p.split > 1) {
+    // K-split partials: every rank parks its accumulators (thread-major) in
+    // its own ring, rank 0 adds ranks 1, 2, ... in order (deterministic) and
+    // scatters; the second barrier keeps the other ranks' shared memory
+    // alive until rank 0 has read it
+    __syncthreads();
+    double* part = sm;
+#pragma unroll
+    for (int a = 0; a < kWM; ++a)
+#pragma unroll
+      for (int n = 0; n < kWN; ++n)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) part[((a * kWN + n) * 2 + h) * kThr + tid] = acc[a][n][h];
+    cg::cluster_group cl = cg::this_cluster();
+    cl.sync();
+    if (z == 0) {
+      for (int r = 1; r < p.split; ++r) {
+        const double* rp = cl.map_shared_rank(part, r);
+#pragma unroll
+        for (int a = 0; a < kWM; ++a)
+#pragma unroll
+          for (int n = 0; n < kWN; ++n)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) acc[a][n][h] += rp[((a * kWN + n) * 2 + h) * kThr + tid];
+      }
+    }
+    cl.sync();
+    if (z != 0) return;
+  }
   // scatter: lane holds P/Q[y][x], [y][x+1] with y = wr0 + 8a + g,
   // x = x0 + 16 wn + 8n + 2t.  The 32 columns meet at most one tile-column
   // boundary (nb >= 32): J = J0 + (x - x0 >= bnd).  One writer per element:
@@ -234,8 +270,31 @@ int update_syrk_dmma(int64_t nb, int64_t ntk, const double* L21, int64_t ldl, co
   a.M2p = (int)((2 * ntk + 7) / 8 * 8);
   const int64_t Mt = a.M2p + (mags ? (ntk + 7) / 8 * 8 : 0);
   const dim3 grid((unsigned)((Mt + kTM - 1) / kTM), (unsigned)(nk / kTN));
-  syrk_rule_dmma_kernel<<<grid, kThr, kRuleSmem, s>>>(a);
-  ABFT_CUDA_TRY(cudaGetLastError());
+  // small grids (the look-ahead's single tile column, late iterations) are
+  // bound by the k-loop's latency, not by the DMMA rate: split K over a
+  // cluster while the grid stays under ~4 CTAs per SM
+  const int64_t ctas = (int64_t)grid.x * grid.y;
+  int split = 1;
+  while (split < 8 && ctas * split * 2 <= 4 * 148 && (nb / kBK) % (split * 2) == 0) split *= 2;
+  a.split = split;
+  if (split == 1) {
+    syrk_rule_dmma_kernel<<<grid, kThr, kRuleSmem, s>>>(a);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    return 0;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid.x, grid.y, (unsigned)split);
+  cfg.blockDim = dim3(kThr, 1, 1);
+  cfg.dynamicSmemBytes = kRuleSmem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = 1;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = (unsigned)split;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  ABFT_CUDA_TRY(cudaLaunchKernelEx(&cfg, syrk_rule_dmma_kernel, a));
   return 0;
 }
 

@@ -1,5 +1,5 @@
 // abft_rule_small.cu — the PD / PU checksum rules with an explicit inverse
-// (a5, `abft_update_trsm_inv`) as ONE launch.
+// (a5, `abft_update_trsm_inv`) as ONE launch on the FP64 tensor cores.
 //
 // Paper: checksums are updated by applying the operation to them (L149,
 // §IV); the PU of Cholesky / LU / QR is a TRSM, so its checksum rule is a
@@ -10,20 +10,18 @@
 //   side R: chk (nvec x nb) <- chk op(W),   mag (nmag x nb) <- mag |op(W)|
 //   side L: chk (nb x nvec) <- op(W) chk,   mag (nb x nmag) <- |op(W)| mag
 //
-// The library route was a GEMM into scratch + a copy back per array plus an
+// The library route is a GEMM into scratch + a copy back per array plus an
 // |W| copy (5-7 launches, 25-35 us of dependent latency on the side chain of
 // the look-ahead drivers).  Here every checksum vector v (a row for side R,
 // a column for side L) is independent: out_v = old_v M with M = op(W) (side
-// R) or op(W)^T (side L), so the update runs IN PLACE as one clustered
-// launch.  A cluster owns VB vectors and spans the nb output columns (JB per
-// CTA); every CTA stages the cluster's old vectors in shared memory, the
-// cluster barrier orders all reads before any write, then each CTA computes
-// and stores its JB columns.  W is streamed through shared memory in
-// QB-row chunks with a register prefetch of the next chunk.  Summation
-// order: q ascending, one FMA chain per output (deterministic).  Each CTA
-// reads its nb x JB slice of W from L2 (512 KB at nb=512 fp64); thread groups
-// whose vectors are all past the end (the 2 + 1 vectors of the PD rule) skip
-// the FMAs.
+// R) or op(W)^T (side L).  A thread-block cluster owns 32 vectors and spans
+// all nb output columns (JB = 32 per CTA, nb / 32 <= 16 CTAs): each CTA runs
+// a DMMA (mma.sync m8n8k4 f64) main loop over q with a 4-stage cp.async ring,
+// then the cluster barrier orders every CTA's reads of the old vectors
+// before any CTA stores its columns — so the update runs IN PLACE, no
+// scratch, no copy back.  Summation order: one DMMA chain per output over q
+// ascending (deterministic).  fp64 only (fp32 and nb = 1024 keep the library
+// route).
 #include <cooperative_groups.h>
 
 #include "abft_common.cuh"
@@ -33,179 +31,150 @@ namespace cg = cooperative_groups;
 namespace abft {
 namespace {
 
-constexpr int kVB = 16;   // vectors per cluster
-constexpr int kThr = 256;
+constexpr int kVB = 32;   // vectors per cluster (rows of the product)
+constexpr int kJB = 32;   // output columns per CTA
+constexpr int kBK = 16;   // q per stage
+constexpr int kStages = 4;
+constexpr int kThr = 128;  // 4 warps: 2 (vectors, 16 each) x 2 (columns, 16 each)
+constexpr int kLd = kVB + 4;  // stage row stride (doubles): 4 (mod 16) keeps fragments conflict-free
+static_assert(kVB == kJB, "one stage layout for both operands");
 
-template <typename T>
 struct SmallRuleArgs {
-  const T* W;
+  const double* W;
   int64_t ldw;
   int tW;     // M[q][j] = tW ? W[j + q ldw] : W[q + j ldw]
   int sideR;  // vector v element q at base[v + q ld] (R) or base[q + v ld] (L)
   int nb;
-  T* chk;
+  double* chk;
   int64_t ldchk;
   int nvec;
-  T* mag;
+  double* mag;
   int64_t ldmag;
   int nmag;
   int nblk_chk;  // vector blocks of chk (the rest are magnitude blocks)
 };
 
-// rows of M per staged chunk: 16 prefetched values per thread
-template <int JB>
-constexpr int qb_of() {
-  return 4096 / JB;
+__device__ __forceinline__ void cp_async8(void* smem, const void* gmem, bool valid) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(smem_u32(smem)), "l"(gmem),
+               "r"(valid ? 8 : 0)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void dmma(double (&d)[2], double a, double b) {
+  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+               : "+d"(d[0]), "+d"(d[1])
+               : "d"(a), "d"(b));
 }
 
-template <typename T, int JB>
-__global__ void __launch_bounds__(kThr) trsm_inv_rule_kernel(SmallRuleArgs<T> a) {
-  constexpr int kQB = qb_of<JB>();
-  extern __shared__ __align__(16) unsigned char rs_smem[];
-  constexpr int WLD = JB + 2;  // row stride of the W chunk (even: 16-B aligned pairs)
-  T* Vs = reinterpret_cast<T*>(rs_smem);  // [kVB][nb]
-  T* Ws = Vs + (size_t)kVB * a.nb;        // [kQB][WLD]
-  const int tid = threadIdx.x;
+__global__ void __launch_bounds__(kThr) trsm_inv_rule_kernel(const __grid_constant__ SmallRuleArgs a) {
+  __shared__ __align__(16) double Vs[kStages][kBK][kLd];  // [q][v]
+  __shared__ __align__(16) double Ms[kStages][kBK][kLd];  // [q][j]
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int wv = warp & 1, wj = warp >> 1;
+  const int g = lane >> 2, t = lane & 3;
   const int nb = a.nb;
   const int vb = blockIdx.y;
   const bool mag = vb >= a.nblk_chk;
-  T* base = mag ? a.mag : a.chk;
+  double* base = mag ? a.mag : a.chk;
   const int64_t ld = mag ? a.ldmag : a.ldchk;
   const int nv = mag ? a.nmag : a.nvec;
   const int v0 = (mag ? vb - a.nblk_chk : vb) * kVB;
-  const int j0 = blockIdx.x * JB;
-
-  // 1. the cluster's old vectors
-  if (a.sideR) {
-    for (int idx = tid; idx < kVB * nb; idx += kThr) {
-      const int v = idx % kVB, q = idx / kVB;
-      Vs[v * nb + q] = v0 + v < nv ? base[(v0 + v) + (int64_t)q * ld] : T(0);
-    }
-  } else {
-    for (int idx = tid; idx < kVB * nb; idx += kThr) {
-      const int q = idx % nb, v = idx / nb;
-      Vs[v * nb + q] = v0 + v < nv ? base[q + (int64_t)(v0 + v) * ld] : T(0);
-    }
-  }
-  // every CTA of the cluster has read the old values before anyone writes
-  cg::this_cluster().sync();
-
-  // 2. out[v][j] = sum_q Vs[v][q] M[q][j]; thread: column pair jp, vector group g
-  constexpr int NP = JB / 2;         // column pairs
-  constexpr int NG = kThr / NP;      // vector groups
-  constexpr int VPG = kVB / NG;      // vectors per thread
-  static_assert(VPG >= 1 && kVB % NG == 0, "tile shape");
-  const int jp = tid % NP, g = tid / NP;
-  const bool active = v0 + g * VPG < nv;  // uniform per group of NP threads
-  T acc[VPG][2];
+  const int j0 = blockIdx.x * kJB;
+  const int64_t sv = a.sideR ? 1 : ld, sq = a.sideR ? ld : 1;  // vector / q strides of base
+  const int64_t mj = a.tW ? 1 : a.ldw, mq = a.tW ? a.ldw : 1;  // column / q strides of M in W
+  // fill roles: 128 threads x 4 elements per operand per stage (16 q x 32);
+  // the contiguous index of each operand runs fastest over the threads
+  auto fill = [&](int kt, int st) {
+    const int q0 = kt * kBK;
 #pragma unroll
-  for (int i = 0; i < VPG; ++i) acc[i][0] = acc[i][1] = T(0);
-  constexpr int PER = kQB * JB / kThr;  // chunk elements loaded per thread
-  T pre[PER];
-  auto load_chunk = [&](int q0) {
-#pragma unroll
-    for (int u = 0; u < PER; ++u) {
+    for (int u = 0; u < 4; ++u) {
       const int idx = tid + u * kThr;
-      int qq, jj;
-      if (a.tW) {  // contiguous along j
-        jj = idx % JB;
-        qq = idx / JB;
-      } else {     // contiguous along q
-        qq = idx % kQB;
-        jj = idx / kQB;
-      }
-      const int q = q0 + qq, j = j0 + jj;
-      pre[u] = q < nb ? (a.tW ? a.W[j + (int64_t)q * a.ldw] : a.W[q + (int64_t)j * a.ldw]) : T(0);
-    }
-  };
-  auto store_chunk = [&]() {
-#pragma unroll
-    for (int u = 0; u < PER; ++u) {
-      const int idx = tid + u * kThr;
-      int qq, jj;
-      if (a.tW) {
-        jj = idx % JB;
-        qq = idx / JB;
+      int x, qq;  // V: x = vector
+      if (a.sideR) {
+        x = idx % kVB;
+        qq = idx / kVB;
       } else {
-        qq = idx % kQB;
-        jj = idx / kQB;
+        qq = idx % kBK;
+        x = idx / kBK;
       }
-      const T w = pre[u];
-      Ws[qq * WLD + jj] = mag ? T(fabs(w)) : w;
+      const bool ok = v0 + x < nv;
+      cp_async8(&Vs[st][qq][x], base + (ok ? (v0 + x) * sv + (int64_t)(q0 + qq) * sq : 0), ok);
+      int y, qm;  // M: y = column
+      if (a.tW) {
+        y = idx % kJB;
+        qm = idx / kJB;
+      } else {
+        qm = idx % kBK;
+        y = idx / kBK;
+      }
+      cp_async8(&Ms[st][qm][y], a.W + (int64_t)(j0 + y) * mj + (int64_t)(q0 + qm) * mq, true);
     }
   };
-  load_chunk(0);
-  for (int q0 = 0; q0 < nb; q0 += kQB) {
-    __syncthreads();  // the previous chunk's readers are done
-    store_chunk();
-    __syncthreads();
-    if (q0 + kQB < nb) load_chunk(q0 + kQB);  // in flight during the FMAs below
-    const int qn = !active ? 0 : (nb - q0 < kQB ? nb - q0 : kQB);
-    for (int qq = 0; qq < qn; ++qq) {
-      const T w0 = Ws[qq * WLD + 2 * jp], w1 = Ws[qq * WLD + 2 * jp + 1];
+  const int ksteps = nb / kBK;
 #pragma unroll
-      for (int i = 0; i < VPG; ++i) {
-        const T x = Vs[(g * VPG + i) * nb + q0 + qq];
-        acc[i][0] = fma(x, w0, acc[i][0]);
-        acc[i][1] = fma(x, w1, acc[i][1]);
+  for (int s = 0; s < kStages - 1; ++s) {
+    if (s < ksteps) fill(s, s);
+    cp_async_commit();
+  }
+  double acc[2][2][2] = {};  // [v-tile][j-tile][2]
+  for (int kt = 0; kt < ksteps; ++kt) {
+    cp_async_wait<kStages - 2>();
+    __syncthreads();
+    const int nx = kt + kStages - 1;
+    if (nx < ksteps) fill(nx, nx % kStages);
+    cp_async_commit();
+    const int st = kt % kStages;
+#pragma unroll
+    for (int k4 = 0; k4 < kBK; k4 += 4) {
+      double bf[2];
+#pragma unroll
+      for (int n = 0; n < 2; ++n) {
+        const double w = Ms[st][k4 + t][wj * 16 + n * 8 + g];
+        bf[n] = mag ? fabs(w) : w;
+      }
+#pragma unroll
+      for (int m = 0; m < 2; ++m) {
+        const double af = Vs[st][k4 + t][wv * 16 + m * 8 + g];
+#pragma unroll
+        for (int n = 0; n < 2; ++n) dmma(acc[m][n], af, bf[n]);
       }
     }
   }
-  // 3. store this CTA's columns of the cluster's vectors
+  cp_async_wait<0>();
+  // every CTA of the cluster has read all of the cluster's old vectors
+  cg::this_cluster().sync();
+  // lane holds out[v][j], out[v][j+1]: v = v0 + 16 wv + 8 m + g, j = j0 + 16 wj + 8 n + 2 t
 #pragma unroll
-  for (int i = 0; i < VPG; ++i) {
-    const int v = v0 + g * VPG + i;
+  for (int m = 0; m < 2; ++m) {
+    const int v = v0 + wv * 16 + m * 8 + g;
     if (v >= nv) continue;
 #pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const int j = j0 + 2 * jp + h;
-      if (a.sideR)
-        base[v + (int64_t)j * ld] = acc[i][h];
-      else
-        base[j + (int64_t)v * ld] = acc[i][h];
-    }
+    for (int n = 0; n < 2; ++n)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int j = j0 + wj * 16 + n * 8 + 2 * t + h;
+        base[(int64_t)v * sv + (int64_t)j * sq] = acc[m][n][h];
+      }
   }
-}
-
-template <typename T, int JB>
-int launch_small_rule(const SmallRuleArgs<T>& a, int nblk, cudaStream_t s) {
-  auto kern = trsm_inv_rule_kernel<T, JB>;
-  const size_t smem = ((size_t)kVB * a.nb + (size_t)qb_of<JB>() * (JB + 2)) * sizeof(T);
-  static size_t attr = 0;
-  if (attr < smem) {
-    ABFT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    attr = smem;
-  }
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)(a.nb / JB), (unsigned)nblk, 1);
-  cfg.blockDim = dim3(kThr, 1, 1);
-  cfg.dynamicSmemBytes = smem;
-  cfg.stream = s;
-  cudaLaunchAttribute at[1];
-  at[0].id = cudaLaunchAttributeClusterDimension;
-  at[0].val.clusterDim.x = (unsigned)(a.nb / JB);
-  at[0].val.clusterDim.y = 1;
-  at[0].val.clusterDim.z = 1;
-  cfg.attrs = at;
-  cfg.numAttrs = 1;
-  ABFT_CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, a));
-  return 0;
 }
 
 }  // namespace
 
-// Returns ABFT_E_UNSUPPORTED for shapes outside nb in {32, ..., 1024} powers
-// of two (the caller then takes the library route).
-template <typename T>
-int trsm_inv_rule(char side, char trans, int64_t nb, const T* W, int64_t ldw, T* chk, int64_t ldchk, int64_t nvec,
-                  T* mag, int64_t ldmag, int64_t nmag, cudaStream_t s) {
-  if (nb < 32 || nb > 1024 || (nb & (nb - 1))) return ABFT_E_UNSUPPORTED;
+// Returns ABFT_E_UNSUPPORTED outside fp64 with nb in {32, ..., 512} powers of
+// two (the caller then takes the library route).
+int trsm_inv_rule(char side, char trans, int64_t nb, const double* W, int64_t ldw, double* chk, int64_t ldchk,
+                  int64_t nvec, double* mag, int64_t ldmag, int64_t nmag, cudaStream_t s) {
+  if (nb < 32 || nb > 16 * kJB || (nb & (nb - 1))) return ABFT_E_UNSUPPORTED;
   const bool right = side == 'R' || side == 'r';
   const bool tr = trans == 'T' || trans == 't';
   if (!mag) nmag = 0;
   if (!chk) nvec = 0;
   if (nvec <= 0 && nmag <= 0) return 0;
-  SmallRuleArgs<T> a{};
+  SmallRuleArgs a{};
   a.W = W;
   a.ldw = ldw;
   a.tW = right ? tr : !tr;
@@ -219,14 +188,26 @@ int trsm_inv_rule(char side, char trans, int64_t nb, const T* W, int64_t ldw, T*
   a.nmag = (int)(nmag > 0 ? nmag : 0);
   a.nblk_chk = (a.nvec + kVB - 1) / kVB;
   const int nblk = a.nblk_chk + (a.nmag + kVB - 1) / kVB;
-  if (nb >= 128) return launch_small_rule<T, 128>(a, nblk, s);
-  if (nb == 64) return launch_small_rule<T, 64>(a, nblk, s);
-  return launch_small_rule<T, 32>(a, nblk, s);
+  const unsigned cs = (unsigned)(nb / kJB);
+  static bool attr = false;
+  if (!attr) {
+    ABFT_CUDA_TRY(cudaFuncSetAttribute(trsm_inv_rule_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+    attr = true;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(cs, (unsigned)nblk, 1);
+  cfg.blockDim = dim3(kThr, 1, 1);
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = cs;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  ABFT_CUDA_TRY(cudaLaunchKernelEx(&cfg, trsm_inv_rule_kernel, a));
+  return 0;
 }
-
-template int trsm_inv_rule<double>(char, char, int64_t, const double*, int64_t, double*, int64_t, int64_t, double*,
-                                   int64_t, int64_t, cudaStream_t);
-template int trsm_inv_rule<float>(char, char, int64_t, const float*, int64_t, float*, int64_t, int64_t, float*,
-                                  int64_t, int64_t, cudaStream_t);
 
 }  // namespace abft

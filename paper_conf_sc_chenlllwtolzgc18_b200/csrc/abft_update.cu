@@ -12,6 +12,7 @@
 #include <cusolverDn.h>
 
 #include <mutex>
+#include <type_traits>
 #include <unordered_map>
 #include <vector>
 
@@ -325,19 +326,21 @@ static int copy_back(T* out, int64_t ldo, const T* tmp, int64_t rows, int64_t co
 // a5 with a precomputed inverse W = T^-1:
 //   side R: chk (nvec x nb) <- chk * op(W);  mag (nmag x nb) <- mag * |op(W)|
 //   side L: chk (nb x nvec) <- op(W) * chk;  mag (nb x nmag) <- |op(W)| * mag
-template <typename T>
-int trsm_inv_rule(char side, char trans, int64_t nb, const T* W, int64_t ldw, T* chk, int64_t ldchk, int64_t nvec,
-                  T* mag, int64_t ldmag, int64_t nmag, cudaStream_t s);  // abft_rule_small.cu
+int trsm_inv_rule(char side, char trans, int64_t nb, const double* W, int64_t ldw, double* chk, int64_t ldchk,
+                  int64_t nvec, double* mag, int64_t ldmag, int64_t nmag, cudaStream_t s);  // abft_rule_small.cu
 
 template <typename T>
 int update_trsm_inv_t(char side, char trans, int64_t nb, const T* W, int64_t ldw, T* chk, int64_t ldchk, int64_t nvec,
                       T* mag, int64_t ldmag, int64_t nmag, cudaStream_t s) {
-  // one clustered in-place launch (abft_rule_small.cu); ABFT_RULE_CUBLAS=1
-  // keeps the library route below (GEMM into scratch + copy back per array)
+  // fp64: one clustered in-place DMMA launch (abft_rule_small.cu);
+  // ABFT_RULE_CUBLAS=1 keeps the library route below (GEMM into scratch +
+  // copy back per array), as fp32 and nb = 1024 do
   static const bool gemm_route = getenv("ABFT_RULE_CUBLAS") != nullptr;
-  if (!gemm_route) {
-    const int r = trsm_inv_rule<T>(side, trans, nb, W, ldw, chk, ldchk, nvec, mag, ldmag, nmag, s);
-    if (r != ABFT_E_UNSUPPORTED) return r;
+  if constexpr (std::is_same<T, double>::value) {
+    if (!gemm_route) {
+      const int r = trsm_inv_rule(side, trans, nb, W, ldw, chk, ldchk, nvec, mag, ldmag, nmag, s);
+      if (r != ABFT_E_UNSUPPORTED) return r;
+    }
   }
   const bool left = side == 'L' || side == 'l';
   const cublasOperation_t oW = op_of(trans);
