@@ -38,7 +38,9 @@ constexpr int kWarps = kThreads / 32;
 template <typename T, int NB, int K, bool VERIFY = false>
 struct PassCfg {
   static constexpr int RK = K * NB;              // rows per CTA
-  static constexpr int GC = NB < 64 ? NB : 64;  // group columns (slab granularity)
+  // group columns (slab granularity): 32 for NB >= 256, so that a single
+  // tile (the drivers' diagonal-tile checks) splits into NB/32 slab CTAs
+  static constexpr int GC = NB < 64 ? NB : (NB >= 256 ? 32 : 64);
   static constexpr int COL_BYTES = RK * (int)sizeof(T);
   // 32 KiB stages for every column size (fp64 nb=1024, 8-KiB columns, had
   // 16 KiB stages of 2 columns: the row-sum chunk CQ fell to 2 columns, the

@@ -15,11 +15,12 @@
 // straight into the four arrays (one writer per element: a fire-and-forget
 // reduction, no P / Q scratch).
 //
-// Tiling (the shape cuBLAS picks for these skinny products): CTA tile 64
-// rows of A x 32 columns, 4 warps of 32 x 16 (4 x 2 DMMA tiles), K = nb in
-// 16-deep stages through a 4-stage cp.async ring (53 KB: 4 CTAs per SM);
-// grid (Mt / 64, nk / 32), row tiles fastest so the CTAs that share an L21
-// slice run together.  Summation order: one fixed DMMA chain per output
+// Tiling: CTA tile 64 rows of A x 32 columns, 4 warps of 32 x 16 (4 x 2
+// DMMA tiles), K = nb in 16-deep stages through a 4-stage cp.async ring
+// (53 KB: 4 CTAs per SM); grid (Mt / 64, nk / 32), row tiles fastest so the
+// CTAs that share an L21 slice run together (a 64 x 64 tile with 32 x 32
+// warps measured no faster: 225 vs 212-231 us at ntk = 59, slower at 30).
+// Small grids split K over a cluster (below).  Summation order: one fixed DMMA chain per output
 // element over k ascending (deterministic; not the cuBLAS order, so P and Q
 // agree with the GEMM route to rounding, well inside the checks' tau).
 #include <cooperative_groups.h>
@@ -40,6 +41,7 @@ constexpr int kStages = 4;
 constexpr int kThr = 128;     // 4 warps: 2 (m, 32 rows) x 2 (n, 16 columns)
 constexpr int kWM = 4;        // m-tiles per warp
 constexpr int kWN = 2;        // n-tiles per warp
+constexpr int kWNC = kWN * 8;  // columns per warp
 constexpr int kLdA = kTM + 4;  // row stride = 4 (mod 16 doubles): conflict-free fragments
 constexpr int kLdB = kTN + 4;
 constexpr size_t kRuleSmem = (size_t)kStages * kBK * (kLdA + kLdB) * sizeof(double);
@@ -61,6 +63,7 @@ struct RuleArgs {
   int nb;
   int M2p;    // checksum rows padded to 8 (magnitude rows start here)
   int split;  // K split over a (1, 1, split) cluster (small grids), partials reduced in rank order
+  int nk;     // columns of the product (rows of L21 used)
 };
 
 __device__ __forceinline__ void cp_async8(void* smem, const void* gmem, bool valid) {
@@ -130,7 +133,8 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
   const double* srcA = isp ? p.cL + ya : (isq ? p.mL + yqa : p.cL);
   const int64_t ldA = isp ? p.ldc : (isq ? p.ldcm : 0);
   const int cb = tid % kTN, kbq = tid / kTN;      // 4 threads per column: k = kbq, kbq + 4, ...
-  const double* srcB = p.L + x0 + cb;
+  const bool bok = x0 + cb < p.nk;
+  const double* srcB = p.L + (bok ? x0 + cb : 0);
   auto fill = [&](int kt, int st) {
     const int64_t kb = (int64_t)(kbeg + kt) * kBK;
     double* as = As + (size_t)st * kBK * kLdA + ra;
@@ -138,7 +142,7 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
     for (int kk = ka; kk < kBK; kk += kThr / kTM) cp_async8(as + kk * kLdA, srcA + (kb + kk) * ldA, isp || isq);
     double* bs = Bs + (size_t)st * kBK * kLdB + cb;
 #pragma unroll
-    for (int kk = kbq; kk < kBK; kk += kThr / kTN) cp_async8(bs + kk * kLdB, srcB + (kb + kk) * p.ldl, true);
+    for (int kk = kbq; kk < kBK; kk += kThr / kTN) cp_async8(bs + kk * kLdB, srcB + (kb + kk) * p.ldl, bok);
   };
 #pragma unroll
   for (int s = 0; s < kStages - 1; ++s) {
@@ -161,7 +165,7 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
     if (nx < ksteps) fill(nx, nx % kStages);
     cp_async_commit();
     const double* as = As + (size_t)(kt % kStages) * kBK * kLdA + wm * 32 + g;
-    const double* bs = Bs + (size_t)(kt % kStages) * kBK * kLdB + wn * 16 + g;
+    const double* bs = Bs + (size_t)(kt % kStages) * kBK * kLdB + wn * kWNC + g;
     switch (aq) {  // warp-uniform
       case 0: stage_mma<0>(acc, as, bs, t); break;
       case 1: stage_mma<1>(acc, as, bs, t); break;
@@ -201,10 +205,8 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
     if (z != 0) return;
   }
   // scatter: lane holds P/Q[y][x], [y][x+1] with y = wr0 + 8a + g,
-  // x = x0 + 16 wn + 8n + 2t.  The 32 columns meet at most one tile-column
-  // boundary (nb >= 32): J = J0 + (x - x0 >= bnd).  One writer per element:
-  // a reduction adds exactly what load + add + store would.
-  const int J0 = x0 / p.nb, bnd = (J0 + 1) * p.nb - x0;
+  // x = x0 + 16 wn + 8n + 2t, tile column J = x / nb.  One writer per
+  // element: a reduction adds exactly what load + add + store would.
 #pragma unroll
   for (int a = 0; a < kWM; ++a) {
     const int y = wr0 + a * 8 + g;
@@ -222,8 +224,9 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
     for (int n = 0; n < kWN; ++n)
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
-        const int xx = wn * 16 + n * 8 + 2 * t + h;
-        const int J = J0 + (xx >= bnd);
+        const int xx = wn * kWNC + n * 8 + 2 * t + h;
+        if (x0 + xx >= p.nk) continue;
+        const int J = (x0 + xx) / p.nb;
         const double v = sgn * acc[a][n][h];
         if (I >= J) atomicAdd(Cp + (int64_t)(x0 + xx) * ldC, v);
         if (Rp && J >= I) atomicAdd(Rp + (x0 + xx) + rowR, v);
@@ -269,7 +272,8 @@ int update_syrk_dmma(int64_t nb, int64_t ntk, const double* L21, int64_t ldl, co
   a.nb = (int)nb;
   a.M2p = (int)((2 * ntk + 7) / 8 * 8);
   const int64_t Mt = a.M2p + (mags ? (ntk + 7) / 8 * 8 : 0);
-  const dim3 grid((unsigned)((Mt + kTM - 1) / kTM), (unsigned)(nk / kTN));
+  a.nk = (int)nk;
+  const dim3 grid((unsigned)((Mt + kTM - 1) / kTM), (unsigned)((nk + kTN - 1) / kTN));
   // small grids (the look-ahead's single tile column, late iterations) are
   // bound by the k-loop's latency, not by the DMMA rate: split K over a
   // cluster while the grid stays under ~4 CTAs per SM
