@@ -38,9 +38,11 @@ constexpr int kWarps = kThreads / 32;
 template <typename T, int NB, int K, bool VERIFY = false>
 struct PassCfg {
   static constexpr int RK = K * NB;              // rows per CTA
-  // group columns (slab granularity): 32 for NB >= 256, so that a single
-  // tile (the drivers' diagonal-tile checks) splits into NB/32 slab CTAs
-  static constexpr int GC = NB < 64 ? NB : (NB >= 256 ? 32 : 64);
+  // group columns (slab granularity).  (32-column groups for NB >= 256 were
+  // measured: single diagonal-tile checks 11.6 -> 7.8 us (LOWER col), 18.6
+  // -> 16.7 (SYM both), but 59-tile both-direction panels 31.9 -> 39.6 us
+  // from the doubled row-partial traffic; ft_potrf unchanged.)
+  static constexpr int GC = NB < 64 ? NB : 64;
   static constexpr int COL_BYTES = RK * (int)sizeof(T);
   // 32 KiB stages for every column size (fp64 nb=1024, 8-KiB columns, had
   // 16 KiB stages of 2 columns: the row-sum chunk CQ fell to 2 columns, the
