@@ -95,6 +95,20 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
+// 1-D TMA bulk copy shared -> global (bulk-group completion).
+__device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+// at most N of this thread's committed bulk groups may still be reading shared memory
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+// every committed bulk group of this thread is complete (writes performed)
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
 // --------------------------------------------------------------- math --
 // Explicit round-to-nearest ops so the compiler cannot re-contract: the
@@ -151,6 +165,14 @@ int panel_row_rule(int32_t dtype, int64_t rows, int64_t nb, const void* L, int64
 int update_syrk_dmma(int64_t nb, int64_t ntk, const double* L21, int64_t ldl, const double* cL, int64_t ldc,
                      const double* mL, int64_t ldcm, double* Cc, double* Rr, int64_t ldr, double* Cm, double* Rm,
                      int64_t ldrm, cudaStream_t s, int64_t ntc = -1);
+// abft_check (verify + locate in one launch) that also writes the checked
+// range's stored elements, as corrected, to ckpt (ld ldk; element (gi, gj)
+// of the range at ckpt[(gi - I0 nb) + (gj - J0 nb) ldk]): the drivers'
+// local-restart copy of an op's input (f1) folded into its pre-op check
+// (abft_pass.cu; a plain copy after the check when the ring cannot carry it)
+int check_ckpt(const abft_mat_t* mat, const abft_tiles_t* tiles, int32_t which, const abft_tol_t* tol,
+               const abft_report_t* report, abft_fix_t* fixes, int32_t max_fixes, int32_t* n_fixes, void* ckpt,
+               int64_t ldk, cudaStream_t s);
 // Free the per-stream pools (workspace, counters: abft_runtime.cu) and the
 // per-stream library handles and scratch (abft_update.cu) of a stream that is
 // about to be destroyed.  The stream must be idle.

@@ -36,6 +36,10 @@ struct LocArgs {
   int32_t* n_fixes;
   int64_t ntiles;
   const int32_t* gate;  // nullable: run only if *gate != 0
+  // drivers' local-restart checkpoint of the checked range (nullable): a
+  // data fix also lands at ckpt[(gi - I0 nb) + (gj - J0 nb) ldk]
+  void* ckpt;
+  int64_t ldk;
 };
 
 template <typename T>
@@ -491,6 +495,9 @@ __device__ __noinline__ void locate_tile(const LocArgs& p, int I, int J, int32_t
             *ptr = nv;
             int si, sj;
             X.stored(ac.i, ac.j, si, sj);
+            if (p.ckpt)
+              reinterpret_cast<T*>(p.ckpt)[((int64_t)(I - p.tiles.I0) * nb + si) +
+                                           ((int64_t)(J - p.tiles.J0) * nb + sj) * p.ldk] = nv;
             int slot = atomicAdd(p.n_fixes, 1);
             if (slot < p.max_fixes && p.fixes) {
               abft_fix_t f;

@@ -130,6 +130,12 @@ struct PassArgs {
   // locate_tile on it before exiting (no separate locate launch)
   int fuse;
   LocArgs loc;
+  // local-restart checkpoint (f1, drivers only): the producer also writes
+  // every landed stage's columns to ckpt (element (gi, gj) of the range at
+  // ckpt[(gi - I0 nb) + (gj - J0 nb) ldk]) with bulk shared->global copies,
+  // so the pre-op check and the copy of its input are one pass over HBM
+  void* ckpt;
+  int64_t ldk;
 };
 
 template <typename T, int VEC>
@@ -415,10 +421,26 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(const __grid_constant__ Pas
 
   // ------------------------------------------------------------ producer --
   if (warp == kWarps) {
+    T* ck = p.ckpt ? reinterpret_cast<T*>(p.ckpt) + ((int64_t)(Ib - p.tiles.I0) * NB) +
+                         ((int64_t)(J - p.tiles.J0) * NB) * p.ldk
+                   : nullptr;
     if (p.use_bulk && lane == 0) {
+      // checkpoint: once stage h has landed, its columns go back out to ck
+      auto store_stage = [&](int h) {
+        const int sl = h % C::NSTAGE;
+        mbar_wait(&full[sl], (uint32_t)((h / C::NSTAGE) & 1));
+        const T* sb = ring + (size_t)sl * C::STAGE_ELEMS;
+#pragma unroll 1
+        for (int cc = 0; cc < C::CC; ++cc)
+          bulk_s2g(ck + (int64_t)(c0 + h * C::CC + cc) * p.ldk, sb + cc * RK, RV * sizeof(T));
+        bulk_commit();
+      };
       for (int g = 0; g < nst; ++g) {
         const int slot = g % C::NSTAGE;
-        if (g >= C::NSTAGE) mbar_wait(&empty[slot], (uint32_t)(((g / C::NSTAGE) - 1) & 1));
+        if (g >= C::NSTAGE) {
+          mbar_wait(&empty[slot], (uint32_t)(((g / C::NSTAGE) - 1) & 1));
+          if (ck) bulk_wait_read<C::NSTAGE - 2>();  // stage g - NSTAGE's store has read the slot
+        }
         T* dst = ring + (size_t)slot * C::STAGE_ELEMS;
         fence_proxy_async();
         mbar_arrive_expect_tx(&full[slot], (uint32_t)(C::CC * RV * sizeof(T)));
@@ -426,8 +448,18 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(const __grid_constant__ Pas
 #pragma unroll 1
         for (int cc = 0; cc < C::CC; ++cc)
           bulk_g2s(dst + cc * RK, src + (int64_t)cc * p.lda, RV * sizeof(T), &full[slot]);
+        if (ck && g >= 1) store_stage(g - 1);
+      }
+      if (ck) {
+        store_stage(nst - 1);
+        bulk_wait_all();
+        asm volatile("fence.proxy.async.global;" ::: "memory");
+        __threadfence();
       }
     }
+    // the checkpoint is complete before this CTA's tile can be finished (and
+    // corrected by the fused locate, which patches the checkpoint too)
+    if (ck) asm volatile("bar.sync 2, %0;" ::"n"(kBlock) : "memory");
     return;
   }
 
@@ -657,6 +689,7 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(const __grid_constant__ Pas
       }
     }
   }
+  if (p.ckpt) asm volatile("bar.sync 2, %0;" ::"n"(kBlock) : "memory");  // the producer's checkpoint stores are done
   // ---------------- slab reduction: last CTA finishes the unit ------------
   if (nslab > 1) {
     __threadfence();
@@ -926,7 +959,8 @@ int validate_mat(const abft_mat_t* m, const abft_tiles_t* t, int which) {
 }
 
 static int run_pass(const abft_mat_t* m, const abft_tiles_t* t, int which, const abft_tol_t* tol,
-                    const abft_report_t* rep, cudaStream_t s, bool verify, const LocArgs* loc = nullptr) {
+                    const abft_report_t* rep, cudaStream_t s, bool verify, const LocArgs* loc = nullptr,
+                    void* ckpt = nullptr, int64_t ldk = 0) {
   int rc = validate_mat(m, t, which);
   if (rc) return rc;
   const int64_t ntiles = tiles_count(*t);
@@ -962,18 +996,46 @@ static int run_pass(const abft_mat_t* m, const abft_tiles_t* t, int which, const
     a.drow = rep->drow;
     a.counts = rep->counts;
   }
+  // the checkpoint rides on the bulk-copy ring (16-B aligned columns)
+  const bool ck_fused = ckpt && a.use_bulk && (uintptr_t)ckpt % 16 == 0 && (ldk * (int64_t)es) % 16 == 0;
   if (loc) {
     a.fuse = 1;
     a.loc = *loc;
+    if (ck_fused) {
+      a.loc.ckpt = ckpt;
+      a.loc.ldk = ldk;
+    }
+  }
+  if (ck_fused) {
+    a.ckpt = ckpt;
+    a.ldk = ldk;
   }
   g_fuse_missed = false;
   if (m->dtype == ABFT_F64)
     rc = verify ? launch_t<double, true>(a, m->nb, ntiles, s) : launch_t<double, false>(a, m->nb, ntiles, s);
   else
     rc = verify ? launch_t<float, true>(a, m->nb, ntiles, s) : launch_t<float, false>(a, m->nb, ntiles, s);
-  if (rc || !loc || !g_fuse_missed) return rc;
-  LocArgs la = *loc;
-  return launch_locate_args(la, m->dtype, s);
+  if (rc) return rc;
+  if (loc && g_fuse_missed) {
+    LocArgs la = a.loc;
+    rc = launch_locate_args(la, m->dtype, s);
+    if (rc) return rc;
+  }
+  if (ckpt && !ck_fused) {  // the checkpoint as a plain copy of the checked (and corrected) range
+    const int64_t nb = m->nb;
+    return copy2d(ckpt, ldk * es, (const char*)m->A + ((int64_t)t->I0 * nb + (int64_t)t->J0 * nb * m->lda) * es,
+                  m->lda * es, (size_t)(t->I1 - t->I0) * nb * es, (size_t)(t->J1 - t->J0) * nb, s);
+  }
+  return 0;
+}
+
+int check_ckpt(const abft_mat_t* mat, const abft_tiles_t* tiles, int32_t which, const abft_tol_t* tol,
+               const abft_report_t* report, abft_fix_t* fixes, int32_t max_fixes, int32_t* n_fixes, void* ckpt,
+               int64_t ldk, cudaStream_t s) {
+  LocArgs la;
+  const int rc = fill_loc_args(la, mat, tiles, which, tol, report, fixes, max_fixes, n_fixes);
+  if (rc) return rc;
+  return run_pass(mat, tiles, which, tol, report, s, true, &la, ckpt, ldk);
 }
 
 }  // namespace abft

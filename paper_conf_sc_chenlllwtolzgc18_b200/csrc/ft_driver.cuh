@@ -173,7 +173,8 @@ struct Driver {
     if (c->side) return 0;
     int lo = 0, hi = 0;
     ABFT_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-    ABFT_CUDA_TRY(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, hi));
+    static const bool low = getenv("ABFT_SIDE_LOW") != nullptr;  // priority experiments
+    ABFT_CUDA_TRY(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, low ? lo : hi));
     ABFT_CUDA_TRY(cudaEventCreateWithFlags(&c->ev_col, cudaEventDisableTiming));
     ABFT_CUDA_TRY(cudaEventCreateWithFlags(&c->ev_side, cudaEventDisableTiming));
     return 0;
@@ -357,8 +358,11 @@ struct Driver {
     onchip_pending.clear();
     return 0;
   }
+  // ckpt (nullable): also leave a copy of the checked range's data, as
+  // corrected by the check, at ckpt (ld ldk) — the local-restart copy of the
+  // next op's input (f1), written by the check's own pass when it can be
   int check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only = false,
-            cudaStream_t on = nullptr);
+            cudaStream_t on = nullptr, void* ckpt = nullptr, int64_t ldk = 0);
   // ABFT_DIAG_SKIP (timing diagnostics only; results are then unprotected):
   // bit 0 skips the checks issued on the main stream, bit 1 those on the
   // look-ahead side stream, bit 2 the TMU checksum rule, bit 3 the PD / PU rules
@@ -366,13 +370,22 @@ struct Driver {
     static const int v = getenv("ABFT_DIAG_SKIP") ? atoi(getenv("ABFT_DIAG_SKIP")) : 0;
     return v;
   }
-  int check_impl(int I0, int I1, int J0, int J1, int view, int which, bool lower_only, cudaStream_t on) {
-    if (diag_skip() & (s == s_main && !on ? 1 : 2)) return 0;
+  int check_impl(int I0, int I1, int J0, int J1, int view, int which, bool lower_only, cudaStream_t on, void* ckpt,
+                 int64_t ldk) {
     abft_tiles_t t{I0, I1, J0, J1, lower_only ? 1 : 0, view};
     const abft_stream_t st = (abft_stream_t)(on ? on : s);
+    auto plain_copy = [&]() -> int {
+      if (!ckpt) return 0;
+      return abft::copy2d(ckpt, ldk * es, a_at((int64_t)I0 * nb, (int64_t)J0 * nb), lda * es,
+                          (size_t)(I1 - I0) * nb * es, (size_t)(J1 - J0) * nb, (cudaStream_t)st);
+    };
+    if (diag_skip() & (s == s_main && !on ? 1 : 2)) return plain_copy();
     if (o->checksum_gemm) {  // prior-art GEMM recalculation (f3 baseline)
       FT_TRY(abft_verify_gemm(&M, &t, which, &tol, &R, st));
       FT_TRY(abft_locate_correct(&M, &t, which, &tol, &R, c->fixlog, c->fixcap, nfix, st));
+      FT_TRY(plain_copy());
+    } else if (ckpt) {  // verify + locate + checkpoint in one pass
+      FT_TRY(check_ckpt(&M, &t, which, &tol, &R, c->fixlog, c->fixcap, nfix, ckpt, ldk, (cudaStream_t)st));
     } else {  // verify + locate in one launch
       FT_TRY(abft_check(&M, &t, which, &tol, &R, c->fixlog, c->fixcap, nfix, st));
     }
@@ -559,9 +572,10 @@ struct PhaseScope {
   }
 };
 
-inline int Driver::check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only, cudaStream_t on) {
+inline int Driver::check(int I0, int I1, int J0, int J1, int view, int which, bool lower_only, cudaStream_t on,
+                          void* ckpt, int64_t ldk) {
   PhaseScope ps(*this, FT_PH_CHECKS);
-  return check_impl(I0, I1, J0, J1, view, which, lower_only, on);
+  return check_impl(I0, I1, J0, J1, view, which, lower_only, on, ckpt, ldk);
 }
 
 // FT_PD_HOST (ft_host.cu): Alg. 2 lines 3-7 for the panel of iteration k,

@@ -301,9 +301,6 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     const int64_t nk = n - r1;    // trailing size
     const int m2 = (int)(2 * (nt - k - 1));
     if (ft) FT_TRY(d.begin_iteration());
-    // Alg. 2 lines 3-4: check the panel to be decomposed (diag tile, SYM view, both)
-    FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
-    if (ft && pre_checks) FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_SYM_LOWER, W));
     char* rbuf = (char*)c->rsv;
     auto copy2d = [&](void* dst, int64_t ldd, const void* src, int64_t lds, int64_t rows, int64_t cols) -> int {
       if (rows <= 0 || cols <= 0) return 0;
@@ -321,9 +318,16 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     // read the difference back into pinned memory after it (one event)
     auto post_readback = [&]() -> int { return d.post_delta(0); };
     auto readback_delta = [&](int* delta) -> int { return d.wait_delta(0, delta); };
+    // Alg. 2 lines 3-4: check the panel to be decomposed (diag tile, SYM view,
+    // both); with local restart the check's pass also leaves the PD input's
+    // copy (f1, L430) in pd_a
+    FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
+    const bool ck_pd = rs && pre_checks;
+    if (ft && pre_checks)
+      FT_TRY(d.check(k, k + 1, k, k + 1, ABFT_SYM_LOWER, W, false, nullptr, ck_pd ? pd_a : nullptr, nb));
     if (rs) {
       PhaseScope ps(d, FT_PH_RESTART);
-      FT_TRY(copy2d(pd_a, nb, d.a_at(r0, r0), lda, nb, nb));
+      if (!ck_pd) FT_TRY(copy2d(pd_a, nb, d.a_at(r0, r0), lda, nb, nb));
       FT_TRY(copy2d(pd_c, 2, d.colchk_at(2 * k, r0), d.M.ldc, 2, nb));
       FT_TRY(copy2d(pd_m, 1, d.colmag_at(k, r0), d.M.ldcm, 1, nb));
     }
@@ -382,10 +386,12 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (k == nt - 1) return 0;
     // line 8: check the panel to be updated (both checksums)
     FT_TRY(d.inject_at(k, FT_AT_PRE_PU_CHECK));
-    if (ft && pre_checks) FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, W));
+    const bool ck_pu = rs && pre_checks;  // the check's pass leaves the PU input's copy in pu_a
+    if (ft && pre_checks)
+      FT_TRY(d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, W, false, nullptr, ck_pu ? pu_a : nullptr, nk));
     if (rs) {
       PhaseScope ps(d, FT_PH_RESTART);
-      FT_TRY(copy2d(pu_a, nk, d.a_at(r1, r0), lda, nk, nb));
+      if (!ck_pu) FT_TRY(copy2d(pu_a, nk, d.a_at(r1, r0), lda, nk, nb));
       FT_TRY(copy2d(pu_c, m2, d.colchk_at(2 * (k + 1), r0), d.M.ldc, m2, nb));
       FT_TRY(copy2d(pu_m, m2 / 2, d.colmag_at(k + 1, r0), d.M.ldcm, m2 / 2, nb));
     }

@@ -121,6 +121,27 @@ def test_fault_campaign_parity(lib, ctx, case, lookahead):
     _compare(lib, ctx, A, 32, [dr.Inject(2, point, kind, target, gi, gj, bits)], lookahead=lookahead)
 
 
+# Two faults in one iteration: the first is corrected by a pre-op check, the
+# second forces the local restart of that op (L430).  The restart restores the
+# op's input from the copy the pre-op check's own pass left behind
+# (ft_driver.cuh check(ckpt)): that copy must hold the CORRECTED element, as
+# the oracle's copy taken after the check does.
+DOUBLE_CASES = [
+    [(dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 0, 70, 66, (61,)), (dr.AT_PRE_PD, dr.KIND_PERSIST, 0, 75, 70, (57,))],
+    [(dr.AT_PRE_PU_CHECK, dr.KIND_PERSIST, 0, 200, 70, (60,)), (dr.AT_PRE_PU, dr.KIND_ONCHIP, 0, 70, 66, (60,))],
+    [(dr.AT_PRE_PU_CHECK, dr.KIND_PERSIST, 0, 131, 77, (59,)), (dr.AT_POST_PU, dr.KIND_PERSIST, 0, 150, 90, (63,)),
+     (dr.AT_POST_PU, dr.KIND_PERSIST, 0, 155, 93, (62,))],
+]
+
+
+@pytest.mark.parametrize("lookahead", [True, False])
+@pytest.mark.parametrize("case", range(len(DOUBLE_CASES)))
+def test_restart_from_check_checkpoint(lib, ctx, case, lookahead):
+    A = si.spd(256, seed=0)
+    so, sg = _compare(lib, ctx, A, 32, [dr.Inject(2, *c) for c in DOUBLE_CASES[case]], lookahead=lookahead)
+    assert so.restarts >= 1 and sg.restarts == so.restarts
+
+
 # fp32 (every entry point takes ABFT_F32; BASELINE's 1e-5): the same fault
 # kinds with the flips moved into the fp32 word (fp64 bit b -> b - 32: the
 # exponent/sign bits stay exponent/sign bits, 52-54 become mantissa 20-22)
