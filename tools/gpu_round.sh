@@ -31,3 +31,7 @@ ABFT_ITER_EVENTS=1 python tools/iter_time.py 30720 512 potrf 2> $out/iter_potrf.
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:checksum_pass -s 2 -c 2 \
    -o $out/prof_pass -f python bench.py --steps 1 --warmup 1 --no-e2e --no-potrf --no-cpu --no-lu-qr --no-mgpu \
    > $out/ncu_full.log 2>&1
+for sk in 0 1 2 3 7 15; do ABFT_DIAG_SKIP=$sk python tools/diag_time.py 30720 512 3 2>&1 | grep skip; done > $out/diag_skip.log
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:dmma -s 1 -c 1 -o $out/prof_rule -f \
+   python tools/rule_ncu.py 59 > $out/ncu_rule.log 2>&1
+python tools/small_pass.py > $out/small_pass.log 2>&1
