@@ -155,6 +155,26 @@ int copy2d(void* dst, size_t dpitch, const void* src, size_t spitch, size_t widt
 // returning at once when *gate == 0 (abft_gated.cu; the local-restart redo).
 int gemm_gated(int32_t dtype, bool ta, bool tb, bool absa, bool absb, int64_t M, int64_t N, int64_t K, const void* A,
                int64_t lda, const void* B, int64_t ldb, void* C, int64_t ldc, const int32_t* gate, cudaStream_t s);
+struct GatedGemm {
+  int64_t M, N, K;
+  const void* A;
+  int64_t lda;
+  const void* B;
+  int64_t ldb;
+  void* C;
+  int64_t ldc;
+  int ta, tb, absa, absb;
+};
+// up to 3 gated products in one launch (same dtype and gate)
+int gemm_gated_multi(int32_t dtype, const GatedGemm* g, int n, const int32_t* gate, cudaStream_t s);
+// up to 4 2-D copies (as copy2d) in one launch; honours launch_gate()
+struct Copy2D {
+  void* dst;
+  size_t dpitch;
+  const void* src;
+  size_t spitch, width, height;
+};
+int copy2d_multi(const Copy2D* c, int n, cudaStream_t s);
 // Cholesky TMU row-checksum rule of one trailing tile column (look-ahead):
 // re/rw (rows) -= L (rows x nb) [ce cw] and rm += |L| mc, ce/cw/mc strided
 // (abft_update.cu).

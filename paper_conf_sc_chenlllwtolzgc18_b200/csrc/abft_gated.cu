@@ -12,16 +12,16 @@
 // of reading c-6) because a library GEMM cannot read a device gate; they run
 // for real only when a restart happens, so they are sized for correctness,
 // not for peak.
+#include <algorithm>
+
 #include "abft_common.cuh"
 
 namespace abft {
 
 template <typename T>
-__global__ void __launch_bounds__(256) gemm_gated_kernel(int64_t M, int64_t N, int64_t K, const T* __restrict__ A,
-                                                         int64_t lda, const T* __restrict__ B, int64_t ldb,
-                                                         T* __restrict__ C, int64_t ldc, int ta, int tb, int absa,
-                                                         int absb, const int32_t* gate) {
-  if (gate && *gate == 0) return;
+__device__ __forceinline__ void gemm_tile(int64_t M, int64_t N, int64_t K, const T* __restrict__ A, int64_t lda,
+                                          const T* __restrict__ B, int64_t ldb, T* __restrict__ C, int64_t ldc, int ta,
+                                          int tb, int absa, int absb) {
   __shared__ T As[16][64 + 1];
   __shared__ T Bs[16][64 + 1];
   const int64_t m0 = (int64_t)blockIdx.x * 64, n0 = (int64_t)blockIdx.y * 64;
@@ -68,18 +68,45 @@ __global__ void __launch_bounds__(256) gemm_gated_kernel(int64_t M, int64_t N, i
   }
 }
 
-int gemm_gated(int32_t dtype, bool ta, bool tb, bool absa, bool absb, int64_t M, int64_t N, int64_t K, const void* A,
-               int64_t lda, const void* B, int64_t ldb, void* C, int64_t ldc, const int32_t* gate, cudaStream_t s) {
-  if (M <= 0 || N <= 0) return 0;
-  const dim3 grid((unsigned)((M + 63) / 64), (unsigned)((N + 63) / 64));
+// up to 3 independent products per launch (blockIdx.z): the restart redo's
+// data, checksum and magnitude GEMMs are one gated launch
+struct GatedBatch {
+  GatedGemm g[3];
+  int n;
+};
+
+template <typename T>
+__global__ void __launch_bounds__(256) gemm_gated_kernel(const __grid_constant__ GatedBatch b, const int32_t* gate) {
+  if (gate && *gate == 0) return;
+  const GatedGemm& q = b.g[blockIdx.z];
+  if ((int64_t)blockIdx.x * 64 >= q.M || (int64_t)blockIdx.y * 64 >= q.N) return;  // uniform per CTA
+  gemm_tile<T>(q.M, q.N, q.K, reinterpret_cast<const T*>(q.A), q.lda, reinterpret_cast<const T*>(q.B), q.ldb,
+               reinterpret_cast<T*>(q.C), q.ldc, q.ta, q.tb, q.absa, q.absb);
+}
+
+int gemm_gated_multi(int32_t dtype, const GatedGemm* g, int n, const int32_t* gate, cudaStream_t s) {
+  GatedBatch b{};
+  int64_t gx = 0, gy = 0;
+  for (int i = 0; i < n; ++i) {
+    if (g[i].M <= 0 || g[i].N <= 0) continue;
+    b.g[b.n++] = g[i];
+    gx = std::max<int64_t>(gx, (g[i].M + 63) / 64);
+    gy = std::max<int64_t>(gy, (g[i].N + 63) / 64);
+  }
+  if (b.n == 0) return 0;
+  const dim3 grid((unsigned)gx, (unsigned)gy, (unsigned)b.n);
   if (dtype == ABFT_F64)
-    gemm_gated_kernel<double><<<grid, 256, 0, s>>>(M, N, K, (const double*)A, lda, (const double*)B, ldb, (double*)C,
-                                                   ldc, ta, tb, absa, absb, gate);
+    gemm_gated_kernel<double><<<grid, 256, 0, s>>>(b, gate);
   else
-    gemm_gated_kernel<float><<<grid, 256, 0, s>>>(M, N, K, (const float*)A, lda, (const float*)B, ldb, (float*)C, ldc,
-                                                  ta, tb, absa, absb, gate);
+    gemm_gated_kernel<float><<<grid, 256, 0, s>>>(b, gate);
   ABFT_CUDA_TRY(cudaGetLastError());
   return 0;
+}
+
+int gemm_gated(int32_t dtype, bool ta, bool tb, bool absa, bool absb, int64_t M, int64_t N, int64_t K, const void* A,
+               int64_t lda, const void* B, int64_t ldb, void* C, int64_t ldc, const int32_t* gate, cudaStream_t s) {
+  const GatedGemm g{M, N, K, A, lda, B, ldb, C, ldc, ta, tb, absa, absb};
+  return gemm_gated_multi(dtype, &g, 1, gate, s);
 }
 
 }  // namespace abft

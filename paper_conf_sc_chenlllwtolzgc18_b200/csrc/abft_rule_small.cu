@@ -33,7 +33,7 @@ namespace {
 
 constexpr int kVB = 32;   // vectors per cluster (rows of the product)
 constexpr int kJB = 32;   // output columns per CTA
-constexpr int kBK = 16;   // q per stage
+constexpr int kBK = 32;   // q per stage (16 measured: 32 dependent stages, 18 us per launch)
 constexpr int kStages = 4;
 constexpr int kThr = 128;  // 4 warps: 2 (vectors, 16 each) x 2 (columns, 16 each)
 constexpr int kLd = kVB + 4;  // stage row stride (doubles): 4 (mod 16) keeps fragments conflict-free
@@ -70,9 +70,12 @@ __device__ __forceinline__ void dmma(double (&d)[2], double a, double b) {
                : "d"(a), "d"(b));
 }
 
+constexpr size_t kSmem = 2 * (size_t)kStages * kBK * kLd * sizeof(double);
+
 __global__ void __launch_bounds__(kThr) trsm_inv_rule_kernel(const __grid_constant__ SmallRuleArgs a) {
-  __shared__ __align__(16) double Vs[kStages][kBK][kLd];  // [q][v]
-  __shared__ __align__(16) double Ms[kStages][kBK][kLd];  // [q][j]
+  extern __shared__ __align__(16) double rs_sm[];
+  double(*Vs)[kBK][kLd] = reinterpret_cast<double(*)[kBK][kLd]>(rs_sm);                         // [q][v]
+  double(*Ms)[kBK][kLd] = reinterpret_cast<double(*)[kBK][kLd]>(rs_sm + kStages * kBK * kLd);  // [q][j]
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int wv = warp & 1, wj = warp >> 1;
   const int g = lane >> 2, t = lane & 3;
@@ -86,12 +89,12 @@ __global__ void __launch_bounds__(kThr) trsm_inv_rule_kernel(const __grid_consta
   const int j0 = blockIdx.x * kJB;
   const int64_t sv = a.sideR ? 1 : ld, sq = a.sideR ? ld : 1;  // vector / q strides of base
   const int64_t mj = a.tW ? 1 : a.ldw, mq = a.tW ? a.ldw : 1;  // column / q strides of M in W
-  // fill roles: 128 threads x 4 elements per operand per stage (16 q x 32);
+  // fill roles: 128 threads x 8 elements per operand per stage (32 q x 32);
   // the contiguous index of each operand runs fastest over the threads
   auto fill = [&](int kt, int st) {
     const int q0 = kt * kBK;
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < kBK * kVB / kThr; ++u) {
       const int idx = tid + u * kThr;
       int x, qq;  // V: x = vector
       if (a.sideR) {
@@ -192,12 +195,13 @@ int trsm_inv_rule(char side, char trans, int64_t nb, const double* W, int64_t ld
   static bool attr = false;
   if (!attr) {
     ABFT_CUDA_TRY(cudaFuncSetAttribute(trsm_inv_rule_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+    ABFT_CUDA_TRY(cudaFuncSetAttribute(trsm_inv_rule_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmem));
     attr = true;
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(cs, (unsigned)nblk, 1);
   cfg.blockDim = dim3(kThr, 1, 1);
-  cfg.dynamicSmemBytes = 0;
+  cfg.dynamicSmemBytes = kSmem;
   cfg.stream = s;
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeClusterDimension;

@@ -788,12 +788,12 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       auto pu_redo = [&](const int32_t* g) -> int {
         {
           PhaseScope ps(d, FT_PH_RESTART);
-          FT_TRY(gemm_gated(dtype, false, false, false, false, nb, nk, nb, c->linv, nb, pu_a, nb, d.a_at(r0, r1), lda,
-                            g, s));
-          FT_TRY(gemm_gated(dtype, false, false, false, false, nb, m2, nb, c->linv, nb, pu_r, nb,
-                            d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, g, s));
-          FT_TRY(gemm_gated(dtype, false, false, true, false, nb, m2 / 2, nb, c->linv, nb, pu_rm, nb,
-                            d.rowmag_at(r0, k + 1), d.M.ldrm, g, s));
+          // data, checksum and magnitude products as one gated launch
+          const GatedGemm gg[3] = {{nb, nk, nb, c->linv, nb, pu_a, nb, d.a_at(r0, r1), lda, 0, 0, 0, 0},
+                                   {nb, m2, nb, c->linv, nb, pu_r, nb, d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, 0, 0, 0, 0},
+                                   {nb, m2 / 2, nb, c->linv, nb, pu_rm, nb, d.rowmag_at(r0, k + 1), d.M.ldrm, 0, 0, 1,
+                                    0}};
+          FT_TRY(gemm_gated_multi(dtype, gg, 3, g, s));
         }
         return d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_ROW);
       };

@@ -8,6 +8,9 @@
 // before/after PD), c-25 (guarded Fig. 4a trailing repair), c-8 (fault hooks).
 #include <dlfcn.h>
 
+#include <initializer_list>
+#include <tuple>
+
 #include "ft_driver.cuh"
 
 // ------------------------------------------------------------ panel potrf --
@@ -314,6 +317,15 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     char* pu_a = pd_m + (size_t)nb * d.es;
     char* pu_c = pu_a + (size_t)nk * nb * d.es;
     char* pu_m = pu_c + (size_t)m2 * nb * d.es;
+    // several restart copies as one launch: (dst, ldd, src, lds, rows, cols) in elements
+    auto copies = [&](std::initializer_list<std::tuple<void*, int64_t, const void*, int64_t, int64_t, int64_t>> l) {
+      Copy2D cs[4];
+      int n = 0;
+      for (const auto& t : l)
+        cs[n++] = Copy2D{std::get<0>(t), (size_t)std::get<1>(t) * d.es, std::get<2>(t), (size_t)std::get<3>(t) * d.es,
+                         (size_t)std::get<4>(t) * d.es, (size_t)std::get<5>(t)};
+      return copy2d_multi(cs, n, s);
+    };
     // PD restart decision: snapshot the uncorrectable count before the check,
     // read the difference back into pinned memory after it (one event)
     auto post_readback = [&]() -> int { return d.post_delta(0); };
@@ -328,8 +340,7 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (rs) {
       PhaseScope ps(d, FT_PH_RESTART);
       if (!ck_pd) FT_TRY(copy2d(pd_a, nb, d.a_at(r0, r0), lda, nb, nb));
-      FT_TRY(copy2d(pd_c, 2, d.colchk_at(2 * k, r0), d.M.ldc, 2, nb));
-      FT_TRY(copy2d(pd_m, 1, d.colmag_at(k, r0), d.M.ldcm, 1, nb));
+      FT_TRY(copies({{pd_c, 2, d.colchk_at(2 * k, r0), d.M.ldc, 2, nb}, {pd_m, 1, d.colmag_at(k, r0), d.M.ldcm, 1, nb}}));
     }
     auto do_pd = [&]() -> int {
       PhaseScope ps(d, FT_PH_PD);
@@ -376,9 +387,9 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       if (delta <= 0) return 0;
       ++d.restarts;
       add_i32_kernel<<<1, 1, 0, s>>>(d.counts + ABFT_CNT_UNCORRECTABLE, -delta);
-      FT_TRY(copy2d(d.a_at(r0, r0), lda, pd_a, nb, nb, nb));
-      FT_TRY(copy2d(d.colchk_at(2 * k, r0), d.M.ldc, pd_c, 2, 2, nb));
-      FT_TRY(copy2d(d.colmag_at(k, r0), d.M.ldcm, pd_m, 1, 1, nb));
+      FT_TRY(copies({{d.a_at(r0, r0), lda, pd_a, nb, nb, nb},
+                     {d.colchk_at(2 * k, r0), d.M.ldc, pd_c, 2, 2, nb},
+                     {d.colmag_at(k, r0), d.M.ldcm, pd_m, 1, 1, nb}}));
       FT_TRY(do_pd());
       return d.check(k, k + 1, k, k + 1, ABFT_LOWER, ABFT_COL);
     };
@@ -392,8 +403,8 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     if (rs) {
       PhaseScope ps(d, FT_PH_RESTART);
       if (!ck_pu) FT_TRY(copy2d(pu_a, nk, d.a_at(r1, r0), lda, nk, nb));
-      FT_TRY(copy2d(pu_c, m2, d.colchk_at(2 * (k + 1), r0), d.M.ldc, m2, nb));
-      FT_TRY(copy2d(pu_m, m2 / 2, d.colmag_at(k + 1, r0), d.M.ldcm, m2 / 2, nb));
+      FT_TRY(copies({{pu_c, m2, d.colchk_at(2 * (k + 1), r0), d.M.ldc, m2, nb},
+                     {pu_m, m2 / 2, d.colmag_at(k + 1, r0), d.M.ldcm, m2 / 2, nb}}));
     }
     if (defer_pd) FT_TRY(pd_restart());
     // Fig. 4b (L359): a 1D pattern fixed by this iteration's pre-PD / pre-PU
@@ -469,12 +480,12 @@ extern "C" int ft_potrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       auto pu_redo = [&](const int32_t* g) -> int {
         {
           PhaseScope ps(d, FT_PH_RESTART);
-          FT_TRY(gemm_gated(dtype, false, true, false, false, nk, nb, nb, pu_a, nk, c->linv, nb, d.a_at(r1, r0), lda,
-                            g, s));
-          FT_TRY(gemm_gated(dtype, false, true, false, false, m2, nb, nb, pu_c, m2, c->linv, nb,
-                            d.colchk_at(2 * (k + 1), r0), d.M.ldc, g, s));
-          FT_TRY(gemm_gated(dtype, false, true, false, true, m2 / 2, nb, nb, pu_m, m2 / 2, c->linv, nb,
-                            d.colmag_at(k + 1, r0), d.M.ldcm, g, s));
+          // data, checksum and magnitude products as one gated launch
+          const GatedGemm gg[3] = {{nk, nb, nb, pu_a, nk, c->linv, nb, d.a_at(r1, r0), lda, 0, 1, 0, 0},
+                                   {m2, nb, nb, pu_c, m2, c->linv, nb, d.colchk_at(2 * (k + 1), r0), d.M.ldc, 0, 1, 0, 0},
+                                   {m2 / 2, nb, nb, pu_m, m2 / 2, c->linv, nb, d.colmag_at(k + 1, r0), d.M.ldcm, 0, 1,
+                                    0, 1}};
+          FT_TRY(gemm_gated_multi(dtype, gg, 3, g, s));
         }
         return d.check(k + 1, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_COL);
       };
