@@ -165,6 +165,11 @@ struct GatedGemm {
   int64_t ldc;
   int ta, tb, absa, absb;
 };
+// fp64 abft_update_gemm on the DMMA rule kernel (abft_rule_dmma.cu);
+// ABFT_E_UNSUPPORTED for shapes it does not take
+int update_gemm_dmma(int which, char transX, char transY, double alpha, const double* X, int64_t ldx,
+                     const double* Y, int64_t ldy, double* C, int64_t ldcc, int64_t M2, int64_t N, int64_t K,
+                     const double* Xm, int64_t ldxm, double* Cm, int64_t ldcm, cudaStream_t s);
 // up to 3 gated products in one launch (same dtype and gate)
 int gemm_gated_multi(int32_t dtype, const GatedGemm* g, int n, const int32_t* gate, cudaStream_t s);
 // up to 4 2-D copies (as copy2d) in one launch; honours launch_gate()

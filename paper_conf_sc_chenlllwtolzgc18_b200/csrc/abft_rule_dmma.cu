@@ -47,23 +47,32 @@ constexpr int kLdB = kTN + 4;
 constexpr size_t kRuleSmem = (size_t)kStages * kBK * (kLdA + kLdB) * sizeof(double);
 
 struct RuleArgs {
-  const double* L;  // L21, nk x nb, ld ldl
-  int64_t ldl;
-  const double* cL;  // c(L21): M2 x nb, ld ldc
-  int64_t ldc;
-  const double* mL;  // m_c(L21): ntk x nb, ld ldcm (nullable: no Q)
-  int64_t ldcm;
-  double* Cc;  // c of the trailing tiles, ld ldc
-  double* Rr;  // r, ld ldr (nullable)
-  int64_t ldr;
-  double* Cm;  // m_c, ld ldcm (nullable)
-  double* Rm;  // m_r, ld ldrm (nullable)
-  int64_t ldrm;
-  int ntk;
-  int nb;
-  int M2p;    // checksum rows padded to 8 (magnitude rows start here)
+  // the product P = A B, A = [checksum rows (M2); pad to M2p; magnitude rows (M)]
+  const double* X;  // A(y, k) = X[y xy + k xk], y < M2
+  int64_t xy, xk;
+  const double* Xm;  // A(M2p + q, k) = Xm[q my + k mk], q < M (nullable: no magnitude rows)
+  int64_t my, mk;
+  const double* Y;  // B(k, x) = Y[k yk + x yx]; the magnitude rows take |B|
+  int64_t yk, yx;
+  int M2, M, M2p;
+  int N, K;   // columns and depth of the product
   int split;  // K split over a (1, 1, split) cluster (small grids), partials reduced in rank order
-  int nk;     // columns of the product (rows of L21 used)
+  int mode;   // 0: Cholesky scatter (c / r of the lower tiles, below); 1: plain (C, Cmo)
+  // mode 0: c(A_IJ) -= P[2I.., cols of J] (I >= J), r(A_IJ) -= P[2J.., cols of I]^T,
+  // m_c += Q[I, cols of J], m_r += Q[J, cols of I]^T
+  double* Cc;  // c of the trailing tiles, ld oldc
+  double* Rr;  // r, ld ldr (nullable)
+  int64_t oldc, ldr;
+  double* Cm;  // m_c, ld oldcm (nullable)
+  double* Rm;  // m_r, ld ldrm (nullable)
+  int64_t oldcm, ldrm;
+  int nb;
+  // mode 1: C[y cy + x cx] += alpha P(y, x), Cmo[q cmy + x cmx] += |alpha| Q(q, x)
+  double* C;
+  int64_t cy, cx;
+  double* Cmo;
+  int64_t cmy, cmx;
+  double alpha;
 };
 
 __device__ __forceinline__ void cp_async8(void* smem, const void* gmem, bool valid) {
@@ -123,26 +132,44 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
   const int r0 = blockIdx.x * kTM;                // first row of A
   const int x0 = blockIdx.y * kTN;                // first column (row of L21)
   // this CTA's k-steps: all of them, or its rank's share of a K-split cluster
-  const int kall = p.nb / kBK, z = blockIdx.z;
+  const int kall = (p.K + kBK - 1) / kBK, z = blockIdx.z;
   const int kbeg = z * kall / p.split, ksteps = (z + 1) * kall / p.split - kbeg;
-  const int M2 = 2 * p.ntk;
-  // fill roles (fixed for the CTA): A row ra (k parity by half), L21 column cb
-  const int ra = tid % kTM, ka = tid / kTM;       // 2 threads per row: k = ka, ka + 2, ...
-  const int ya = r0 + ra, yqa = ya - p.M2p;
-  const bool isp = ya < M2, isq = p.mL && yqa >= 0 && yqa < p.ntk;
-  const double* srcA = isp ? p.cL + ya : (isq ? p.mL + yqa : p.cL);
-  const int64_t ldA = isp ? p.ldc : (isq ? p.ldcm : 0);
-  const int cb = tid % kTN, kbq = tid / kTN;      // 4 threads per column: k = kbq, kbq + 4, ...
-  const bool bok = x0 + cb < p.nk;
-  const double* srcB = p.L + (bok ? x0 + cb : 0);
+  const int M2 = p.M2;
+  // fill roles (fixed for the CTA), the contiguous index of each operand
+  // fastest over the threads: A 64 rows x 16 k (8 loads), B 16 k x 32 x (4)
+  const bool akf = p.xk == 1, bkf = p.yk == 1;
+  auto a_src = [&](int y, int64_t k, bool& ok) -> const double* {
+    const int q = y - p.M2p;
+    if (y < M2 && k < p.K) {
+      ok = true;
+      return p.X + y * p.xy + k * p.xk;
+    }
+    if (p.Xm && q >= 0 && q < p.M && k < p.K) {
+      ok = true;
+      return p.Xm + q * p.my + k * p.mk;
+    }
+    ok = false;
+    return p.Y;  // any valid address (zero-filled)
+  };
   auto fill = [&](int kt, int st) {
     const int64_t kb = (int64_t)(kbeg + kt) * kBK;
-    double* as = As + (size_t)st * kBK * kLdA + ra;
+    double* as = As + (size_t)st * kBK * kLdA;
 #pragma unroll
-    for (int kk = ka; kk < kBK; kk += kThr / kTM) cp_async8(as + kk * kLdA, srcA + (kb + kk) * ldA, isp || isq);
-    double* bs = Bs + (size_t)st * kBK * kLdB + cb;
+    for (int u = 0; u < kTM * kBK / kThr; ++u) {
+      const int idx = tid + u * kThr;
+      const int rr = akf ? idx / kBK : idx % kTM, kk = akf ? idx % kBK : idx / kTM;
+      bool ok;
+      const double* src = a_src(r0 + rr, kb + kk, ok);
+      cp_async8(as + kk * kLdA + rr, src, ok);
+    }
+    double* bs = Bs + (size_t)st * kBK * kLdB;
 #pragma unroll
-    for (int kk = kbq; kk < kBK; kk += kThr / kTN) cp_async8(bs + kk * kLdB, srcB + (kb + kk) * p.ldl, bok);
+    for (int u = 0; u < kTN * kBK / kThr; ++u) {
+      const int idx = tid + u * kThr;
+      const int cc = bkf ? idx / kBK : idx % kTN, kk = bkf ? idx % kBK : idx / kTN;
+      const bool ok = x0 + cc < p.N && kb + kk < p.K;
+      cp_async8(bs + kk * kLdB + cc, ok ? p.Y + (kb + kk) * p.yk + (int64_t)(x0 + cc) * p.yx : p.Y, ok);
+    }
   };
 #pragma unroll
   for (int s = 0; s < kStages - 1; ++s) {
@@ -204,6 +231,29 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
     cl.sync();
     if (z != 0) return;
   }
+  if (p.mode == 1) {  // plain: C += alpha P, Cmo += |alpha| Q (one writer per element)
+    const double aa = fabs(p.alpha);
+#pragma unroll
+    for (int a = 0; a < kWM; ++a) {
+      const int y = wr0 + a * 8 + g;
+      const bool q = a >= aq;
+      const int yq = y - p.M2p;
+      if (!q && y >= M2) continue;
+      if (q && (!p.Cmo || yq >= p.M)) continue;
+#pragma unroll
+      for (int n = 0; n < kWN; ++n)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int x = x0 + wn * kWNC + n * 8 + 2 * t + h;
+          if (x >= p.N) continue;
+          if (q)
+            atomicAdd(p.Cmo + (int64_t)yq * p.cmy + (int64_t)x * p.cmx, aa * acc[a][n][h]);
+          else
+            atomicAdd(p.C + (int64_t)y * p.cy + (int64_t)x * p.cx, p.alpha * acc[a][n][h]);
+        }
+    }
+    return;
+  }
   // scatter: lane holds P/Q[y][x], [y][x+1] with y = wr0 + 8a + g,
   // x = x0 + 16 wn + 8n + 2t, tile column J = x / nb.  One writer per
   // element: a reduction adds exactly what load + add + store would.
@@ -213,11 +263,11 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
     const bool q = a >= aq;
     const int yq = y - p.M2p;
     if (!q && y >= M2) continue;
-    if (q && (!p.Cm || yq >= p.ntk)) continue;
+    if (q && (!p.Cm || yq >= p.M)) continue;
     const int I = q ? yq : y / 2;
     double* Cp = q ? p.Cm + yq : p.Cc + y;  // + x * ldC
     double* Rp = q ? p.Rm : p.Rr;           // + x + row * ldR
-    const int64_t ldC = q ? p.ldcm : p.ldc;
+    const int64_t ldC = q ? p.oldcm : p.oldc;
     const int64_t rowR = (int64_t)(q ? yq : y) * (q ? p.ldrm : p.ldr);
     const double sgn = q ? 1.0 : -1.0;
 #pragma unroll
@@ -225,7 +275,7 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         const int xx = wn * kWNC + n * 8 + 2 * t + h;
-        if (x0 + xx >= p.nk) continue;
+        if (x0 + xx >= p.N) continue;
         const int J = (x0 + xx) / p.nb;
         const double v = sgn * acc[a][n][h];
         if (I >= J) atomicAdd(Cp + (int64_t)(x0 + xx) * ldC, v);
@@ -234,52 +284,22 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
   }
 }
 
-}  // namespace
-
-// Returns ABFT_E_UNSUPPORTED when the shape is not covered (the caller takes
-// the cuBLAS route): nb must be a multiple of 32.  ntc < ntk restricts the
-// product to the first ntc tile columns (x < ntc nb; the look-ahead's single
-// tile column: ntc = 1 with Rr = Rm = null, c and m_c of every tile I >= J0).
-int update_syrk_dmma(int64_t nb, int64_t ntk, const double* L21, int64_t ldl, const double* cL, int64_t ldc,
-                     const double* mL, int64_t ldcm, double* Cc, double* Rr, int64_t ldr, double* Cm, double* Rm,
-                     int64_t ldrm, cudaStream_t s, int64_t ntc) {
-  if (nb % kTN || nb <= 0) return ABFT_E_UNSUPPORTED;
-  if (ntc < 0) ntc = ntk;
-  const int64_t nk = ntc * nb;  // columns: the first ntc tiles of L21's rows
-  if (nk == 0) return 0;
-  if (nk > (1LL << 30)) return ABFT_E_UNSUPPORTED;  // 32-bit column indices inside the kernel
+static int launch_rule(RuleArgs& a, cudaStream_t s) {
   static bool attr = false;
   if (!attr) {
     ABFT_CUDA_TRY(cudaFuncSetAttribute(syrk_rule_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)kRuleSmem));
     attr = true;
   }
-  RuleArgs a{};
-  a.L = L21;
-  a.ldl = ldl;
-  a.cL = cL;
-  a.ldc = ldc;
-  const bool mags = mL && Cm;
-  a.mL = mags ? mL : nullptr;
-  a.ldcm = ldcm;
-  a.Cc = Cc;
-  a.Rr = Rr;
-  a.ldr = ldr;
-  a.Cm = mags ? Cm : nullptr;
-  a.Rm = mags ? Rm : nullptr;
-  a.ldrm = ldrm;
-  a.ntk = (int)ntk;
-  a.nb = (int)nb;
-  a.M2p = (int)((2 * ntk + 7) / 8 * 8);
-  const int64_t Mt = a.M2p + (mags ? (ntk + 7) / 8 * 8 : 0);
-  a.nk = (int)nk;
-  const dim3 grid((unsigned)((Mt + kTM - 1) / kTM), (unsigned)((nk + kTN - 1) / kTN));
+  const int64_t Mt = a.M2p + (a.Xm ? (a.M + 7) / 8 * 8 : 0);
+  const dim3 grid((unsigned)((Mt + kTM - 1) / kTM), (unsigned)((a.N + kTN - 1) / kTN));
   // small grids (the look-ahead's single tile column, late iterations) are
   // bound by the k-loop's latency, not by the DMMA rate: split K over a
   // cluster while the grid stays under ~4 CTAs per SM
   const int64_t ctas = (int64_t)grid.x * grid.y;
+  const int kall = (a.K + kBK - 1) / kBK;
   int split = 1;
-  while (split < 8 && ctas * split * 2 <= 4 * 148 && (nb / kBK) % (split * 2) == 0) split *= 2;
+  while (split < 8 && ctas * split * 2 <= 4 * 148 && kall % (split * 2) == 0) split *= 2;
   a.split = split;
   if (split == 1) {
     syrk_rule_dmma_kernel<<<grid, kThr, kRuleSmem, s>>>(a);
@@ -300,6 +320,95 @@ int update_syrk_dmma(int64_t nb, int64_t ntk, const double* L21, int64_t ldl, co
   cfg.numAttrs = 1;
   ABFT_CUDA_TRY(cudaLaunchKernelEx(&cfg, syrk_rule_dmma_kernel, a));
   return 0;
+}
+
+}  // namespace
+
+// Returns ABFT_E_UNSUPPORTED when the shape is not covered (the caller takes
+// the cuBLAS route): nb must be a multiple of 32.  ntc < ntk restricts the
+// product to the first ntc tile columns (x < ntc nb; the look-ahead's single
+// tile column: ntc = 1 with Rr = Rm = null, c and m_c of every tile I >= J0).
+int update_syrk_dmma(int64_t nb, int64_t ntk, const double* L21, int64_t ldl, const double* cL, int64_t ldc,
+                     const double* mL, int64_t ldcm, double* Cc, double* Rr, int64_t ldr, double* Cm, double* Rm,
+                     int64_t ldrm, cudaStream_t s, int64_t ntc) {
+  if (nb % kTN || nb <= 0) return ABFT_E_UNSUPPORTED;
+  if (ntc < 0) ntc = ntk;
+  const int64_t nk = ntc * nb;  // columns: the first ntc tiles of L21's rows
+  if (nk == 0) return 0;
+  if (nk > (1LL << 30)) return ABFT_E_UNSUPPORTED;  // 32-bit column indices inside the kernel
+  RuleArgs a{};
+  const bool mags = mL && Cm;
+  a.X = cL;  // c(L21): 2 ntk x nb, ld ldc
+  a.xy = 1;
+  a.xk = ldc;
+  a.Xm = mags ? mL : nullptr;  // m_c(L21): ntk x nb, ld ldcm
+  a.my = 1;
+  a.mk = ldcm;
+  a.Y = L21;  // B(k, x) = L21[x, k]
+  a.yk = ldl;
+  a.yx = 1;
+  a.M2 = (int)(2 * ntk);
+  a.M = mags ? (int)ntk : 0;
+  a.M2p = (int)((2 * ntk + 7) / 8 * 8);
+  a.N = (int)nk;
+  a.K = (int)nb;
+  a.mode = 0;
+  a.Cc = Cc;
+  a.Rr = Rr;
+  a.oldc = ldc;
+  a.ldr = ldr;
+  a.Cm = mags ? Cm : nullptr;
+  a.Rm = mags ? Rm : nullptr;
+  a.oldcm = ldcm;
+  a.ldrm = ldrm;
+  a.nb = (int)nb;
+  return launch_rule(a, s);
+}
+
+// abft_update_gemm (a6) in fp64 on the same kernel: the COL rule
+//   C (M2 x N) += alpha op(X) op(Y),  Cm (M2/2 x N) += |alpha| op(Xm) |op(Y)|
+// and the ROW rule as its transpose
+//   C^T (M2 x N) += alpha op(X)^T op(Y)^T,  Cm^T += |alpha| op(Xm)^T |op(Y)^T|
+// (LU's c(A22) -= c(L21) U12 and r(A22) -= L21 r(U12), QR's c(A2) -= c(V) W
+// with their magnitudes, c-6 / c-13): one launch instead of the |op(Y)| copy
+// and two library GEMMs.
+int update_gemm_dmma(int which, char transX, char transY, double alpha, const double* X, int64_t ldx,
+                     const double* Y, int64_t ldy, double* C, int64_t ldcc, int64_t M2, int64_t N, int64_t K,
+                     const double* Xm, int64_t ldxm, double* Cm, int64_t ldcm, cudaStream_t s) {
+  if (M2 <= 0 || N <= 0) return 0;
+  if (N > (1LL << 30) || M2 > (1 << 20) || K > (1 << 20)) return ABFT_E_UNSUPPORTED;
+  const bool tX = transX == 'T' || transX == 't', tY = transY == 'T' || transY == 't';
+  const bool col = which == ABFT_COL;
+  RuleArgs a{};
+  const bool mags = Xm && Cm;
+  // A(y, k): COL op(X)(y, k); ROW op(X)(k, y)
+  const bool x_yfast = col ? !tX : tX;  // y runs along X's leading dimension
+  a.X = X;
+  a.xy = x_yfast ? 1 : ldx;
+  a.xk = x_yfast ? ldx : 1;
+  a.Xm = mags ? Xm : nullptr;
+  a.my = x_yfast ? 1 : ldxm;
+  a.mk = x_yfast ? ldxm : 1;
+  // B(k, x): COL op(Y)(k, x); ROW op(Y)(x, k)
+  const bool y_kfast = col ? !tY : tY;  // k runs along Y's leading dimension
+  a.Y = Y;
+  a.yk = y_kfast ? 1 : ldy;
+  a.yx = y_kfast ? ldy : 1;
+  a.M2 = (int)M2;
+  a.M = mags ? (int)(M2 / 2) : 0;
+  a.M2p = (int)((M2 + 7) / 8 * 8);
+  a.N = (int)N;
+  a.K = (int)K;
+  a.mode = 1;
+  a.C = C;
+  a.cy = col ? 1 : ldcc;
+  a.cx = col ? ldcc : 1;
+  a.Cmo = mags ? Cm : nullptr;
+  a.cmy = col ? 1 : ldcm;
+  a.cmx = col ? ldcm : 1;
+  a.alpha = alpha;
+  a.nb = 1;
+  return launch_rule(a, s);
 }
 
 }  // namespace abft

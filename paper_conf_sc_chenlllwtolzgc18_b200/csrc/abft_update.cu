@@ -517,6 +517,16 @@ int update_gemm_t(int which, char transX, char transY, double alpha, const void*
                   int64_t ldy, void* Cv, int64_t ldcc, int64_t M2, int64_t N, int64_t K, const void* Xmv,
                   int64_t ldxm, void* Cmv, int64_t ldcm, cudaStream_t s) {
   if (M2 == 0 || N == 0) return 0;
+  // fp64: one DMMA launch (abft_rule_dmma.cu); ABFT_RULE_CUBLAS=1 keeps the
+  // library route below (|op(Y)| copy + two GEMMs), as fp32 does
+  static const bool gemm_route = getenv("ABFT_RULE_CUBLAS") != nullptr;
+  if constexpr (std::is_same<T, double>::value) {
+    if (!gemm_route) {
+      const int r = update_gemm_dmma(which, transX, transY, alpha, (const double*)Xv, ldx, (const double*)Yv, ldy,
+                                     (double*)Cv, ldcc, M2, N, K, (const double*)Xmv, ldxm, (double*)Cmv, ldcm, s);
+      if (r != ABFT_E_UNSUPPORTED) return r;
+    }
+  }
   std::unique_lock<std::mutex> lk;
   cublasHandle_t h = blas_handle(s, lk);
   const T* X = reinterpret_cast<const T*>(Xv);

@@ -86,9 +86,12 @@ def test_update_trsm_inv_padded(lib, prec, side, trans, nb, nvec):
     assert np.abs(host(Md) - mref).max() <= tol * np.abs(mref).max()
 
 
-@pytest.mark.parametrize("which,tX,tY", [(1, "N", "T"), (2, "T", "N"), (1, "N", "N"), (2, "N", "N")])
-def test_update_gemm_matches_matmul(lib, which, tX, tY):
-    M2, N, K = 12, 96, 32
+# fp64 runs the DMMA rule kernel (abft_rule_dmma.cu, mode 1): a small case, a
+# ragged one (N, K off the 32 / 16 tiles), and a 60-tile LU panel's rule
+@pytest.mark.parametrize("M2,N,K", [(12, 96, 32), (6, 75, 40), (118, 2000, 512)])
+@pytest.mark.parametrize("which,tX,tY", [(1, "N", "T"), (2, "T", "N"), (1, "N", "N"), (2, "N", "N"), (1, "T", "N"),
+                                         (2, "N", "T"), (1, "T", "T"), (2, "T", "T")])
+def test_update_gemm_matches_matmul(lib, which, tX, tY, M2, N, K):
     X = si.general(*((M2, K) if (which == 1) == (tX == "N") else (K, M2)), seed=4)
     Y = si.general(*((K, N) if (which == 1) == (tY == "N") else (N, K)), seed=5)
     C = si.general(*((M2, N) if which == 1 else (N, M2)), seed=6)
