@@ -135,40 +135,69 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
   const int kall = (p.K + kBK - 1) / kBK, z = blockIdx.z;
   const int kbeg = z * kall / p.split, ksteps = (z + 1) * kall / p.split - kbeg;
   const int M2 = p.M2;
-  // fill roles (fixed for the CTA), the contiguous index of each operand
-  // fastest over the threads: A 64 rows x 16 k (8 loads), B 16 k x 32 x (4)
+  // fill roles, the contiguous index of each operand fastest over the
+  // threads: A 64 rows x 16 k (8 loads), B 16 k x 32 x (4 loads).  With rows
+  // (columns) fastest a thread keeps one row (column) for the whole loop, so
+  // its source pointer is computed once (the Cholesky and LU-COL shapes).
   const bool akf = p.xk == 1, bkf = p.yk == 1;
-  auto a_src = [&](int y, int64_t k, bool& ok) -> const double* {
+  auto a_row = [&](int y, const double*& src, int64_t& kst) -> bool {
     const int q = y - p.M2p;
-    if (y < M2 && k < p.K) {
-      ok = true;
-      return p.X + y * p.xy + k * p.xk;
+    if (y < M2) {
+      src = p.X + y * p.xy;
+      kst = p.xk;
+      return true;
     }
-    if (p.Xm && q >= 0 && q < p.M && k < p.K) {
-      ok = true;
-      return p.Xm + q * p.my + k * p.mk;
+    if (p.Xm && q >= 0 && q < p.M) {
+      src = p.Xm + q * p.my;
+      kst = p.mk;
+      return true;
     }
-    ok = false;
-    return p.Y;  // any valid address (zero-filled)
+    src = p.Y;  // any valid address (zero-filled)
+    kst = 0;
+    return false;
   };
+  const double* srcA0 = p.Y;
+  int64_t kA0 = 0;
+  const bool okA0 = akf ? false : a_row(r0 + tid % kTM, srcA0, kA0);
+  const int xb = tid % kTN;
+  const bool okB0 = !bkf && x0 + xb < p.N;
+  const double* srcB0 = p.Y + (okB0 ? (int64_t)(x0 + xb) * p.yx : 0);
   auto fill = [&](int kt, int st) {
     const int64_t kb = (int64_t)(kbeg + kt) * kBK;
     double* as = As + (size_t)st * kBK * kLdA;
+    if (!akf) {
+      const int ra = tid % kTM;
 #pragma unroll
-    for (int u = 0; u < kTM * kBK / kThr; ++u) {
-      const int idx = tid + u * kThr;
-      const int rr = akf ? idx / kBK : idx % kTM, kk = akf ? idx % kBK : idx / kTM;
-      bool ok;
-      const double* src = a_src(r0 + rr, kb + kk, ok);
-      cp_async8(as + kk * kLdA + rr, src, ok);
+      for (int u = 0; u < kTM * kBK / kThr; ++u) {
+        const int kk = tid / kTM + u * (kThr / kTM);
+        cp_async8(as + kk * kLdA + ra, srcA0 + (kb + kk) * kA0, okA0);
+      }
+    } else {
+      const int kk = tid % kBK;
+#pragma unroll 1
+      for (int u = 0; u < kTM * kBK / kThr; ++u) {
+        const int rr = tid / kBK + u * (kThr / kBK);
+        const double* src;
+        int64_t kst;
+        const bool ok = a_row(r0 + rr, src, kst);
+        cp_async8(as + kk * kLdA + rr, src + (kb + kk) * kst, ok);
+      }
     }
     double* bs = Bs + (size_t)st * kBK * kLdB;
+    if (!bkf) {
 #pragma unroll
-    for (int u = 0; u < kTN * kBK / kThr; ++u) {
-      const int idx = tid + u * kThr;
-      const int cc = bkf ? idx / kBK : idx % kTN, kk = bkf ? idx % kBK : idx / kTN;
-      const bool ok = x0 + cc < p.N && kb + kk < p.K;
-      cp_async8(bs + kk * kLdB + cc, ok ? p.Y + (kb + kk) * p.yk + (int64_t)(x0 + cc) * p.yx : p.Y, ok);
+      for (int u = 0; u < kTN * kBK / kThr; ++u) {
+        const int kk = tid / kTN + u * (kThr / kTN);
+        cp_async8(bs + kk * kLdB + xb, srcB0 + (kb + kk) * p.yk, okB0);
+      }
+    } else {
+      const int kk = tid % kBK;
+#pragma unroll
+      for (int u = 0; u < kTN * kBK / kThr; ++u) {
+        const int cc = tid / kBK + u * (kThr / kBK);
+        const bool ok = x0 + cc < p.N;
+        cp_async8(bs + kk * kLdB + cc, ok ? p.Y + (kb + kk) + (int64_t)(x0 + cc) * p.yx : p.Y, ok);
+      }
     }
   };
 #pragma unroll
@@ -376,7 +405,7 @@ int update_gemm_dmma(int which, char transX, char transY, double alpha, const do
                      const double* Y, int64_t ldy, double* C, int64_t ldcc, int64_t M2, int64_t N, int64_t K,
                      const double* Xm, int64_t ldxm, double* Cm, int64_t ldcm, cudaStream_t s) {
   if (M2 <= 0 || N <= 0) return 0;
-  if (N > (1LL << 30) || M2 > (1 << 20) || K > (1 << 20)) return ABFT_E_UNSUPPORTED;
+  if (N > (1LL << 30) || M2 > (1 << 20) || K > (1 << 20) || K % kBK) return ABFT_E_UNSUPPORTED;
   const bool tX = transX == 'T' || transX == 't', tY = transY == 'T' || transY == 't';
   const bool col = which == ABFT_COL;
   RuleArgs a{};
