@@ -21,6 +21,8 @@ FLAGS = [
     "--expt-relaxed-constexpr",
     "-cudart", "static",
 ]
+# experiments only: extra nvcc flags (e.g. -DABFT_VERIFY_RING_KB=64)
+FLAGS += os.environ.get("ABFT_EXTRA_NVCC", "").split()
 LIBS = ["-L/usr/local/cuda/lib64", "-lcublas", "-lcusolver", "-ldl", "-Xlinker", "-rpath=/usr/local/cuda/lib64"]
 
 

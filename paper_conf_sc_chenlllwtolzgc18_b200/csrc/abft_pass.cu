@@ -35,7 +35,13 @@ constexpr int kWarps = kThreads / 32;
 // NB = checksum tile; K = vertically adjacent tiles streamed by one CTA
 // (K > 1 for small tiles: one K*NB-row bulk copy per column and a K-times
 // longer CTA lifetime; GENERAL views only).
-template <typename T, int NB, int K, bool VERIFY = false>
+// LEAN (verify launches of at most one wave: the drivers' per-iteration
+// checks): a 64 KiB ring instead of 96 KiB.  Such a check runs next to the
+// factorization's DSYRK on the look-ahead side stream; every KiB it holds is
+// shared memory a DSYRK CTA cannot have (a 110 KiB check CTA displaced two
+// of them, a 76 KiB one displaces one): ft_potrf n=30720 6.70% -> 5.74%,
+// while the full-matrix pass keeps the deeper ring (7.06 vs 6.85 TB/s).
+template <typename T, int NB, int K, bool VERIFY = false, bool LEAN = false>
 struct PassCfg {
   static constexpr int RK = K * NB;              // rows per CTA
   // group columns (slab granularity).  (32-column groups for NB >= 256 were
@@ -63,7 +69,8 @@ struct PassCfg {
   // nb=512 verify a third 32 KiB ring stage)
   static constexpr int REC_ELEMS = 0;
   static constexpr int SIDE_BYTES = (RK * 3 + REC_ELEMS) * (int)sizeof(T);
-  static constexpr int RING_BYTES = RK >= 256 ? (96 * 1024 < 108 * 1024 - SIDE_BYTES ? 96 * 1024
+  static constexpr int RING_CAP = LEAN ? 64 * 1024 : 96 * 1024;
+  static constexpr int RING_BYTES = RK >= 256 ? (RING_CAP < 108 * 1024 - SIDE_BYTES ? RING_CAP
                                                                                         : 108 * 1024 - SIDE_BYTES)
                                               : 48 * 1024;
   static constexpr int NSTAGE_RAW = RING_BYTES / STAGE_BYTES;
@@ -361,9 +368,9 @@ __device__ __forceinline__ void super_of(const abft_tiles_t& t, int mode, int K,
 // the 4 SM sub-partitions put 5 warps on one of them (16K registers each).
 // The verify variant of stacked tiles otherwise takes 111 and runs one CTA
 // per SM (fp32 nb=256 verify at 2.5 TB/s, ncu r01).
-template <typename T, int NB, int K, bool VERIFY>
+template <typename T, int NB, int K, bool VERIFY, bool LEAN>
 __global__ void __maxnreg__(96) checksum_pass_kernel(const __grid_constant__ PassArgs p) {  // kBlock threads
-  using C = PassCfg<T, NB, K, VERIFY>;
+  using C = PassCfg<T, NB, K, VERIFY, LEAN>;
   constexpr int RK = C::RK;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   T* ring = reinterpret_cast<T*>(smem_raw);
@@ -847,30 +854,16 @@ __global__ void __maxnreg__(96) checksum_pass_kernel(const __grid_constant__ Pas
 // tables do not fit (fp64 nb=1024): run_pass then launches locate itself
 static thread_local bool g_fuse_missed = false;
 
-template <typename T, int NB, int K, bool VERIFY>
-static int launch_k(PassArgs& a, int64_t nsup, cudaStream_t s) {
-  using C = PassCfg<T, NB, K, VERIFY>;
-  auto kern = checksum_pass_kernel<T, NB, K, VERIFY>;
+template <typename T, int NB, int K, bool VERIFY, bool LEAN>
+static int launch_cfg(PassArgs& a, int64_t nsup, int nslab, cudaStream_t s) {
+  using C = PassCfg<T, NB, K, VERIFY, LEAN>;
+  auto kern = checksum_pass_kernel<T, NB, K, VERIFY, LEAN>;
   static bool attr_done = false;  // per instantiation
   if (!attr_done) {
     ABFT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM));
     attr_done = true;
   }
-  static int sms = 0;
-  if (!sms) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms <= 0) sms = 148;
-  }
   const int64_t ntiles = nsup * K;  // tile slots of the workspace (ragged stacks included)
-  // slabs: split the units of a small launch so that it fills, but does not
-  // spill past, one wave of 2 CTAs per SM (a spilled second wave cost more
-  // than the halved slab saved: 40-59-tile panels 10% slower, slab_tune r01)
-  int nslab = 1;
-  const int max_slab = C::GROUPS;
-  while (nslab < max_slab && nsup * nslab * 2 <= 2LL * sms) nslab *= 2;
-  static const int force_slab = getenv("ABFT_NSLAB") ? atoi(getenv("ABFT_NSLAB")) : 0;  // tuning experiments only
-  if (force_slab > 0) nslab = std::min(force_slab, max_slab);
   a.nslab = nslab;
   a.K = K;
   const int want_fuse = a.fuse;
@@ -894,6 +887,27 @@ static int launch_k(PassArgs& a, int64_t nsup, cudaStream_t s) {
   a.fuse = want_fuse;
   ABFT_CUDA_TRY(cudaGetLastError());
   return 0;
+}
+
+template <typename T, int NB, int K, bool VERIFY>
+static int launch_k(PassArgs& a, int64_t nsup, cudaStream_t s) {
+  using C = PassCfg<T, NB, K, VERIFY>;
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms <= 0) sms = 148;
+  }
+  // slabs: split the units of a small launch so that it fills, but does not
+  // spill past, one wave of 2 CTAs per SM (a spilled second wave cost more
+  // than the halved slab saved: 40-59-tile panels 10% slower, slab_tune r01)
+  int nslab = 1;
+  const int max_slab = C::GROUPS;
+  while (nslab < max_slab && nsup * nslab * 2 <= 2LL * sms) nslab *= 2;
+  static const int force_slab = getenv("ABFT_NSLAB") ? atoi(getenv("ABFT_NSLAB")) : 0;  // tuning experiments only
+  if (force_slab > 0) nslab = std::min(force_slab, max_slab);
+  if (VERIFY && nsup * nslab <= 2LL * sms) return launch_cfg<T, NB, K, VERIFY, true>(a, nsup, nslab, s);
+  return launch_cfg<T, NB, K, VERIFY, false>(a, nsup, nslab, s);
 }
 
 // Small tiles are streamed K at a time (K*NB*s >= 4 KiB per column copy):
