@@ -37,7 +37,10 @@ namespace {
 constexpr int kTM = 64;       // rows of A per CTA
 constexpr int kTN = 32;       // columns per CTA
 constexpr int kBK = 16;       // k per stage
-constexpr int kStages = 4;
+#ifndef ABFT_RULE_STAGES
+#define ABFT_RULE_STAGES 4
+#endif
+constexpr int kStages = ABFT_RULE_STAGES;
 constexpr int kThr = 128;     // 4 warps: 2 (m, 32 rows) x 2 (n, 16 columns)
 constexpr int kWM = 4;        // m-tiles per warp
 constexpr int kWN = 2;        // n-tiles per warp

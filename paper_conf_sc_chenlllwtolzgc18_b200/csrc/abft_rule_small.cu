@@ -33,7 +33,10 @@ namespace {
 
 constexpr int kVB = 32;   // vectors per cluster (rows of the product)
 constexpr int kJB = 32;   // output columns per CTA
-constexpr int kBK = 32;   // q per stage (16 measured: 32 dependent stages, 18 us per launch)
+#ifndef ABFT_SMALL_RULE_BK
+#define ABFT_SMALL_RULE_BK 16
+#endif
+constexpr int kBK = ABFT_SMALL_RULE_BK;  // q per stage (32: 73 KB of shared memory next to the DSYRK, ft_potrf 0.1-0.4 ms slower)
 constexpr int kStages = 4;
 constexpr int kThr = 128;  // 4 warps: 2 (vectors, 16 each) x 2 (columns, 16 each)
 constexpr int kLd = kVB + 4;  // stage row stride (doubles): 4 (mod 16) keeps fragments conflict-free
