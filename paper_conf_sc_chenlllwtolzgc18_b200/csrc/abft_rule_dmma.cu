@@ -165,16 +165,23 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
   const int xb = tid % kTN;
   const bool okB0 = !bkf && x0 + xb < p.N;
   const double* srcB0 = p.Y + (okB0 ? (int64_t)(x0 + xb) * p.yx : 0);
+  // running source pointers of the row- / column-fastest fills (fill() is
+  // called for k-steps 0, 1, 2, ... in order)
+  const int64_t sA = (int64_t)(kThr / kTM) * kA0, sB = (int64_t)(kThr / kTN) * p.yk;
+  const double* pA = srcA0 + ((int64_t)kbeg * kBK + tid / kTM) * kA0;
+  const double* pB = srcB0 + ((int64_t)kbeg * kBK + tid / kTN) * p.yk;
   auto fill = [&](int kt, int st) {
     const int64_t kb = (int64_t)(kbeg + kt) * kBK;
     double* as = As + (size_t)st * kBK * kLdA;
-    if (!akf) {
-      const int ra = tid % kTM;
+    if (!akf) {  // running pointer: one 64-bit add per load, compile-time smem offsets
+      double* ad = as + (tid / kTM) * kLdA + tid % kTM;
+      const double* ag = pA;
 #pragma unroll
       for (int u = 0; u < kTM * kBK / kThr; ++u) {
-        const int kk = tid / kTM + u * (kThr / kTM);
-        cp_async8(as + kk * kLdA + ra, srcA0 + (kb + kk) * kA0, okA0);
+        cp_async8(ad + u * (kThr / kTM) * kLdA, ag, okA0);
+        ag += sA;
       }
+      pA += sA * (kTM * kBK / kThr);
     } else {
       const int kk = tid % kBK;
 #pragma unroll 1
@@ -188,11 +195,14 @@ __global__ void __launch_bounds__(kThr, 4) syrk_rule_dmma_kernel(RuleArgs p) {
     }
     double* bs = Bs + (size_t)st * kBK * kLdB;
     if (!bkf) {
+      double* bd = bs + (tid / kTN) * kLdB + xb;
+      const double* bg = pB;
 #pragma unroll
       for (int u = 0; u < kTN * kBK / kThr; ++u) {
-        const int kk = tid / kTN + u * (kThr / kTN);
-        cp_async8(bs + kk * kLdB + xb, srcB0 + (kb + kk) * p.yk, okB0);
+        cp_async8(bd + u * (kThr / kTN) * kLdB, bg, okB0);
+        bg += sB;
       }
+      pB += sB * (kTN * kBK / kThr);
     } else {
       const int kk = tid % kBK;
 #pragma unroll
