@@ -172,7 +172,7 @@ int update_gemm_dmma(int which, char transX, char transY, double alpha, const do
                      const double* Xm, int64_t ldxm, double* Cm, int64_t ldcm, cudaStream_t s);
 // up to 3 gated products in one launch (same dtype and gate)
 int gemm_gated_multi(int32_t dtype, const GatedGemm* g, int n, const int32_t* gate, cudaStream_t s);
-// up to 4 2-D copies (as copy2d) in one launch; honours launch_gate()
+// up to 6 2-D copies (as copy2d) in one launch; honours launch_gate()
 struct Copy2D {
   void* dst;
   size_t dpitch;

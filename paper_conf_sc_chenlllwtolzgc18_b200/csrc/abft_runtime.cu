@@ -112,7 +112,7 @@ int copy2d(void* dst, size_t dpitch, const void* src, size_t spitch, size_t widt
 }
 
 struct CopyBatch {
-  Copy2D c[4];
+  Copy2D c[6];
   int n;
 };
 // blockIdx.z = copy; 8-byte words when every copy allows them (checksum
@@ -134,6 +134,7 @@ int copy2d_multi(const Copy2D* c, int n, cudaStream_t s) {
   CopyBatch b{};
   uintptr_t al = 0;
   size_t wmax = 0, hmax = 0;
+  if (n > 6) return ABFT_E_UNSUPPORTED;
   for (int i = 0; i < n; ++i) {
     if (c[i].width == 0 || c[i].height == 0) continue;
     b.c[b.n++] = c[i];

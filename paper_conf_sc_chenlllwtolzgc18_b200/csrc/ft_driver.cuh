@@ -10,6 +10,8 @@
 #include <cstring>
 #include <mutex>
 #include <string>
+#include <initializer_list>
+#include <tuple>
 #include <vector>
 
 #include "abft_common.cuh"
@@ -448,6 +450,18 @@ struct Driver {
   int copy(void* dst, int64_t ldd, const void* src, int64_t lds, int64_t rows, int64_t cols) {
     if (rows <= 0 || cols <= 0) return 0;
     return abft::copy2d(dst, ldd * es, src, lds * es, rows * es, cols, s);
+  }
+  // up to 6 such copies as one launch: (dst, ldd, src, lds, rows, cols) in elements
+  using CopySpec = std::tuple<void*, int64_t, const void*, int64_t, int64_t, int64_t>;
+  int copies(std::initializer_list<CopySpec> l) {
+    Copy2D cs[6];
+    int n = 0;
+    for (const CopySpec& t : l) {
+      if (n == 6) return ABFT_E_UNSUPPORTED;
+      cs[n++] = Copy2D{std::get<0>(t), (size_t)std::get<1>(t) * es, std::get<2>(t), (size_t)std::get<3>(t) * es,
+                       (size_t)std::get<4>(t) * es, (size_t)std::get<5>(t)};
+    }
+    return copy2d_multi(cs, n, s);
   }
   // f1 hooks: the fix-log position at the start of iteration k; the Fig. 4b
   // check (gated on a 1D fix since then); the periodic trailing check.

@@ -643,10 +643,9 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     const int64_t r0 = k * nb;
     if (ft) FT_TRY(d.begin_iteration());
     // Alg. 2 lines 3-4: check the column panel to be decomposed (c + r)
-    FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
-    if (ft) FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH));
     // Local restart (f1, L430): the column panel with its checksums is copied
-    // after its pre-op check; layout in rsv: panel | c | m_c | r | m_r
+    // after its pre-op check (the panel by the check's own pass); layout in
+    // rsv: panel | c | m_c | r | m_r
     const int64_t mk = n - r0;
     const int ntk = (int)(nt - k);
     char* rb = (char*)c->rsv;
@@ -655,13 +654,14 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     char* cp_m = cp_c + (size_t)2 * ntk * nb * d.es;
     char* cp_r = cp_m + (size_t)ntk * nb * d.es;
     char* cp_rm = cp_r + (size_t)mk * 2 * d.es;
+    FT_TRY(d.inject_at(k, FT_AT_PRE_PD_CHECK));
+    if (ft) FT_TRY(d.check(k, (int)nt, k, k + 1, ABFT_GENERAL, ABFT_BOTH, false, nullptr, rs ? cp_a : nullptr, mk));
     if (rs) {
       PhaseScope ps(d, FT_PH_RESTART);
-      FT_TRY(d.copy(cp_a, mk, d.a_at(r0, r0), lda, mk, nb));
-      FT_TRY(d.copy(cp_c, 2 * ntk, d.colchk_at(2 * k, r0), d.M.ldc, 2 * ntk, nb));
-      FT_TRY(d.copy(cp_m, ntk, d.colmag_at(k, r0), d.M.ldcm, ntk, nb));
-      FT_TRY(d.copy(cp_r, mk, d.rowchk_at(r0, 2 * k), d.M.ldr, mk, 2));
-      FT_TRY(d.copy(cp_rm, mk, d.rowmag_at(r0, k), d.M.ldrm, mk, 1));
+      FT_TRY(d.copies({{cp_c, 2 * ntk, d.colchk_at(2 * k, r0), d.M.ldc, 2 * ntk, nb},
+                       {cp_m, ntk, d.colmag_at(k, r0), d.M.ldcm, ntk, nb},
+                       {cp_r, mk, d.rowchk_at(r0, 2 * k), d.M.ldr, mk, 2},
+                       {cp_rm, mk, d.rowmag_at(r0, k), d.M.ldrm, mk, 1}}));
     }
     // line 5: PD with pivoting, swap rule, c(L), r(U_kk)
     auto do_pd = [&]() -> int {
@@ -688,11 +688,11 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
       auto pd_redo = [&]() -> int {  // 2D after the PD: undo its swaps, restore the copy, redo
         PhaseScope ps(d, FT_PH_RESTART);
         if (!split) FT_TRY(panel_getrf_undo(&d.M, k, s, perm));  // split: nothing outside the panel moved yet
-        FT_TRY(d.copy(d.a_at(r0, r0), lda, cp_a, mk, mk, nb));
-        FT_TRY(d.copy(d.colchk_at(2 * k, r0), d.M.ldc, cp_c, 2 * ntk, 2 * ntk, nb));
-        FT_TRY(d.copy(d.colmag_at(k, r0), d.M.ldcm, cp_m, ntk, ntk, nb));
-        FT_TRY(d.copy(d.rowchk_at(r0, 2 * k), d.M.ldr, cp_r, mk, mk, 2));
-        FT_TRY(d.copy(d.rowmag_at(r0, k), d.M.ldrm, cp_rm, mk, mk, 1));
+        FT_TRY(d.copies({{d.a_at(r0, r0), lda, cp_a, mk, mk, nb},
+                         {d.colchk_at(2 * k, r0), d.M.ldc, cp_c, 2 * ntk, 2 * ntk, nb},
+                         {d.colmag_at(k, r0), d.M.ldcm, cp_m, ntk, ntk, nb},
+                         {d.rowchk_at(r0, 2 * k), d.M.ldr, cp_r, mk, mk, 2},
+                         {d.rowmag_at(r0, k), d.M.ldrm, cp_rm, mk, mk, 1}}));
         return 0;
       };
       // (The PD redo stays a host decision: cuSOLVER's getrf cannot read a
@@ -725,17 +725,17 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
     const int m2 = (int)(2 * (nt - k - 1));
     char* rb = (char*)c->rsv;
     // line 8: check the row panel to be updated (c + r)
-    FT_TRY(d.inject_at(k, FT_AT_PRE_PU_CHECK));
-    if (ft) FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_BOTH));
-    // local restart copy of the row panel: A12 | r(A12) | m_r(A12)
+    // local restart copy of the row panel: A12 (by the check's own pass) |
+    // r(A12) | m_r(A12)
     char* pu_a = rb;
     char* pu_r = pu_a + (size_t)nb * nk * d.es;
     char* pu_rm = pu_r + (size_t)nb * m2 * d.es;
+    FT_TRY(d.inject_at(k, FT_AT_PRE_PU_CHECK));
+    if (ft) FT_TRY(d.check(k, k + 1, k + 1, (int)nt, ABFT_GENERAL, ABFT_BOTH, false, nullptr, rs ? pu_a : nullptr, nb));
     if (rs) {
       PhaseScope ps(d, FT_PH_RESTART);
-      FT_TRY(d.copy(pu_a, nb, d.a_at(r0, r1), lda, nb, nk));
-      FT_TRY(d.copy(pu_r, nb, d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, nb, m2));
-      FT_TRY(d.copy(pu_rm, nb, d.rowmag_at(r0, k + 1), d.M.ldrm, nb, m2 / 2));
+      FT_TRY(d.copies({{pu_r, nb, d.rowchk_at(r0, 2 * (k + 1)), d.M.ldr, nb, m2},
+                       {pu_rm, nb, d.rowmag_at(r0, k + 1), d.M.ldrm, nb, m2 / 2}}));
     }
     // Fig. 4b (L359): a 1D pattern fixed in this iteration -> check the trailing matrix
     if (ft) FT_TRY(d.fig4b_check(k + 1, (int)nt, k + 1, (int)nt, ABFT_GENERAL, ABFT_BOTH, false));

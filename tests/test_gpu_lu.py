@@ -190,6 +190,24 @@ def _gpu_getrf_rs(lib, ctx, A_np, nb, inject, restart):
     return host(A), ipiv.cpu().numpy() - 1, rc, stats
 
 
+# Two faults in one iteration: the first corrected by the pre-PD / pre-PU
+# check, the second forcing the restart of that op.  The restart restores
+# the input from the copy the check's own pass wrote (ft_driver.cuh
+# check(ckpt)), which must hold the corrected element as the oracle's does.
+LU_DOUBLE = [
+    [(1, dr.AT_PRE_PD_CHECK, dr.KIND_PERSIST, 0, 150, 70, (61,)), (1, dr.AT_PRE_PD, dr.KIND_PERSIST, 0, 130, 70, (60,))],
+    [(2, dr.AT_PRE_PU_CHECK, dr.KIND_PERSIST, 0, 130, 200, (60,)), (2, dr.AT_PRE_PU, dr.KIND_ONCHIP, 0, 140, 130, (60,))],
+]
+
+
+@pytest.mark.parametrize("lookahead", [True, False])
+@pytest.mark.parametrize("case", range(len(LU_DOUBLE)))
+def test_lu_restart_from_check_checkpoint(lib, ctx, case, lookahead):
+    A = si.general(256, seed=31)
+    so, sg = _compare(lib, ctx, A, 64, [dr.Inject(*c) for c in LU_DOUBLE[case]], lookahead=lookahead)
+    assert so.restarts == 1 and sg.restarts == so.restarts
+
+
 @pytest.mark.parametrize("k,point,kind,gi,gj,bit", [
     (1, dr.AT_PRE_PD, dr.KIND_PERSIST, 200, 66, 62),   # consumed by getrf, other pivots
     (1, dr.AT_PRE_PD, dr.KIND_PERSIST, 130, 70, 60),
