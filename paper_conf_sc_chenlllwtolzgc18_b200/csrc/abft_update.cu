@@ -633,10 +633,93 @@ __global__ void __launch_bounds__(256) panel_row_rule_kernel(int64_t rows, int n
   }
 }
 
+// The same rule with two rows per lane (16-B / 8-B vector loads: a warp
+// reads 64 consecutive rows of a column, 512 B for fp64) and 8 loads in
+// flight per lane; a block owns 64 rows.  The scalar version above ran the
+// n=30720 first-iteration panel (124 MB) at 3.0 TB/s, latency-bound (ncu:
+// 25 cycles per issued instruction, 43% occupancy).
+template <typename T, typename V2>
+__global__ void __launch_bounds__(256) panel_row_rule2_kernel(int64_t rows, int nb, const T* __restrict__ L,
+                                                              int64_t ldl, const T* __restrict__ ce,
+                                                              const T* __restrict__ cw, int64_t ldc,
+                                                              const T* __restrict__ mc, int64_t ldcm,
+                                                              T* __restrict__ re, T* __restrict__ rw,
+                                                              T* __restrict__ rm) {
+  __shared__ T sv[3][1024];
+  __shared__ T part[8][3][64];
+  for (int q = threadIdx.x; q < nb; q += blockDim.x) {
+    sv[0][q] = ce[(int64_t)q * ldc];
+    sv[1][q] = cw[(int64_t)q * ldc];
+    sv[2][q] = mc ? mc[(int64_t)q * ldcm] : T(0);
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t x = (int64_t)blockIdx.x * 64 + 2 * lane;  // this lane's rows x, x + 1
+  const int qn = nb / 8, q0 = warp * qn;
+  T se0 = T(0), sw0 = T(0), sm0 = T(0), se1 = T(0), sw1 = T(0), sm1 = T(0);
+  if (x < rows) {  // rows is even: both rows exist
+    const T* Lx = L + x + (int64_t)q0 * ldl;
+    for (int q = 0; q < qn; q += 8) {
+      V2 l[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (q + u < qn) l[u] = __ldg(reinterpret_cast<const V2*>(Lx + (int64_t)(q + u) * ldl));
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        if (q + u < qn) {
+          const T a = sv[0][q0 + q + u], b = sv[1][q0 + q + u], c = sv[2][q0 + q + u];
+          se0 = fma(l[u].x, a, se0);
+          sw0 = fma(l[u].x, b, sw0);
+          sm0 = fma(fabs(l[u].x), c, sm0);
+          se1 = fma(l[u].y, a, se1);
+          sw1 = fma(l[u].y, b, sw1);
+          sm1 = fma(fabs(l[u].y), c, sm1);
+        }
+      }
+    }
+  }
+  part[warp][0][2 * lane] = se0;
+  part[warp][1][2 * lane] = sw0;
+  part[warp][2][2 * lane] = sm0;
+  part[warp][0][2 * lane + 1] = se1;
+  part[warp][1][2 * lane + 1] = sw1;
+  part[warp][2][2 * lane + 1] = sm1;
+  __syncthreads();
+  // 64 rows x 3 sums, warp order (deterministic); threads 0..63 finish one row each
+  const int r = threadIdx.x;
+  const int64_t xr = (int64_t)blockIdx.x * 64 + r;
+  if (r < 64 && xr < rows) {
+    T e = T(0), w = T(0), m = T(0);
+#pragma unroll
+    for (int g = 0; g < 8; ++g) {
+      e += part[g][0][r];
+      w += part[g][1][r];
+      m += part[g][2][r];
+    }
+    re[xr] -= e;
+    rw[xr] -= w;
+    if (rm) rm[xr] += m;
+  }
+}
+
 int panel_row_rule(int32_t dtype, int64_t rows, int64_t nb, const void* L, int64_t ldl, const void* ce, const void* cw,
                    int64_t ldc, const void* mc, int64_t ldcm, void* re, void* rw, void* rm, cudaStream_t s) {
   if (rows <= 0) return 0;
   if (nb % 8 || nb > 1024) return ABFT_E_UNSUPPORTED;
+  const size_t es = dtype == ABFT_F64 ? 8 : 4;
+  if (rows % 2 == 0 && (uintptr_t)L % (2 * es) == 0 && (ldl * es) % (2 * es) == 0) {
+    const unsigned grid2 = (unsigned)((rows + 63) / 64);
+    if (dtype == ABFT_F64)
+      panel_row_rule2_kernel<double, double2><<<grid2, 256, 0, s>>>(
+          rows, (int)nb, (const double*)L, ldl, (const double*)ce, (const double*)cw, ldc, (const double*)mc, ldcm,
+          (double*)re, (double*)rw, (double*)rm);
+    else
+      panel_row_rule2_kernel<float, float2><<<grid2, 256, 0, s>>>(
+          rows, (int)nb, (const float*)L, ldl, (const float*)ce, (const float*)cw, ldc, (const float*)mc, ldcm,
+          (float*)re, (float*)rw, (float*)rm);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    return 0;
+  }
   const unsigned grid = (unsigned)((rows + 31) / 32);
   if (dtype == ABFT_F64)
     panel_row_rule_kernel<double><<<grid, 256, 0, s>>>(rows, (int)nb, (const double*)L, ldl, (const double*)ce,
