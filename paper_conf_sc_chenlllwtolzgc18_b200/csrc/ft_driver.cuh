@@ -59,6 +59,10 @@ struct ft_ctx {
   // private stream (high priority) and its events
   cudaStream_t side = nullptr;
   cudaEvent_t ev_col = nullptr, ev_side = nullptr;
+  // ft_potrf look-ahead: the TMU checksum rule of the trailing rest on its own
+  // stream, next to the DSYRK it does not depend on (ft_opts_t.rule_stream)
+  cudaStream_t rule = nullptr;
+  cudaEvent_t ev_rule = nullptr;
   void* putmp2 = nullptr;  // PU scratch of the side stream
   size_t putmp2_bytes = 0;
   std::vector<cudaEvent_t> evpool;  // opts->timing: per-phase span events (reused across calls)
@@ -179,6 +183,12 @@ struct Driver {
     ABFT_CUDA_TRY(cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, low ? lo : hi));
     ABFT_CUDA_TRY(cudaEventCreateWithFlags(&c->ev_col, cudaEventDisableTiming));
     ABFT_CUDA_TRY(cudaEventCreateWithFlags(&c->ev_side, cudaEventDisableTiming));
+    return 0;
+  }
+  int rule_setup() {
+    if (c->rule) return 0;
+    ABFT_CUDA_TRY(cudaStreamCreateWithFlags(&c->rule, cudaStreamNonBlocking));
+    ABFT_CUDA_TRY(cudaEventCreateWithFlags(&c->ev_rule, cudaEventDisableTiming));
     return 0;
   }
   int ctf_flagged = 0, ctf_recomputed = 0;
