@@ -903,10 +903,28 @@ extern "C" int ft_getrf(ft_ctx_t* c, int32_t dtype, int64_t n, void* dA, int64_t
         FT_TRY(recheck(k, r1, r2));
       }
       ABFT_CUDA_TRY(cudaEventRecord(c->ev_col, d.s));
+      // the rest's checksum rules on a stream of its own next to the DGEMM
+      // (they read the re-checked panels L21, U12 and their checksums and
+      // write the checksums of tile columns >= k+2, which neither the DGEMM
+      // nor the side chain's panel k+1 touches), joined before the re-check;
+      // runs with a fault plan keep Alg. 2's sequential order
+      static const bool rule_seq = getenv("ABFT_RULE_STREAM") && atoi(getenv("ABFT_RULE_STREAM")) == 0;
+      const bool par = ft && !rule_seq && o->n_inject == 0;
+      if (par) {
+        FT_TRY(d.rule_setup());
+        ABFT_CUDA_TRY(cudaStreamWaitEvent(c->rule, c->ev_col, 0));
+        cudaStream_t keep = d.s;
+        d.s = c->rule;
+        const int rc = tmu_chk(k, r2, n);
+        d.s = keep;
+        FT_TRY(rc);
+        ABFT_CUDA_TRY(cudaEventRecord(c->ev_rule, c->rule));
+      }
       FT_TRY(tmu_data(k, r2, n));
       if (ft) {
-        FT_TRY(tmu_chk(k, r2, n));
+        if (!par) FT_TRY(tmu_chk(k, r2, n));
         FT_TRY(d.inject_at(k, FT_AT_POST_TMU));
+        if (par) ABFT_CUDA_TRY(cudaStreamWaitEvent(d.s, c->ev_rule, 0));
         FT_TRY(recheck(k, r2, n));
       }
       ABFT_CUDA_TRY(cudaStreamWaitEvent(c->side, c->ev_col, 0));
