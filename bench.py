@@ -511,6 +511,9 @@ def potrf_overhead(abft, si, n, nb, reps, host_pd=True):
             "overhead_pct": 100.0 * (ft_ms - plain_ms) / plain_ms, "cusolver_potrf_ms": cus,
             "overhead_vs_cusolver_pct": 100.0 * (ft_ms - cus) / cus,
             "lookahead": True, "phases_ms": phases,
+            "phases_note": "device spans per phase on the stream each phase runs on; side-stream and rule-stream "
+                           "spans overlap the main stream (the trailing checksum rule interleaves with the DSYRK, "
+                           "so its span is about the DSYRK's)",
             "no_lookahead": {"ms_ft": nola_ft, "ms_plain": nola_plain,
                              "overhead_pct": 100.0 * (nola_ft - nola_plain) / nola_plain},
             "ms_ft_no_restart": nors_ms, "overhead_pct_no_restart": 100.0 * (nors_ms - plain_ms) / plain_ms,
