@@ -142,6 +142,17 @@ def test_restart_from_check_checkpoint(lib, ctx, case, lookahead):
     assert so.restarts >= 1 and sg.restarts == so.restarts
 
 
+def test_restart_from_check_checkpoint_nb1024(lib, ctx):
+    """fp64 nb=1024: the locate tables do not fit the pass kernel (separate
+    locate launch), and the check's copy of the PU input is patched by that
+    standalone locate (abft_pass.cu run_pass)."""
+    A = si.spd(4096, seed=0)
+    inj = [dr.Inject(1, dr.AT_PRE_PU_CHECK, dr.KIND_PERSIST, 0, 3000, 1500, (60,)),
+           dr.Inject(1, dr.AT_PRE_PU, dr.KIND_ONCHIP, 0, 1100, 1050, (60,))]
+    so, sg = _compare(lib, ctx, A, 1024, inj)
+    assert so.restarts == 1 and sg.restarts == 1
+
+
 # fp32 (every entry point takes ABFT_F32; BASELINE's 1e-5): the same fault
 # kinds with the flips moved into the fp32 word (fp64 bit b -> b - 32: the
 # exponent/sign bits stay exponent/sign bits, 52-54 become mantissa 20-22)
