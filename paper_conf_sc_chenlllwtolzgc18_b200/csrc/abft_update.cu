@@ -239,28 +239,45 @@ __global__ void __launch_bounds__(256) tri_inv_base_kernel(const T* __restrict__
     Xs[i][j] = (i == j) ? T(1) : T(0);
   }
   __syncthreads();
-  // column j of X = Ls^-1 by forward substitution, one thread per column, no
-  // barriers: x_j = 1 / l_jj, x_i = -(sum_{j<=k<i} l_ik x_k) / l_ii (i > j),
-  // the sum in four interleaved partial chains.  (The column-oriented
-  // elimination it replaces took two CTA barriers per step: 51 us per
-  // 512x512 inverse on B200, 8 CTAs of 64x64.)
-  const int j = tid;
-  if (j < bs) {
-    Xs[j][j] = T(1) / Ls[j][j];
-    for (int i = j + 1; i < bs; ++i) {
-      T a0 = T(0), a1 = T(0), a2 = T(0), a3 = T(0);
-      int k = j;
-      for (; k + 3 < i; k += 4) {
-        a0 = fma(Ls[i][k], Xs[k][j], a0);
-        a1 = fma(Ls[i][k + 1], Xs[k + 1][j], a1);
-        a2 = fma(Ls[i][k + 2], Xs[k + 2][j], a2);
-        a3 = fma(Ls[i][k + 3], Xs[k + 3][j], a3);
+  // X = Ls^-1 blocked inside the CTA: the 16x16 diagonal blocks by forward
+  // substitution (one thread per column), then the pairs merged level by
+  // level, X21 = -X22 (L21 X11), as products over all 256 threads (three
+  // barriers per level).  (A single forward substitution per column of the
+  // 64x64 block was a 64-long dependent chain per thread: 51 us per 512x512
+  // inverse, as was the column-oriented elimination before it.)
+  T* Tmp = &Xs[0][0] + (size_t)kInvBS * (kInvBS + 1);  // [bs * 16] products of one level
+  if (tid < bs) {
+    const int b0l = tid & ~15, col = tid;
+    Xs[col][col] = T(1) / Ls[col][col];
+    for (int i = col + 1; i < b0l + 16 && i < bs; ++i) {
+      T a0 = T(0), a1 = T(0);
+      int k = col;
+      for (; k + 1 < i; k += 2) {
+        a0 = fma(Ls[i][k], Xs[k][col], a0);
+        a1 = fma(Ls[i][k + 1], Xs[k + 1][col], a1);
       }
-      for (; k < i; ++k) a0 = fma(Ls[i][k], Xs[k][j], a0);
-      Xs[i][j] = -((a0 + a1) + (a2 + a3)) / Ls[i][i];
+      if (k < i) a0 = fma(Ls[i][k], Xs[k][col], a0);
+      Xs[i][col] = -(a0 + a1) / Ls[i][i];
     }
   }
   __syncthreads();
+  for (int h = 16; h < bs; h *= 2) {
+    const int hh = h * h, nout = (bs / (2 * h)) * hh;
+    for (int idx = tid; idx < nout; idx += blockDim.x) {  // Tmp_p = L21_p X11_p
+      const int pp = idx / hh, e = idx - pp * hh, r = e % h, c = e / h, o = 2 * h * pp;
+      T acc = T(0);
+      for (int t = c; t < h; ++t) acc = fma(Ls[o + h + r][o + t], Xs[o + t][o + c], acc);  // X11 lower
+      Tmp[idx] = acc;
+    }
+    __syncthreads();
+    for (int idx = tid; idx < nout; idx += blockDim.x) {  // X21_p = -X22_p Tmp_p
+      const int pp = idx / hh, e = idx - pp * hh, r = e % h, c = e / h, o = 2 * h * pp;
+      T acc = T(0);
+      for (int t = 0; t <= r; ++t) acc = fma(Xs[o + h + r][o + h + t], Tmp[pp * hh + t + c * h], acc);  // X22 lower
+      Xs[o + h + r][o + c] = -acc;
+    }
+    __syncthreads();
+  }
   for (int idx = tid; idx < bs * bs; idx += blockDim.x) {
     const int i = idx % bs, jj = idx / bs;
     if (upper)  // W = X^T
@@ -287,7 +304,7 @@ int tri_inverse_t(char uplo, char diag, int nb, const T* Tm, int ldt, T* W, int 
   const int bs = nb < kInvBS ? nb : kInvBS;
   if (nb % bs) return ABFT_E_UNSUPPORTED;
   ABFT_CUDA_TRY(cudaMemset2DAsync(W, (size_t)ldw * sizeof(T), 0, (size_t)nb * sizeof(T), nb, s));
-  const size_t smem = 2 * kInvBS * (kInvBS + 1) * sizeof(T);
+  const size_t smem = (2 * kInvBS * (kInvBS + 1) + (size_t)kInvBS * 16) * sizeof(T);
   static bool attr = false;
   if (!attr) {
     ABFT_CUDA_TRY(cudaFuncSetAttribute(tri_inv_base_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
