@@ -51,8 +51,8 @@ struct ft_ctx {
   int32_t* hpin_dev = nullptr;  // device alias of hpin (a kernel writes read-back words straight to the host)
   cudaEvent_t ev = nullptr;  // marks the PD-check read-back (restart decision)
   // The drivers run on a private non-blocking stream joined to `stream` at
-  // entry and exit: the device-decided restart captures its redo into a
-  // graph, and the legacy default stream cannot be captured.
+  // entry and exit (the look-ahead's side and rule streams fork from and join
+  // back into it; library handles and scratch are per stream).
   cudaStream_t drv = nullptr;
   cudaEvent_t join = nullptr;
   // look-ahead (the next panel's PD / PU next to the current TMU): a second
