@@ -20,7 +20,10 @@
 // (53 KB: 4 CTAs per SM); grid (Mt / 64, nk / 32), row tiles fastest so the
 // CTAs that share an L21 slice run together (a 64 x 64 tile with 32 x 32
 // warps measured no faster: 225 vs 212-231 us at ntk = 59, slower at 30).
-// Small grids split K over a cluster (below).  Summation order: one fixed DMMA chain per output
+// Small grids split K over a cluster (below).  (A bulk-copy fill — one
+// thread issuing a cp.async.bulk per k-row of the checksum rows and of B,
+// 32 small copies per stage on an mbarrier — measured 1.6x slower than the
+// per-thread 8-byte cp.async: 365 vs 230 us at ntk = 59.)  Summation order: one fixed DMMA chain per output
 // element over k ascending (deterministic; not the cuBLAS order, so P and Q
 // agree with the GEMM route to rounding, well inside the checks' tau).
 #include <cooperative_groups.h>
