@@ -19,6 +19,17 @@ import synth_inputs as si
 from paper_conf_sc_chenlllwtolzgc18_b200 import abft
 
 L2 = torch.cuda.get_device_properties(0).L2_cache_size
+try:  # SM clock right after each timed set (a record, not a filter)
+    import pynvml
+
+    pynvml.nvmlInit()
+    _nvh = pynvml.nvmlDeviceGetHandleByIndex(torch.cuda.current_device())
+
+    def sm_clock():
+        return pynvml.nvmlDeviceGetClockInfo(_nvh, pynvml.NVML_CLOCK_SM)
+except Exception:  # noqa: BLE001
+    def sm_clock():
+        return None
 flush = torch.empty(4 * L2, dtype=torch.uint8, device="cuda")
 evict = torch.empty(4 * L2 // 8, dtype=torch.float64, device="cuda")
 
@@ -69,11 +80,14 @@ def main():
                     small = bytes_pass < 16 * L2  # re-read after a (clean) flush below 2 GB
                     reps = 20 if n <= 16384 else 8
                     te = timed(lambda: abft.abft_encode(mat, t), reps, small)
+                    clk_e = sm_clock()
                     tv = timed(lambda: abft.abft_verify(mat, t, abft.BOTH, tol, rep), reps, small)
+                    clk_v = sm_clock()
                     assert int(rep.counts.sum().item()) == 0
                     rec = {"dtype": str(dt).split(".")[-1], "n": n, "nb": nb, "lower_only": lower,
                            "encode_GBs": bytes_pass / te / 1e6, "verify_GBs": bytes_pass / tv / 1e6,
-                           "encode_verify_GBs": 2 * bytes_pass / (te + tv) / 1e6, "l2_flushed": small}
+                           "encode_verify_GBs": 2 * bytes_pass / (te + tv) / 1e6, "l2_flushed": small,
+                           "sm_mhz_after_encode": clk_e, "sm_mhz_after_verify": clk_v}
                     if not lower:
                         V = torch.stack([torch.ones(nb, dtype=dt, device="cuda"),
                                          torch.arange(1, nb + 1, dtype=dt, device="cuda")], 1)
