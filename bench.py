@@ -2,8 +2,9 @@
 """Benchmark of the 2D weighted-checksum hot path (BASELINE.json metric:
 "checksum encode+verify GB/s vs HBM peak; ft_potrf overhead % at n=30720").
 
-One timed STEP = abft_encode + abft_verify + abft_locate_correct (a no-op
-launch when nothing is flagged) over the whole fp64 n=30720, nb=512 matrix
+One timed STEP = abft_encode + abft_check (verify with the locate / correct
+rounds fused into the same launch; they do nothing when no tile is flagged)
+over the whole fp64 n=30720, nb=512 matrix
 (7.55 GB per pass, larger than the 126 MB L2, so no flush is needed).  The
 ft_potrf overhead half of the metric is measured in the same run: the
 fault-tolerant driver (all §8(a) rows, Alg. 2 order) vs the same driver with
@@ -309,10 +310,9 @@ def run_ours(args):
         abft.abft_encode(mat, t_all)
         if ev:
             ev[1].record()
-        abft.abft_verify(mat, t_all, abft.BOTH, tol, rep)
+        abft.abft_check(mat, t_all, abft.BOTH, tol, rep, fixbuf, nfix)  # verify + fused locate
         if ev:
             ev[2].record()
-        abft.abft_locate_correct(mat, t_all, abft.BOTH, tol, rep, fixbuf, nfix)
         if world > 1:
             D.reduce_counts(rep.counts)  # error-report exchange (L361-L363)
 
@@ -421,7 +421,7 @@ def run_ours(args):
                          "encode_GBs": pass_bytes / (enc_ms / 1e3) / 1e9,
                          "verify_GBs": pass_bytes / (ver_ms / 1e3) / 1e9,
                          "torch_sum_GBs": read_only_gbs},
-            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": 3 * args.steps, "clocks": clk.summary(),
+            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": 2 * args.steps, "clocks": clk.summary(),
             "ft_potrf": ftp, "ft_getrf_geqrf": lq, "ft_potrf_mgpu": mg,
         }
         print(json.dumps(line), flush=True)
