@@ -174,14 +174,12 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
         lcol_idx.append((len(srcs), per))
 
     def check(m, tl, which):
-        abft.abft_verify(m, tl, which, tol, rep)
-        abft.abft_locate_correct(m, tl, which, tol, rep, fixes, nfix)
+        abft.abft_check(m, tl, which, tol, rep, fixes, nfix)  # verify + fused locate, one launch
 
     def check_recv(m, tl, acc):
         """Post-broadcast check of a received copy (L355) into the round's
         counters `acc` (added to the run's totals once the round is decided)."""
-        abft.abft_verify(m, tl, abft.COL, tol, rep_b)
-        abft.abft_locate_correct(m, tl, abft.COL, tol, rep_b, fixes, nfix)
+        abft.abft_check(m, tl, abft.COL, tol, rep_b, fixes, nfix)
         acc.add_(rep_b.counts)
         rep_b.counts.zero_()
 
@@ -436,9 +434,7 @@ def ft_potrf_mgpu(A_loc: torch.Tensor, lay: Layout, abft_on=True, tol_scale=1.0,
             if abft_on:
                 before = nfix.clone()
                 for buf in (Lrow, Lcol):
-                    abft.abft_verify(buf.mat(), abft.tiles(0, buf.cnt, 0, 1), abft.COL, tol, rep_b)
-                    abft.abft_locate_correct(buf.mat(), abft.tiles(0, buf.cnt, 0, 1), abft.COL, tol, rep_b, fixes,
-                                             nfix)
+                    abft.abft_check(buf.mat(), abft.tiles(0, buf.cnt, 0, 1), abft.COL, tol, rep_b, fixes, nfix)
                 consumed.add_(nfix - before)
                 cb_total.add_(rep_b.counts)
                 rep_b.counts.zero_()
