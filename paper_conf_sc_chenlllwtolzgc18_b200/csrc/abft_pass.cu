@@ -906,7 +906,9 @@ static int launch_k(PassArgs& a, int64_t nsup, cudaStream_t s) {
   while (nslab < max_slab && nsup * nslab * 2 <= 2LL * sms) nslab *= 2;
   static const int force_slab = getenv("ABFT_NSLAB") ? atoi(getenv("ABFT_NSLAB")) : 0;  // tuning experiments only
   if (force_slab > 0) nslab = std::min(force_slab, max_slab);
-  if (VERIFY && nsup * nslab <= 2LL * sms) return launch_cfg<T, NB, K, VERIFY, true>(a, nsup, nslab, s);
+  if constexpr (VERIFY) {
+    if (nsup * nslab <= 2LL * sms) return launch_cfg<T, NB, K, VERIFY, true>(a, nsup, nslab, s);
+  }
   return launch_cfg<T, NB, K, VERIFY, false>(a, nsup, nslab, s);
 }
 
